@@ -1,0 +1,352 @@
+#!/usr/bin/env python
+"""FastPSO hot-path benchmark (BASELINE.json metric: particle-dim updates/sec and
+% of HBM roofline at 1/2/4/8 B200).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--workload NS|C1|C2|C3|C4|C5]
+    python -m torch.distributed.run --nproc-per-node N ... bench.py --gpus N ...
+    python bench.py --impl reference ...   # the CPU oracle on a bounded sample
+
+A "step" is one PSO iteration over the whole swarm: the fused kernel (move,
+evaluate, pbest, gbest) plus, for N > 1, the NCCL all-gather + select of the
+gbest exchange.  Default workload: the north_star swarm, Rastrigin 100,000
+particles x 2,000 dims (2.4 GB of fp32 state, larger than the 126 MB L2, so no
+L2 flush is needed between steps).  N > 1 splits the same swarm by particles
+(strong scaling).  Prints ONE JSON line on rank 0.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+from synth import OBJ_NAMES, WORKLOADS  # noqa: E402
+
+METRIC = "particle-dim updates/sec and % of HBM roofline at 1/2/4/8 B200"
+UNIT = "particle-dim updates/s"
+L2_BYTES = 126 * 2**20
+FALLBACK_HBM_GBS = 6650.0  # B200_PROFILING.md fallback, used only without MEASURED_PEAKS.json
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=1000)
+    ap.add_argument("--warmup", type=int, default=20)
+    ap.add_argument("--workload", default="NS", choices=sorted(WORKLOADS))
+    ap.add_argument("--impl", default="fastpso", choices=["fastpso", "reference"])
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-seconds", type=float, default=15.0,
+                    help="CPU budget of the cpu_baseline oracle sample")
+    return ap.parse_args()
+
+
+def hbm_peak():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        with open(p) as fh:
+            return float(json.load(fh)["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    except Exception:
+        return FALLBACK_HBM_GBS, "fallback (B200_PROFILING.md)"
+
+
+def ncu_traffic(workload_name):
+    """DRAM bytes per launch of the step kernel from the committed ncu --set full summary."""
+    p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    try:
+        with open(p) as fh:
+            return json.load(fh).get(workload_name)
+    except Exception:
+        return None
+
+
+# ------------------------------------------------------------------ clocks
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled during the timed region."""
+
+    FIELDS = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+              "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, device: int):
+        self.device = device
+        self.proc = None
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.device), f"--query-gpu={self.FIELDS}",
+                 "--format=csv,noheader,nounits", "-lms", "100"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            time.sleep(0.3)
+        except Exception:
+            self.proc = None
+        return self
+
+    def __exit__(self, *exc):
+        self.result = None
+        if self.proc is None:
+            return
+        time.sleep(0.15)
+        self.proc.terminate()
+        try:
+            out, _ = self.proc.communicate(timeout=5)
+        except Exception:
+            self.proc.kill()
+            out = ""
+        sm, mx, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for line in out.splitlines():
+            parts = [p.strip() for p in line.split(",")]
+            if len(parts) < 7:
+                continue
+            try:
+                sm.append(float(parts[0]))
+                mx.append(float(parts[1]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, parts[3:7]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        if sm:
+            self.result = {"sm_mhz": statistics.median(sm), "sm_max_mhz": max(mx),
+                           "reasons": sorted(reasons), "samples": len(sm)}
+
+
+# ------------------------------------------------------------------ CPU oracle
+def oracle_sample(w, budget_s: float, steps_hint: int | None = None):
+    """Time the oracle (as it stands) on a bounded sample of workload w:
+    the first rows of the same swarm (same d, objective, parameters), stepping
+    `k` iterations.  Returns (rate, seconds, description, (rows, k, sec/step))."""
+    import oracle as orc
+    rows = 64
+    probe = orc.OracleSwarm(rows, w.d, w.w, w.c1, w.c2, w.lo, w.hi, w.objective, w.seed,
+                            vmax=w.vmax)
+    t0 = time.perf_counter()
+    probe.step(1)
+    per_elem = (time.perf_counter() - t0) / (rows * w.d)
+    if steps_hint is None:
+        k = 5
+        rows = max(1, min(w.n, int(budget_s / (per_elem * w.d * k))))
+    else:
+        k = steps_hint
+        rows = max(1, min(w.n, int(budget_s / (per_elem * w.d * k))))
+    s = orc.OracleSwarm(rows, w.d, w.w, w.c1, w.c2, w.lo, w.hi, w.objective, w.seed, vmax=w.vmax)
+    return s, rows, k
+
+
+def cpu_baseline(w, budget_s: float):
+    s, rows, k = oracle_sample(w, budget_s)
+    t0 = time.perf_counter()
+    s.step(k)
+    dt = time.perf_counter() - t0
+    rate = rows * w.d * k / dt
+    return {"value": rate, "unit": UNIT, "cores": 1, "kind": "oracle",
+            "sample": f"oracle (single-threaded C++ -O3 -ffp-contract=off) on the first {rows} of "
+                      f"{w.n} particles x {w.d} dims, {k} iterations ({dt:.1f} s), create excluded",
+            "host_cpu": _cpu_model()}
+
+
+def _cpu_model():
+    try:
+        with open("/proc/cpuinfo") as fh:
+            for line in fh:
+                if line.startswith("model name"):
+                    return line.split(":", 1)[1].strip() + f" ({os.cpu_count()} logical cpus)"
+    except Exception:
+        pass
+    return None
+
+
+def run_reference(args, w):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    K, W = args.steps, args.warmup
+    budget = 150.0  # whole --steps K --warmup W run
+    s, rows, _ = oracle_sample(w, budget / max(K + W, 1), steps_hint=1)
+    s.step(W)
+    t0 = time.perf_counter()
+    s.step(K)
+    dt = time.perf_counter() - t0
+    rate = rows * w.d * K / dt
+    sample = (f"oracle (single-threaded C++ -O3 -ffp-contract=off) on the first {rows} of {w.n} "
+              f"particles x {w.d} dims; {W} warm-up + {K} timed iterations ({dt:.1f} s)")
+    line = {
+        "impl": "reference", "metric": METRIC, "value": rate, "unit": UNIT,
+        "n_gpus": args.gpus, "steps": K, "warmup": W, "ms_per_step": dt * 1e3 / K,
+        "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f32",
+        "data": "synthetic", "config": _config(w, args.gpus, K, extra={"sample_rows": rows}),
+        "cpu_baseline": {"value": rate, "unit": UNIT, "cores": 1, "kind": "oracle",
+                         "sample": sample, "host_cpu": _cpu_model()},
+        "e2e": {"value": rate, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def _config(w, n_gpus, K, extra=None):
+    state = 3 * w.n * w.d * 4
+    cfg = {"workload": w.name, "objective": OBJ_NAMES[w.objective], "n": w.n, "d": w.d,
+           "w": w.w, "c1": w.c1, "c2": w.c2, "lo": w.lo, "hi": w.hi,
+           "vmax": w.vmax if w.vmax > 0 else 1.0, "seed": w.seed, "timed_iterations": K,
+           "parallelism": f"particle-split x{n_gpus}" if n_gpus > 1 else "single GPU",
+           "l2": ("inputs larger than L2 (%.2f GB state vs 126 MB L2); no flush" % (state / 1e9))
+           if state / max(n_gpus, 1) > L2_BYTES else
+           ("state (%.1f MB/GPU) fits in L2: L2-resident, not an HBM number" % (state / n_gpus / 1e6))}
+    if extra:
+        cfg.update(extra)
+    return cfg
+
+
+# ------------------------------------------------------------------ GPU arm
+def run_gpu(args, w):
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_icpp_liuwc21_b200 as fp
+    from paper_conf_icpp_liuwc21_b200.distributed import destroy_comm, init_comm
+
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world != args.gpus:
+        raise SystemExit(f"--gpus {args.gpus} but WORLD_SIZE={world}")
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    comm = None
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+        comm = init_comm(local)
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    def max_over_ranks(x: float) -> float:
+        if world == 1:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    stream = torch.cuda.Stream(device=dev)  # the library enqueues on this stream
+    torch.cuda.set_stream(stream)
+    K, W = args.steps, args.warmup
+    sw = fp.Swarm(w.n, w.d, w.w, w.c1, w.c2, w.lo, w.hi, w.objective, w.seed, vmax=w.vmax,
+                  device=local, stream=stream, nccl_comm=comm, timing=True)
+    sw.step(W)
+    sw.synchronize()
+    sw.reset_counters()
+
+    # ---------------- device-timed region
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with ClockSampler(local) as clk:
+        barrier()
+        ev0.record(stream)
+        sw.step(K)
+        ev1.record(stream)
+        barrier()
+    ms = max_over_ranks(ev0.elapsed_time(ev1))
+    info = sw.info()
+    kern_ms = max_over_ranks(info["step_kernel_ms"] / max(info["step_kernel_count"], 1))
+    launches = int(info["launches"])
+    improvements = info["improvements"]
+    n_local = info["n_local"]
+    gf, gi, _ = sw.gbest(pos=False)
+
+    total_updates = w.n * w.d * K
+    value = total_updates / (ms / 1e3)
+    rho = improvements / max(n_local * K, 1)
+    # algorithmic bytes per launch of the step kernel
+    bytes_per_update = 20.0 + 4.0 * rho
+    alg_bytes = n_local * w.d * bytes_per_update + n_local * (4.0 + 4.0 * rho)
+    achieved = alg_bytes / (kern_ms / 1e3) / 1e9
+    peak, peak_src = hbm_peak()
+
+    # ---------------- end to end through the public API, host buffers
+    e2e = None
+    clk_e2e = None
+    if not args.no_e2e:
+        X = torch.empty((n_local, w.d), dtype=torch.float32).pin_memory()
+        V = torch.empty_like(X).pin_memory()
+        PB = torch.empty_like(X).pin_memory()
+        pf = torch.empty((n_local,), dtype=torch.float32).pin_memory()
+        _, _, _, _, t_ck = sw.get_state(out=(X, V, PB, pf))  # a host checkpoint of the swarm
+        sw.close()
+        sw2 = fp.Swarm(w.n, w.d, w.w, w.c1, w.c2, w.lo, w.hi, w.objective, w.seed, vmax=w.vmax,
+                       device=local, stream=stream, nccl_comm=comm)
+        gpos = torch.empty((w.d,), dtype=torch.float32).pin_memory()
+        with ClockSampler(local) as clk2:
+            barrier()
+            t0 = time.perf_counter()
+            sw2.set_state(X, V, PB, pf, t=t_ck)  # H2D of the whole swarm state
+            sw2.step(K)
+            res = sw2.gbest(out=gpos)            # D2H of the result (synchronises)
+            barrier()
+            e2e_s = max_over_ranks(time.perf_counter() - t0)
+        clk_e2e = clk2.result
+        sw2.close()
+        h2d = 3 * n_local * w.d * 4 + n_local * 4
+        d2h = 4 + 8 + 4 * w.d
+        e2e = {"value": total_updates / e2e_s, "unit": UNIT,
+               "h2d_bytes_per_step": h2d / K, "d2h_bytes_per_step": d2h / K,
+               "seconds": e2e_s,
+               "path": "pso_set_state(pinned host X,V,PB,pf) + pso_step(K) + pso_get_gbest(pinned host)",
+               "gbest": res[0]}
+    else:
+        sw.close()
+    if comm:
+        destroy_comm(comm)
+
+    line = None
+    if rank == 0:
+        cpu = None
+        if world == 1 and not args.no_cpu_baseline:
+            cpu = cpu_baseline(w, args.cpu_seconds)
+        state_per_gpu = 3 * n_local * w.d * 4
+        line = {
+            "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": K,
+            "warmup": W, "ms_per_step": ms / K, "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None, "dtype": "f32",
+            "data": "synthetic (swarm initialised from Philox streams, seed %d)" % w.seed,
+            "config": _config(w, world, K),
+            "gpu_launches": launches,
+            "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                         "frac": achieved / peak, "peak_source": peak_src,
+                         "traffic": ncu_traffic(w.name),
+                         "kernel": "k_step (fused move+eval+pbest+gbest)",
+                         "kernel_avg_us": kern_ms * 1e3,
+                         "bytes_per_update": bytes_per_update, "rho": rho,
+                         "alg_bytes_per_launch": alg_bytes,
+                         "l2_resident": state_per_gpu <= L2_BYTES,
+                         "cta": {"threads": info["threads_per_cta"], "vpt": info["vec_per_thread"],
+                                 "grid": info["grid"], "ctas_per_sm": info["ctas_per_sm"]}},
+            "clocks": clk.result, "e2e": e2e, "clocks_e2e": clk_e2e,
+            "cpu_baseline": cpu, "gbest": {"fitness": gf, "index": gi},
+        }
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+    return 0
+
+
+def main():
+    args = parse()
+    w = WORKLOADS[args.workload]
+    if args.impl == "reference":
+        return run_reference(args, w)
+    return run_gpu(args, w)
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -1,0 +1,200 @@
+/*
+ * fastpso.h — C ABI of the B200-native FastPSO hot path.
+ *
+ * The library runs the per-iteration swarm update of FastPSO (Liu, Wen, Cai,
+ * ICPP'21) as ONE fused sm_100a kernel per iteration: counter-based random
+ * weights, the velocity/position update, the objective evaluation, the pbest
+ * compare-and-copy and the gbest argmin.  Citations are PAPER.md lines (P:Lnnn):
+ *
+ *   Alg. 1, P:L81-103   inputs n, omega, c1, c2, max_iter; output "the optimal
+ *                       positions of the particles"
+ *   Eq. 1,  P:L105-109  v' = omega v + c1 l (.) (pbest - p) + c2 g (.) (gbest - p)
+ *   Eq. 2,  P:L111-115  p' = p + v'
+ *   Eq. 4,  P:L171-253  the same on the n x d matrices V, P, L, G, E_l, E_g
+ *   Eq. 5,  P:L255-265  user-defined velocity bounds (here: |v| <= vmax)
+ *   Sec 3.1 P:L135      random swarm initialisation and per-iteration L, G
+ *   Sec 3.2 P:L137-147  swarm evaluation; user-defined evaluation schema
+ *   Sec 3.3 P:L149-153  pbest update; gbest = min and its index by reduction
+ *   P:L281              multi-GPU by particle splitting (made synchronous here)
+ *   P:L667              one cached device allocation (one arena per handle)
+ *
+ * Conventions (all entry points):
+ *   - Every call returns a pso_status; nothing aborts or throws across the ABI.
+ *     pso_last_error() gives a thread-local detail string for the last failure.
+ *   - Host buffers are owned by the caller, dense row-major (rows of d floats,
+ *     no padding).  Device memory is owned by the handle (one arena).
+ *   - pso_step only enqueues work on the handle's stream.  Launch errors are
+ *     returned at once; asynchronous faults surface at the next synchronising
+ *     call (pso_get_gbest / pso_get_state / pso_get_info / pso_synchronize).
+ *   - After any CUDA or NCCL error the handle is POISONED: every later call
+ *     except pso_destroy returns PSO_ERR_POISONED.
+ *   - A handle is not thread-safe; different handles are independent.
+ *   - Multi-GPU (opts.nccl_comm != NULL, world k > 1): n is the GLOBAL swarm
+ *     size, rank r owns global rows [floor(n r / k), floor(n (r+1) / k)).  All
+ *     calls except get_* / destroy are collective: every rank must make the
+ *     same sequence.  The gbest is bitwise identical on every rank, and every
+ *     result is bitwise independent of k.
+ *   - Determinism: the same arguments and seed give bitwise identical results;
+ *     pso_step(h, a); pso_step(h, b) is bitwise pso_step(h, a + b).
+ *   - Numerics: fp32 state; the update (Eq. 1, 5, 2) is evaluated in the fixed
+ *     order a = w*v; b = (c1*r1)*(pb-x); c = (c2*r2)*(g-x); v' = (a+b)+c,
+ *     v' = clamp(v', -vmax, vmax), x' = clamp(x + v', lo, hi), each op rounded
+ *     once (no FMA contraction).  Fitness is fp32 (tree-reduced per particle).
+ */
+#ifndef FASTPSO_H
+#define FASTPSO_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define FASTPSO_VERSION_MAJOR 0
+#define FASTPSO_VERSION_MINOR 1
+#define PSO_D_MAX 8192 /* max dimension held per fused row (one CTA per row) */
+
+typedef struct pso_swarm* pso_handle; /* opaque; owns all device memory */
+
+typedef enum {
+  PSO_OK = 0,
+  PSO_ERR_INVALID = 1,     /* bad argument (nothing was changed) */
+  PSO_ERR_NOMEM = 2,       /* device (or host) allocation failed */
+  PSO_ERR_CUDA = 3,        /* CUDA runtime error (handle is poisoned) */
+  PSO_ERR_NCCL = 4,        /* NCCL error or NCCL unavailable (poisoned) */
+  PSO_ERR_UNSUPPORTED = 5, /* valid but not supported (e.g. d > PSO_D_MAX) */
+  PSO_ERR_POISONED = 6     /* an earlier CUDA/NCCL error poisoned the handle */
+} pso_status;
+
+/* Objectives (Sec 3.2).  Definitions (k = 1..d):
+ *   SPHERE      sum x_k^2
+ *   RASTRIGIN   sum (x_k^2 + 10 - 10 cos(2 pi x_k))               ([20])
+ *   ROSENBROCK  sum_{k<d} 100 (x_{k+1} - x_k^2)^2 + (x_k - 1)^2   ([20])
+ *   GRIEWANK    1 + sum x_k^2 / 4000 - prod cos(x_k / sqrt(k))
+ *   ACKLEY      -20 exp(-0.2 sqrt(sum x^2/d)) - exp(sum cos(2 pi x)/d) + 20 + e
+ *               ([20]); compiled through the user-functor schema
+ *               (csrc/user_objectives.cuh), as a user objective would be
+ *   EASOM       -(-1)^d prod cos^2(x_k) exp(-sum (x_k - pi)^2)
+ * Ids >= PSO_OBJ_CUSTOM_BASE are user functors registered at compile time in
+ * csrc/user_objectives.cuh (the paper's evaluation_kernel<L> schema,
+ * P:L139-145, realised as compile-time device functors). */
+enum {
+  PSO_OBJ_SPHERE = 1,
+  PSO_OBJ_RASTRIGIN = 2,
+  PSO_OBJ_ROSENBROCK = 3,
+  PSO_OBJ_GRIEWANK = 4,
+  PSO_OBJ_ACKLEY = 5,
+  PSO_OBJ_EASOM = 6,
+  PSO_OBJ_CUSTOM_BASE = 64
+};
+
+/* Option flags. */
+enum {
+  PSO_FLAG_TIMING = 1 /* record CUDA events around every step kernel launch;
+                         totals are reported by pso_get_info */
+};
+
+/* Options; a zero-initialised struct means "defaults". */
+typedef struct {
+  float vmax;      /* Eq. 5 bound |v| <= vmax; <= 0 -> 1.0 (reading 3) */
+  int32_t device;  /* CUDA ordinal; < 0 -> the caller's current device.  NOTE:
+                      zero-initialised means device 0 unless set to -1 */
+  void* stream;    /* cudaStream_t to enqueue on; NULL -> a library-owned stream */
+  void* nccl_comm; /* ncclComm_t (see pso_nccl_comm_init); NULL -> single GPU */
+  uint32_t flags;  /* PSO_FLAG_* */
+} pso_opts;
+
+/* Create a swarm of n particles in d dimensions and initialise it (Alg. 1
+ * lines 1-3, Sec 3.1): x0 ~ U[lo, hi], v0 ~ U[-vmax, vmax] from the Philox
+ * streams keyed on (seed, particle, dim); the first evaluation; pbest = x0;
+ * gbest = the lowest index attaining min f(x0).
+ *   out        receives the handle (set to NULL on failure)
+ *   n          global swarm size, 1 <= n < 2^32
+ *   d          dimension, 1 <= d <= PSO_D_MAX (else PSO_ERR_UNSUPPORTED)
+ *   w, c1, c2  Eq. 1 parameters, finite
+ *   lo < hi    finite domain bounds; positions are clamped to [lo, hi]
+ *   objective  PSO_OBJ_* or a registered custom id (else PSO_ERR_INVALID)
+ *   seed       64-bit Philox key
+ * Blocks until initialisation has completed (errors are reported here). */
+pso_status pso_create(pso_handle* out, int64_t n, int32_t d, float w, float c1, float c2,
+                      float lo, float hi, int32_t objective, uint64_t seed);
+pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c1, float c2,
+                         float lo, float hi, int32_t objective, uint64_t seed,
+                         const pso_opts* opts);
+
+/* Enqueue iters >= 0 iterations; each is one fused kernel: move (Eq. 1, 5,
+ * 2), evaluate (Sec 3.2), pbest (Sec 3.3, strict <) and gbest (strict <,
+ * lowest index among equal new minima).  With world > 1 each iteration adds
+ * one NCCL all-gather of (key, candidate row) and a select kernel. */
+pso_status pso_step(pso_handle h, int64_t iters);
+
+/* Wait for all enqueued work and report asynchronous errors. */
+pso_status pso_synchronize(pso_handle h);
+
+/* Synchronise and read the global best: fitness, global particle index, and
+ * (if pos != NULL) its d-float position.  Any output pointer may be NULL.
+ * Host pointers.  Identical bits on every rank. */
+pso_status pso_get_gbest(pso_handle h, float* fitness, int64_t* index, float* pos);
+
+/* Synchronise and copy the rank-local state to host buffers (any may be NULL):
+ * x, v, pb: n_local x d floats; pf: n_local floats; t: iterations done. */
+pso_status pso_get_state(pso_handle h, float* x, float* v, float* pb, float* pf, uint64_t* t);
+
+/* Replace the rank-local state from host buffers (all required: x, v, pb are
+ * n_local x d, pf is n_local; NaN pf is read as +inf) and set the iteration
+ * counter to t.  The gbest is recomputed from pf/pb exactly as after create.
+ * Collective when world > 1.  Synchronous. */
+pso_status pso_set_state(pso_handle h, const float* x, const float* v, const float* pb,
+                         const float* pf, uint64_t t);
+
+/* Information and counters. */
+typedef struct {
+  int64_t n, n_local, row_begin; /* global size, local rows, first global row */
+  int32_t d, pitch;              /* dimension, row pitch in floats (16-B rows) */
+  int32_t rank, world;
+  int32_t threads_per_cta, vec_per_thread, grid, ctas_per_sm;
+  float vmax;
+  uint64_t t;                    /* iterations done */
+  uint64_t launches;             /* kernels launched by this handle so far */
+  uint64_t improvements;         /* pbest improvements (rows) so far, all steps */
+  double step_kernel_ms;         /* PSO_FLAG_TIMING: summed step-kernel time */
+  uint64_t step_kernel_count;    /* PSO_FLAG_TIMING: step kernels timed */
+  size_t arena_bytes;            /* device bytes owned by the handle */
+} pso_info;
+pso_status pso_get_info(pso_handle h, pso_info* info);
+/* Reset launches / improvements / timing counters. */
+pso_status pso_reset_counters(pso_handle h);
+
+/* Destroy the handle and free its device memory.  NULL-safe. */
+void pso_destroy(pso_handle h);
+
+const char* pso_status_string(pso_status s);
+const char* pso_last_error(void);
+/* 1 if objective id is compiled in, else 0. */
+int pso_objective_registered(int32_t objective);
+
+/* --- NCCL plumbing for the particle-split multi-GPU path --------- *
+ * NCCL is resolved at run time (dlopen of libnccl.so.2, or $PSO_NCCL_LIB), so
+ * the library has no link-time NCCL dependency; inside a PyTorch process this
+ * is the NCCL torch already loaded.  id is a 128-byte ncclUniqueId blob. */
+pso_status pso_nccl_get_unique_id(void* id128);
+pso_status pso_nccl_comm_init(void** comm, int32_t nranks, const void* id128, int32_t rank,
+                              int32_t device);
+pso_status pso_nccl_comm_destroy(void* comm);
+
+/* --- Device-side primitives exposed for parity tests ---------------------- */
+/* out[k] = word(tag, t, i, j0 + k) computed on the device (k < m), with the
+ * library's Philox (use_curand = 0) or with curand_Philox4x32_10 (1).
+ * word(tag,t,i,j) = Philox4x32-10(ctr = {j>>2, i, t, tag}, key = {seed lo, hi})[j&3]. */
+pso_status pso_debug_philox(uint64_t seed, uint32_t tag, uint32_t t, uint32_t i, uint32_t j0,
+                            int64_t m, uint32_t* out, int32_t use_curand, int32_t device);
+/* Evaluate m rows (dense m x d host matrix X) on the device with the same
+ * functor + CTA reduction the fused kernel uses; out receives m floats. */
+pso_status pso_debug_objective(int32_t objective, const float* X, int64_t m, int32_t d,
+                               float* out, int32_t device);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* FASTPSO_H */

@@ -1,0 +1,675 @@
+// api.cpp — the C ABI of include/fastpso.h: validation, the per-handle device
+// arena (the paper's GPU memory caching: one allocation reused for the
+// whole run), the iteration loop of Alg. 1 as kernel launches,
+// the synchronous particle-split gbest exchange over NCCL, state I/O,
+// counters and error handling.
+#include "fastpso.h"
+
+#include <cuda_runtime.h>
+#include <dlfcn.h>
+
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <limits>
+#include <string>
+#include <utility>
+#include <vector>
+
+#include "kernels.h"
+
+using namespace fastpso;
+
+namespace {
+
+thread_local std::string g_last_error;
+
+pso_status fail(pso_status s, const char* fmt, ...) {
+  char buf[512];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof(buf), fmt, ap);
+  va_end(ap);
+  g_last_error = buf;
+  return s;
+}
+
+// ------------------------------------------------------------ NCCL (dlopen)
+// Minimal ABI subset of nccl.h (stable across NCCL 2.x).
+typedef struct ncclComm* ncclComm_t;
+typedef struct {
+  char internal[128];
+} ncclUniqueId;
+typedef int ncclResult_t;  // ncclSuccess == 0
+enum { kNcclUint8 = 1 };
+
+struct NcclApi {
+  void* handle = nullptr;
+  ncclResult_t (*GetUniqueId)(ncclUniqueId*) = nullptr;
+  ncclResult_t (*CommInitRank)(ncclComm_t*, int, ncclUniqueId, int) = nullptr;
+  ncclResult_t (*CommDestroy)(ncclComm_t) = nullptr;
+  ncclResult_t (*CommCount)(ncclComm_t, int*) = nullptr;
+  ncclResult_t (*CommUserRank)(ncclComm_t, int*) = nullptr;
+  ncclResult_t (*CommGetAsyncError)(ncclComm_t, ncclResult_t*) = nullptr;
+  ncclResult_t (*AllGather)(const void*, void*, size_t, int, ncclComm_t, cudaStream_t) = nullptr;
+  const char* (*GetErrorString)(ncclResult_t) = nullptr;
+  std::string error;
+};
+
+NcclApi* nccl() {
+  static NcclApi api;
+  static bool tried = false;
+  if (tried) return api.handle ? &api : nullptr;
+  tried = true;
+  const char* env = std::getenv("PSO_NCCL_LIB");
+  const char* names[] = {env, "libnccl.so.2", "libnccl.so"};
+  for (const char* n : names) {
+    if (!n || !*n) continue;
+    // Prefer an NCCL already loaded into the process (e.g. by PyTorch).
+    api.handle = dlopen(n, RTLD_NOW | RTLD_GLOBAL | RTLD_NOLOAD);
+    if (!api.handle) api.handle = dlopen(n, RTLD_NOW | RTLD_GLOBAL);
+    if (api.handle) break;
+  }
+  if (!api.handle) {
+    const char* e = dlerror();
+    api.error = e ? e : "libnccl.so.2 not found";
+    return nullptr;
+  }
+#define PSO_SYM(field, name)                                       \
+  *(void**)(&api.field) = dlsym(api.handle, name);                 \
+  if (!api.field) {                                                \
+    api.error = std::string("missing NCCL symbol ") + name;        \
+    api.handle = nullptr;                                          \
+    return nullptr;                                                \
+  }
+  PSO_SYM(GetUniqueId, "ncclGetUniqueId")
+  PSO_SYM(CommInitRank, "ncclCommInitRank")
+  PSO_SYM(CommDestroy, "ncclCommDestroy")
+  PSO_SYM(CommCount, "ncclCommCount")
+  PSO_SYM(CommUserRank, "ncclCommUserRank")
+  PSO_SYM(CommGetAsyncError, "ncclCommGetAsyncError")
+  PSO_SYM(AllGather, "ncclAllGather")
+  PSO_SYM(GetErrorString, "ncclGetErrorString")
+#undef PSO_SYM
+  return &api;
+}
+
+const char* nccl_str(ncclResult_t r) {
+  NcclApi* a = nccl();
+  return (a && a->GetErrorString) ? a->GetErrorString(r) : "nccl error";
+}
+
+// ------------------------------------------------------------ the handle
+size_t align_up(size_t v, size_t a) { return (v + a - 1) / a * a; }
+
+}  // namespace
+
+struct pso_swarm {
+  // problem
+  int64_t n = 0, n_local = 0, row_begin = 0;
+  int32_t d = 0, pitch = 0, objective = 0;
+  float w = 0, c1 = 0, c2 = 0, lo = 0, hi = 0, vmax = 1;
+  uint64_t seed = 0;
+  // placement
+  int device = 0, sm_count = 0, rank = 0, world = 1;
+  cudaStream_t stream = nullptr;
+  bool own_stream = false;
+  ncclComm_t comm = nullptr;
+  uint32_t flags = 0;
+  // memory
+  void* arena = nullptr;
+  size_t arena_bytes = 0;
+  SwarmArgs args{};
+  LaunchCfg cfg{};
+  // run state
+  uint64_t t = 0;
+  bool poisoned = false;
+  uint64_t launches = 0;
+  std::vector<std::pair<cudaEvent_t, cudaEvent_t>> events;
+  size_t events_used = 0;
+  double timed_ms = 0;
+  uint64_t timed_count = 0;
+};
+
+namespace {
+
+pso_status cuda_fail(pso_swarm* h, cudaError_t e, const char* what) {
+  if (h) h->poisoned = true;
+  cudaGetLastError();  // clear a sticky launch error where possible
+  return fail(PSO_ERR_CUDA, "%s: %s (%s)", what, cudaGetErrorString(e), cudaGetErrorName(e));
+}
+
+#define PSO_CUDA(h, call)                                      \
+  do {                                                         \
+    cudaError_t _e = (call);                                   \
+    if (_e != cudaSuccess) return cuda_fail((h), _e, #call);   \
+  } while (0)
+
+pso_status check_handle(pso_swarm* h) {
+  if (!h) return fail(PSO_ERR_INVALID, "NULL handle");
+  if (h->poisoned) return fail(PSO_ERR_POISONED, "handle poisoned by an earlier CUDA/NCCL error");
+  return PSO_OK;
+}
+
+// Make the handle's device current for this call.
+pso_status use_device(pso_swarm* h) {
+  PSO_CUDA(h, cudaSetDevice(h->device));
+  return PSO_OK;
+}
+
+pso_status exchange(pso_swarm* h) {
+  if (h->world <= 1) return PSO_OK;
+  NcclApi* a = nccl();
+  if (!a) {
+    h->poisoned = true;
+    return fail(PSO_ERR_NCCL, "NCCL unavailable");
+  }
+  const size_t rec = record_bytes(h->pitch);
+  ncclResult_t r = a->AllGather(h->args.send, const_cast<unsigned char*>(h->args.recv), rec,
+                                kNcclUint8, h->comm, h->stream);
+  if (r != 0) {
+    h->poisoned = true;
+    return fail(PSO_ERR_NCCL, "ncclAllGather: %s", nccl_str(r));
+  }
+  PSO_CUDA(h, launch_select(h->args, h->stream));
+  ++h->launches;
+  return PSO_OK;
+}
+
+pso_status sync_and_check(pso_swarm* h) {
+  cudaError_t e = cudaStreamSynchronize(h->stream);
+  if (e != cudaSuccess) return cuda_fail(h, e, "cudaStreamSynchronize");
+  if (h->world > 1) {
+    NcclApi* a = nccl();
+    ncclResult_t ar = 0;
+    if (a && a->CommGetAsyncError(h->comm, &ar) == 0 && ar != 0) {
+      h->poisoned = true;
+      return fail(PSO_ERR_NCCL, "NCCL async error: %s", nccl_str(ar));
+    }
+  }
+  return PSO_OK;
+}
+
+// Reset the gbest control words before a full re-selection (create / set_state).
+pso_status reset_ctl(pso_swarm* h, uint32_t t) {
+  DevCtl c{};
+  c.key_cur = ~0ull;
+  c.key_acc = ~0ull;
+  c.improvements = 0;
+  c.done = 0;
+  c.t = t;
+  // improvements are preserved across set_state: read-modify-write
+  DevCtl old{};
+  PSO_CUDA(h, cudaMemcpyAsync(&old, h->args.ctl, sizeof(DevCtl), cudaMemcpyDeviceToHost, h->stream));
+  PSO_CUDA(h, cudaStreamSynchronize(h->stream));
+  c.improvements = old.improvements;
+  PSO_CUDA(h, cudaMemcpyAsync(h->args.ctl, &c, sizeof(DevCtl), cudaMemcpyHostToDevice, h->stream));
+  PSO_CUDA(h, cudaStreamSynchronize(h->stream));
+  return PSO_OK;
+}
+
+float decode_fitness(unsigned long long key) {
+  uint32_t o = (uint32_t)(key >> 32);
+  uint32_t u = (o & 0x80000000u) ? (o & 0x7FFFFFFFu) : ~o;
+  float f;
+  std::memcpy(&f, &u, 4);
+  return f;
+}
+
+bool finite(float v) { return std::isfinite(v); }
+
+}  // namespace
+
+// ============================================================== C ABI
+extern "C" {
+
+const char* pso_status_string(pso_status s) {
+  switch (s) {
+    case PSO_OK: return "PSO_OK";
+    case PSO_ERR_INVALID: return "PSO_ERR_INVALID";
+    case PSO_ERR_NOMEM: return "PSO_ERR_NOMEM";
+    case PSO_ERR_CUDA: return "PSO_ERR_CUDA";
+    case PSO_ERR_NCCL: return "PSO_ERR_NCCL";
+    case PSO_ERR_UNSUPPORTED: return "PSO_ERR_UNSUPPORTED";
+    case PSO_ERR_POISONED: return "PSO_ERR_POISONED";
+  }
+  return "PSO_ERR_UNKNOWN";
+}
+
+const char* pso_last_error(void) { return g_last_error.c_str(); }
+
+int pso_objective_registered(int32_t objective) { return objective_registered(objective) ? 1 : 0; }
+
+pso_status pso_create(pso_handle* out, int64_t n, int32_t d, float w, float c1, float c2, float lo,
+                      float hi, int32_t objective, uint64_t seed) {
+  pso_opts o{};
+  o.device = -1;
+  return pso_create_ex(out, n, d, w, c1, c2, lo, hi, objective, seed, &o);
+}
+
+pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c1, float c2,
+                         float lo, float hi, int32_t objective, uint64_t seed,
+                         const pso_opts* opts) {
+  if (!out) return fail(PSO_ERR_INVALID, "out is NULL");
+  *out = nullptr;
+  pso_opts o{};
+  o.device = -1;
+  if (opts) o = *opts;
+  // ---- validation (nothing touches the GPU before this passes)
+  if (n < 1 || n >= (int64_t)1 << 32) return fail(PSO_ERR_INVALID, "n=%lld outside [1, 2^32)", (long long)n);
+  if (d < 1) return fail(PSO_ERR_INVALID, "d=%d < 1", d);
+  if (d > PSO_D_MAX) return fail(PSO_ERR_UNSUPPORTED, "d=%d > PSO_D_MAX=%d", d, PSO_D_MAX);
+  if (!finite(w) || !finite(c1) || !finite(c2))
+    return fail(PSO_ERR_INVALID, "w, c1, c2 must be finite");
+  if (!finite(lo) || !finite(hi) || !(lo < hi))
+    return fail(PSO_ERR_INVALID, "need finite lo < hi (got %g, %g)", lo, hi);
+  if (!(o.vmax == o.vmax) || std::isinf(o.vmax)) return fail(PSO_ERR_INVALID, "vmax must be finite");
+  if (!objective_registered(objective))
+    return fail(PSO_ERR_INVALID, "objective %d is not registered", objective);
+  if (o.flags & ~(uint32_t)PSO_FLAG_TIMING) return fail(PSO_ERR_INVALID, "unknown flags 0x%x", o.flags);
+
+  pso_swarm* h = new (std::nothrow) pso_swarm();
+  if (!h) return fail(PSO_ERR_NOMEM, "host allocation failed");
+  h->n = n;
+  h->d = d;
+  h->pitch = (d + 3) / 4 * 4;
+  h->objective = objective;
+  h->w = w;
+  h->c1 = c1;
+  h->c2 = c2;
+  h->lo = lo;
+  h->hi = hi;
+  h->vmax = o.vmax > 0.f ? o.vmax : 1.0f;  // reading 3
+  h->seed = seed;
+  h->flags = o.flags;
+
+  auto bail = [&](pso_status s) {
+    pso_destroy(h);
+    return s;
+  };
+
+  // ---- device and stream
+  if (o.device >= 0) {
+    cudaError_t e = cudaSetDevice(o.device);
+    if (e != cudaSuccess) return bail(cuda_fail(nullptr, e, "cudaSetDevice"));
+    h->device = o.device;
+  } else {
+    cudaError_t e = cudaGetDevice(&h->device);
+    if (e != cudaSuccess) return bail(cuda_fail(nullptr, e, "cudaGetDevice"));
+    if ((e = cudaSetDevice(h->device)) != cudaSuccess) return bail(cuda_fail(nullptr, e, "cudaSetDevice"));
+  }
+  {
+    cudaError_t e = cudaDeviceGetAttribute(&h->sm_count, cudaDevAttrMultiProcessorCount, h->device);
+    if (e != cudaSuccess) return bail(cuda_fail(nullptr, e, "cudaDeviceGetAttribute"));
+    int major = 0;
+    cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, h->device);
+    if (major != 10)
+      return bail(fail(PSO_ERR_UNSUPPORTED, "device %d has compute capability %d.x; this build is sm_100a only",
+                       h->device, major));
+  }
+  if (o.stream) {
+    h->stream = (cudaStream_t)o.stream;
+  } else {
+    cudaError_t e = cudaStreamCreateWithFlags(&h->stream, cudaStreamNonBlocking);
+    if (e != cudaSuccess) return bail(cuda_fail(nullptr, e, "cudaStreamCreate"));
+    h->own_stream = true;
+  }
+
+  // ---- world (particle split)
+  if (o.nccl_comm) {
+    NcclApi* a = nccl();
+    if (!a) return bail(fail(PSO_ERR_NCCL, "NCCL unavailable: %s", "dlopen failed"));
+    h->comm = (ncclComm_t)o.nccl_comm;
+    int cnt = 1, rk = 0;
+    if (a->CommCount(h->comm, &cnt) != 0 || a->CommUserRank(h->comm, &rk) != 0)
+      return bail(fail(PSO_ERR_NCCL, "ncclCommCount/UserRank failed"));
+    h->world = cnt;
+    h->rank = rk;
+  }
+  h->row_begin = (n * h->rank) / h->world;
+  h->n_local = (n * (h->rank + 1)) / h->world - h->row_begin;
+
+  // ---- launch plan
+  int vpt_override = 0;
+  if (const char* v = std::getenv("PSO_VPT")) vpt_override = std::atoi(v);
+  {
+    cudaError_t e = plan_launch(objective, d, h->n_local > 0 ? h->n_local : 1, h->sm_count,
+                                vpt_override, &h->cfg);
+    if (e != cudaSuccess) return bail(cuda_fail(nullptr, e, "plan_launch"));
+  }
+
+  // ---- one arena: X, V, PB, pf, G, ctl, exchange records
+  const size_t rows = (size_t)(h->n_local > 0 ? h->n_local : 1);
+  const size_t mat = align_up(rows * (size_t)h->pitch * 4, 256);
+  const size_t pfb = align_up(rows * 4, 256);
+  const size_t gb = align_up((size_t)h->pitch * 4, 256);
+  const size_t ctlb = align_up(sizeof(DevCtl), 256);
+  const size_t rec = align_up(record_bytes(h->pitch), 256);
+  const size_t sendb = h->world > 1 ? rec : 0;
+  const size_t recvb = h->world > 1 ? (size_t)h->world * record_bytes(h->pitch) : 0;
+  h->arena_bytes = 3 * mat + pfb + gb + ctlb + sendb + align_up(recvb, 256);
+  {
+    cudaError_t e = cudaMalloc(&h->arena, h->arena_bytes);
+    if (e == cudaErrorMemoryAllocation) {
+      cudaGetLastError();
+      return bail(fail(PSO_ERR_NOMEM, "cudaMalloc(%zu bytes) failed", h->arena_bytes));
+    }
+    if (e != cudaSuccess) return bail(cuda_fail(nullptr, e, "cudaMalloc"));
+  }
+  unsigned char* p = (unsigned char*)h->arena;
+  SwarmArgs& A = h->args;
+  A.X = (float*)p; p += mat;
+  A.V = (float*)p; p += mat;
+  A.PB = (float*)p; p += mat;
+  A.pf = (float*)p; p += pfb;
+  A.G = (float*)p; p += gb;
+  A.ctl = (DevCtl*)p; p += ctlb;
+  A.send = h->world > 1 ? p : nullptr; p += sendb;
+  A.recv = h->world > 1 ? p : nullptr;
+  A.n_local = h->n_local;
+  A.row_begin = h->row_begin;
+  A.d = d;
+  A.nvec = h->pitch / 4;
+  A.world = h->world;
+  A.w = w; A.c1 = c1; A.c2 = c2; A.lo = lo; A.hi = hi; A.vmax = h->vmax;
+  A.seed_lo = (unsigned)seed;
+  A.seed_hi = (unsigned)(seed >> 32);
+
+  {
+    cudaError_t e = cudaMemsetAsync(A.G, 0, gb + ctlb, h->stream);  // G and ctl
+    if (e != cudaSuccess) return bail(cuda_fail(nullptr, e, "cudaMemsetAsync"));
+    if (h->world > 1) {
+      e = cudaMemsetAsync(A.send, 0, sendb, h->stream);
+      if (e != cudaSuccess) return bail(cuda_fail(nullptr, e, "cudaMemsetAsync"));
+    }
+  }
+  pso_status st = reset_ctl(h, 0);
+  if (st != PSO_OK) return bail(st);
+
+  // ---- Alg. 1 lines 1-3 + first evaluation and best update
+  if (h->n_local > 0) {
+    cudaError_t e = launch_init(objective, A, h->cfg, h->stream);
+    if (e != cudaSuccess) return bail(cuda_fail(nullptr, e, "launch_init"));
+    ++h->launches;
+  } else if (h->world > 1) {
+    // empty shard: contribute "no candidate"
+    unsigned long long none[2] = {~0ull, 0ull};
+    cudaError_t e = cudaMemcpyAsync(A.send, none, 16, cudaMemcpyHostToDevice, h->stream);
+    if (e != cudaSuccess) return bail(cuda_fail(nullptr, e, "cudaMemcpyAsync"));
+  }
+  if ((st = exchange(h)) != PSO_OK) return bail(st);
+  if ((st = sync_and_check(h)) != PSO_OK) return bail(st);
+  h->t = 0;
+  *out = h;
+  return PSO_OK;
+}
+
+pso_status pso_step(pso_handle h, int64_t iters) {
+  pso_status st = check_handle(h);
+  if (st != PSO_OK) return st;
+  if (iters < 0) return fail(PSO_ERR_INVALID, "iters=%lld < 0", (long long)iters);
+  if (iters == 0) return PSO_OK;
+  if ((st = use_device(h)) != PSO_OK) return st;
+  const bool timing = (h->flags & PSO_FLAG_TIMING) != 0;
+  for (int64_t it = 0; it < iters; ++it) {
+    if (h->n_local > 0) {
+      std::pair<cudaEvent_t, cudaEvent_t>* ev = nullptr;
+      if (timing) {
+        if (h->events_used == h->events.size()) {
+          cudaEvent_t a, b;
+          PSO_CUDA(h, cudaEventCreate(&a));
+          PSO_CUDA(h, cudaEventCreate(&b));
+          h->events.emplace_back(a, b);
+        }
+        ev = &h->events[h->events_used++];
+        PSO_CUDA(h, cudaEventRecord(ev->first, h->stream));
+      }
+      PSO_CUDA(h, launch_step(h->objective, h->args, h->cfg, h->stream));
+      ++h->launches;
+      if (ev) PSO_CUDA(h, cudaEventRecord(ev->second, h->stream));
+    }
+    if ((st = exchange(h)) != PSO_OK) return st;
+    if (timing && h->events_used >= 4096) {  // bound the event pool: fold into totals
+      PSO_CUDA(h, cudaStreamSynchronize(h->stream));
+      for (size_t k = 0; k < h->events_used; ++k) {
+        float ms = 0;
+        PSO_CUDA(h, cudaEventElapsedTime(&ms, h->events[k].first, h->events[k].second));
+        h->timed_ms += ms;
+      }
+      h->timed_count += h->events_used;
+      h->events_used = 0;
+    }
+  }
+  h->t += (uint64_t)iters;
+  return PSO_OK;
+}
+
+pso_status pso_synchronize(pso_handle h) {
+  pso_status st = check_handle(h);
+  if (st != PSO_OK) return st;
+  if ((st = use_device(h)) != PSO_OK) return st;
+  return sync_and_check(h);
+}
+
+pso_status pso_get_gbest(pso_handle h, float* fitness, int64_t* index, float* pos) {
+  pso_status st = check_handle(h);
+  if (st != PSO_OK) return st;
+  if ((st = use_device(h)) != PSO_OK) return st;
+  unsigned long long key = 0;
+  PSO_CUDA(h, cudaMemcpyAsync(&key, &h->args.ctl->key_cur, 8, cudaMemcpyDeviceToHost, h->stream));
+  if (pos) PSO_CUDA(h, cudaMemcpyAsync(pos, h->args.G, (size_t)h->d * 4, cudaMemcpyDeviceToHost, h->stream));
+  if ((st = sync_and_check(h)) != PSO_OK) return st;
+  if (fitness) *fitness = decode_fitness(key);
+  if (index) *index = (int64_t)(uint32_t)key;
+  return PSO_OK;
+}
+
+pso_status pso_get_state(pso_handle h, float* x, float* v, float* pb, float* pf, uint64_t* t) {
+  pso_status st = check_handle(h);
+  if (st != PSO_OK) return st;
+  if ((st = use_device(h)) != PSO_OK) return st;
+  const size_t w = (size_t)h->d * 4, sp = (size_t)h->pitch * 4, rows = (size_t)h->n_local;
+  if (rows > 0) {
+    if (x) PSO_CUDA(h, cudaMemcpy2DAsync(x, w, h->args.X, sp, w, rows, cudaMemcpyDeviceToHost, h->stream));
+    if (v) PSO_CUDA(h, cudaMemcpy2DAsync(v, w, h->args.V, sp, w, rows, cudaMemcpyDeviceToHost, h->stream));
+    if (pb) PSO_CUDA(h, cudaMemcpy2DAsync(pb, w, h->args.PB, sp, w, rows, cudaMemcpyDeviceToHost, h->stream));
+    if (pf) PSO_CUDA(h, cudaMemcpyAsync(pf, h->args.pf, rows * 4, cudaMemcpyDeviceToHost, h->stream));
+  }
+  if ((st = sync_and_check(h)) != PSO_OK) return st;
+  if (t) *t = h->t;
+  return PSO_OK;
+}
+
+pso_status pso_set_state(pso_handle h, const float* x, const float* v, const float* pb,
+                         const float* pf, uint64_t t) {
+  pso_status st = check_handle(h);
+  if (st != PSO_OK) return st;
+  if (h->n_local > 0 && (!x || !v || !pb || !pf))
+    return fail(PSO_ERR_INVALID, "set_state needs x, v, pb and pf");
+  if (t >= ((uint64_t)1 << 32)) return fail(PSO_ERR_INVALID, "t=%llu >= 2^32", (unsigned long long)t);
+  if ((st = use_device(h)) != PSO_OK) return st;
+  const size_t w = (size_t)h->d * 4, sp = (size_t)h->pitch * 4, rows = (size_t)h->n_local;
+  if (rows > 0) {
+    const size_t mat = rows * sp;
+    if (h->pitch != h->d) {  // zero the row padding
+      PSO_CUDA(h, cudaMemsetAsync(h->args.X, 0, mat, h->stream));
+      PSO_CUDA(h, cudaMemsetAsync(h->args.V, 0, mat, h->stream));
+      PSO_CUDA(h, cudaMemsetAsync(h->args.PB, 0, mat, h->stream));
+    }
+    PSO_CUDA(h, cudaMemcpy2DAsync(h->args.X, sp, x, w, w, rows, cudaMemcpyHostToDevice, h->stream));
+    PSO_CUDA(h, cudaMemcpy2DAsync(h->args.V, sp, v, w, w, rows, cudaMemcpyHostToDevice, h->stream));
+    PSO_CUDA(h, cudaMemcpy2DAsync(h->args.PB, sp, pb, w, w, rows, cudaMemcpyHostToDevice, h->stream));
+    PSO_CUDA(h, cudaMemcpyAsync(h->args.pf, pf, rows * 4, cudaMemcpyHostToDevice, h->stream));
+  }
+  if ((st = reset_ctl(h, (uint32_t)t)) != PSO_OK) return st;
+  if (rows > 0) {
+    PSO_CUDA(h, launch_rebest(h->args, (unsigned)t, h->stream));
+    ++h->launches;
+  } else if (h->world > 1) {
+    unsigned long long none[2] = {~0ull, 0ull};
+    PSO_CUDA(h, cudaMemcpyAsync(h->args.send, none, 16, cudaMemcpyHostToDevice, h->stream));
+  }
+  if ((st = exchange(h)) != PSO_OK) return st;
+  if ((st = sync_and_check(h)) != PSO_OK) return st;
+  h->t = t;
+  return PSO_OK;
+}
+
+pso_status pso_get_info(pso_handle h, pso_info* info) {
+  if (!h) return fail(PSO_ERR_INVALID, "NULL handle");
+  if (!info) return fail(PSO_ERR_INVALID, "info is NULL");
+  pso_status st = check_handle(h);
+  if (st != PSO_OK) return st;
+  if ((st = use_device(h)) != PSO_OK) return st;
+  if ((st = sync_and_check(h)) != PSO_OK) return st;
+  for (size_t k = 0; k < h->events_used; ++k) {
+    float ms = 0;
+    PSO_CUDA(h, cudaEventElapsedTime(&ms, h->events[k].first, h->events[k].second));
+    h->timed_ms += ms;
+  }
+  h->timed_count += h->events_used;
+  h->events_used = 0;
+  DevCtl c{};
+  PSO_CUDA(h, cudaMemcpy(&c, h->args.ctl, sizeof(DevCtl), cudaMemcpyDeviceToHost));
+  std::memset(info, 0, sizeof(*info));
+  info->n = h->n;
+  info->n_local = h->n_local;
+  info->row_begin = h->row_begin;
+  info->d = h->d;
+  info->pitch = h->pitch;
+  info->rank = h->rank;
+  info->world = h->world;
+  info->threads_per_cta = h->cfg.threads;
+  info->vec_per_thread = h->cfg.vpt;
+  info->grid = h->cfg.grid;
+  info->ctas_per_sm = h->cfg.ctas_per_sm;
+  info->vmax = h->vmax;
+  info->t = h->t;
+  info->launches = h->launches;
+  info->improvements = c.improvements;
+  info->step_kernel_ms = h->timed_ms;
+  info->step_kernel_count = h->timed_count;
+  info->arena_bytes = h->arena_bytes;
+  return PSO_OK;
+}
+
+pso_status pso_reset_counters(pso_handle h) {
+  pso_status st = check_handle(h);
+  if (st != PSO_OK) return st;
+  if ((st = use_device(h)) != PSO_OK) return st;
+  if ((st = sync_and_check(h)) != PSO_OK) return st;
+  h->launches = 0;
+  h->timed_ms = 0;
+  h->timed_count = 0;
+  h->events_used = 0;
+  unsigned long long zero = 0;
+  PSO_CUDA(h, cudaMemcpy(&h->args.ctl->improvements, &zero, 8, cudaMemcpyHostToDevice));
+  return PSO_OK;
+}
+
+void pso_destroy(pso_handle h) {
+  if (!h) return;
+  cudaSetDevice(h->device);
+  if (h->stream) cudaStreamSynchronize(h->stream);
+  for (auto& e : h->events) {
+    cudaEventDestroy(e.first);
+    cudaEventDestroy(e.second);
+  }
+  if (h->arena) cudaFree(h->arena);
+  if (h->own_stream && h->stream) cudaStreamDestroy(h->stream);
+  cudaGetLastError();
+  delete h;
+}
+
+// ------------------------------------------------------------ NCCL helpers
+pso_status pso_nccl_get_unique_id(void* id128) {
+  if (!id128) return fail(PSO_ERR_INVALID, "id is NULL");
+  NcclApi* a = nccl();
+  if (!a) return fail(PSO_ERR_NCCL, "NCCL unavailable");
+  ncclUniqueId id;
+  ncclResult_t r = a->GetUniqueId(&id);
+  if (r != 0) return fail(PSO_ERR_NCCL, "ncclGetUniqueId: %s", nccl_str(r));
+  std::memcpy(id128, &id, sizeof(id));
+  return PSO_OK;
+}
+
+pso_status pso_nccl_comm_init(void** comm, int32_t nranks, const void* id128, int32_t rank,
+                              int32_t device) {
+  if (!comm || !id128) return fail(PSO_ERR_INVALID, "comm/id is NULL");
+  if (nranks < 1 || rank < 0 || rank >= nranks) return fail(PSO_ERR_INVALID, "bad rank/nranks");
+  NcclApi* a = nccl();
+  if (!a) return fail(PSO_ERR_NCCL, "NCCL unavailable");
+  if (device >= 0) {
+    cudaError_t e = cudaSetDevice(device);
+    if (e != cudaSuccess) return cuda_fail(nullptr, e, "cudaSetDevice");
+  }
+  ncclUniqueId id;
+  std::memcpy(&id, id128, sizeof(id));
+  ncclComm_t c = nullptr;
+  ncclResult_t r = a->CommInitRank(&c, nranks, id, rank);
+  if (r != 0) return fail(PSO_ERR_NCCL, "ncclCommInitRank: %s", nccl_str(r));
+  *comm = c;
+  return PSO_OK;
+}
+
+pso_status pso_nccl_comm_destroy(void* comm) {
+  if (!comm) return PSO_OK;
+  NcclApi* a = nccl();
+  if (!a) return fail(PSO_ERR_NCCL, "NCCL unavailable");
+  ncclResult_t r = a->CommDestroy((ncclComm_t)comm);
+  if (r != 0) return fail(PSO_ERR_NCCL, "ncclCommDestroy: %s", nccl_str(r));
+  return PSO_OK;
+}
+
+// ------------------------------------------------------------ debug entry points
+pso_status pso_debug_philox(uint64_t seed, uint32_t tag, uint32_t t, uint32_t i, uint32_t j0,
+                            int64_t m, uint32_t* out, int32_t use_curand, int32_t device) {
+  if (m < 0 || (m > 0 && !out)) return fail(PSO_ERR_INVALID, "bad m/out");
+  if (m == 0) return PSO_OK;
+  if (device >= 0) {
+    cudaError_t e = cudaSetDevice(device);
+    if (e != cudaSuccess) return cuda_fail(nullptr, e, "cudaSetDevice");
+  }
+  unsigned* dev = nullptr;
+  cudaError_t e = cudaMalloc(&dev, (size_t)m * 4);
+  if (e != cudaSuccess) return cuda_fail(nullptr, e, "cudaMalloc");
+  e = debug_philox(seed, tag, t, i, j0, m, dev, use_curand, 0);
+  if (e == cudaSuccess) e = cudaMemcpy(out, dev, (size_t)m * 4, cudaMemcpyDeviceToHost);
+  cudaFree(dev);
+  if (e != cudaSuccess) return cuda_fail(nullptr, e, "debug_philox");
+  return PSO_OK;
+}
+
+pso_status pso_debug_objective(int32_t objective, const float* X, int64_t m, int32_t d, float* out,
+                               int32_t device) {
+  if (m < 0 || d < 1 || d > PSO_D_MAX || (m > 0 && (!X || !out)))
+    return fail(PSO_ERR_INVALID, "bad arguments");
+  if (!objective_registered(objective)) return fail(PSO_ERR_INVALID, "objective %d not registered", objective);
+  if (m == 0) return PSO_OK;
+  if (device >= 0) {
+    cudaError_t e = cudaSetDevice(device);
+    if (e != cudaSuccess) return cuda_fail(nullptr, e, "cudaSetDevice");
+  }
+  int dev_id = 0, sms = 148;
+  cudaGetDevice(&dev_id);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev_id);
+  const int pitch = (d + 3) / 4 * 4;
+  float* dX = nullptr;
+  float* dO = nullptr;
+  cudaError_t e = cudaMalloc(&dX, (size_t)m * pitch * 4);
+  if (e == cudaSuccess) e = cudaMalloc(&dO, (size_t)m * 4);
+  if (e == cudaSuccess) e = cudaMemset(dX, 0, (size_t)m * pitch * 4);
+  if (e == cudaSuccess)
+    e = cudaMemcpy2D(dX, (size_t)pitch * 4, X, (size_t)d * 4, (size_t)d * 4, (size_t)m,
+                     cudaMemcpyHostToDevice);
+  if (e == cudaSuccess) e = debug_objective(objective, dX, m, d, pitch, dO, sms, 0);
+  if (e == cudaSuccess) e = cudaMemcpy(out, dO, (size_t)m * 4, cudaMemcpyDeviceToHost);
+  cudaFree(dX);
+  cudaFree(dO);
+  if (e != cudaSuccess) return cuda_fail(nullptr, e, "debug_objective");
+  return PSO_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,65 @@
+// kernels.h — internal interface between the C ABI (api.cpp) and the CUDA
+// kernels (swarm_kernels.cu, debug_kernels.cu).  Not part of the public ABI.
+#pragma once
+#include <cuda_runtime.h>
+
+#include <cstddef>
+#include <cstdint>
+
+namespace fastpso {
+
+// Per-handle control block in device memory (one cache line).
+struct DevCtl {
+  unsigned long long key_cur;       // incumbent gbest key: ord(gf) << 32 | gi
+  unsigned long long key_acc;       // atomicMin accumulator of this iteration
+  unsigned long long improvements;  // pbest improvements, summed
+  unsigned int done;                // last-CTA ticket counter
+  unsigned int t;                   // iterations done (low 32 bits; Philox ctr[2])
+  unsigned long long pad[4];
+};
+
+// Exchange record for world > 1: the local candidate key and its PB row.
+// Layout: [u64 key][u64 pad][pitch floats].
+__host__ __device__ inline size_t record_bytes(int pitch) { return 16 + (size_t)pitch * 4; }
+
+struct SwarmArgs {
+  float* X;   // n_local x pitch
+  float* V;
+  float* PB;
+  float* pf;  // n_local
+  float* G;   // pitch (gbest position)
+  unsigned char* send;        // world > 1: this rank's exchange record
+  const unsigned char* recv;  // world > 1: world records after the all-gather
+  DevCtl* ctl;
+  long long n_local;
+  long long row_begin;
+  int d, nvec;                // nvec = pitch / 4
+  int world;
+  float w, c1, c2, lo, hi, vmax;
+  unsigned int seed_lo, seed_hi;
+};
+
+struct LaunchCfg {
+  int vpt = 1;       // float4 per thread per row
+  int threads = 32;  // CTA size
+  int grid = 1;      // persistent grid
+  int ctas_per_sm = 1;
+  size_t smem = 0;   // dynamic shared memory bytes
+};
+
+bool objective_registered(int objective);
+// Choose the CTA shape for d and size the persistent grid for n_local rows.
+cudaError_t plan_launch(int objective, int d, long long n_local, int sm_count, int vpt_override,
+                        LaunchCfg* cfg);
+cudaError_t launch_init(int objective, const SwarmArgs& a, const LaunchCfg& c, cudaStream_t s);
+cudaError_t launch_step(int objective, const SwarmArgs& a, const LaunchCfg& c, cudaStream_t s);
+cudaError_t launch_rebest(const SwarmArgs& a, unsigned t, cudaStream_t s);
+cudaError_t launch_select(const SwarmArgs& a, cudaStream_t s);
+
+cudaError_t debug_philox(unsigned long long seed, unsigned tag, unsigned t, unsigned i,
+                         unsigned j0, long long m, unsigned* out_dev, int use_curand,
+                         cudaStream_t s);
+cudaError_t debug_objective(int objective, const float* X_dev, long long m, int d, int pitch,
+                            float* out_dev, int sm_count, cudaStream_t s);
+
+}  // namespace fastpso

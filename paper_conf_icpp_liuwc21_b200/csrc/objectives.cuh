@@ -1,0 +1,124 @@
+// objectives.cuh — compile-time objective functors (the paper's user-defined
+// evaluation schema, Sec 3.2, without an extended lambda or a JIT).
+//
+// A functor F describes a per-particle fitness as map -> reduce -> finalize
+// over the particle's d coordinates, so it can be fused into the swarm-update
+// kernel: each thread maps the coordinates it just updated into kAcc fp32
+// accumulators, the CTA tree-reduces them with F::combine, and one thread
+// calls F::finalize.  Interface:
+//
+//   static constexpr int  kAcc;        // accumulators per thread (1 or 2)
+//   static constexpr bool kNeighbor;   // map() needs x_{j+1} (Rosenbrock)
+//   __device__ static void  init(float* a);                 // identities
+//   __device__ static void  map(float* a, float x, float xnext, int j, int d);
+//                                      // j: 0-based dim; xnext valid iff kNeighbor && j+1 < d
+//   __device__ static void  combine(float* a, const float* b);   // associative
+//   __device__ static float finalize(const float* a, int d);
+//
+// The reduction order is fixed by the launch shape, which depends only on d,
+// so fitness bits do not depend on the grid or on the number of GPUs.
+// Formulas are rearranged for fp32 accuracy where that is free (noted below);
+// all are mathematically the definitions in include/fastpso.h.
+#pragma once
+
+namespace fastpso {
+
+// Sphere: sum x_k^2.
+struct Sphere {
+  static constexpr int kAcc = 1;
+  static constexpr bool kNeighbor = false;
+  __device__ static void init(float* a) { a[0] = 0.f; }
+  __device__ static void map(float* a, float x, float, int, int) { a[0] = fmaf(x, x, a[0]); }
+  __device__ static void combine(float* a, const float* b) { a[0] += b[0]; }
+  __device__ static float finalize(const float* a, int) { return a[0]; }
+};
+
+// Rastrigin ([20]): sum x^2 + 10 - 10 cos(2 pi x) = sum x^2 + 20 sin^2(pi x).
+// The sin^2 form has no cancellation, so every term is computed to ~1 ulp.
+struct Rastrigin {
+  static constexpr int kAcc = 1;
+  static constexpr bool kNeighbor = false;
+  __device__ static void init(float* a) { a[0] = 0.f; }
+  __device__ static void map(float* a, float x, float, int, int) {
+    const float s = sinpif(x);
+    a[0] += fmaf(x, x, 20.f * (s * s));
+  }
+  __device__ static void combine(float* a, const float* b) { a[0] += b[0]; }
+  __device__ static float finalize(const float* a, int) { return a[0]; }
+};
+
+// Rosenbrock ([20]): sum_{k<d} 100 (x_{k+1} - x_k^2)^2 + (x_k - 1)^2.
+struct Rosenbrock {
+  static constexpr int kAcc = 1;
+  static constexpr bool kNeighbor = true;
+  __device__ static void init(float* a) { a[0] = 0.f; }
+  __device__ static void map(float* a, float x, float xn, int j, int d) {
+    if (j + 1 < d) {
+      const float t = fmaf(-x, x, xn);
+      const float u = x - 1.f;
+      a[0] += fmaf(100.f * t, t, u * u);
+    }
+  }
+  __device__ static void combine(float* a, const float* b) { a[0] += b[0]; }
+  __device__ static float finalize(const float* a, int) { return a[0]; }
+};
+
+// Griewank: 1 + sum x_k^2 / 4000 - prod cos(x_k / sqrt(k)), k = j + 1.
+struct Griewank {
+  static constexpr int kAcc = 2;
+  static constexpr bool kNeighbor = false;
+  __device__ static void init(float* a) {
+    a[0] = 0.f;
+    a[1] = 1.f;
+  }
+  __device__ static void map(float* a, float x, float, int j, int) {
+    a[0] = fmaf(x, x, a[0]);
+    a[1] *= cosf(x * rsqrtf((float)(j + 1)));
+  }
+  __device__ static void combine(float* a, const float* b) {
+    a[0] += b[0];
+    a[1] *= b[1];
+  }
+  __device__ static float finalize(const float* a, int) {
+    return a[0] * (1.f / 4000.f) + (1.f - a[1]);
+  }
+};
+
+// Easom: -(-1)^d prod cos^2(x_k) exp(-sum (x_k - pi)^2).
+struct Easom {
+  static constexpr int kAcc = 2;
+  static constexpr bool kNeighbor = false;
+  __device__ static void init(float* a) {
+    a[0] = 1.f;
+    a[1] = 0.f;
+  }
+  __device__ static void map(float* a, float x, float, int, int) {
+    const float c = cosf(x);
+    const float e = x - 3.14159265358979f;
+    a[0] *= c * c;
+    a[1] = fmaf(e, e, a[1]);
+  }
+  __device__ static void combine(float* a, const float* b) {
+    a[0] *= b[0];
+    a[1] += b[1];
+  }
+  __device__ static float finalize(const float* a, int d) {
+    const float v = a[0] * expf(-a[1]);
+    return (d & 1) ? v : -v;
+  }
+};
+
+}  // namespace fastpso
+
+#include "user_objectives.cuh"
+
+// Built-in objective registry: X(id, Functor).  User functors are listed in
+// PSO_USER_OBJECTIVES (user_objectives.cuh).
+#define PSO_BUILTIN_OBJECTIVES(X)     \
+  X(1, ::fastpso::Sphere)             \
+  X(2, ::fastpso::Rastrigin)          \
+  X(3, ::fastpso::Rosenbrock)         \
+  X(4, ::fastpso::Griewank)           \
+  X(6, ::fastpso::Easom)
+
+#define PSO_ALL_OBJECTIVES(X) PSO_BUILTIN_OBJECTIVES(X) PSO_USER_OBJECTIVES(X)

@@ -1,0 +1,58 @@
+// philox.cuh — counter-based random weights in registers.
+//
+// The paper materialises two n x d random matrices L, G per iteration with
+// Thrust (Sec 3.1; Eq. 4, L and G at P:L195-211) — 16 B of HBM
+// traffic per element (write + read).  Here every weight is recomputed from
+// (seed, t, particle, dim) by Philox4x32-10 in registers: 0 B of HBM.
+// One call yields the 4 weights of one float4 of dimensions for one tag.
+//
+// Stream layout (reading 6):
+//   word(tag, t, i, j) = Philox4x32-10(ctr = {j>>2, i, t, tag}, key = {seed lo, seed hi})[j&3]
+//   tags: R1 = 0 (l_ij of Eq. 1), R2 = 1 (g_ij), X0 = 2, V0 = 3 (init, t = 0)
+//   U(w) = (w >> 8) * 2^-24  in [0, 1 - 2^-24]  (reading 5)
+#pragma once
+#include <cstdint>
+
+namespace fastpso {
+
+enum : uint32_t { kTagR1 = 0, kTagR2 = 1, kTagX0 = 2, kTagV0 = 3 };
+
+struct PhiloxKey {
+  uint32_t k0, k1;
+};
+
+// Philox4x32-10 (Salmon et al., SC'11): 10 rounds of two 32x32->64 products;
+// the key is bumped by the Weyl constants between rounds.
+__device__ __forceinline__ uint4 philox4x32_10(uint4 c, PhiloxKey key) {
+  uint32_t k0 = key.k0, k1 = key.k1;
+#pragma unroll
+  for (int r = 0; r < 10; ++r) {
+    if (r > 0) {
+      k0 += 0x9E3779B9u;
+      k1 += 0xBB67AE85u;
+    }
+    const uint32_t lo0 = 0xD2511F53u * c.x;
+    const uint32_t hi0 = __umulhi(0xD2511F53u, c.x);
+    const uint32_t lo1 = 0xCD9E8D57u * c.z;
+    const uint32_t hi1 = __umulhi(0xCD9E8D57u, c.z);
+    c = make_uint4(hi1 ^ c.y ^ k0, lo1, hi0 ^ c.w ^ k1, lo0);
+  }
+  return c;
+}
+
+// 24-bit uniform: exact conversion (w >> 8 < 2^24) times an exact power of 2.
+__device__ __forceinline__ float u01(uint32_t w) {
+  return __uint2float_rn(w >> 8) * 0x1p-24f;
+}
+
+__device__ __forceinline__ float4 u01x4(uint4 w) {
+  return make_float4(u01(w.x), u01(w.y), u01(w.z), u01(w.w));
+}
+
+// The 4 uniforms of float4 q (dims 4q..4q+3) of particle i at iteration t.
+__device__ __forceinline__ float4 uniforms4(PhiloxKey key, uint32_t tag, uint32_t t,
+                                            uint32_t i, uint32_t q) {
+  return u01x4(philox4x32_10(make_uint4(q, i, t, tag), key));
+}
+
+}  // namespace fastpso

@@ -1,0 +1,290 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle.
+
+Acceptance (north_star):
+  * Philox words and init state: bit-exact
+  * single step from identical injected state: X, V bit-exact (<= 1e-5 rel
+    required); fitness within the derived tolerance; PB / pbest decisions
+    equal except ambiguous rows (|f - pf| within tolerance); gbest index exact
+    unless ambiguous
+  * C1 after 100 iterations: gbest fitness within relative 1e-4
+Sizes span several CTA tiles, ragged d (d % 4 != 0), every CTA shape
+(VPT 1/2/4/8) and the degenerate n = 1, d = 1.
+"""
+import numpy as np
+import pytest
+
+import oracle as orc
+import paper_conf_icpp_liuwc21_b200 as fp
+from synth import (ACKLEY, DOMAINS, EASOM, GRIEWANK, RASTRIGIN, ROSENBROCK, SPHERE, WORKLOADS,
+                   random_state, sample_rows)
+from tests.helpers import assert_bitwise, assert_fitness_close, fit_tol
+
+pytestmark = pytest.mark.gpu
+
+OBJS = [SPHERE, RASTRIGIN, ROSENBROCK, GRIEWANK, ACKLEY, EASOM]
+# (n, d): C1; ragged d over several tiles; VPT 1, 2, 4, 8 shapes; degenerate
+SHAPES = [(32, 10), (257, 13), (300, 1000), (70, 2000), (9, 4096), (3, 8192), (1, 1), (5, 3),
+          (40, 999)]
+
+
+def gpu_swarm(n, d, obj, seed=2021, w=0.9, c1=2.0, c2=2.0, vmax=0.0, **kw):
+    lo, hi = DOMAINS[obj]
+    return fp.Swarm(n, d, w, c1, c2, lo, hi, obj, seed, vmax=vmax, device=0, **kw)
+
+
+def cpu_swarm(n, d, obj, seed=2021, w=0.9, c1=2.0, c2=2.0, vmax=0.0, create=True):
+    lo, hi = DOMAINS[obj]
+    return orc.OracleSwarm(n, d, w, c1, c2, lo, hi, obj, seed, vmax=vmax, create=create)
+
+
+# ------------------------------------------------------------------ Philox
+@pytest.mark.parametrize("tag,t,i,j0,m", [(0, 1, 0, 0, 4096), (1, 7, 123456, 5, 1001),
+                                          (2, 0, 2**32 - 1, 0, 64), (3, 0, 77, 8189, 3),
+                                          (0, 2**32 - 1, 5, 1, 513)])
+@pytest.mark.parametrize("seed", [0, 2021, 2**64 - 1])
+def test_philox_words_bitexact(tag, t, i, j0, m, seed):
+    ref = orc.words(seed, tag, t, i, j0, m)
+    got = fp.debug_philox(seed, tag, t, i, j0, m, device=0)
+    np.testing.assert_array_equal(got, ref)
+    cur = fp.debug_philox(seed, tag, t, i, j0, m, use_curand=True, device=0)
+    np.testing.assert_array_equal(cur, ref)  # NVIDIA's curand_Philox4x32_10, same counters
+
+
+# ------------------------------------------------------------------ objectives
+@pytest.mark.parametrize("obj", OBJS)
+@pytest.mark.parametrize("d", [1, 2, 7, 64, 1000, 2000, 4096, 8192])
+def test_objective_matches_oracle(obj, d):
+    lo, hi = DOMAINS[obj]
+    rng = np.random.default_rng(d * 10 + obj)
+    X = rng.uniform(lo, hi, size=(17, d)).astype(np.float32)
+    X[0] = 0.0
+    X[1] = np.float32(1.0) if obj == ROSENBROCK else X[1]
+    got = fp.debug_objective(obj, X, device=0)
+    ref = orc.objective_rows(obj, X)
+    assert_fitness_close(obj, X, got, ref)
+
+
+def test_objective_closed_forms_on_gpu():
+    assert fp.debug_objective(SPHERE, np.array([[1, 2, 3]], np.float32))[0] == 14.0
+    assert fp.debug_objective(ROSENBROCK, np.ones((1, 33), np.float32))[0] == 0.0
+    assert fp.debug_objective(ROSENBROCK, np.zeros((1, 33), np.float32))[0] == 32.0
+    assert fp.debug_objective(RASTRIGIN, np.zeros((1, 100), np.float32))[0] == 0.0
+    assert fp.debug_objective(GRIEWANK, np.zeros((1, 100), np.float32))[0] == 0.0
+    assert abs(fp.debug_objective(ACKLEY, np.zeros((1, 100), np.float32))[0]) <= 1e-6
+    x = np.arange(-5, 5, dtype=np.float32)[None, :]
+    assert fp.debug_objective(RASTRIGIN, x)[0] == pytest.approx(float((x.astype(np.float64) ** 2).sum()),
+                                                                 rel=1e-6)
+
+
+# ------------------------------------------------------------------ init
+@pytest.mark.parametrize("obj", OBJS)
+@pytest.mark.parametrize("n,d", SHAPES)
+def test_init_bitexact(obj, n, d):
+    g = gpu_swarm(n, d, obj, seed=11 * n + d)
+    c = cpu_swarm(n, d, obj, seed=11 * n + d)
+    X, V, PB, pf, t = g.get_state()
+    assert t == 0
+    assert_bitwise(X, c.X, "X0")
+    assert_bitwise(V, c.V, "V0")
+    assert_bitwise(PB, c.PB, "PB0")
+    assert_fitness_close(obj, c.X, pf, c.pf, "pf0")
+    gf, gi, G = g.gbest()
+    assert_bitwise(G, PB[gi], "G == PB[gi]")
+    assert pf[gi] == gf and gf == pf.min() and gi == int(np.argmin(pf))
+    tol = fit_tol(obj, c.X, c.pf)
+    ambiguous = np.abs(c.pf.astype(np.float64) - c.gf) <= tol + fit_tol(obj, c.X[[c.gi]], [c.gf])[0]
+    if ambiguous.sum() <= 1:
+        assert gi == c.gi
+    else:
+        assert ambiguous[gi]
+
+
+# ------------------------------------------------------------------ single step
+def _step_and_compare(obj, n, d, seed, pf_mode, t0=0):
+    lo, hi = DOMAINS[obj]
+    X, V, PB, pf = random_state(n, d, lo, hi, 1.0, seed, pf_mode="inf")
+    if pf_mode == "mixed":
+        # pf around the oracle's next f, +-50%: both pbest branches, clear margins
+        probe = cpu_swarm(n, d, obj, seed=seed, create=False).set_state(X, V, PB, pf, t=t0)
+        probe.step(1)
+        rng = np.random.default_rng(seed + 1)
+        pf = (probe.f * rng.choice([0.5, 1.5], size=n)).astype(np.float32)
+        pf[probe.f < 0] = probe.f[probe.f < 0] * 0.5
+    g = gpu_swarm(n, d, obj, seed=seed).set_state(X, V, PB, pf, t=t0)
+    c = cpu_swarm(n, d, obj, seed=seed, create=False).set_state(X, V, PB, pf, t=t0)
+    gf0, gi0, G0 = g.gbest()
+    assert gi0 == c.gi and gf0 == c.gf
+    assert_bitwise(G0, c.G, "G after set_state")
+    g.step(1)
+    c.step(1)
+    gX, gV, gPB, gpf, gt = g.get_state()
+    assert gt == t0 + 1 == c.t
+    assert_bitwise(gX, c.X, "X")
+    assert_bitwise(gV, c.V, "V")
+    # pbest decisions: equal unless ambiguous
+    tol = fit_tol(obj, c.X, c.f)
+    amb = np.abs(c.f.astype(np.float64) - pf.astype(np.float64)) <= tol
+    c_imp = c.f < pf
+    g_imp = (gpf.view(np.uint32) != pf.view(np.uint32)) | (gPB != PB).any(axis=1)
+    assert ((g_imp == c_imp) | amb).all(), np.argwhere((g_imp != c_imp) & ~amb)[:5]
+    agree = (g_imp == c_imp) & ~amb
+    assert_bitwise(gPB[agree], c.PB[agree], "PB")
+    imp = agree & c_imp
+    assert_fitness_close(obj, c.X[imp], gpf[imp], c.pf[imp], "pf (improved rows)")
+    assert_bitwise(gpf[agree & ~c_imp], pf[agree & ~c_imp], "pf (kept rows)")
+    gf, gi, G = g.gbest()
+    assert_bitwise(G, gPB[gi], "G == PB[gi]")
+    if not amb.any():
+        assert gi == c.gi
+    return g, c
+
+
+@pytest.mark.parametrize("obj", OBJS)
+@pytest.mark.parametrize("n,d", SHAPES)
+def test_single_step_all_improve(obj, n, d):
+    _step_and_compare(obj, n, d, seed=1000 + 7 * n + d, pf_mode="inf", t0=0)
+
+
+@pytest.mark.parametrize("obj", [SPHERE, RASTRIGIN, ROSENBROCK, GRIEWANK, ACKLEY])
+@pytest.mark.parametrize("n,d", [(257, 13), (300, 1000), (70, 2000), (9, 4096)])
+def test_single_step_mixed_pbest(obj, n, d):
+    _step_and_compare(obj, n, d, seed=2000 + n + d, pf_mode="mixed", t0=41)
+
+
+# ------------------------------------------------------------------ multi-step
+def test_lockstep_c1_100_iterations():
+    """C1 (Sphere 32x10): at every one of 100 iterations the oracle, restarted
+    from the GPU's state, must reproduce the GPU's next state."""
+    w = WORKLOADS["C1"]
+    g = gpu_swarm(w.n, w.d, w.objective, seed=w.seed)
+    c = cpu_swarm(w.n, w.d, w.objective, seed=w.seed)
+    for it in range(w.iters):
+        X, V, PB, pf, t = g.get_state()
+        gf, gi, G = g.gbest()
+        c.set_state(X, V, PB, pf, t=t)
+        assert c.gi == gi
+        g.step(1)
+        c.step(1)
+        X2, V2, PB2, pf2, _ = g.get_state()
+        assert_bitwise(X2, c.X, f"X it={it}")
+        assert_bitwise(V2, c.V, f"V it={it}")
+        assert_fitness_close(SPHERE, c.PB, pf2, c.pf, f"pf it={it}")
+
+
+def test_end_to_end_c1_100_iterations():
+    w = WORKLOADS["C1"]
+    g = gpu_swarm(w.n, w.d, w.objective, seed=w.seed)
+    c = cpu_swarm(w.n, w.d, w.objective, seed=w.seed)
+    g.step(w.iters)
+    c.step(w.iters)
+    gf, gi, G = g.gbest()
+    assert gf == pytest.approx(c.gf, rel=1e-4)
+    X, V, PB, pf, t = g.get_state()
+    assert t == w.iters
+    assert gi == c.gi
+    assert_bitwise(X, c.X, "X after 100 iterations")
+
+
+@pytest.mark.parametrize("obj", [RASTRIGIN, ROSENBROCK, GRIEWANK, ACKLEY])
+def test_end_to_end_independent_runs(obj):
+    n, d, T = 64, 37, 50
+    g = gpu_swarm(n, d, obj, seed=5)
+    c = cpu_swarm(n, d, obj, seed=5)
+    g.step(T)
+    c.step(T)
+    gf, gi, G = g.gbest()
+    assert gf == pytest.approx(c.gf, rel=1e-4, abs=1e-5)
+
+
+# ------------------------------------------------------------------ invariants
+@pytest.mark.parametrize("obj,n,d", [(RASTRIGIN, 1024, 1000), (ROSENBROCK, 500, 1001),
+                                     (GRIEWANK, 300, 2000), (ACKLEY, 100, 4096)])
+def test_invariants_over_run(obj, n, d):
+    lo, hi = DOMAINS[obj]
+    g = gpu_swarm(n, d, obj, seed=n)
+    prev_pf, prev_gf = g.get_state()[3], g.gbest(pos=False)[0]
+    for _ in range(10):
+        g.step(3)
+        X, V, PB, pf, t = g.get_state()
+        gf, gi, G = g.gbest()
+        assert (X >= np.float32(lo)).all() and (X <= np.float32(hi)).all()
+        assert (np.abs(V) <= g.vmax).all()
+        assert (pf <= prev_pf).all() and gf <= prev_gf
+        assert gf == pf.min() and pf[gi] == gf
+        assert_bitwise(G, PB[gi], "G == PB[gi]")
+        prev_pf, prev_gf = pf, gf
+
+
+# ------------------------------------------------------------------ API semantics
+def test_step_splitting_and_determinism():
+    a = gpu_swarm(200, 300, RASTRIGIN, seed=9)
+    b = gpu_swarm(200, 300, RASTRIGIN, seed=9)
+    a.step(7)
+    b.step(3).step(0).step(4)
+    for x, y in zip(a.get_state()[:4], b.get_state()[:4]):
+        assert_bitwise(x, y, "split")
+    assert a.gbest()[:2] == b.gbest()[:2]
+    c = gpu_swarm(200, 300, RASTRIGIN, seed=10)
+    assert not np.array_equal(a.get_state()[0], c.step(7).get_state()[0])
+
+
+def test_launch_counter_and_improvements():
+    g = gpu_swarm(1000, 256, SPHERE, seed=3, timing=True)
+    g.reset_counters()
+    g.step(20)
+    info = g.info()
+    assert info["launches"] == 20
+    assert info["step_kernel_count"] == 20 and info["step_kernel_ms"] > 0
+    assert 0 < info["improvements"] <= 20 * 1000
+
+
+def test_errors_do_not_abort():
+    with pytest.raises(fp.PsoError) as e:
+        gpu_swarm(0, 10, SPHERE)
+    assert e.value.status == 1
+    with pytest.raises(fp.PsoError) as e:
+        gpu_swarm(10, 10000, SPHERE)
+    assert e.value.status == 5
+    g = gpu_swarm(10, 10, SPHERE)
+    with pytest.raises(fp.PsoError):
+        g.step(-1)
+    with pytest.raises(ValueError):
+        g.set_state(np.zeros((9, 10)), np.zeros((10, 10)), np.zeros((10, 10)), np.zeros(10))
+    fp.lib().pso_destroy(None)
+
+
+# ------------------------------------------------------------------ full size, sampled
+@pytest.mark.parametrize("key", ["NS", "C4"])
+def test_full_size_sampled_rows(key):
+    """Bench configuration (100k x 2000) in the bench's launch shape: the
+    oracle recomputes sampled rows of one iteration exactly (rows are
+    independent given G), and the gbest invariants hold over the whole swarm."""
+    w = WORKLOADS[key]
+    g = gpu_swarm(w.n, w.d, w.objective, seed=w.seed)
+    idx = sample_rows(w.n, 48, seed=7)
+    X0, V0, _, _, _ = g.get_state()
+    # init rows are bit-exact
+    for i in idx[:8]:
+        c = orc.OracleSwarm(w.n, w.d, w.w, w.c1, w.c2, w.lo, w.hi, w.objective, w.seed,
+                            row_begin=int(i), nrows=1, create=False)
+        c.init_local()
+        assert_bitwise(X0[i], c.X[0], f"X0 row {i}")
+        assert_bitwise(V0[i], c.V[0], f"V0 row {i}")
+    del X0, V0
+    g.step(2)
+    X, V, PB, pf, t = g.get_state()
+    _, _, G = g.gbest()
+    g.step(1)
+    X2, V2, PB2, pf2, t2 = g.get_state()
+    gf, gi, G2 = g.gbest()
+    c = cpu_swarm(w.n, w.d, w.objective, seed=w.seed, create=False)
+    cX, cV, cPB, cpf, cf = c.rows_step(t + 1, G, idx, X[idx], V[idx], PB[idx], pf[idx])
+    assert_bitwise(X2[idx], cX, "X rows")
+    assert_bitwise(V2[idx], cV, "V rows")
+    tol = fit_tol(w.objective, cX, cf)
+    amb = np.abs(cf.astype(np.float64) - pf[idx].astype(np.float64)) <= tol
+    ok = ~amb
+    assert_bitwise(PB2[idx][ok], cPB[ok], "PB rows")
+    assert_fitness_close(w.objective, cPB[ok], pf2[idx][ok], cpf[ok], "pf rows")
+    assert gf == pf2.min() and gi == int(np.argmin(pf2))
+    assert_bitwise(G2, PB2[gi], "G == PB[gi]")
