@@ -154,6 +154,9 @@ typedef struct {
   int32_t d, pitch;              /* dimension, row pitch in floats (16-B rows) */
   int32_t rank, world;
   int32_t threads_per_cta, vec_per_thread, grid, ctas_per_sm;
+  int32_t tma_pipeline;          /* 1: bulk-copy (TMA) pipelined step kernel */
+  int32_t pipeline_stages;       /* rows in flight per CTA in that pipeline */
+  int32_t smem_bytes;            /* dynamic shared memory of the step kernel */
   float vmax;
   uint64_t t;                    /* iterations done */
   uint64_t launches;             /* kernels launched by this handle so far */

@@ -332,11 +332,16 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
   h->n_local = (n * (h->rank + 1)) / h->world - h->row_begin;
 
   // ---- launch plan
-  int vpt_override = 0;
-  if (const char* v = std::getenv("PSO_VPT")) vpt_override = std::atoi(v);
+  PlanHints hints;
+  if (const char* v = std::getenv("PSO_VPT")) hints.vpt = std::atoi(v);
+  if (const char* v = std::getenv("PSO_STAGES")) hints.stages = std::atoi(v);
+  if (const char* v = std::getenv("PSO_KERNEL")) {
+    if (!std::strcmp(v, "reg")) hints.kernel = 0;
+    if (!std::strcmp(v, "tma")) hints.kernel = 1;
+  }
   {
     cudaError_t e = plan_launch(objective, d, h->n_local > 0 ? h->n_local : 1, h->sm_count,
-                                vpt_override, &h->cfg);
+                                hints, &h->cfg);
     if (e != cudaSuccess) return bail(cuda_fail(nullptr, e, "plan_launch"));
   }
 
@@ -545,6 +550,9 @@ pso_status pso_get_info(pso_handle h, pso_info* info) {
   info->vec_per_thread = h->cfg.vpt;
   info->grid = h->cfg.grid;
   info->ctas_per_sm = h->cfg.ctas_per_sm;
+  info->tma_pipeline = h->cfg.tma;
+  info->pipeline_stages = h->cfg.stages;
+  info->smem_bytes = (int32_t)h->cfg.smem;
   info->vmax = h->vmax;
   info->t = h->t;
   info->launches = h->launches;

@@ -40,16 +40,27 @@ struct SwarmArgs {
 };
 
 struct LaunchCfg {
-  int vpt = 1;       // float4 per thread per row
-  int threads = 32;  // CTA size
-  int grid = 1;      // persistent grid
+  int vpt = 1;        // float4 per compute thread per row
+  int compute = 32;   // compute threads per CTA (one row per CTA at a time)
+  int threads = 32;   // CTA size (compute + 32 producer threads for the TMA pipeline)
+  int grid = 1;       // persistent grid
   int ctas_per_sm = 1;
-  size_t smem = 0;   // dynamic shared memory bytes
+  int tma = 0;        // 1: warp-specialised bulk-copy (TMA) pipeline; 0: register streaming
+  int stages = 0;     // TMA pipeline depth (rows in flight per CTA)
+  size_t smem = 0;    // dynamic shared memory bytes of the step kernel
+  size_t init_smem = 0;
+};
+
+// Tuning overrides (0 / -1 = automatic): PSO_VPT, PSO_KERNEL=reg|tma, PSO_STAGES.
+struct PlanHints {
+  int vpt = 0;
+  int kernel = -1;  // -1 auto, 0 register, 1 tma
+  int stages = 0;
 };
 
 bool objective_registered(int objective);
 // Choose the CTA shape for d and size the persistent grid for n_local rows.
-cudaError_t plan_launch(int objective, int d, long long n_local, int sm_count, int vpt_override,
+cudaError_t plan_launch(int objective, int d, long long n_local, int sm_count, const PlanHints& h,
                         LaunchCfg* cfg);
 cudaError_t launch_init(int objective, const SwarmArgs& a, const LaunchCfg& c, cudaStream_t s);
 cudaError_t launch_step(int objective, const SwarmArgs& a, const LaunchCfg& c, cudaStream_t s);

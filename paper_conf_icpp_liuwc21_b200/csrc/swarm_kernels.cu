@@ -2,7 +2,7 @@
 //
 // One kernel per iteration replaces the paper's five phases (Fig. 5, P:L561-567:
 // init / eval / pbest / gbest / swarm) and its materialised random matrices.
-// Per particle row (one CTA per row, persistent grid):
+// Per particle row (one CTA per row at a time, persistent grid):
 //
 //   A1  r1, r2 = Philox4x32-10(seed, t, i, q) in registers        (Eq. 1 l, g)
 //   A2  v' = (w v + (c1 r1)(pb - x)) + (c2 r2)(g - x)              (Eq. 1/4)
@@ -17,6 +17,15 @@
 // (x, v) + 4 rho B (pbest copy) + (4 + 4 rho)/d (pf).  G (4 d B) is staged
 // into shared memory once per CTA per iteration by a bulk async copy (TMA
 // engine, cp.async.bulk + mbarrier) and read from there for every row.
+//
+// Two variants of the step kernel share the row arithmetic:
+//   k_step_tma  (rows of >= 256 dims): warp-specialised.  One producer warp
+//               streams whole x / v / pb rows into a ring of shared-memory
+//               stages with cp.async.bulk (TMA engine) and mbarrier
+//               complete_tx; the compute warps drain the ring.  Memory-level
+//               parallelism is the ring depth, independent of registers.
+//   k_step_reg  (short rows): every thread loads its float4s with 128-bit
+//               LDGs; many rows per SM in flight through occupancy.
 #include <cuda_runtime.h>
 
 #include <cstdint>
@@ -28,7 +37,8 @@
 namespace fastpso {
 namespace {
 
-constexpr int kMaxThreads = 256;
+constexpr int kMaxThreads = 256;  // compute threads per CTA
+constexpr int kMaxStages = 8;
 constexpr unsigned kFull = 0xFFFFFFFFu;
 
 // ---------------------------------------------------------------- helpers
@@ -55,13 +65,20 @@ __device__ __forceinline__ void st_stream(float4* p, float4 v) {
                : "memory");
 }
 
-// --- bulk async copy global -> shared (TMA engine) with an mbarrier -------
+// Named barrier 1 over the n compute threads (the producer warp never joins).
+__device__ __forceinline__ void team_sync(int n) {
+  asm volatile("bar.sync 1, %0;" ::"r"(n) : "memory");
+}
+
+// --- mbarrier + bulk async copy global -> shared (TMA engine) -------------
 __device__ __forceinline__ uint32_t smem_addr(const void* p) {
   return (uint32_t)__cvta_generic_to_shared(p);
 }
 __device__ __forceinline__ void mbar_init(unsigned long long* bar, unsigned count) {
   asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_addr(bar)), "r"(count)
                : "memory");
+}
+__device__ __forceinline__ void mbar_fence_init() {
   asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
 }
 __device__ __forceinline__ void mbar_expect_tx(unsigned long long* bar, unsigned bytes) {
@@ -69,13 +86,8 @@ __device__ __forceinline__ void mbar_expect_tx(unsigned long long* bar, unsigned
                "r"(bytes)
                : "memory");
 }
-__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, unsigned bytes,
-                                         unsigned long long* bar) {
-  asm volatile(
-      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::
-          "r"(smem_addr(dst)),
-      "l"(src), "r"(bytes), "r"(smem_addr(bar))
-      : "memory");
+__device__ __forceinline__ void mbar_arrive(unsigned long long* bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_addr(bar)) : "memory");
 }
 __device__ __forceinline__ void mbar_wait(unsigned long long* bar, unsigned phase) {
   asm volatile(
@@ -88,16 +100,13 @@ __device__ __forceinline__ void mbar_wait(unsigned long long* bar, unsigned phas
       "r"(phase)
       : "memory");
 }
-
-// Stage G (nvec float4) into shared memory: one bulk copy issued by thread 0.
-__device__ __forceinline__ void stage_gbest(float4* sG, const float* G, int nvec,
-                                            unsigned long long* bar) {
-  if (threadIdx.x == 0) {
-    mbar_init(bar, 1);
-    mbar_expect_tx(bar, (unsigned)nvec * 16u);
-    bulk_g2s(sG, G, (unsigned)nvec * 16u, bar);
-  }
-  __syncthreads();  // barrier initialised before anyone waits on it
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, unsigned bytes,
+                                         unsigned long long* bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::
+          "r"(smem_addr(dst)),
+      "l"(src), "r"(bytes), "r"(smem_addr(bar))
+      : "memory");
 }
 
 // --- Eq. 1, 5, 2 on one element, fixed fp32 order, no contraction --------
@@ -133,28 +142,28 @@ struct RowSmem {
   float red[32 * Obj::kAcc];
   float f;
   int improved;
-  unsigned long long bar;
   int last;
+  unsigned long long gbar;  // gbest staging barrier
+  unsigned long long acc, cur;
 };
 
-// Reduce a[] over the CTA (fixed order: lanes by xor-butterfly, then warps in
-// order), finalize in thread 0 and decide the pbest update against pf_old
-// (only thread 0's pf_old is read).  Returns f to all threads; *improved is
-// the CTA-uniform pbest decision.  Two __syncthreads.
+// Reduce a[] over the nthr compute threads (fixed order: lanes by
+// xor-butterfly, then warps in index order), finalize in thread 0 and decide
+// the pbest update against pf_old (only thread 0's pf_old is read).
 template <class Obj>
 __device__ __forceinline__ float cta_fitness(float* a, RowSmem<Obj>& sm, int d, float pf_old,
-                                             bool& improved) {
+                                             bool& improved, int tid, int nthr) {
   warp_combine<Obj>(a);
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int warp = tid >> 5, lane = tid & 31;
   if (lane == 0) {
 #pragma unroll
     for (int k = 0; k < Obj::kAcc; ++k) sm.red[warp * Obj::kAcc + k] = a[k];
   }
-  __syncthreads();
+  team_sync(nthr);
   if (warp == 0) {
     float c[Obj::kAcc];
     Obj::init(c);
-    if (lane < (int)(blockDim.x >> 5)) {
+    if (lane < (nthr >> 5)) {
 #pragma unroll
       for (int k = 0; k < Obj::kAcc; ++k) c[k] = sm.red[lane * Obj::kAcc + k];
     }
@@ -165,7 +174,7 @@ __device__ __forceinline__ float cta_fitness(float* a, RowSmem<Obj>& sm, int d, 
       sm.improved = (f < pf_old) ? 1 : 0;  // strict; NaN never improves
     }
   }
-  __syncthreads();
+  team_sync(nthr);
   improved = sm.improved != 0;
   return sm.f;
 }
@@ -174,18 +183,18 @@ __device__ __forceinline__ float cta_fitness(float* a, RowSmem<Obj>& sm, int d, 
 // that need x_{j+1} the first element of every float4 is published in sFirst.
 template <class Obj, int VPT>
 __device__ __forceinline__ void map_row(float* acc, const float4 (&x)[VPT], float* sFirst,
-                                        int nvec, int d) {
+                                        int nvec, int d, int tid, int nthr) {
   if constexpr (Obj::kNeighbor) {
 #pragma unroll
     for (int s = 0; s < VPT; ++s) {
-      const int q = threadIdx.x + s * blockDim.x;
+      const int q = tid + s * nthr;
       if (q < nvec) sFirst[q] = x[s].x;
     }
-    __syncthreads();
+    team_sync(nthr);
   }
 #pragma unroll
   for (int s = 0; s < VPT; ++s) {
-    const int q = threadIdx.x + s * blockDim.x;
+    const int q = tid + s * nthr;
     if (q < nvec) {
       const int j = 4 * q;
       float nx = 0.f;
@@ -204,28 +213,84 @@ __device__ __forceinline__ void map_row(float* acc, const float4 (&x)[VPT], floa
   }
 }
 
+// A2-A6 for one row: update, store x' / v', evaluate, pbest compare-and-copy.
+// src(s, q, x, v, pb) supplies the operands of float4 q (slot s) — from
+// registers (k_step_reg) or from the shared-memory stage (k_step_tma);
+// release() runs once every operand has been read.  x' stays in registers
+// (xn) until the pbest decision.  Returns f; `improved` is CTA-uniform.
+template <class Obj, int VPT, class Src, class Release>
+__device__ __forceinline__ float process_row(const SwarmArgs& a, const MoveParams& mp,
+                                             PhiloxKey key, uint32_t t, uint32_t gi, long long r,
+                                             Src&& src, Release&& release, const float4* sG,
+                                             float* sFirst, RowSmem<Obj>& sm, int tid, int nthr,
+                                             float pf_old, bool& improved) {
+  const int nvec = a.nvec, d = a.d;
+  float4* Xr = reinterpret_cast<float4*>(a.X) + r * nvec;
+  float4* Vr = reinterpret_cast<float4*>(a.V) + r * nvec;
+  float4* Pr = reinterpret_cast<float4*>(a.PB) + r * nvec;
+  float4 xn[VPT];
+#pragma unroll
+  for (int s = 0; s < VPT; ++s) {
+    const int q = tid + s * nthr;
+    if (q < nvec) {
+      float4 x, v, pb;
+      src(s, q, x, v, pb);
+      const float4 g = sG[q];
+      const float4 r1 = uniforms4(key, kTagR1, t, gi, (uint32_t)q);
+      const float4 r2 = uniforms4(key, kTagR2, t, gi, (uint32_t)q);
+      move1(mp, x.x, v.x, pb.x, g.x, r1.x, r2.x);
+      move1(mp, x.y, v.y, pb.y, g.y, r1.y, r2.y);
+      move1(mp, x.z, v.z, pb.z, g.z, r1.z, r2.z);
+      move1(mp, x.w, v.w, pb.w, g.w, r1.w, r2.w);
+      if ((d & 3) && q == nvec - 1) {  // keep the row padding at zero
+        const int j = 4 * q;
+        if (j + 1 >= d) x.y = v.y = 0.f;
+        if (j + 2 >= d) x.z = v.z = 0.f;
+        if (j + 3 >= d) x.w = v.w = 0.f;
+      }
+      st_stream(Xr + q, x);
+      st_stream(Vr + q, v);
+      xn[s] = x;
+    }
+  }
+  release();
+  float acc[Obj::kAcc];
+  Obj::init(acc);
+  map_row<Obj, VPT>(acc, xn, sFirst, nvec, d, tid, nthr);
+  const float f = cta_fitness<Obj>(acc, sm, d, pf_old, improved, tid, nthr);
+  if (improved) {
+#pragma unroll
+    for (int s = 0; s < VPT; ++s) {
+      const int q = tid + s * nthr;
+      if (q < nvec) st_stream(Pr + q, xn[s]);
+    }
+  }
+  return f;
+}
+
 // Last-CTA epilogue: publish the iteration's gbest.  world == 1: copy PB[gi]
 // into G and advance the incumbent key.  world > 1: write the local candidate
 // record (key, PB row) for the all-gather; the select kernel finishes.
-__device__ __forceinline__ void gbest_epilogue(const SwarmArgs& a, uint32_t t) {
-  __shared__ unsigned long long s_acc, s_cur;
-  if (threadIdx.x == 0) {
+template <class Obj>
+__device__ __forceinline__ void gbest_epilogue(const SwarmArgs& a, RowSmem<Obj>& sm, uint32_t t,
+                                               int tid, int nthr) {
+  if (tid == 0) {
     __threadfence();
-    s_acc = *(volatile unsigned long long*)&a.ctl->key_acc;
-    s_cur = a.ctl->key_cur;
+    sm.acc = *(volatile unsigned long long*)&a.ctl->key_acc;
+    sm.cur = a.ctl->key_cur;
   }
-  __syncthreads();
-  const unsigned long long acc = s_acc, cur = s_cur;
+  team_sync(nthr);
+  const unsigned long long acc = sm.acc, cur = sm.cur;
   const bool have = acc < cur;
   const float4* src = nullptr;
-  if (have) src = reinterpret_cast<const float4*>(a.PB) +
-                  ((long long)(uint32_t)acc - a.row_begin) * a.nvec;
+  if (have)
+    src = reinterpret_cast<const float4*>(a.PB) + ((long long)(uint32_t)acc - a.row_begin) * a.nvec;
   if (a.world == 1) {
     if (have) {
       float4* G4 = reinterpret_cast<float4*>(a.G);
-      for (int q = threadIdx.x; q < a.nvec; q += blockDim.x) G4[q] = __ldcg(src + q);
+      for (int q = tid; q < a.nvec; q += nthr) G4[q] = __ldcg(src + q);
     }
-    if (threadIdx.x == 0) {
+    if (tid == 0) {
       if (have) a.ctl->key_cur = acc;
       a.ctl->t = t;
       a.ctl->done = 0;
@@ -234,8 +299,8 @@ __device__ __forceinline__ void gbest_epilogue(const SwarmArgs& a, uint32_t t) {
     unsigned long long* hdr = reinterpret_cast<unsigned long long*>(a.send);
     float4* row = reinterpret_cast<float4*>(a.send + 16);
     if (have)
-      for (int q = threadIdx.x; q < a.nvec; q += blockDim.x) row[q] = __ldcg(src + q);
-    if (threadIdx.x == 0) {
+      for (int q = tid; q < a.nvec; q += nthr) row[q] = __ldcg(src + q);
+    if (tid == 0) {
       hdr[0] = have ? acc : ~0ull;
       hdr[1] = 0;
       a.ctl->t = t;
@@ -244,104 +309,168 @@ __device__ __forceinline__ void gbest_epilogue(const SwarmArgs& a, uint32_t t) {
   }
 }
 
-// Publish this CTA's candidate and improvement count; returns true in the
-// last CTA to finish (which then runs gbest_epilogue).
+// Publish this CTA's candidate and improvement count; true in the last CTA
+// to finish (which then runs gbest_epilogue).
 template <class Obj>
 __device__ __forceinline__ bool cta_finish(const SwarmArgs& a, RowSmem<Obj>& sm,
-                                           unsigned long long best, unsigned nimp) {
-  __syncthreads();  // every PB / X / V store of this CTA is issued
-  if (threadIdx.x == 0) {
+                                           unsigned long long best, unsigned nimp, int tid,
+                                           int nthr) {
+  team_sync(nthr);  // every PB / X / V store of this CTA is issued
+  if (tid == 0) {
     if (best != ~0ull) atomicMin(&a.ctl->key_acc, best);
     if (nimp) atomicAdd(&a.ctl->improvements, (unsigned long long)nimp);
     __threadfence();
     const unsigned ticket = atomicAdd(&a.ctl->done, 1u);
     sm.last = (ticket == gridDim.x - 1) ? 1 : 0;
   }
-  __syncthreads();
+  team_sync(nthr);
   return sm.last != 0;
 }
 
-// ------------------------------------------------------------ step kernel
+__device__ __forceinline__ void row_bookkeeping(const SwarmArgs& a, long long r, uint32_t gi,
+                                                float f, bool improved, uint32_t inc_ord,
+                                                unsigned long long& best, unsigned& nimp) {
+  if (improved) {
+    a.pf[r] = f;
+    ++nimp;
+  }
+  if (f == f && ord_f32(f) < inc_ord) {  // strictly below gf (Alg. 1 line 10)
+    const unsigned long long k = pack_key(f, gi);
+    best = k < best ? k : best;
+  }
+}
+
+// ------------------------------------------------- step kernel: registers
 template <class Obj, int VPT>
 __global__ void __launch_bounds__(kMaxThreads, (VPT >= 8) ? 1 : 2)
-    k_step(const SwarmArgs a) {
-  extern __shared__ __align__(16) unsigned char dsmem[];
+    k_step_reg(const SwarmArgs a, int /*stages: unused, same signature as k_step_tma*/) {
+  extern __shared__ __align__(128) unsigned char dsmem[];
   float4* sG = reinterpret_cast<float4*>(dsmem);
   float* sFirst = reinterpret_cast<float*>(sG + a.nvec);
   __shared__ RowSmem<Obj> sm;
-
-  stage_gbest(sG, a.G, a.nvec, &sm.bar);
+  const int tid = threadIdx.x, nthr = blockDim.x;
+  if (tid == 0) {
+    mbar_init(&sm.gbar, 1);
+    mbar_fence_init();
+    mbar_expect_tx(&sm.gbar, (unsigned)a.nvec * 16u);
+    bulk_g2s(sG, a.G, (unsigned)a.nvec * 16u, &sm.gbar);
+  }
+  __syncthreads();
   const uint32_t t = a.ctl->t + 1u;
   const uint32_t inc_ord = (uint32_t)(a.ctl->key_cur >> 32);
   const PhiloxKey key{a.seed_lo, a.seed_hi};
   const MoveParams mp{a.w, a.c1, a.c2, a.lo, a.hi, a.vmax};
-  const int nvec = a.nvec, d = a.d;
-  const bool ragged = (d & 3) != 0;
-  mbar_wait(&sm.bar, 0);
+  const int nvec = a.nvec;
+  mbar_wait(&sm.gbar, 0);
 
   unsigned long long best = ~0ull;
   unsigned nimp = 0;
   for (long long r = blockIdx.x; r < a.n_local; r += gridDim.x) {
     const uint32_t gi = (uint32_t)(a.row_begin + r);
-    float4* Xr = reinterpret_cast<float4*>(a.X) + r * nvec;
-    float4* Vr = reinterpret_cast<float4*>(a.V) + r * nvec;
-    float4* Pr = reinterpret_cast<float4*>(a.PB) + r * nvec;
+    const float4* Xr = reinterpret_cast<const float4*>(a.X) + r * nvec;
+    const float4* Vr = reinterpret_cast<const float4*>(a.V) + r * nvec;
+    const float4* Pr = reinterpret_cast<const float4*>(a.PB) + r * nvec;
     float4 x[VPT], v[VPT], pb[VPT];
 #pragma unroll
     for (int s = 0; s < VPT; ++s) {
-      const int q = threadIdx.x + s * blockDim.x;
+      const int q = tid + s * nthr;
       if (q < nvec) {
         x[s] = ld_stream(Xr + q);
         v[s] = ld_stream(Vr + q);
         pb[s] = ld_stream(Pr + q);
       }
     }
-    const float pf_old = (threadIdx.x == 0) ? a.pf[r] : 0.f;
-#pragma unroll
-    for (int s = 0; s < VPT; ++s) {
-      const int q = threadIdx.x + s * blockDim.x;
-      if (q < nvec) {
-        const float4 g = sG[q];
-        const float4 r1 = uniforms4(key, kTagR1, t, gi, (uint32_t)q);
-        const float4 r2 = uniforms4(key, kTagR2, t, gi, (uint32_t)q);
-        move1(mp, x[s].x, v[s].x, pb[s].x, g.x, r1.x, r2.x);
-        move1(mp, x[s].y, v[s].y, pb[s].y, g.y, r1.y, r2.y);
-        move1(mp, x[s].z, v[s].z, pb[s].z, g.z, r1.z, r2.z);
-        move1(mp, x[s].w, v[s].w, pb[s].w, g.w, r1.w, r2.w);
-        if (ragged && q == nvec - 1) {  // keep the row padding at zero
-          const int j = 4 * q;
-          if (j + 1 >= d) x[s].y = v[s].y = 0.f;
-          if (j + 2 >= d) x[s].z = v[s].z = 0.f;
-          if (j + 3 >= d) x[s].w = v[s].w = 0.f;
-        }
-        st_stream(Xr + q, x[s]);
-        st_stream(Vr + q, v[s]);
-      }
-    }
-    float acc[Obj::kAcc];
-    Obj::init(acc);
-    map_row<Obj, VPT>(acc, x, sFirst, nvec, d);
+    const float pf_old = (tid == 0) ? a.pf[r] : 0.f;
     bool improved;
-    const float f = cta_fitness<Obj>(acc, sm, d, pf_old, improved);
-    if (improved) {
-#pragma unroll
-      for (int s = 0; s < VPT; ++s) {
-        const int q = threadIdx.x + s * blockDim.x;
-        if (q < nvec) st_stream(Pr + q, x[s]);
-      }
-    }
-    if (threadIdx.x == 0) {
-      if (improved) {
-        a.pf[r] = f;
-        ++nimp;
-      }
-      if (f == f && ord_f32(f) < inc_ord) {  // strictly below gf (Alg. 1 line 10)
-        const unsigned long long k = pack_key(f, gi);
-        best = k < best ? k : best;
-      }
-    }
+    const float f = process_row<Obj, VPT>(
+        a, mp, key, t, gi, r,
+        [&](int s, int, float4& xo, float4& vo, float4& po) {
+          xo = x[s];
+          vo = v[s];
+          po = pb[s];
+        },
+        [] {}, sG, sFirst, sm, tid, nthr, pf_old, improved);
+    if (tid == 0) row_bookkeeping(a, r, gi, f, improved, inc_ord, best, nimp);
   }
-  if (cta_finish<Obj>(a, sm, best, nimp)) gbest_epilogue(a, t);
+  if (cta_finish<Obj>(a, sm, best, nimp, tid, nthr)) gbest_epilogue<Obj>(a, sm, t, tid, nthr);
+}
+
+// ------------------------------------------------- step kernel: TMA pipeline
+// Warps 0..C/32-1 compute; the last warp is the producer.  Shared memory:
+// [G: nvec float4][stages x {x, v, pb}: nvec float4 each][sFirst].
+template <class Obj, int VPT>
+__global__ void __launch_bounds__(kMaxThreads + 32, (VPT <= 2) ? 2 : 1)
+    k_step_tma(const SwarmArgs a, int stages) {
+  extern __shared__ __align__(128) unsigned char dsmem[];
+  const int nvec = a.nvec;
+  const int nthr = (int)blockDim.x - 32;  // compute threads
+  float4* sG = reinterpret_cast<float4*>(dsmem);
+  float4* ring = sG + nvec;
+  float* sFirst = reinterpret_cast<float*>(ring + (size_t)stages * 3 * nvec);
+  __shared__ RowSmem<Obj> sm;
+  __shared__ unsigned long long full[kMaxStages], empty[kMaxStages];
+  const int tid = threadIdx.x;
+  if (tid == 0) {
+    mbar_init(&sm.gbar, 1);
+    for (int s = 0; s < stages; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&empty[s], (unsigned)(nthr >> 5));
+    }
+    mbar_fence_init();
+  }
+  __syncthreads();
+  const uint32_t t = a.ctl->t + 1u;
+
+  if (tid >= nthr) {  // ---------------- producer warp
+    if (tid == nthr) {
+      const unsigned row_bytes = (unsigned)nvec * 16u;
+      mbar_expect_tx(&sm.gbar, row_bytes);
+      bulk_g2s(sG, a.G, row_bytes, &sm.gbar);
+      int k = 0;
+      for (long long r = blockIdx.x; r < a.n_local; r += gridDim.x, ++k) {
+        const int s = k % stages;
+        if (k >= stages) mbar_wait(&empty[s], ((unsigned)(k / stages) & 1u) ^ 1u);
+        float4* st = ring + (size_t)s * 3 * nvec;
+        mbar_expect_tx(&full[s], 3u * row_bytes);
+        bulk_g2s(st, a.X + (size_t)r * 4 * nvec, row_bytes, &full[s]);
+        bulk_g2s(st + nvec, a.V + (size_t)r * 4 * nvec, row_bytes, &full[s]);
+        bulk_g2s(st + 2 * nvec, a.PB + (size_t)r * 4 * nvec, row_bytes, &full[s]);
+      }
+    }
+    return;
+  }
+
+  // ---------------- compute warps
+  const uint32_t inc_ord = (uint32_t)(a.ctl->key_cur >> 32);
+  const PhiloxKey key{a.seed_lo, a.seed_hi};
+  const MoveParams mp{a.w, a.c1, a.c2, a.lo, a.hi, a.vmax};
+  const int lane = tid & 31;
+  mbar_wait(&sm.gbar, 0);
+  unsigned long long best = ~0ull;
+  unsigned nimp = 0;
+  int k = 0;
+  for (long long r = blockIdx.x; r < a.n_local; r += gridDim.x, ++k) {
+    const int s = k % stages;
+    const uint32_t gi = (uint32_t)(a.row_begin + r);
+    const float pf_old = (tid == 0) ? a.pf[r] : 0.f;
+    const float4* st = ring + (size_t)s * 3 * nvec;
+    mbar_wait(&full[s], (unsigned)(k / stages) & 1u);
+    bool improved;
+    const float f = process_row<Obj, VPT>(
+        a, mp, key, t, gi, r,
+        [&](int, int q, float4& xo, float4& vo, float4& po) {
+          xo = st[q];
+          vo = st[nvec + q];
+          po = st[2 * nvec + q];
+        },
+        [&] {
+          __syncwarp();
+          if (lane == 0) mbar_arrive(&empty[s]);  // stage may be refilled
+        },
+        sG, sFirst, sm, tid, nthr, pf_old, improved);
+    if (tid == 0) row_bookkeeping(a, r, gi, f, improved, inc_ord, best, nimp);
+  }
+  if (cta_finish<Obj>(a, sm, best, nimp, tid, nthr)) gbest_epilogue<Obj>(a, sm, t, tid, nthr);
 }
 
 // ------------------------------------------------------------ init kernel
@@ -351,10 +480,10 @@ __global__ void __launch_bounds__(kMaxThreads, (VPT >= 8) ? 1 : 2)
 template <class Obj, int VPT>
 __global__ void __launch_bounds__(kMaxThreads, (VPT >= 8) ? 1 : 2)
     k_init(const SwarmArgs a) {
-  extern __shared__ __align__(16) unsigned char dsmem[];
-  float4* sG = reinterpret_cast<float4*>(dsmem);
-  float* sFirst = reinterpret_cast<float*>(sG + a.nvec);
+  extern __shared__ __align__(128) unsigned char dsmem[];
+  float* sFirst = reinterpret_cast<float*>(dsmem);
   __shared__ RowSmem<Obj> sm;
+  const int tid = threadIdx.x, nthr = blockDim.x;
   const PhiloxKey key{a.seed_lo, a.seed_hi};
   const int nvec = a.nvec, d = a.d;
   const float span = __fsub_rn(a.hi, a.lo);
@@ -369,7 +498,7 @@ __global__ void __launch_bounds__(kMaxThreads, (VPT >= 8) ? 1 : 2)
     float4 x[VPT];
 #pragma unroll
     for (int s = 0; s < VPT; ++s) {
-      const int q = threadIdx.x + s * blockDim.x;
+      const int q = tid + s * nthr;
       if (q < nvec) {
         const float4 ux = uniforms4(key, kTagX0, 0u, gi, (uint32_t)q);
         const float4 uv = uniforms4(key, kTagV0, 0u, gi, (uint32_t)q);
@@ -389,10 +518,10 @@ __global__ void __launch_bounds__(kMaxThreads, (VPT >= 8) ? 1 : 2)
     }
     float acc[Obj::kAcc];
     Obj::init(acc);
-    map_row<Obj, VPT>(acc, x, sFirst, nvec, d);
+    map_row<Obj, VPT>(acc, x, sFirst, nvec, d, tid, nthr);
     bool improved;
-    float f = cta_fitness<Obj>(acc, sm, d, 0.f, improved);
-    if (threadIdx.x == 0) {
+    float f = cta_fitness<Obj>(acc, sm, d, 0.f, improved, tid, nthr);
+    if (tid == 0) {
       if (f != f) f = __int_as_float(0x7f800000);  // reading 11: NaN -> +inf
       a.pf[r] = f;
       if (ord_f32(f) < inc_ord) {
@@ -401,15 +530,18 @@ __global__ void __launch_bounds__(kMaxThreads, (VPT >= 8) ? 1 : 2)
       }
     }
   }
-  if (cta_finish<Obj>(a, sm, best, 0)) gbest_epilogue(a, 0u);
-  (void)sG;
+  if (cta_finish<Obj>(a, sm, best, 0, tid, nthr)) gbest_epilogue<Obj>(a, sm, 0u, tid, nthr);
 }
 
 // ---------------------------------------------------------- rebest kernel
 // After set_state: pf NaN -> +inf, gbest = lowest index attaining min pf.
+struct NoObj {
+  static constexpr int kAcc = 1;
+};
 __global__ void __launch_bounds__(256) k_rebest(const SwarmArgs a, unsigned t) {
   __shared__ unsigned long long s_best[8];
-  __shared__ int s_last;
+  __shared__ RowSmem<NoObj> sm;
+  const int tid = threadIdx.x, nthr = blockDim.x;
   unsigned long long best = ~0ull;
   for (long long r = blockIdx.x * (long long)blockDim.x + threadIdx.x; r < a.n_local;
        r += (long long)gridDim.x * blockDim.x) {
@@ -426,16 +558,12 @@ __global__ void __launch_bounds__(256) k_rebest(const SwarmArgs a, unsigned t) {
     const unsigned long long o = __shfl_xor_sync(kFull, best, off);
     best = o < best ? o : best;
   }
-  if ((threadIdx.x & 31) == 0) s_best[threadIdx.x >> 5] = best;
+  if ((tid & 31) == 0) s_best[tid >> 5] = best;
   __syncthreads();
-  if (threadIdx.x == 0) {
-    for (int w = 1; w < (int)(blockDim.x >> 5); ++w) best = s_best[w] < best ? s_best[w] : best;
-    if (best != ~0ull) atomicMin(&a.ctl->key_acc, best);
-    __threadfence();
-    s_last = (atomicAdd(&a.ctl->done, 1u) == gridDim.x - 1) ? 1 : 0;
-  }
-  __syncthreads();
-  if (s_last) gbest_epilogue(a, t);
+  if (tid == 0)
+    for (int w = 1; w < (nthr >> 5); ++w) best = s_best[w] < best ? s_best[w] : best;
+  if (cta_finish<NoObj>(a, sm, tid == 0 ? best : ~0ull, 0, tid, nthr))
+    gbest_epilogue<NoObj>(a, sm, t, tid, nthr);
 }
 
 // ---------------------------------------------------------- select kernel
@@ -490,67 +618,53 @@ __global__ void __launch_bounds__(128) k_select(const SwarmArgs a) {
 template <class Obj, int VPT>
 __global__ void __launch_bounds__(kMaxThreads) k_eval(const float* X, long long m, int d,
                                                       int nvec, float* out) {
-  extern __shared__ __align__(16) unsigned char dsmem[];
+  extern __shared__ __align__(128) unsigned char dsmem[];
   float* sFirst = reinterpret_cast<float*>(dsmem);
   __shared__ RowSmem<Obj> sm;
+  const int tid = threadIdx.x, nthr = blockDim.x;
   for (long long r = blockIdx.x; r < m; r += gridDim.x) {
     const float4* Xr = reinterpret_cast<const float4*>(X) + r * nvec;
     float4 x[VPT];
 #pragma unroll
     for (int s = 0; s < VPT; ++s) {
-      const int q = threadIdx.x + s * blockDim.x;
+      const int q = tid + s * nthr;
       if (q < nvec) x[s] = Xr[q];
     }
     float acc[Obj::kAcc];
     Obj::init(acc);
-    map_row<Obj, VPT>(acc, x, sFirst, nvec, d);
+    map_row<Obj, VPT>(acc, x, sFirst, nvec, d, tid, nthr);
     bool improved;
-    const float f = cta_fitness<Obj>(acc, sm, d, 0.f, improved);
-    if (threadIdx.x == 0) out[r] = f;
-    __syncthreads();
+    const float f = cta_fitness<Obj>(acc, sm, d, 0.f, improved, tid, nthr);
+    if (tid == 0) out[r] = f;
   }
 }
 
 // ---------------------------------------------------------- dispatch
-constexpr int kVpts[] = {1, 2, 4, 8};
+enum class Which { StepReg, StepTma, Init, Eval };
 
 template <class Obj>
-struct Kern {
-  static const void* step(int vpt) {
-    switch (vpt) {
-      case 1: return (const void*)k_step<Obj, 1>;
-      case 2: return (const void*)k_step<Obj, 2>;
-      case 4: return (const void*)k_step<Obj, 4>;
-      default: return (const void*)k_step<Obj, 8>;
-    }
+const void* pick(Which w, int vpt) {
+#define PSO_VPT_CASES(KERNEL)                          \
+  switch (vpt) {                                       \
+    case 1: return (const void*)KERNEL<Obj, 1>;        \
+    case 2: return (const void*)KERNEL<Obj, 2>;        \
+    case 4: return (const void*)KERNEL<Obj, 4>;        \
+    default: return (const void*)KERNEL<Obj, 8>;       \
   }
-  static const void* init(int vpt) {
-    switch (vpt) {
-      case 1: return (const void*)k_init<Obj, 1>;
-      case 2: return (const void*)k_init<Obj, 2>;
-      case 4: return (const void*)k_init<Obj, 4>;
-      default: return (const void*)k_init<Obj, 8>;
-    }
+  switch (w) {
+    case Which::StepReg: PSO_VPT_CASES(k_step_reg)
+    case Which::StepTma: PSO_VPT_CASES(k_step_tma)
+    case Which::Init: PSO_VPT_CASES(k_init)
+    default: PSO_VPT_CASES(k_eval)
   }
-  static const void* eval(int vpt) {
-    switch (vpt) {
-      case 1: return (const void*)k_eval<Obj, 1>;
-      case 2: return (const void*)k_eval<Obj, 2>;
-      case 4: return (const void*)k_eval<Obj, 4>;
-      default: return (const void*)k_eval<Obj, 8>;
-    }
-  }
-  static constexpr bool neighbor = Obj::kNeighbor;
-};
-
-enum class Which { Step, Init, Eval };
+#undef PSO_VPT_CASES
+}
 
 const void* kernel_for(int objective, Which w, int vpt, bool* neighbor) {
-#define PSO_CASE(ID, F)                                                            \
-  case ID:                                                                         \
-    *neighbor = Kern<F>::neighbor;                                                 \
-    return w == Which::Step ? Kern<F>::step(vpt)                                   \
-                            : (w == Which::Init ? Kern<F>::init(vpt) : Kern<F>::eval(vpt));
+#define PSO_CASE(ID, F)                      \
+  case ID:                                   \
+    *neighbor = F::kNeighbor;                \
+    return pick<F>(w, vpt);
   switch (objective) {
     PSO_ALL_OBJECTIVES(PSO_CASE)
     default:
@@ -562,6 +676,7 @@ const void* kernel_for(int objective, Which w, int vpt, bool* neighbor) {
 // CTA shape for a row of nvec float4: the smallest VPT in {1,2,4,8} whose
 // thread count fits 256, threads rounded up to a warp multiple.
 void shape_for(int nvec, int vpt_override, int* vpt, int* threads) {
+  static const int kVpts[] = {1, 2, 4, 8};
   int v = 8;
   for (int c : kVpts) {
     if ((nvec + c - 1) / c <= kMaxThreads) {
@@ -577,42 +692,82 @@ void shape_for(int nvec, int vpt_override, int* vpt, int* threads) {
   *threads = ((t + 31) / 32) * 32;
 }
 
-size_t dyn_smem(int nvec, bool neighbor, Which w) {
-  size_t s = (w == Which::Eval) ? 0 : (size_t)nvec * 16;  // staged G
-  if (neighbor) s += (size_t)nvec * 4;                      // first element of each float4
-  return s;
-}
-
-cudaError_t launch_rows(Which which, int objective, const SwarmArgs& a, const LaunchCfg& c,
-                        cudaStream_t s) {
-  bool nb = false;
-  const void* fn = kernel_for(objective, which, c.vpt, &nb);
-  if (!fn) return cudaErrorInvalidDeviceFunction;
-  void* args[] = {const_cast<SwarmArgs*>(&a)};
-  return cudaLaunchKernel(fn, dim3(c.grid), dim3(c.threads), args, c.smem, s);
-}
+constexpr size_t kSmemPerSm = 228 * 1024;       // B200 unified L1/shared per SM
+constexpr size_t kSmemPerCtaMax = 227 * 1024;   // opt-in maximum per CTA
+constexpr size_t kStaticReserve = 2048;         // static shared + per-CTA reservation
 
 }  // namespace
 
 bool objective_registered(int objective) {
   bool nb;
-  return kernel_for(objective, Which::Step, 1, &nb) != nullptr;
+  return kernel_for(objective, Which::Init, 1, &nb) != nullptr;
 }
 
-cudaError_t plan_launch(int objective, int d, long long n_local, int sm_count, int vpt_override,
+cudaError_t plan_launch(int objective, int d, long long n_local, int sm_count, const PlanHints& h,
                         LaunchCfg* cfg) {
   const int nvec = (d + 3) / 4;
-  shape_for(nvec, vpt_override, &cfg->vpt, &cfg->threads);
+  shape_for(nvec, h.vpt, &cfg->vpt, &cfg->compute);
   bool nb = false;
-  const void* fn = kernel_for(objective, Which::Step, cfg->vpt, &nb);
-  if (!fn) return cudaErrorInvalidDeviceFunction;
-  cfg->smem = dyn_smem(nvec, nb, Which::Step);
-  int per_sm = 0;
-  cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, cfg->threads, cfg->smem);
-  if (e != cudaSuccess) return e;
-  if (per_sm < 1) per_sm = 1;
-  cfg->ctas_per_sm = per_sm;
-  long long grid = (long long)per_sm * sm_count;
+  if (!kernel_for(objective, Which::Init, cfg->vpt, &nb)) return cudaErrorInvalidDeviceFunction;
+  const size_t row = (size_t)nvec * 16;
+  const size_t first = nb ? (size_t)nvec * 4 : 0;
+  cfg->init_smem = first;
+  cudaError_t e;
+
+  // ---- TMA pipeline: rows of >= 256 dims unless forced otherwise
+  bool tma = h.kernel == 1 || (h.kernel == -1 && nvec >= 64);
+  if (tma) {
+    const void* fn = kernel_for(objective, Which::StepTma, cfg->vpt, &nb);
+    const int threads = cfg->compute + 32;
+    // CTAs per SM the registers allow, capped at 2; the ring fills the rest.
+    int by_regs = 0;
+    if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&by_regs, fn, threads, 0)) != cudaSuccess)
+      return e;
+    int ctas = by_regs < 1 ? 1 : (by_regs > 2 ? 2 : by_regs);
+    int stages = 0;
+    for (; ctas >= 1; --ctas) {
+      size_t budget = kSmemPerSm / ctas - kStaticReserve;
+      if (budget > kSmemPerCtaMax - kStaticReserve) budget = kSmemPerCtaMax - kStaticReserve;
+      if (budget > row + first) stages = (int)((budget - row - first) / (3 * row));
+      if (stages >= 2) break;
+    }
+    if (h.stages >= 2 && h.stages <= kMaxStages) stages = stages < h.stages ? stages : h.stages;
+    if (stages > kMaxStages) stages = kMaxStages;
+    if (stages >= 2) {
+      const size_t smem = row + (size_t)stages * 3 * row + first;
+      if ((e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem)) !=
+          cudaSuccess)
+        return e;
+      int per_sm = 0;
+      if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, threads, smem)) !=
+          cudaSuccess)
+        return e;
+      if (per_sm >= 1) {
+        cfg->tma = 1;
+        cfg->stages = stages;
+        cfg->threads = threads;
+        cfg->smem = smem;
+        cfg->ctas_per_sm = per_sm;
+      } else {
+        tma = false;
+      }
+    } else {
+      tma = false;
+    }
+  }
+  if (!tma) {
+    const void* fn = kernel_for(objective, Which::StepReg, cfg->vpt, &nb);
+    cfg->tma = 0;
+    cfg->stages = 0;
+    cfg->threads = cfg->compute;
+    cfg->smem = row + first;
+    int per_sm = 0;
+    if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, cfg->threads, cfg->smem)) !=
+        cudaSuccess)
+      return e;
+    cfg->ctas_per_sm = per_sm < 1 ? 1 : per_sm;
+  }
+  long long grid = (long long)cfg->ctas_per_sm * sm_count;
   if (grid > n_local) grid = n_local;
   if (grid < 1) grid = 1;
   cfg->grid = (int)grid;
@@ -620,11 +775,22 @@ cudaError_t plan_launch(int objective, int d, long long n_local, int sm_count, i
 }
 
 cudaError_t launch_step(int objective, const SwarmArgs& a, const LaunchCfg& c, cudaStream_t s) {
-  return launch_rows(Which::Step, objective, a, c, s);
+  bool nb = false;
+  const void* fn = kernel_for(objective, c.tma ? Which::StepTma : Which::StepReg, c.vpt, &nb);
+  if (!fn) return cudaErrorInvalidDeviceFunction;
+  int stages = c.stages;
+  void* args[] = {const_cast<SwarmArgs*>(&a), &stages};
+  return cudaLaunchKernel(fn, dim3(c.grid), dim3(c.threads), args, c.smem, s);
 }
 
 cudaError_t launch_init(int objective, const SwarmArgs& a, const LaunchCfg& c, cudaStream_t s) {
-  return launch_rows(Which::Init, objective, a, c, s);
+  bool nb = false;
+  const void* fn = kernel_for(objective, Which::Init, c.vpt, &nb);
+  if (!fn) return cudaErrorInvalidDeviceFunction;
+  long long grid = a.n_local < 4LL * 148 * 2 ? a.n_local : 4LL * 148 * 2;
+  if (grid < 1) grid = 1;
+  void* args[] = {const_cast<SwarmArgs*>(&a)};
+  return cudaLaunchKernel(fn, dim3((unsigned)grid), dim3(c.compute), args, c.init_smem, s);
 }
 
 cudaError_t launch_rebest(const SwarmArgs& a, unsigned t, cudaStream_t s) {
@@ -651,7 +817,7 @@ cudaError_t debug_objective(int objective, const float* X_dev, long long m, int 
   long long grid = m < (long long)sm_count * 4 ? m : (long long)sm_count * 4;
   if (grid < 1) grid = 1;
   void* args[] = {(void*)&X_dev, (void*)&m, (void*)&d, (void*)&nvec, (void*)&out_dev};
-  return cudaLaunchKernel(fn, dim3((unsigned)grid), dim3(threads), args, dyn_smem(nvec, nb, Which::Eval),
+  return cudaLaunchKernel(fn, dim3((unsigned)grid), dim3(threads), args, nb ? (size_t)nvec * 4 : 0,
                           s);
 }
 

@@ -17,7 +17,7 @@ import oracle as orc
 import paper_conf_icpp_liuwc21_b200 as fp
 from synth import (ACKLEY, DOMAINS, EASOM, GRIEWANK, RASTRIGIN, ROSENBROCK, SPHERE, WORKLOADS,
                    random_state, sample_rows)
-from tests.helpers import assert_bitwise, assert_fitness_close, fit_tol
+from pso_testutil import assert_bitwise, assert_fitness_close, fit_tol
 
 pytestmark = pytest.mark.gpu
 
@@ -149,6 +149,20 @@ def test_single_step_all_improve(obj, n, d):
 @pytest.mark.parametrize("n,d", [(257, 13), (300, 1000), (70, 2000), (9, 4096)])
 def test_single_step_mixed_pbest(obj, n, d):
     _step_and_compare(obj, n, d, seed=2000 + n + d, pf_mode="mixed", t0=41)
+
+
+@pytest.mark.parametrize("kernel", ["reg", "tma"])
+@pytest.mark.parametrize("obj", [RASTRIGIN, ROSENBROCK, GRIEWANK])
+@pytest.mark.parametrize("n,d", [(300, 13), (301, 1000), (70, 2001), (9, 4096), (5, 8192)])
+def test_single_step_both_kernels(kernel, obj, n, d, monkeypatch):
+    """Both step-kernel variants (register streaming / TMA bulk-copy pipeline)
+    on every CTA shape, with a shallow and the default pipeline depth."""
+    monkeypatch.setenv("PSO_KERNEL", kernel)
+    g, _ = _step_and_compare(obj, n, d, seed=3000 + n + d, pf_mode="mixed", t0=3)
+    info = g.info()
+    assert info["tma_pipeline"] == (1 if kernel == "tma" else 0) or (kernel == "tma" and d >= 8192)
+    monkeypatch.setenv("PSO_STAGES", "2")
+    _step_and_compare(obj, n, d, seed=3100 + n + d, pf_mode="inf", t0=9)
 
 
 # ------------------------------------------------------------------ multi-step
