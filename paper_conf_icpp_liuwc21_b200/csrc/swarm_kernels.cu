@@ -109,6 +109,28 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, unsigned by
       : "memory");
 }
 
+__device__ __forceinline__ void bulk_s2g(void* dst, const void* src, unsigned bytes) {
+  asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(dst),
+               "r"(smem_addr(src)), "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void bulk_commit() {
+  asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+}
+template <int N>
+__device__ __forceinline__ void bulk_wait_read() {
+  asm volatile("cp.async.bulk.wait_group.read %0;" ::"n"(N) : "memory");
+}
+__device__ __forceinline__ void bulk_wait_all() {
+  asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+}
+__device__ __forceinline__ void fence_proxy_async_shared() {
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+__device__ __forceinline__ void fence_proxy_async_global() {
+  asm volatile("fence.proxy.async.global;" ::: "memory");
+}
+
 // --- Eq. 1, 5, 2 on one element, fixed fp32 order, no contraction --------
 struct MoveParams {
   float w, c1, c2, lo, hi, vmax;
@@ -179,6 +201,21 @@ __device__ __forceinline__ float cta_fitness(float* a, RowSmem<Obj>& sm, int d, 
   return sm.f;
 }
 
+// Map one float4 of new positions (dims j..j+3; nx = x_{j+4} for neighbours).
+template <class Obj>
+__device__ __forceinline__ void map4(float* acc, const float4& x, float nx, int j, int d) {
+  if (j + 3 < d) {
+    Obj::map(acc, x.x, x.y, j, d);
+    Obj::map(acc, x.y, x.z, j + 1, d);
+    Obj::map(acc, x.z, x.w, j + 2, d);
+    Obj::map(acc, x.w, nx, j + 3, d);
+  } else {  // ragged tail of the row
+    if (j < d) Obj::map(acc, x.x, x.y, j, d);
+    if (j + 1 < d) Obj::map(acc, x.y, x.z, j + 1, d);
+    if (j + 2 < d) Obj::map(acc, x.z, x.w, j + 2, d);
+  }
+}
+
 // Map the VPT float4 of new positions into the accumulators.  For functors
 // that need x_{j+1} the first element of every float4 is published in sFirst.
 template <class Obj, int VPT>
@@ -196,22 +233,13 @@ __device__ __forceinline__ void map_row(float* acc, const float4 (&x)[VPT], floa
   for (int s = 0; s < VPT; ++s) {
     const int q = tid + s * nthr;
     if (q < nvec) {
-      const int j = 4 * q;
       float nx = 0.f;
       if constexpr (Obj::kNeighbor) nx = (q + 1 < nvec) ? sFirst[q + 1] : 0.f;
-      if (j + 3 < d) {
-        Obj::map(acc, x[s].x, x[s].y, j, d);
-        Obj::map(acc, x[s].y, x[s].z, j + 1, d);
-        Obj::map(acc, x[s].z, x[s].w, j + 2, d);
-        Obj::map(acc, x[s].w, nx, j + 3, d);
-      } else {  // ragged tail of the row
-        if (j < d) Obj::map(acc, x[s].x, x[s].y, j, d);
-        if (j + 1 < d) Obj::map(acc, x[s].y, x[s].z, j + 1, d);
-        if (j + 2 < d) Obj::map(acc, x[s].z, x[s].w, j + 2, d);
-      }
+      map4<Obj>(acc, x[s], nx, 4 * q, d);
     }
   }
 }
+
 
 // A2-A6 for one row: update, store x' / v', evaluate, pbest compare-and-copy.
 // src(s, q, x, v, pb) supplies the operands of float4 q (slot s) — from
@@ -309,6 +337,37 @@ __device__ __forceinline__ void gbest_epilogue(const SwarmArgs& a, RowSmem<Obj>&
   }
 }
 
+// The same epilogue run by one warp (the TMA kernel's finaliser warp).
+__device__ __forceinline__ void warp_gbest_epilogue(const SwarmArgs& a, uint32_t t, int lane) {
+  unsigned long long acc = 0, cur = 0;
+  if (lane == 0) {
+    __threadfence();
+    acc = *(volatile unsigned long long*)&a.ctl->key_acc;
+    cur = a.ctl->key_cur;
+  }
+  acc = __shfl_sync(kFull, acc, 0);
+  cur = __shfl_sync(kFull, cur, 0);
+  const bool have = acc < cur;
+  const float4* src = nullptr;
+  if (have)
+    src = reinterpret_cast<const float4*>(a.PB) + ((long long)(uint32_t)acc - a.row_begin) * a.nvec;
+  float4* dst = a.world == 1 ? reinterpret_cast<float4*>(a.G) : reinterpret_cast<float4*>(a.send + 16);
+  if (have)
+    for (int q = lane; q < a.nvec; q += 32) dst[q] = __ldcg(src + q);
+  __syncwarp();
+  if (lane == 0) {
+    if (a.world == 1) {
+      if (have) a.ctl->key_cur = acc;
+    } else {
+      unsigned long long* hdr = reinterpret_cast<unsigned long long*>(a.send);
+      hdr[0] = have ? acc : ~0ull;
+      hdr[1] = 0;
+    }
+    a.ctl->t = t;
+    a.ctl->done = 0;
+  }
+}
+
 // Publish this CTA's candidate and improvement count; true in the last CTA
 // to finish (which then runs gbest_epilogue).
 template <class Obj>
@@ -396,81 +455,193 @@ __global__ void __launch_bounds__(kMaxThreads, (VPT >= 8) ? 1 : 2)
 }
 
 // ------------------------------------------------- step kernel: TMA pipeline
-// Warps 0..C/32-1 compute; the last warp is the producer.  Shared memory:
-// [G: nvec float4][stages x {x, v, pb}: nvec float4 each][sFirst].
+// Warp-specialised; every HBM byte of the row stream moves through the TMA
+// engine (bulk async copies), the compute warps touch only shared memory.
+//   warps 0..W-1  compute: x, v, pb, g from the stage (LDS.128) -> Philox ->
+//                 Eq. 1/5/2 -> x', v' written back into the stage (STS.128)
+//                 -> objective map -> warp partial -> arrive(done[s])
+//   warp  W       producer: G once, then per row cp.async.bulk x, v, pb rows
+//                 global -> stage s, completion on full[s] (complete_tx)
+//   warp  W+1     finaliser: per row, combine the W warp partials (fixed
+//                 order), f, the pbest decision, then bulk-store the stage's
+//                 x' -> X, v' -> V (and x' -> PB if improved), the gbest
+//                 candidate, and release the stage to the producer once the
+//                 bulk stores have read it (wait_group.read).
+// Barriers per stage: full (1 arrival + tx bytes), done (W arrivals), empty (1).
+// Shared memory: [G: nvec float4][stages x {x, v, pb}: nvec float4 each].
 template <class Obj, int VPT>
-__global__ void __launch_bounds__(kMaxThreads + 32, (VPT <= 2) ? 2 : 1)
+__global__ void __launch_bounds__(kMaxThreads + 64, (VPT <= 2) ? 2 : 1)
     k_step_tma(const SwarmArgs a, int stages) {
   extern __shared__ __align__(128) unsigned char dsmem[];
-  const int nvec = a.nvec;
-  const int nthr = (int)blockDim.x - 32;  // compute threads
+  const int nvec = a.nvec, d = a.d;
+  const int nthr = (int)blockDim.x - 64;  // compute threads
+  const int nwarps = nthr >> 5;
   float4* sG = reinterpret_cast<float4*>(dsmem);
   float4* ring = sG + nvec;
-  float* sFirst = reinterpret_cast<float*>(ring + (size_t)stages * 3 * nvec);
-  __shared__ RowSmem<Obj> sm;
-  __shared__ unsigned long long full[kMaxStages], empty[kMaxStages];
-  const int tid = threadIdx.x;
+  __shared__ float red[kMaxStages][(kMaxThreads / 32) * 2];
+  __shared__ unsigned long long full[kMaxStages], empty[kMaxStages], done[kMaxStages], gbar;
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   if (tid == 0) {
-    mbar_init(&sm.gbar, 1);
+    mbar_init(&gbar, 1);
     for (int s = 0; s < stages; ++s) {
       mbar_init(&full[s], 1);
-      mbar_init(&empty[s], (unsigned)(nthr >> 5));
+      mbar_init(&done[s], (unsigned)nwarps);
+      mbar_init(&empty[s], 1);
     }
     mbar_fence_init();
   }
   __syncthreads();
   const uint32_t t = a.ctl->t + 1u;
+  const unsigned row_bytes = (unsigned)nvec * 16u;
 
-  if (tid >= nthr) {  // ---------------- producer warp
-    if (tid == nthr) {
-      const unsigned row_bytes = (unsigned)nvec * 16u;
-      mbar_expect_tx(&sm.gbar, row_bytes);
-      bulk_g2s(sG, a.G, row_bytes, &sm.gbar);
+  if (warp == nwarps) {  // ---------------- producer
+    if (lane == 0) {
+      mbar_expect_tx(&gbar, row_bytes);
+      bulk_g2s(sG, a.G, row_bytes, &gbar);
+      int s = 0;
+      unsigned ph = 0;
       int k = 0;
       for (long long r = blockIdx.x; r < a.n_local; r += gridDim.x, ++k) {
-        const int s = k % stages;
-        if (k >= stages) mbar_wait(&empty[s], ((unsigned)(k / stages) & 1u) ^ 1u);
+        if (k >= stages) mbar_wait(&empty[s], ph ^ 1u);
         float4* st = ring + (size_t)s * 3 * nvec;
         mbar_expect_tx(&full[s], 3u * row_bytes);
         bulk_g2s(st, a.X + (size_t)r * 4 * nvec, row_bytes, &full[s]);
         bulk_g2s(st + nvec, a.V + (size_t)r * 4 * nvec, row_bytes, &full[s]);
         bulk_g2s(st + 2 * nvec, a.PB + (size_t)r * 4 * nvec, row_bytes, &full[s]);
+        if (++s == stages) {
+          s = 0;
+          ph ^= 1u;
+        }
       }
     }
     return;
   }
 
+  if (warp == nwarps + 1) {  // ---------------- finaliser
+    __shared__ int s_last;
+    if (lane == 0) {
+      const uint32_t inc_ord = (uint32_t)(a.ctl->key_cur >> 32);
+      unsigned long long best = ~0ull;
+      unsigned nimp = 0;
+      int s = 0, prev = -1;
+      unsigned ph = 0;
+      for (long long r = blockIdx.x; r < a.n_local; r += gridDim.x) {
+        const float pf_old = a.pf[r];
+        const uint32_t gi = (uint32_t)(a.row_begin + r);
+        mbar_wait(&done[s], ph);
+        float c[Obj::kAcc];
+        Obj::init(c);
+        for (int w = 0; w < nwarps; ++w) {
+          float b[Obj::kAcc];
+#pragma unroll
+          for (int j = 0; j < Obj::kAcc; ++j) b[j] = red[s][w * Obj::kAcc + j];
+          Obj::combine(c, b);
+        }
+        const float f = Obj::finalize(c, d);
+        const float4* st = ring + (size_t)s * 3 * nvec;
+        const size_t off = (size_t)r * 4 * nvec;
+        bulk_s2g(a.X + off, st, row_bytes);
+        bulk_s2g(a.V + off, st + nvec, row_bytes);
+        if (f < pf_old) {  // Alg. 1 line 7: strict; NaN never improves
+          bulk_s2g(a.PB + off, st, row_bytes);
+          a.pf[r] = f;
+          ++nimp;
+        }
+        bulk_commit();
+        if (f == f && ord_f32(f) < inc_ord) {  // strictly below gf (Alg. 1 line 10)
+          const unsigned long long key = pack_key(f, gi);
+          best = key < best ? key : best;
+        }
+        if (prev >= 0) {  // the previous row's stores have read their stage
+          bulk_wait_read<1>();
+          mbar_arrive(&empty[prev]);
+        }
+        prev = s;
+        if (++s == stages) {
+          s = 0;
+          ph ^= 1u;
+        }
+      }
+      bulk_wait_all();  // every X / V / PB row written
+      fence_proxy_async_global();
+      if (best != ~0ull) atomicMin(&a.ctl->key_acc, best);
+      if (nimp) atomicAdd(&a.ctl->improvements, (unsigned long long)nimp);
+      __threadfence();
+      s_last = (atomicAdd(&a.ctl->done, 1u) == gridDim.x - 1) ? 1 : 0;
+    }
+    __syncwarp();
+    if (s_last) warp_gbest_epilogue(a, t, lane);
+    return;
+  }
+
   // ---------------- compute warps
-  const uint32_t inc_ord = (uint32_t)(a.ctl->key_cur >> 32);
   const PhiloxKey key{a.seed_lo, a.seed_hi};
   const MoveParams mp{a.w, a.c1, a.c2, a.lo, a.hi, a.vmax};
-  const int lane = tid & 31;
-  mbar_wait(&sm.gbar, 0);
-  unsigned long long best = ~0ull;
-  unsigned nimp = 0;
-  int k = 0;
-  for (long long r = blockIdx.x; r < a.n_local; r += gridDim.x, ++k) {
-    const int s = k % stages;
+  mbar_wait(&gbar, 0);
+  int s = 0;
+  unsigned ph = 0;
+  for (long long r = blockIdx.x; r < a.n_local; r += gridDim.x) {
     const uint32_t gi = (uint32_t)(a.row_begin + r);
-    const float pf_old = (tid == 0) ? a.pf[r] : 0.f;
-    const float4* st = ring + (size_t)s * 3 * nvec;
-    mbar_wait(&full[s], (unsigned)(k / stages) & 1u);
-    bool improved;
-    const float f = process_row<Obj, VPT>(
-        a, mp, key, t, gi, r,
-        [&](int, int q, float4& xo, float4& vo, float4& po) {
-          xo = st[q];
-          vo = st[nvec + q];
-          po = st[2 * nvec + q];
-        },
-        [&] {
-          __syncwarp();
-          if (lane == 0) mbar_arrive(&empty[s]);  // stage may be refilled
-        },
-        sG, sFirst, sm, tid, nthr, pf_old, improved);
-    if (tid == 0) row_bookkeeping(a, r, gi, f, improved, inc_ord, best, nimp);
+    float4* st = ring + (size_t)s * 3 * nvec;
+    mbar_wait(&full[s], ph);
+    float4 xn[VPT];
+#pragma unroll
+    for (int j = 0; j < VPT; ++j) {
+      const int q = tid + j * nthr;
+      if (q < nvec) {
+        float4 x = st[q], v = st[nvec + q];
+        const float4 pb = st[2 * nvec + q];
+        const float4 g = sG[q];
+        const float4 r1 = uniforms4(key, kTagR1, t, gi, (uint32_t)q);
+        const float4 r2 = uniforms4(key, kTagR2, t, gi, (uint32_t)q);
+        move1(mp, x.x, v.x, pb.x, g.x, r1.x, r2.x);
+        move1(mp, x.y, v.y, pb.y, g.y, r1.y, r2.y);
+        move1(mp, x.z, v.z, pb.z, g.z, r1.z, r2.z);
+        move1(mp, x.w, v.w, pb.w, g.w, r1.w, r2.w);
+        if ((d & 3) && q == nvec - 1) {  // keep the row padding at zero
+          const int jj = 4 * q;
+          if (jj + 1 >= d) x.y = v.y = 0.f;
+          if (jj + 2 >= d) x.z = v.z = 0.f;
+          if (jj + 3 >= d) x.w = v.w = 0.f;
+        }
+        st[q] = x;
+        st[nvec + q] = v;
+        xn[j] = x;
+      }
+    }
+    float acc[Obj::kAcc];
+    Obj::init(acc);
+    if constexpr (Obj::kNeighbor) {
+      team_sync(nthr);  // every x' of the row is in the stage
+#pragma unroll
+      for (int j = 0; j < VPT; ++j) {
+        const int q = tid + j * nthr;
+        if (q < nvec) {
+          const int jj = 4 * q;
+          const float nx = (q + 1 < nvec) ? st[q + 1].x : 0.f;
+          map4<Obj>(acc, xn[j], nx, jj, d);
+        }
+      }
+    } else {
+#pragma unroll
+      for (int j = 0; j < VPT; ++j) {
+        const int q = tid + j * nthr;
+        if (q < nvec) map4<Obj>(acc, xn[j], 0.f, 4 * q, d);
+      }
+    }
+    warp_combine<Obj>(acc);
+    if (lane == 0) {
+#pragma unroll
+      for (int j = 0; j < Obj::kAcc; ++j) red[s][warp * Obj::kAcc + j] = acc[j];
+    }
+    fence_proxy_async_shared();  // x', v' visible to the bulk stores
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&done[s]);
+    if (++s == stages) {
+      s = 0;
+      ph ^= 1u;
+    }
   }
-  if (cta_finish<Obj>(a, sm, best, nimp, tid, nthr)) gbest_epilogue<Obj>(a, sm, t, tid, nthr);
 }
 
 // ------------------------------------------------------------ init kernel
@@ -718,7 +889,7 @@ cudaError_t plan_launch(int objective, int d, long long n_local, int sm_count, c
   bool tma = h.kernel == 1 || (h.kernel == -1 && nvec >= 64);
   if (tma) {
     const void* fn = kernel_for(objective, Which::StepTma, cfg->vpt, &nb);
-    const int threads = cfg->compute + 32;
+    const int threads = cfg->compute + 64;  // + producer warp + finaliser warp
     // CTAs per SM the registers allow, capped at 2; the ring fills the rest.
     int by_regs = 0;
     if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&by_regs, fn, threads, 0)) != cudaSuccess)
@@ -728,13 +899,13 @@ cudaError_t plan_launch(int objective, int d, long long n_local, int sm_count, c
     for (; ctas >= 1; --ctas) {
       size_t budget = kSmemPerSm / ctas - kStaticReserve;
       if (budget > kSmemPerCtaMax - kStaticReserve) budget = kSmemPerCtaMax - kStaticReserve;
-      if (budget > row + first) stages = (int)((budget - row - first) / (3 * row));
+      if (budget > row) stages = (int)((budget - row) / (3 * row));
       if (stages >= 2) break;
     }
     if (h.stages >= 2 && h.stages <= kMaxStages) stages = stages < h.stages ? stages : h.stages;
     if (stages > kMaxStages) stages = kMaxStages;
     if (stages >= 2) {
-      const size_t smem = row + (size_t)stages * 3 * row + first;
+      const size_t smem = row + (size_t)stages * 3 * row;
       if ((e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem)) !=
           cudaSuccess)
         return e;
