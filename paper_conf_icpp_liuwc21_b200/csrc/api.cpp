@@ -114,6 +114,7 @@ struct pso_swarm {
   uint64_t seed = 0;
   // placement
   int device = 0, sm_count = 0, rank = 0, world = 1;
+  bool xchg = false;  // run the all-gather + select exchange (world > 1, or forced for testing)
   cudaStream_t stream = nullptr;
   bool own_stream = false;
   ncclComm_t comm = nullptr;
@@ -160,7 +161,7 @@ pso_status use_device(pso_swarm* h) {
 }
 
 pso_status exchange(pso_swarm* h) {
-  if (h->world <= 1) return PSO_OK;
+  if (!h->xchg) return PSO_OK;
   NcclApi* a = nccl();
   if (!a) {
     h->poisoned = true;
@@ -327,6 +328,8 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
       return bail(fail(PSO_ERR_NCCL, "ncclCommCount/UserRank failed"));
     h->world = cnt;
     h->rank = rk;
+    const char* fx = std::getenv("PSO_FORCE_EXCHANGE");
+    h->xchg = cnt > 1 || (fx && *fx && *fx != '0');
   }
   h->row_begin = (n * h->rank) / h->world;
   h->n_local = (n * (h->rank + 1)) / h->world - h->row_begin;
@@ -352,8 +355,8 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
   const size_t gb = align_up((size_t)h->pitch * 4, 256);
   const size_t ctlb = align_up(sizeof(DevCtl), 256);
   const size_t rec = align_up(record_bytes(h->pitch), 256);
-  const size_t sendb = h->world > 1 ? rec : 0;
-  const size_t recvb = h->world > 1 ? (size_t)h->world * record_bytes(h->pitch) : 0;
+  const size_t sendb = h->xchg ? rec : 0;
+  const size_t recvb = h->xchg ? (size_t)h->world * record_bytes(h->pitch) : 0;
   h->arena_bytes = 3 * mat + pfb + gb + ctlb + sendb + align_up(recvb, 256);
   {
     cudaError_t e = cudaMalloc(&h->arena, h->arena_bytes);
@@ -371,13 +374,14 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
   A.pf = (float*)p; p += pfb;
   A.G = (float*)p; p += gb;
   A.ctl = (DevCtl*)p; p += ctlb;
-  A.send = h->world > 1 ? p : nullptr; p += sendb;
-  A.recv = h->world > 1 ? p : nullptr;
+  A.send = h->xchg ? p : nullptr; p += sendb;
+  A.recv = h->xchg ? p : nullptr;
   A.n_local = h->n_local;
   A.row_begin = h->row_begin;
   A.d = d;
   A.nvec = h->pitch / 4;
   A.world = h->world;
+  A.exchange = h->xchg ? 1 : 0;
   A.w = w; A.c1 = c1; A.c2 = c2; A.lo = lo; A.hi = hi; A.vmax = h->vmax;
   A.seed_lo = (unsigned)seed;
   A.seed_hi = (unsigned)(seed >> 32);
@@ -385,7 +389,7 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
   {
     cudaError_t e = cudaMemsetAsync(A.G, 0, gb + ctlb, h->stream);  // G and ctl
     if (e != cudaSuccess) return bail(cuda_fail(nullptr, e, "cudaMemsetAsync"));
-    if (h->world > 1) {
+    if (h->xchg) {
       e = cudaMemsetAsync(A.send, 0, sendb, h->stream);
       if (e != cudaSuccess) return bail(cuda_fail(nullptr, e, "cudaMemsetAsync"));
     }
@@ -398,7 +402,7 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
     cudaError_t e = launch_init(objective, A, h->cfg, h->stream);
     if (e != cudaSuccess) return bail(cuda_fail(nullptr, e, "launch_init"));
     ++h->launches;
-  } else if (h->world > 1) {
+  } else if (h->xchg) {
     // empty shard: contribute "no candidate"
     unsigned long long none[2] = {~0ull, 0ull};
     cudaError_t e = cudaMemcpyAsync(A.send, none, 16, cudaMemcpyHostToDevice, h->stream);
@@ -512,7 +516,7 @@ pso_status pso_set_state(pso_handle h, const float* x, const float* v, const flo
   if (rows > 0) {
     PSO_CUDA(h, launch_rebest(h->args, (unsigned)t, h->stream));
     ++h->launches;
-  } else if (h->world > 1) {
+  } else if (h->xchg) {
     unsigned long long none[2] = {~0ull, 0ull};
     PSO_CUDA(h, cudaMemcpyAsync(h->args.send, none, 16, cudaMemcpyHostToDevice, h->stream));
   }

@@ -35,6 +35,7 @@ struct SwarmArgs {
   long long row_begin;
   int d, nvec;                // nvec = pitch / 4
   int world;
+  int exchange;               // 1: publish (key, row) records for the all-gather + select
   float w, c1, c2, lo, hi, vmax;
   unsigned int seed_lo, seed_hi;
 };

@@ -313,7 +313,7 @@ __device__ __forceinline__ void gbest_epilogue(const SwarmArgs& a, RowSmem<Obj>&
   const float4* src = nullptr;
   if (have)
     src = reinterpret_cast<const float4*>(a.PB) + ((long long)(uint32_t)acc - a.row_begin) * a.nvec;
-  if (a.world == 1) {
+  if (!a.exchange) {
     if (have) {
       float4* G4 = reinterpret_cast<float4*>(a.G);
       for (int q = tid; q < a.nvec; q += nthr) G4[q] = __ldcg(src + q);
@@ -351,12 +351,12 @@ __device__ __forceinline__ void warp_gbest_epilogue(const SwarmArgs& a, uint32_t
   const float4* src = nullptr;
   if (have)
     src = reinterpret_cast<const float4*>(a.PB) + ((long long)(uint32_t)acc - a.row_begin) * a.nvec;
-  float4* dst = a.world == 1 ? reinterpret_cast<float4*>(a.G) : reinterpret_cast<float4*>(a.send + 16);
+  float4* dst = !a.exchange ? reinterpret_cast<float4*>(a.G) : reinterpret_cast<float4*>(a.send + 16);
   if (have)
     for (int q = lane; q < a.nvec; q += 32) dst[q] = __ldcg(src + q);
   __syncwarp();
   if (lane == 0) {
-    if (a.world == 1) {
+    if (!a.exchange) {
       if (have) a.ctl->key_cur = acc;
     } else {
       unsigned long long* hdr = reinterpret_cast<unsigned long long*>(a.send);

@@ -302,3 +302,33 @@ def test_full_size_sampled_rows(key):
     assert_fitness_close(w.objective, cPB[ok], pf2[idx][ok], cpf[ok], "pf rows")
     assert gf == pf2.min() and gi == int(np.argmin(pf2))
     assert_bitwise(G2, PB2[gi], "G == PB[gi]")
+
+
+# ------------------------------------------------------------------ exchange path
+@pytest.mark.parametrize("obj,n,d", [(RASTRIGIN, 300, 1000), (GRIEWANK, 50, 13)])
+def test_exchange_path_with_single_rank_comm(obj, n, d, monkeypatch):
+    """The multi-GPU exchange (records -> ncclAllGather -> k_select) forced on a
+    1-rank NCCL communicator must give the single-GPU results bitwise."""
+    import torch  # noqa: F401  (loads the NCCL the library resolves)
+    monkeypatch.setenv("PSO_FORCE_EXCHANGE", "1")
+    comm = fp.nccl_comm_init(1, fp.nccl_unique_id(), 0, 0)
+    try:
+        g = gpu_swarm(n, d, obj, seed=5, nccl_comm=comm)
+        ref = gpu_swarm(n, d, obj, seed=5)
+        assert g.gbest()[:2] == ref.gbest()[:2]
+        g.reset_counters()
+        g.step(20)
+        ref.step(20)
+        assert g.info()["launches"] == 40  # step kernel + select kernel per iteration
+        for x, y in zip(g.get_state()[:4], ref.get_state()[:4]):
+            assert_bitwise(x, y, "exchange path state")
+        gf, gi, G = g.gbest()
+        rf, ri, RG = ref.gbest()
+        assert (gf, gi) == (rf, ri)
+        assert_bitwise(G, RG, "G")
+        X, V, PB, pf, t = g.get_state()
+        g.set_state(X, V, PB, pf, t=t)  # rebest through the exchange
+        assert g.gbest()[:2] == (rf, ri)
+        g.close()
+    finally:
+        fp.nccl_comm_destroy(comm)
