@@ -112,7 +112,9 @@ typedef struct {
  *   out        receives the handle (set to NULL on failure)
  *   n          global swarm size, 1 <= n < 2^32
  *   d          dimension, 1 <= d <= PSO_D_MAX (else PSO_ERR_UNSUPPORTED)
- *   w, c1, c2  Eq. 1 parameters, finite
+ *   w, c1, c2  Eq. 1 parameters, finite; c1, c2 = 0 or |c| >= 2^-100 (else
+ *              PSO_ERR_UNSUPPORTED: the kernel folds the 2^-24 of the uniform
+ *              into c, exact only away from the subnormal range)
  *   lo < hi    finite domain bounds; positions are clamped to [lo, hi]
  *   objective  PSO_OBJ_* or a registered custom id (else PSO_ERR_INVALID)
  *   seed       64-bit Philox key

@@ -264,6 +264,8 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
   if (d > PSO_D_MAX) return fail(PSO_ERR_UNSUPPORTED, "d=%d > PSO_D_MAX=%d", d, PSO_D_MAX);
   if (!finite(w) || !finite(c1) || !finite(c2))
     return fail(PSO_ERR_INVALID, "w, c1, c2 must be finite");
+  if ((c1 != 0.f && std::fabs(c1) < 0x1p-100f) || (c2 != 0.f && std::fabs(c2) < 0x1p-100f))
+    return fail(PSO_ERR_UNSUPPORTED, "0 < |c1| or |c2| < 2^-100 is not supported");
   if (!finite(lo) || !finite(hi) || !(lo < hi))
     return fail(PSO_ERR_INVALID, "need finite lo < hi (got %g, %g)", lo, hi);
   if (!(o.vmax == o.vmax) || std::isinf(o.vmax)) return fail(PSO_ERR_INVALID, "vmax must be finite");
@@ -338,6 +340,7 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
   PlanHints hints;
   if (const char* v = std::getenv("PSO_VPT")) hints.vpt = std::atoi(v);
   if (const char* v = std::getenv("PSO_STAGES")) hints.stages = std::atoi(v);
+  if (const char* v = std::getenv("PSO_CTAS")) hints.ctas = std::atoi(v);
   if (const char* v = std::getenv("PSO_KERNEL")) {
     if (!std::strcmp(v, "reg")) hints.kernel = 0;
     if (!std::strcmp(v, "tma")) hints.kernel = 1;

@@ -52,11 +52,12 @@ struct LaunchCfg {
   size_t init_smem = 0;
 };
 
-// Tuning overrides (0 / -1 = automatic): PSO_VPT, PSO_KERNEL=reg|tma, PSO_STAGES.
+// Tuning overrides (0 / -1 = automatic): PSO_VPT, PSO_KERNEL=reg|tma, PSO_STAGES, PSO_CTAS.
 struct PlanHints {
   int vpt = 0;
   int kernel = -1;  // -1 auto, 0 register, 1 tma
   int stages = 0;
+  int ctas = 0;     // max CTAs per SM for the TMA pipeline (0: auto = 2)
 };
 
 bool objective_registered(int objective);

@@ -49,6 +49,18 @@ __device__ __forceinline__ float4 u01x4(uint4 w) {
   return make_float4(u01(w.x), u01(w.y), u01(w.z), u01(w.w));
 }
 
+// The 24-bit integers m = w >> 8 of one call, as exact floats (U = m 2^-24).
+__device__ __forceinline__ float4 raw24x4(uint4 w) {
+  return make_float4(__uint2float_rn(w.x >> 8), __uint2float_rn(w.y >> 8),
+                     __uint2float_rn(w.z >> 8), __uint2float_rn(w.w >> 8));
+}
+
+// m of float4 q (dims 4q..4q+3) of particle i at iteration t.
+__device__ __forceinline__ float4 raw24x4(PhiloxKey key, uint32_t tag, uint32_t t, uint32_t i,
+                                          uint32_t q) {
+  return raw24x4(philox4x32_10(make_uint4(q, i, t, tag), key));
+}
+
 // The 4 uniforms of float4 q (dims 4q..4q+3) of particle i at iteration t.
 __device__ __forceinline__ float4 uniforms4(PhiloxKey key, uint32_t tag, uint32_t t,
                                             uint32_t i, uint32_t q) {

@@ -132,14 +132,22 @@ __device__ __forceinline__ void fence_proxy_async_global() {
 }
 
 // --- Eq. 1, 5, 2 on one element, fixed fp32 order, no contraction --------
+// The oracle computes b = (c1 * r1) * (pb - x) with r1 = m 2^-24 (m the 24-bit
+// Philox integer).  Here c1s = c1 2^-24 is folded once per kernel, and
+// c1s * m == c1 * r1 bit for bit: scaling by a power of two commutes with
+// round-to-nearest while no operand or result is subnormal, which the ABI
+// guarantees by accepting only c1, c2 = 0 or |c1|, |c2| >= 2^-100.
 struct MoveParams {
-  float w, c1, c2, lo, hi, vmax;
+  float w, c1s, c2s, lo, hi, vmax;
 };
+__device__ __forceinline__ MoveParams move_params(const SwarmArgs& a) {
+  return MoveParams{a.w, __fmul_rn(a.c1, 0x1p-24f), __fmul_rn(a.c2, 0x1p-24f), a.lo, a.hi, a.vmax};
+}
 __device__ __forceinline__ void move1(const MoveParams& m, float& x, float& v, float pb, float g,
-                                      float r1, float r2) {
+                                      float m1, float m2) {
   const float a = __fmul_rn(m.w, v);
-  const float b = __fmul_rn(__fmul_rn(m.c1, r1), __fsub_rn(pb, x));
-  const float c = __fmul_rn(__fmul_rn(m.c2, r2), __fsub_rn(g, x));
+  const float b = __fmul_rn(__fmul_rn(m.c1s, m1), __fsub_rn(pb, x));
+  const float c = __fmul_rn(__fmul_rn(m.c2s, m2), __fsub_rn(g, x));
   float vn = __fadd_rn(__fadd_rn(a, b), c);
   vn = fminf(fmaxf(vn, -m.vmax), m.vmax);
   x = fminf(fmaxf(__fadd_rn(x, vn), m.lo), m.hi);
@@ -264,8 +272,8 @@ __device__ __forceinline__ float process_row(const SwarmArgs& a, const MoveParam
       float4 x, v, pb;
       src(s, q, x, v, pb);
       const float4 g = sG[q];
-      const float4 r1 = uniforms4(key, kTagR1, t, gi, (uint32_t)q);
-      const float4 r2 = uniforms4(key, kTagR2, t, gi, (uint32_t)q);
+      const float4 r1 = raw24x4(key, kTagR1, t, gi, (uint32_t)q);
+      const float4 r2 = raw24x4(key, kTagR2, t, gi, (uint32_t)q);
       move1(mp, x.x, v.x, pb.x, g.x, r1.x, r2.x);
       move1(mp, x.y, v.y, pb.y, g.y, r1.y, r2.y);
       move1(mp, x.z, v.z, pb.z, g.z, r1.z, r2.z);
@@ -418,7 +426,7 @@ __global__ void __launch_bounds__(kMaxThreads, (VPT >= 8) ? 1 : 2)
   const uint32_t t = a.ctl->t + 1u;
   const uint32_t inc_ord = (uint32_t)(a.ctl->key_cur >> 32);
   const PhiloxKey key{a.seed_lo, a.seed_hi};
-  const MoveParams mp{a.w, a.c1, a.c2, a.lo, a.hi, a.vmax};
+  const MoveParams mp = move_params(a);
   const int nvec = a.nvec;
   mbar_wait(&sm.gbar, 0);
 
@@ -470,7 +478,7 @@ __global__ void __launch_bounds__(kMaxThreads, (VPT >= 8) ? 1 : 2)
 // Barriers per stage: full (1 arrival + tx bytes), done (W arrivals), empty (1).
 // Shared memory: [G: nvec float4][stages x {x, v, pb}: nvec float4 each].
 template <class Obj, int VPT>
-__global__ void __launch_bounds__(kMaxThreads + 64, (VPT <= 2) ? 2 : 1)
+__global__ void __launch_bounds__(kMaxThreads + 64, 2)
     k_step_tma(const SwarmArgs a, int stages) {
   extern __shared__ __align__(128) unsigned char dsmem[];
   const int nvec = a.nvec, d = a.d;
@@ -576,7 +584,7 @@ __global__ void __launch_bounds__(kMaxThreads + 64, (VPT <= 2) ? 2 : 1)
 
   // ---------------- compute warps
   const PhiloxKey key{a.seed_lo, a.seed_hi};
-  const MoveParams mp{a.w, a.c1, a.c2, a.lo, a.hi, a.vmax};
+  const MoveParams mp = move_params(a);
   mbar_wait(&gbar, 0);
   int s = 0;
   unsigned ph = 0;
@@ -584,16 +592,18 @@ __global__ void __launch_bounds__(kMaxThreads + 64, (VPT <= 2) ? 2 : 1)
     const uint32_t gi = (uint32_t)(a.row_begin + r);
     float4* st = ring + (size_t)s * 3 * nvec;
     mbar_wait(&full[s], ph);
-    float4 xn[VPT];
-#pragma unroll
+    float acc[Obj::kAcc];
+    Obj::init(acc);
+    // VPT <= 2: fully unrolled for ILP; larger VPT: pairs, to bound registers.
+#pragma unroll(VPT <= 2 ? VPT : 2)
     for (int j = 0; j < VPT; ++j) {
       const int q = tid + j * nthr;
       if (q < nvec) {
         float4 x = st[q], v = st[nvec + q];
         const float4 pb = st[2 * nvec + q];
         const float4 g = sG[q];
-        const float4 r1 = uniforms4(key, kTagR1, t, gi, (uint32_t)q);
-        const float4 r2 = uniforms4(key, kTagR2, t, gi, (uint32_t)q);
+        const float4 r1 = raw24x4(key, kTagR1, t, gi, (uint32_t)q);
+        const float4 r2 = raw24x4(key, kTagR2, t, gi, (uint32_t)q);
         move1(mp, x.x, v.x, pb.x, g.x, r1.x, r2.x);
         move1(mp, x.y, v.y, pb.y, g.y, r1.y, r2.y);
         move1(mp, x.z, v.z, pb.z, g.z, r1.z, r2.z);
@@ -606,27 +616,15 @@ __global__ void __launch_bounds__(kMaxThreads + 64, (VPT <= 2) ? 2 : 1)
         }
         st[q] = x;
         st[nvec + q] = v;
-        xn[j] = x;
+        if constexpr (!Obj::kNeighbor) map4<Obj>(acc, x, 0.f, 4 * q, d);
       }
     }
-    float acc[Obj::kAcc];
-    Obj::init(acc);
     if constexpr (Obj::kNeighbor) {
       team_sync(nthr);  // every x' of the row is in the stage
-#pragma unroll
+#pragma unroll(VPT <= 2 ? VPT : 2)
       for (int j = 0; j < VPT; ++j) {
         const int q = tid + j * nthr;
-        if (q < nvec) {
-          const int jj = 4 * q;
-          const float nx = (q + 1 < nvec) ? st[q + 1].x : 0.f;
-          map4<Obj>(acc, xn[j], nx, jj, d);
-        }
-      }
-    } else {
-#pragma unroll
-      for (int j = 0; j < VPT; ++j) {
-        const int q = tid + j * nthr;
-        if (q < nvec) map4<Obj>(acc, xn[j], 0.f, 4 * q, d);
+        if (q < nvec) map4<Obj>(acc, st[q], (q + 1 < nvec) ? st[q + 1].x : 0.f, 4 * q, d);
       }
     }
     warp_combine<Obj>(acc);
@@ -894,7 +892,8 @@ cudaError_t plan_launch(int objective, int d, long long n_local, int sm_count, c
     int by_regs = 0;
     if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&by_regs, fn, threads, 0)) != cudaSuccess)
       return e;
-    int ctas = by_regs < 1 ? 1 : (by_regs > 2 ? 2 : by_regs);
+    const int cap = (h.ctas >= 1 && h.ctas <= 8) ? h.ctas : 2;
+    int ctas = by_regs < 1 ? 1 : (by_regs > cap ? cap : by_regs);
     int stages = 0;
     for (; ctas >= 1; --ctas) {
       size_t budget = kSmemPerSm / ctas - kStaticReserve;
