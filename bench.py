@@ -329,7 +329,10 @@ def run_gpu(args, w):
                          "alg_bytes_per_launch": alg_bytes,
                          "l2_resident": state_per_gpu <= L2_BYTES,
                          "cta": {"threads": info["threads_per_cta"], "vpt": info["vec_per_thread"],
-                                 "grid": info["grid"], "ctas_per_sm": info["ctas_per_sm"]}},
+                                 "grid": info["grid"], "ctas_per_sm": info["ctas_per_sm"],
+                                 "tma_pipeline": info["tma_pipeline"],
+                                 "stages": info["pipeline_stages"],
+                                 "smem_bytes": info["smem_bytes"]}},
             "clocks": clk.result, "e2e": e2e, "clocks_e2e": clk_e2e,
             "cpu_baseline": cpu, "gbest": {"fitness": gf, "index": gi},
         }

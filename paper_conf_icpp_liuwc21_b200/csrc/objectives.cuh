@@ -42,7 +42,6 @@ __device__ __forceinline__ float sinpi_sq(float x) {
 }
 
 constexpr float kInv2Pi = 0.15915494309189535f;
-constexpr float kInvPi = 0.3183098861837907f;
 
 // Sphere: sum x_k^2.
 struct Sphere {
@@ -114,8 +113,9 @@ struct Easom {
     a[1] = 0.f;
   }
   __device__ static void map(float* a, float x, float, int, int) {
+    const float c = cosf(x);  // accurate near its zeros (cos^2 is relative here)
     const float e = x - 3.14159265358979f;
-    a[0] *= 1.f - sinpi_sq(x * kInvPi);  // cos^2(x)
+    a[0] *= c * c;
     a[1] = fmaf(e, e, a[1]);
   }
   __device__ static void combine(float* a, const float* b) {

@@ -894,13 +894,26 @@ cudaError_t plan_launch(int objective, int d, long long n_local, int sm_count, c
       return e;
     const int cap = (h.ctas >= 1 && h.ctas <= 8) ? h.ctas : 2;
     int ctas = by_regs < 1 ? 1 : (by_regs > cap ? cap : by_regs);
-    int stages = 0;
-    for (; ctas >= 1; --ctas) {
-      size_t budget = kSmemPerSm / ctas - kStaticReserve;
+    // The most CTAs per SM (<= cap) that still keep >= 3 rows in flight per
+    // CTA; two rows only if nothing else fits (measured: 2-stage rings leave
+    // HBM idle between rows, 3-4 stages saturate it).
+    auto stages_for = [&](int c) -> int {
+      size_t budget = kSmemPerSm / c - kStaticReserve;
       if (budget > kSmemPerCtaMax - kStaticReserve) budget = kSmemPerCtaMax - kStaticReserve;
-      if (budget > row) stages = (int)((budget - row) / (3 * row));
-      if (stages >= 2) break;
+      return budget > row ? (int)((budget - row) / (3 * row)) : 0;
+    };
+    int stages = 0;
+    int c = ctas;
+    for (; c >= 1; --c)
+      if (stages_for(c) >= 3) break;
+    if (c >= 1) {
+      ctas = c;
+    } else {
+      for (c = ctas; c >= 1 && stages_for(c) < 2; --c) {
+      }
+      ctas = c < 1 ? 1 : c;
     }
+    stages = stages_for(ctas);
     if (h.stages >= 2 && h.stages <= kMaxStages) stages = stages < h.stages ? stages : h.stages;
     if (stages > kMaxStages) stages = kMaxStages;
     if (stages >= 2) {

@@ -19,10 +19,11 @@ def fit_atol(obj: int, X: np.ndarray) -> np.ndarray:
     X = np.atleast_2d(np.asarray(X, dtype=np.float64))
     m, d = X.shape
     if obj == GRIEWANK:
-        # product of d cosines: each factor's argument x*rsqrt(k) carries <= 3 eps
-        # relative error, cosf <= 2 eps: |dP| <= eps * sum(3|x|/sqrt k + 3) + d eps
+        # product of d cosines: each factor's argument y = x*rsqrt(k) carries <= 3 eps
+        # relative error and t = y/(2 pi) 2 more; cos = 1 - 2 sin^2(pi t) is within
+        # ~10 eps absolute of cos(t 2 pi) -> |dP| <= eps * sum(5 |y| + 10) + d eps
         k = np.arange(1, d + 1, dtype=np.float64)
-        return 2.0 ** -21 * (np.abs(X) / np.sqrt(k)).sum(axis=1) + 2.0 ** -21 * d
+        return 2.0 ** -21 * (np.abs(X) / np.sqrt(k)).sum(axis=1) + 2.0 ** -20 * d
     if obj == ACKLEY:
         # C/d carries <= (32 + log2 d + 4) eps absolute; times e
         return np.full(m, np.e * (36.0 + np.log2(max(d, 2))) * EPS * 2)
