@@ -40,7 +40,7 @@ class pso_info(C.Structure):
         ("d", C.c_int32), ("pitch", C.c_int32), ("rank", C.c_int32), ("world", C.c_int32),
         ("threads_per_cta", C.c_int32), ("vec_per_thread", C.c_int32), ("grid", C.c_int32),
         ("ctas_per_sm", C.c_int32), ("tma_pipeline", C.c_int32), ("pipeline_stages", C.c_int32),
-        ("smem_bytes", C.c_int32), ("vmax", C.c_float), ("t", C.c_uint64),
+        ("smem_bytes", C.c_int32), ("resident", C.c_int32), ("vmax", C.c_float), ("t", C.c_uint64),
         ("launches", C.c_uint64), ("improvements", C.c_uint64),
         ("step_kernel_ms", C.c_double), ("step_kernel_count", C.c_uint64),
         ("arena_bytes", C.c_size_t),

@@ -128,7 +128,11 @@ struct pso_swarm {
   uint64_t t = 0;
   bool poisoned = false;
   uint64_t launches = 0;
-  std::vector<std::pair<cudaEvent_t, cudaEvent_t>> events;
+  struct Timed {
+    cudaEvent_t start, stop;
+    uint64_t steps;  // step kernels (iterations) between the two events
+  };
+  std::vector<Timed> events;
   size_t events_used = 0;
   double timed_ms = 0;
   uint64_t timed_count = 0;
@@ -208,6 +212,36 @@ pso_status reset_ctl(pso_swarm* h, uint32_t t) {
   c.improvements = old.improvements;
   PSO_CUDA(h, cudaMemcpyAsync(h->args.ctl, &c, sizeof(DevCtl), cudaMemcpyHostToDevice, h->stream));
   PSO_CUDA(h, cudaStreamSynchronize(h->stream));
+  return PSO_OK;
+}
+
+// Sum the recorded step-kernel times into the totals (synchronises on them).
+pso_status fold_events(pso_swarm* h) {
+  for (size_t k = 0; k < h->events_used; ++k) {
+    float ms = 0;
+    PSO_CUDA(h, cudaEventSynchronize(h->events[k].stop));
+    PSO_CUDA(h, cudaEventElapsedTime(&ms, h->events[k].start, h->events[k].stop));
+    h->timed_ms += ms;
+    h->timed_count += h->events[k].steps;
+  }
+  h->events_used = 0;
+  return PSO_OK;
+}
+
+// Next event pair of the timing pool (bounded: folds into the totals when full).
+pso_status next_event(pso_swarm* h, pso_swarm::Timed** out, uint64_t steps) {
+  if (h->events_used == 4096) {
+    pso_status st = fold_events(h);
+    if (st != PSO_OK) return st;
+  }
+  if (h->events_used == h->events.size()) {
+    pso_swarm::Timed e{};
+    PSO_CUDA(h, cudaEventCreate(&e.start));
+    PSO_CUDA(h, cudaEventCreate(&e.stop));
+    h->events.push_back(e);
+  }
+  *out = &h->events[h->events_used++];
+  (*out)->steps = steps;
   return PSO_OK;
 }
 
@@ -346,6 +380,10 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
     if (!std::strcmp(v, "tma")) hints.kernel = 1;
   }
   {
+    const char* v = std::getenv("PSO_RESIDENT");
+    hints.allow_resident = !h->xchg && hints.kernel == -1 && !(v && !std::strcmp(v, "0"));
+  }
+  {
     cudaError_t e = plan_launch(objective, d, h->n_local > 0 ? h->n_local : 1, h->sm_count,
                                 hints, &h->cfg);
     if (e != cudaSuccess) return bail(cuda_fail(nullptr, e, "plan_launch"));
@@ -425,34 +463,30 @@ pso_status pso_step(pso_handle h, int64_t iters) {
   if (iters == 0) return PSO_OK;
   if ((st = use_device(h)) != PSO_OK) return st;
   const bool timing = (h->flags & PSO_FLAG_TIMING) != 0;
+  if (h->cfg.resident) {  // tiny swarm: the whole call is one single-CTA launch
+    for (int64_t done = 0; done < iters;) {
+      const int chunk = (int)((iters - done) < (1 << 30) ? (iters - done) : (1 << 30));
+      pso_swarm::Timed* ev = nullptr;
+      if (timing && (st = next_event(h, &ev, (uint64_t)chunk)) != PSO_OK) return st;
+      if (ev) PSO_CUDA(h, cudaEventRecord(ev->start, h->stream));
+      PSO_CUDA(h, launch_resident(h->objective, h->args, h->cfg, chunk, h->stream));
+      ++h->launches;
+      if (ev) PSO_CUDA(h, cudaEventRecord(ev->stop, h->stream));
+      done += chunk;
+    }
+    h->t += (uint64_t)iters;
+    return PSO_OK;
+  }
   for (int64_t it = 0; it < iters; ++it) {
     if (h->n_local > 0) {
-      std::pair<cudaEvent_t, cudaEvent_t>* ev = nullptr;
-      if (timing) {
-        if (h->events_used == h->events.size()) {
-          cudaEvent_t a, b;
-          PSO_CUDA(h, cudaEventCreate(&a));
-          PSO_CUDA(h, cudaEventCreate(&b));
-          h->events.emplace_back(a, b);
-        }
-        ev = &h->events[h->events_used++];
-        PSO_CUDA(h, cudaEventRecord(ev->first, h->stream));
-      }
+      pso_swarm::Timed* ev = nullptr;
+      if (timing && (st = next_event(h, &ev, 1)) != PSO_OK) return st;
+      if (ev) PSO_CUDA(h, cudaEventRecord(ev->start, h->stream));
       PSO_CUDA(h, launch_step(h->objective, h->args, h->cfg, h->stream));
       ++h->launches;
-      if (ev) PSO_CUDA(h, cudaEventRecord(ev->second, h->stream));
+      if (ev) PSO_CUDA(h, cudaEventRecord(ev->stop, h->stream));
     }
     if ((st = exchange(h)) != PSO_OK) return st;
-    if (timing && h->events_used >= 4096) {  // bound the event pool: fold into totals
-      PSO_CUDA(h, cudaStreamSynchronize(h->stream));
-      for (size_t k = 0; k < h->events_used; ++k) {
-        float ms = 0;
-        PSO_CUDA(h, cudaEventElapsedTime(&ms, h->events[k].first, h->events[k].second));
-        h->timed_ms += ms;
-      }
-      h->timed_count += h->events_used;
-      h->events_used = 0;
-    }
   }
   h->t += (uint64_t)iters;
   return PSO_OK;
@@ -536,13 +570,7 @@ pso_status pso_get_info(pso_handle h, pso_info* info) {
   if (st != PSO_OK) return st;
   if ((st = use_device(h)) != PSO_OK) return st;
   if ((st = sync_and_check(h)) != PSO_OK) return st;
-  for (size_t k = 0; k < h->events_used; ++k) {
-    float ms = 0;
-    PSO_CUDA(h, cudaEventElapsedTime(&ms, h->events[k].first, h->events[k].second));
-    h->timed_ms += ms;
-  }
-  h->timed_count += h->events_used;
-  h->events_used = 0;
+  if ((st = fold_events(h)) != PSO_OK) return st;
   DevCtl c{};
   PSO_CUDA(h, cudaMemcpy(&c, h->args.ctl, sizeof(DevCtl), cudaMemcpyDeviceToHost));
   std::memset(info, 0, sizeof(*info));
@@ -559,7 +587,8 @@ pso_status pso_get_info(pso_handle h, pso_info* info) {
   info->ctas_per_sm = h->cfg.ctas_per_sm;
   info->tma_pipeline = h->cfg.tma;
   info->pipeline_stages = h->cfg.stages;
-  info->smem_bytes = (int32_t)h->cfg.smem;
+  info->smem_bytes = (int32_t)(h->cfg.resident ? h->cfg.resident_smem : h->cfg.smem);
+  info->resident = h->cfg.resident;
   info->vmax = h->vmax;
   info->t = h->t;
   info->launches = h->launches;
@@ -589,8 +618,8 @@ void pso_destroy(pso_handle h) {
   cudaSetDevice(h->device);
   if (h->stream) cudaStreamSynchronize(h->stream);
   for (auto& e : h->events) {
-    cudaEventDestroy(e.first);
-    cudaEventDestroy(e.second);
+    cudaEventDestroy(e.start);
+    cudaEventDestroy(e.stop);
   }
   if (h->arena) cudaFree(h->arena);
   if (h->own_stream && h->stream) cudaStreamDestroy(h->stream);

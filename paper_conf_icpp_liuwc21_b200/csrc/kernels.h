@@ -49,6 +49,9 @@ struct LaunchCfg {
   int tma = 0;        // 1: warp-specialised bulk-copy (TMA) pipeline; 0: register streaming
   int stages = 0;     // TMA pipeline depth (rows in flight per CTA)
   size_t smem = 0;    // dynamic shared memory bytes of the step kernel
+  int resident = 0;   // 1: tiny swarm, whole pso_step in one single-CTA launch
+  int resident_threads = 0;
+  size_t resident_smem = 0;
   size_t init_smem = 0;
 };
 
@@ -58,6 +61,7 @@ struct PlanHints {
   int kernel = -1;  // -1 auto, 0 register, 1 tma
   int stages = 0;
   int ctas = 0;     // max CTAs per SM for the TMA pipeline (0: auto = 2)
+  bool allow_resident = false;  // single-GPU tiny swarms (PSO_RESIDENT=0 disables)
 };
 
 bool objective_registered(int objective);
@@ -66,6 +70,8 @@ cudaError_t plan_launch(int objective, int d, long long n_local, int sm_count, c
                         LaunchCfg* cfg);
 cudaError_t launch_init(int objective, const SwarmArgs& a, const LaunchCfg& c, cudaStream_t s);
 cudaError_t launch_step(int objective, const SwarmArgs& a, const LaunchCfg& c, cudaStream_t s);
+cudaError_t launch_resident(int objective, const SwarmArgs& a, const LaunchCfg& c, int iters,
+                            cudaStream_t s);
 cudaError_t launch_rebest(const SwarmArgs& a, unsigned t, cudaStream_t s);
 cudaError_t launch_select(const SwarmArgs& a, cudaStream_t s);
 

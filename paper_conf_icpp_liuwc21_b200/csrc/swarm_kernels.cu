@@ -642,6 +642,132 @@ __global__ void __launch_bounds__(kMaxThreads + 64, 2)
   }
 }
 
+// ------------------------------------------------- resident kernel (small swarms)
+// NEXT-1 latency path: for tiny swarms (d <= 128, n d <= 8192)
+// one CTA keeps X, V, PB, pf and G in shared memory for all `iters`
+// iterations of a pso_step call, with one __syncthreads pair per iteration
+// instead of a kernel launch.  One warp per row (rows round-robin over warps),
+// lane q owns float4 q: the per-row reduction is exactly k_step_reg's for
+// its one-warp shape (lane butterfly; the cross-warp step only combines
+// identities), so fitness, decisions and state are bitwise those of the
+// streaming kernels.
+template <class Obj>
+__global__ void __launch_bounds__(1024, 1) k_resident(const SwarmArgs a, int iters) {
+  extern __shared__ __align__(16) unsigned char dsmem[];
+  const int nvec = a.nvec, d = a.d;
+  const int n = (int)a.n_local;
+  const int cells = n * nvec;
+  float4* sX = reinterpret_cast<float4*>(dsmem);
+  float4* sV = sX + cells;
+  float4* sP = sV + cells;
+  float4* sG = sP + cells;
+  float* spf = reinterpret_cast<float*>(sG + nvec);
+  __shared__ unsigned long long s_acc;
+  __shared__ unsigned s_imp;
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, nwarps = blockDim.x >> 5;
+  const float4* X4 = reinterpret_cast<const float4*>(a.X);
+  const float4* V4 = reinterpret_cast<const float4*>(a.V);
+  const float4* P4 = reinterpret_cast<const float4*>(a.PB);
+  for (int i = tid; i < cells; i += blockDim.x) {
+    sX[i] = X4[i];
+    sV[i] = V4[i];
+    sP[i] = P4[i];
+  }
+  for (int i = tid; i < nvec; i += blockDim.x) sG[i] = reinterpret_cast<const float4*>(a.G)[i];
+  for (int i = tid; i < n; i += blockDim.x) spf[i] = a.pf[i];
+  const unsigned long long cur0 = a.ctl->key_cur;
+  const uint32_t t0 = a.ctl->t;
+  if (tid == 0) {
+    s_acc = cur0;
+    s_imp = 0;
+  }
+  __syncthreads();
+  const PhiloxKey key{a.seed_lo, a.seed_hi};
+  const MoveParams mp = move_params(a);
+  unsigned long long cur = cur0;
+  for (int it = 0; it < iters; ++it) {
+    const uint32_t t = t0 + 1u + (uint32_t)it;
+    const uint32_t inc_ord = (uint32_t)(cur >> 32);
+    unsigned long long best = ~0ull;
+    unsigned nimp = 0;
+    for (int r = warp; r < n; r += nwarps) {
+      const uint32_t gi = (uint32_t)(a.row_begin + r);
+      const int c = r * nvec + lane;
+      float4 x = make_float4(0.f, 0.f, 0.f, 0.f);
+      if (lane < nvec) {
+        float4 v = sV[c];
+        const float4 pb = sP[c], g = sG[lane];
+        x = sX[c];
+        const float4 r1 = raw24x4(key, kTagR1, t, gi, (uint32_t)lane);
+        const float4 r2 = raw24x4(key, kTagR2, t, gi, (uint32_t)lane);
+        move1(mp, x.x, v.x, pb.x, g.x, r1.x, r2.x);
+        move1(mp, x.y, v.y, pb.y, g.y, r1.y, r2.y);
+        move1(mp, x.z, v.z, pb.z, g.z, r1.z, r2.z);
+        move1(mp, x.w, v.w, pb.w, g.w, r1.w, r2.w);
+        if ((d & 3) && lane == nvec - 1) {
+          const int jj = 4 * lane;
+          if (jj + 1 >= d) x.y = v.y = 0.f;
+          if (jj + 2 >= d) x.z = v.z = 0.f;
+          if (jj + 3 >= d) x.w = v.w = 0.f;
+        }
+        sX[c] = x;
+        sV[c] = v;
+      }
+      float acc[Obj::kAcc];
+      Obj::init(acc);
+      float nx = 0.f;
+      if constexpr (Obj::kNeighbor) {
+        nx = __shfl_down_sync(kFull, x.x, 1);
+        if (lane + 1 >= nvec) nx = 0.f;
+      }
+      if (lane < nvec) map4<Obj>(acc, x, nx, 4 * lane, d);
+      warp_combine<Obj>(acc);
+      const float f = Obj::finalize(acc, d);
+      const bool improved = f < spf[r];  // strict; NaN never improves
+      __syncwarp();
+      if (improved) {
+        if (lane < nvec) sP[c] = x;
+        if (lane == 0) {
+          spf[r] = f;
+          ++nimp;
+        }
+      }
+      if (lane == 0 && f == f && ord_f32(f) < inc_ord) {
+        const unsigned long long k = pack_key(f, gi);
+        best = k < best ? k : best;
+      }
+    }
+    if (lane == 0) {
+      if (best != ~0ull) atomicMin(&s_acc, best);
+      if (nimp) atomicAdd(&s_imp, nimp);
+    }
+    __syncthreads();
+    const unsigned long long acc_k = s_acc;
+    if (acc_k < cur) {
+      const int lr = (int)((long long)(uint32_t)acc_k - a.row_begin);
+      for (int q = tid; q < nvec; q += blockDim.x) sG[q] = sP[lr * nvec + q];
+      cur = acc_k;
+    }
+    __syncthreads();
+  }
+  float4* X4w = reinterpret_cast<float4*>(a.X);
+  float4* V4w = reinterpret_cast<float4*>(a.V);
+  float4* P4w = reinterpret_cast<float4*>(a.PB);
+  for (int i = tid; i < cells; i += blockDim.x) {
+    X4w[i] = sX[i];
+    V4w[i] = sV[i];
+    P4w[i] = sP[i];
+  }
+  for (int i = tid; i < nvec; i += blockDim.x) reinterpret_cast<float4*>(a.G)[i] = sG[i];
+  for (int i = tid; i < n; i += blockDim.x) a.pf[i] = spf[i];
+  if (tid == 0) {
+    a.ctl->key_cur = cur;
+    a.ctl->key_acc = cur;
+    a.ctl->t = t0 + (uint32_t)iters;
+    a.ctl->improvements += s_imp;
+  }
+}
+
 // ------------------------------------------------------------ init kernel
 // Alg. 1 lines 1-3 (Sec 3.1): x0 = clamp(lo + span U, lo, hi), v0 = -vmax +
 // 2 vmax U from the X0 / V0 streams at t = 0; f = F(x0); pf = f (NaN -> +inf);
@@ -829,6 +955,18 @@ const void* pick(Which w, int vpt) {
 #undef PSO_VPT_CASES
 }
 
+const void* resident_kernel_for(int objective) {
+#define PSO_CASE(ID, F) \
+  case ID:              \
+    return (const void*)k_resident<F>;
+  switch (objective) {
+    PSO_ALL_OBJECTIVES(PSO_CASE)
+    default:
+      return nullptr;
+  }
+#undef PSO_CASE
+}
+
 const void* kernel_for(int objective, Which w, int vpt, bool* neighbor) {
 #define PSO_CASE(ID, F)                      \
   case ID:                                   \
@@ -864,6 +1002,7 @@ void shape_for(int nvec, int vpt_override, int* vpt, int* threads) {
 constexpr size_t kSmemPerSm = 228 * 1024;       // B200 unified L1/shared per SM
 constexpr size_t kSmemPerCtaMax = 227 * 1024;   // opt-in maximum per CTA
 constexpr size_t kStaticReserve = 2048;         // static shared + per-CTA reservation
+constexpr long long kResidentElems = 8192;      // resident path: n d <= this
 
 }  // namespace
 
@@ -882,6 +1021,22 @@ cudaError_t plan_launch(int objective, int d, long long n_local, int sm_count, c
   const size_t first = nb ? (size_t)nvec * 4 : 0;
   cfg->init_smem = first;
   cudaError_t e;
+
+  // ---- resident single-CTA path for tiny swarms (single GPU only)
+  cfg->resident = 0;
+  if (h.allow_resident && nvec <= 32 && n_local * nvec * 4 <= kResidentElems) {
+    const size_t smem = (size_t)n_local * nvec * 16 * 3 + (size_t)nvec * 16 + (size_t)n_local * 4;
+    const void* fn = resident_kernel_for(objective);
+    if (smem <= kSmemPerCtaMax - kStaticReserve &&
+        cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) ==
+            cudaSuccess) {
+      int warps = (int)(n_local < 32 ? n_local : 32);
+      cfg->resident = 1;
+      cfg->resident_threads = 32 * (warps < 1 ? 1 : warps);
+      cfg->resident_smem = smem;
+    }
+    cudaGetLastError();
+  }
 
   // ---- TMA pipeline: rows of >= 256 dims unless forced otherwise
   bool tma = h.kernel == 1 || (h.kernel == -1 && nvec >= 64);
@@ -964,6 +1119,14 @@ cudaError_t launch_step(int objective, const SwarmArgs& a, const LaunchCfg& c, c
   int stages = c.stages;
   void* args[] = {const_cast<SwarmArgs*>(&a), &stages};
   return cudaLaunchKernel(fn, dim3(c.grid), dim3(c.threads), args, c.smem, s);
+}
+
+cudaError_t launch_resident(int objective, const SwarmArgs& a, const LaunchCfg& c, int iters,
+                            cudaStream_t s) {
+  const void* fn = resident_kernel_for(objective);
+  if (!fn) return cudaErrorInvalidDeviceFunction;
+  void* args[] = {const_cast<SwarmArgs*>(&a), &iters};
+  return cudaLaunchKernel(fn, dim3(1), dim3(c.resident_threads), args, c.resident_smem, s);
 }
 
 cudaError_t launch_init(int objective, const SwarmArgs& a, const LaunchCfg& c, cudaStream_t s) {

@@ -332,3 +332,30 @@ def test_exchange_path_with_single_rank_comm(obj, n, d, monkeypatch):
         g.close()
     finally:
         fp.nccl_comm_destroy(comm)
+
+
+# ------------------------------------------------------------------ resident path (NEXT-1)
+@pytest.mark.parametrize("obj,n,d", [(SPHERE, 32, 10), (ROSENBROCK, 100, 16), (GRIEWANK, 7, 13),
+                                     (ACKLEY, 64, 128), (RASTRIGIN, 1, 1), (RASTRIGIN, 200, 40)])
+def test_resident_path_bitwise_equals_streaming(obj, n, d, monkeypatch):
+    """The single-CTA shared-memory path for tiny swarms gives the streaming
+    kernel's results bit for bit (same per-row reduction order), in one launch
+    per pso_step call."""
+    a = gpu_swarm(n, d, obj, seed=31)
+    assert a.info()["resident"] == 1
+    monkeypatch.setenv("PSO_RESIDENT", "0")
+    b = gpu_swarm(n, d, obj, seed=31)
+    assert b.info()["resident"] == 0
+    a.reset_counters()
+    for k in (1, 7, 42):
+        a.step(k)
+        b.step(k)
+        for x, y in zip(a.get_state()[:4], b.get_state()[:4]):
+            assert_bitwise(x, y, f"resident vs streaming after +{k}")
+        fa, ia, Ga = a.gbest()
+        fb, ib, Gb = b.gbest()
+        assert (fa, ia) == (fb, ib)
+        assert_bitwise(Ga, Gb, "G")
+    info = a.info()
+    assert info["launches"] == 3 and info["t"] == 50
+    assert info["improvements"] > 0
