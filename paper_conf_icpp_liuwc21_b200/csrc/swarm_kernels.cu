@@ -646,11 +646,12 @@ __global__ void __launch_bounds__(kMaxThreads + 64, 2)
 // NEXT-1 latency path: for tiny swarms (d <= 128, n d <= 8192)
 // one CTA keeps X, V, PB, pf and G in shared memory for all `iters`
 // iterations of a pso_step call, with one __syncthreads pair per iteration
-// instead of a kernel launch.  One warp per row (rows round-robin over warps),
-// lane q owns float4 q: the per-row reduction is exactly k_step_reg's for
-// its one-warp shape (lane butterfly; the cross-warp step only combines
-// identities), so fitness, decisions and state are bitwise those of the
-// streaming kernels.
+// instead of a kernel launch.  Rows are packed into warps in lane groups of
+// gs = pow2ceil(nvec) lanes (lane q of a group owns float4 q).  The per-row
+// reduction is the xor butterfly over the group, which is exactly the order
+// k_step_reg's one-warp shape produces for these rows (its wider butterfly
+// steps only add the identities of idle lanes), so fitness, decisions and
+// state are bitwise those of the streaming kernels.
 template <class Obj>
 __global__ void __launch_bounds__(1024, 1) k_resident(const SwarmArgs a, int iters) {
   extern __shared__ __align__(16) unsigned char dsmem[];
@@ -665,6 +666,11 @@ __global__ void __launch_bounds__(1024, 1) k_resident(const SwarmArgs a, int ite
   __shared__ unsigned long long s_acc;
   __shared__ unsigned s_imp;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, nwarps = blockDim.x >> 5;
+  int gs = 1;
+  while (gs < nvec) gs <<= 1;
+  const int rpw = 32 / gs;              // rows per warp pass
+  const int sub = lane & (gs - 1);      // float4 index within the row
+  const int leader = lane & ~(gs - 1);  // lane holding the row's result
   const float4* X4 = reinterpret_cast<const float4*>(a.X);
   const float4* V4 = reinterpret_cast<const float4*>(a.V);
   const float4* P4 = reinterpret_cast<const float4*>(a.PB);
@@ -690,22 +696,25 @@ __global__ void __launch_bounds__(1024, 1) k_resident(const SwarmArgs a, int ite
     const uint32_t inc_ord = (uint32_t)(cur >> 32);
     unsigned long long best = ~0ull;
     unsigned nimp = 0;
-    for (int r = warp; r < n; r += nwarps) {
+    for (int base = warp * rpw; base < n; base += nwarps * rpw) {  // warp-uniform loop
+      const int r = base + (lane / gs);
+      const bool row_ok = r < n;
+      const bool act = row_ok && sub < nvec;
       const uint32_t gi = (uint32_t)(a.row_begin + r);
-      const int c = r * nvec + lane;
+      const int c = r * nvec + sub;
       float4 x = make_float4(0.f, 0.f, 0.f, 0.f);
-      if (lane < nvec) {
+      if (act) {
         float4 v = sV[c];
-        const float4 pb = sP[c], g = sG[lane];
+        const float4 pb = sP[c], g = sG[sub];
         x = sX[c];
-        const float4 r1 = raw24x4(key, kTagR1, t, gi, (uint32_t)lane);
-        const float4 r2 = raw24x4(key, kTagR2, t, gi, (uint32_t)lane);
+        const float4 r1 = raw24x4(key, kTagR1, t, gi, (uint32_t)sub);
+        const float4 r2 = raw24x4(key, kTagR2, t, gi, (uint32_t)sub);
         move1(mp, x.x, v.x, pb.x, g.x, r1.x, r2.x);
         move1(mp, x.y, v.y, pb.y, g.y, r1.y, r2.y);
         move1(mp, x.z, v.z, pb.z, g.z, r1.z, r2.z);
         move1(mp, x.w, v.w, pb.w, g.w, r1.w, r2.w);
-        if ((d & 3) && lane == nvec - 1) {
-          const int jj = 4 * lane;
+        if ((d & 3) && sub == nvec - 1) {
+          const int jj = 4 * sub;
           if (jj + 1 >= d) x.y = v.y = 0.f;
           if (jj + 2 >= d) x.z = v.z = 0.f;
           if (jj + 3 >= d) x.w = v.w = 0.f;
@@ -718,24 +727,35 @@ __global__ void __launch_bounds__(1024, 1) k_resident(const SwarmArgs a, int ite
       float nx = 0.f;
       if constexpr (Obj::kNeighbor) {
         nx = __shfl_down_sync(kFull, x.x, 1);
-        if (lane + 1 >= nvec) nx = 0.f;
+        if (sub + 1 >= nvec) nx = 0.f;
       }
-      if (lane < nvec) map4<Obj>(acc, x, nx, 4 * lane, d);
-      warp_combine<Obj>(acc);
+      if (act) map4<Obj>(acc, x, nx, 4 * sub, d);
+      for (int off = gs >> 1; off > 0; off >>= 1) {
+        float o[Obj::kAcc];
+#pragma unroll
+        for (int k = 0; k < Obj::kAcc; ++k) o[k] = __shfl_xor_sync(kFull, acc[k], off);
+        Obj::combine(acc, o);
+      }
       const float f = Obj::finalize(acc, d);
-      const bool improved = f < spf[r];  // strict; NaN never improves
+      const int imp_l = (row_ok && lane == leader && f < spf[r]) ? 1 : 0;  // strict
+      const bool improved = __shfl_sync(kFull, imp_l, leader) != 0;
       __syncwarp();
       if (improved) {
-        if (lane < nvec) sP[c] = x;
-        if (lane == 0) {
+        if (act) sP[c] = x;
+        if (lane == leader) {
           spf[r] = f;
           ++nimp;
         }
       }
-      if (lane == 0 && f == f && ord_f32(f) < inc_ord) {
+      if (row_ok && lane == leader && f == f && ord_f32(f) < inc_ord) {
         const unsigned long long k = pack_key(f, gi);
         best = k < best ? k : best;
       }
+    }
+    for (int off = 16; off > 0; off >>= 1) {
+      const unsigned long long o = __shfl_xor_sync(kFull, best, off);
+      best = o < best ? o : best;
+      nimp += __shfl_xor_sync(kFull, nimp, off);
     }
     if (lane == 0) {
       if (best != ~0ull) atomicMin(&s_acc, best);
@@ -1030,9 +1050,13 @@ cudaError_t plan_launch(int objective, int d, long long n_local, int sm_count, c
     if (smem <= kSmemPerCtaMax - kStaticReserve &&
         cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) ==
             cudaSuccess) {
-      int warps = (int)(n_local < 32 ? n_local : 32);
+      int gs = 1;
+      while (gs < nvec) gs <<= 1;
+      const long long rpw = 32 / gs;
+      long long warps = (n_local + rpw - 1) / rpw;
+      if (warps > 32) warps = 32;
       cfg->resident = 1;
-      cfg->resident_threads = 32 * (warps < 1 ? 1 : warps);
+      cfg->resident_threads = 32 * (int)(warps < 1 ? 1 : warps);
       cfg->resident_smem = smem;
     }
     cudaGetLastError();
