@@ -222,12 +222,15 @@ def run_gpu(args, w):
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     comm = None
-    if world > 1:
+    # PSO_FORCE_EXCHANGE=1 runs the multi-GPU exchange (process group, NCCL
+    # communicator, all-gather + select every step) even on one rank.
+    use_comm = world > 1 or os.environ.get("PSO_FORCE_EXCHANGE", "0") not in ("", "0")
+    if use_comm:
         dist.init_process_group("nccl", device_id=dev)
         comm = init_comm(local)
 
     def barrier():
-        if world > 1:
+        if use_comm:
             dist.barrier()
         torch.cuda.synchronize()
 
@@ -337,7 +340,7 @@ def run_gpu(args, w):
             "cpu_baseline": cpu, "gbest": {"fitness": gf, "index": gi},
         }
         print(json.dumps(line), flush=True)
-    if world > 1:
+    if use_comm:
         dist.barrier()
         dist.destroy_process_group()
     return 0
