@@ -159,8 +159,11 @@ typedef struct {
   int32_t tma_pipeline;          /* 1: bulk-copy (TMA) pipelined step kernel */
   int32_t pipeline_stages;       /* rows in flight per CTA in that pipeline */
   int32_t smem_bytes;            /* dynamic shared memory of the step kernel */
-  int32_t resident;              /* 1: tiny swarm held in one CTA's shared memory for
-                                    a whole pso_step call (one launch per call) */
+  int32_t resident;              /* 0: streaming kernel, one launch per iteration;
+                                    1: tiny swarm held in one CTA's shared memory,
+                                    2: swarm held in the whole grid's shared memory
+                                    (cooperative launch); 1 and 2 run a whole
+                                    pso_step call in one launch (single GPU only) */
   float vmax;
   uint64_t t;                    /* iterations done */
   uint64_t launches;             /* kernels launched by this handle so far */

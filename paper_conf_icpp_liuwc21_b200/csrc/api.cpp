@@ -205,6 +205,8 @@ pso_status reset_ctl(pso_swarm* h, uint32_t t) {
   c.improvements = 0;
   c.done = 0;
   c.t = t;
+  c.key_par[0] = c.key_par[1] = ~0ull;
+  c.bar_count = 0;
   // improvements are preserved across set_state: read-modify-write
   DevCtl old{};
   PSO_CUDA(h, cudaMemcpyAsync(&old, h->args.ctl, sizeof(DevCtl), cudaMemcpyDeviceToHost, h->stream));
@@ -396,9 +398,10 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
   const size_t gb = align_up((size_t)h->pitch * 4, 256);
   const size_t ctlb = align_up(sizeof(DevCtl), 256);
   const size_t rec = align_up(record_bytes(h->pitch), 256);
+  const size_t candb = h->cfg.gridres ? align_up(2 * (size_t)h->cfg.gridres_grid * h->pitch * 4, 256) : 0;
   const size_t sendb = h->xchg ? rec : 0;
   const size_t recvb = h->xchg ? (size_t)h->world * record_bytes(h->pitch) : 0;
-  h->arena_bytes = 3 * mat + pfb + gb + ctlb + sendb + align_up(recvb, 256);
+  h->arena_bytes = 3 * mat + pfb + gb + ctlb + candb + sendb + align_up(recvb, 256);
   {
     cudaError_t e = cudaMalloc(&h->arena, h->arena_bytes);
     if (e == cudaErrorMemoryAllocation) {
@@ -415,6 +418,7 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
   A.pf = (float*)p; p += pfb;
   A.G = (float*)p; p += gb;
   A.ctl = (DevCtl*)p; p += ctlb;
+  A.cand = h->cfg.gridres ? (float*)p : nullptr; p += candb;
   A.send = h->xchg ? p : nullptr; p += sendb;
   A.recv = h->xchg ? p : nullptr;
   A.n_local = h->n_local;
@@ -463,13 +467,16 @@ pso_status pso_step(pso_handle h, int64_t iters) {
   if (iters == 0) return PSO_OK;
   if ((st = use_device(h)) != PSO_OK) return st;
   const bool timing = (h->flags & PSO_FLAG_TIMING) != 0;
-  if (h->cfg.resident) {  // tiny swarm: the whole call is one single-CTA launch
+  if (h->cfg.resident || h->cfg.gridres) {  // the whole call is one launch
     for (int64_t done = 0; done < iters;) {
       const int chunk = (int)((iters - done) < (1 << 30) ? (iters - done) : (1 << 30));
       pso_swarm::Timed* ev = nullptr;
       if (timing && (st = next_event(h, &ev, (uint64_t)chunk)) != PSO_OK) return st;
       if (ev) PSO_CUDA(h, cudaEventRecord(ev->start, h->stream));
-      PSO_CUDA(h, launch_resident(h->objective, h->args, h->cfg, chunk, h->stream));
+      if (h->cfg.resident)
+        PSO_CUDA(h, launch_resident(h->objective, h->args, h->cfg, chunk, h->stream));
+      else
+        PSO_CUDA(h, launch_gridres(h->objective, h->args, h->cfg, chunk, h->stream));
       ++h->launches;
       if (ev) PSO_CUDA(h, cudaEventRecord(ev->stop, h->stream));
       done += chunk;
@@ -588,7 +595,11 @@ pso_status pso_get_info(pso_handle h, pso_info* info) {
   info->tma_pipeline = h->cfg.tma;
   info->pipeline_stages = h->cfg.stages;
   info->smem_bytes = (int32_t)(h->cfg.resident ? h->cfg.resident_smem : h->cfg.smem);
-  info->resident = h->cfg.resident;
+  info->resident = h->cfg.resident ? 1 : (h->cfg.gridres ? 2 : 0);
+  if (h->cfg.gridres) {
+    info->grid = h->cfg.gridres_grid;
+    info->smem_bytes = (int32_t)h->cfg.gridres_smem;
+  }
   info->vmax = h->vmax;
   info->t = h->t;
   info->launches = h->launches;

@@ -15,8 +15,11 @@ struct DevCtl {
   unsigned long long improvements;  // pbest improvements, summed
   unsigned int done;                // last-CTA ticket counter
   unsigned int t;                   // iterations done (low 32 bits; Philox ctr[2])
-  unsigned long long pad[4];
+  unsigned long long key_par[2];    // grid-resident kernel: per-iteration-parity accumulators
+  unsigned int bar_count, bar_gen;  // grid-resident kernel: grid barrier
+  unsigned long long pad;
 };
+static_assert(sizeof(DevCtl) == 64, "DevCtl is one 64-byte block");
 
 // Exchange record for world > 1: the local candidate key and its PB row.
 // Layout: [u64 key][u64 pad][pitch floats].
@@ -28,6 +31,7 @@ struct SwarmArgs {
   float* PB;
   float* pf;  // n_local
   float* G;   // pitch (gbest position)
+  float* cand;                // grid-resident kernel: [2][grid][pitch] candidate rows
   unsigned char* send;        // world > 1: this rank's exchange record
   const unsigned char* recv;  // world > 1: world records after the all-gather
   DevCtl* ctl;
@@ -50,6 +54,10 @@ struct LaunchCfg {
   int stages = 0;     // TMA pipeline depth (rows in flight per CTA)
   size_t smem = 0;    // dynamic shared memory bytes of the step kernel
   int resident = 0;   // 1: tiny swarm, whole pso_step in one single-CTA launch
+  int gridres = 0;    // 1: swarm held in the grid's shared memory (cooperative launch)
+  int gridres_grid = 0;
+  int gridres_rows = 0;     // max rows per CTA
+  size_t gridres_smem = 0;
   int resident_threads = 0;
   size_t resident_smem = 0;
   size_t init_smem = 0;
@@ -72,6 +80,8 @@ cudaError_t launch_init(int objective, const SwarmArgs& a, const LaunchCfg& c, c
 cudaError_t launch_step(int objective, const SwarmArgs& a, const LaunchCfg& c, cudaStream_t s);
 cudaError_t launch_resident(int objective, const SwarmArgs& a, const LaunchCfg& c, int iters,
                             cudaStream_t s);
+cudaError_t launch_gridres(int objective, const SwarmArgs& a, const LaunchCfg& c, int iters,
+                           cudaStream_t s);
 cudaError_t launch_rebest(const SwarmArgs& a, unsigned t, cudaStream_t s);
 cudaError_t launch_select(const SwarmArgs& a, cudaStream_t s);
 

@@ -788,6 +788,212 @@ __global__ void __launch_bounds__(1024, 1) k_resident(const SwarmArgs a, int ite
   }
 }
 
+// ------------------------------------------------- grid-resident kernel
+// NEXT-1 for mid-size swarms whose state fits in the GPU's aggregate shared
+// memory (e.g. C2, 1024 x 1000 = 12 MB): a cooperative persistent grid; CTA b
+// owns rows b, b + grid, ... and keeps their x, v, pb (and pf) in shared
+// memory for all `iters` iterations of a pso_step call, so an iteration moves
+// no row data through L2/HBM at all.  Per row the arithmetic and the
+// reduction order are k_step_tma's (thread-sequential over its float4s, warp
+// butterfly, warps combined in index order by one thread), so results are
+// bitwise those of the streaming kernel.  Per iteration: each CTA publishes
+// its best candidate row to cand[parity][cta] and its key to key_par[parity];
+// a grid barrier (atomic ticket + generation flag; the last CTA resets the
+// other parity's accumulator); then every CTA pulls the winner's row into its
+// shared-memory G.
+__device__ __forceinline__ unsigned ld_acquire_u32(const unsigned* p) {
+  unsigned v;
+  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+
+template <class Obj, int VPT>
+__global__ void __launch_bounds__(kMaxThreads, 1) k_gridres(const SwarmArgs a, int iters) {
+  extern __shared__ __align__(16) unsigned char dsmem[];
+  const int nvec = a.nvec, d = a.d;
+  const int nthr = blockDim.x, tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int nwarps = nthr >> 5;
+  const int grid = gridDim.x, b = blockIdx.x;
+  const long long n = a.n_local;
+  const int myrows = (int)((n - b + grid - 1) / grid);  // rows b, b+grid, ...
+  float4* sG = reinterpret_cast<float4*>(dsmem);
+  float4* sRows = sG + nvec;  // [myrows][3][nvec]
+  float* spf = reinterpret_cast<float*>(sRows + (size_t)myrows * 3 * nvec);
+  __shared__ float red[(kMaxThreads / 32) * 2];
+  __shared__ float s_f;
+  __shared__ int s_imp;
+  __shared__ unsigned long long s_best;
+  __shared__ int s_best_row;
+
+  // ---- load this CTA's rows and G
+  for (int k = 0; k < myrows; ++k) {
+    const long long r = b + (long long)k * grid;
+    const float4* X4 = reinterpret_cast<const float4*>(a.X) + r * nvec;
+    const float4* V4 = reinterpret_cast<const float4*>(a.V) + r * nvec;
+    const float4* P4 = reinterpret_cast<const float4*>(a.PB) + r * nvec;
+    float4* st = sRows + (size_t)k * 3 * nvec;
+    for (int q = tid; q < nvec; q += nthr) {
+      st[q] = X4[q];
+      st[nvec + q] = V4[q];
+      st[2 * nvec + q] = P4[q];
+    }
+    if (tid == 0) spf[k] = a.pf[r];
+  }
+  for (int q = tid; q < nvec; q += nthr) sG[q] = reinterpret_cast<const float4*>(a.G)[q];
+  const unsigned long long cur0 = a.ctl->key_cur;
+  const uint32_t t0 = a.ctl->t;
+  __syncthreads();
+
+  const PhiloxKey key{a.seed_lo, a.seed_hi};
+  const MoveParams mp = move_params(a);
+  unsigned long long cur = cur0;
+  unsigned nimp = 0;
+  for (int it = 0; it < iters; ++it) {
+    const uint32_t t = t0 + 1u + (uint32_t)it;
+    const int par = (int)(t & 1u);
+    const uint32_t inc_ord = (uint32_t)(cur >> 32);
+    unsigned long long best = ~0ull;
+    int best_row = -1;
+    for (int k = 0; k < myrows; ++k) {
+      const long long r = b + (long long)k * grid;
+      const uint32_t gi = (uint32_t)(a.row_begin + r);
+      float4* st = sRows + (size_t)k * 3 * nvec;
+      float acc[Obj::kAcc];
+      Obj::init(acc);
+#pragma unroll(VPT <= 2 ? VPT : 2)
+      for (int j = 0; j < VPT; ++j) {
+        const int q = tid + j * nthr;
+        if (q < nvec) {
+          float4 x = st[q], v = st[nvec + q];
+          const float4 pb = st[2 * nvec + q];
+          const float4 g = sG[q];
+          const float4 r1 = raw24x4(key, kTagR1, t, gi, (uint32_t)q);
+          const float4 r2 = raw24x4(key, kTagR2, t, gi, (uint32_t)q);
+          move1(mp, x.x, v.x, pb.x, g.x, r1.x, r2.x);
+          move1(mp, x.y, v.y, pb.y, g.y, r1.y, r2.y);
+          move1(mp, x.z, v.z, pb.z, g.z, r1.z, r2.z);
+          move1(mp, x.w, v.w, pb.w, g.w, r1.w, r2.w);
+          if ((d & 3) && q == nvec - 1) {
+            const int jj = 4 * q;
+            if (jj + 1 >= d) x.y = v.y = 0.f;
+            if (jj + 2 >= d) x.z = v.z = 0.f;
+            if (jj + 3 >= d) x.w = v.w = 0.f;
+          }
+          st[q] = x;
+          st[nvec + q] = v;
+          if constexpr (!Obj::kNeighbor) map4<Obj>(acc, x, 0.f, 4 * q, d);
+        }
+      }
+      if constexpr (Obj::kNeighbor) {
+        __syncthreads();
+#pragma unroll(VPT <= 2 ? VPT : 2)
+        for (int j = 0; j < VPT; ++j) {
+          const int q = tid + j * nthr;
+          if (q < nvec) map4<Obj>(acc, st[q], (q + 1 < nvec) ? st[q + 1].x : 0.f, 4 * q, d);
+        }
+      }
+      warp_combine<Obj>(acc);
+      if (lane == 0) {
+#pragma unroll
+        for (int j = 0; j < Obj::kAcc; ++j) red[warp * Obj::kAcc + j] = acc[j];
+      }
+      __syncthreads();
+      if (tid == 0) {
+        float c[Obj::kAcc];
+        Obj::init(c);
+        for (int w = 0; w < nwarps; ++w) {
+          float o[Obj::kAcc];
+#pragma unroll
+          for (int j = 0; j < Obj::kAcc; ++j) o[j] = red[w * Obj::kAcc + j];
+          Obj::combine(c, o);
+        }
+        const float f = Obj::finalize(c, d);
+        s_f = f;
+        s_imp = (f < spf[k]) ? 1 : 0;  // strict; NaN never improves
+        if (s_imp) {
+          spf[k] = f;
+          ++nimp;
+        }
+        if (f == f && ord_f32(f) < inc_ord) {
+          const unsigned long long kk = pack_key(f, gi);
+          if (kk < best) {
+            best = kk;
+            best_row = k;
+          }
+        }
+      }
+      __syncthreads();
+      if (s_imp) {
+        for (int q = tid; q < nvec; q += nthr) st[2 * nvec + q] = st[q];
+      }
+    }
+    // ---- publish the CTA's candidate, grid barrier, pull the winner into G
+    if (tid == 0) {
+      s_best = best;
+      s_best_row = best_row;
+    }
+    __syncthreads();
+    if (s_best_row >= 0) {
+      const float4* src = sRows + (size_t)s_best_row * 3 * nvec;  // x' == pb' (it improved)
+      float4* dst = reinterpret_cast<float4*>(a.cand) + ((size_t)par * grid + b) * nvec;
+      for (int q = tid; q < nvec; q += nthr) dst[q] = src[q];
+    }
+    __syncthreads();
+    if (tid == 0) {
+      if (s_best != ~0ull) atomicMin(&a.ctl->key_par[par], s_best);
+      __threadfence();
+      const unsigned gen = ld_acquire_u32(&a.ctl->bar_gen);
+      if (atomicAdd(&a.ctl->bar_count, 1u) == (unsigned)grid - 1) {
+        a.ctl->bar_count = 0;
+        // the other parity serves the next iteration: reset it to the new incumbent
+        const unsigned long long winner = *(volatile unsigned long long*)&a.ctl->key_par[par];
+        a.ctl->key_par[par ^ 1] = winner < cur ? winner : cur;
+        __threadfence();
+        atomicAdd(&a.ctl->bar_gen, 1u);
+      } else {
+        while (ld_acquire_u32(&a.ctl->bar_gen) == gen) {
+        }
+      }
+      __threadfence();
+      s_best = *(volatile unsigned long long*)&a.ctl->key_par[par];
+    }
+    __syncthreads();
+    const unsigned long long win = s_best;
+    if (win < cur) {
+      const long long wr = (long long)(uint32_t)win - a.row_begin;
+      const int owner = (int)(wr % grid);
+      const float4* src = reinterpret_cast<const float4*>(a.cand) + ((size_t)par * grid + owner) * nvec;
+      for (int q = tid; q < nvec; q += nthr) sG[q] = __ldcg(src + q);
+      cur = win;
+    }
+    __syncthreads();
+  }
+
+  // ---- write back
+  for (int k = 0; k < myrows; ++k) {
+    const long long r = b + (long long)k * grid;
+    float4* X4 = reinterpret_cast<float4*>(a.X) + r * nvec;
+    float4* V4 = reinterpret_cast<float4*>(a.V) + r * nvec;
+    float4* P4 = reinterpret_cast<float4*>(a.PB) + r * nvec;
+    const float4* st = sRows + (size_t)k * 3 * nvec;
+    for (int q = tid; q < nvec; q += nthr) {
+      X4[q] = st[q];
+      V4[q] = st[nvec + q];
+      P4[q] = st[2 * nvec + q];
+    }
+    if (tid == 0) a.pf[r] = spf[k];
+  }
+  if (tid == 0 && nimp) atomicAdd(&a.ctl->improvements, (unsigned long long)nimp);
+  if (b == 0) {
+    for (int q = tid; q < nvec; q += nthr) reinterpret_cast<float4*>(a.G)[q] = sG[q];
+    if (tid == 0) {
+      a.ctl->key_cur = cur;
+      a.ctl->key_acc = cur;
+      a.ctl->t = t0 + (uint32_t)iters;
+    }
+  }
+}
+
 // ------------------------------------------------------------ init kernel
 // Alg. 1 lines 1-3 (Sec 3.1): x0 = clamp(lo + span U, lo, hi), v0 = -vmax +
 // 2 vmax U from the X0 / V0 streams at t = 0; f = F(x0); pf = f (NaN -> +inf);
@@ -955,7 +1161,7 @@ __global__ void __launch_bounds__(kMaxThreads) k_eval(const float* X, long long 
 }
 
 // ---------------------------------------------------------- dispatch
-enum class Which { StepReg, StepTma, Init, Eval };
+enum class Which { StepReg, StepTma, Init, Eval, GridRes };
 
 template <class Obj>
 const void* pick(Which w, int vpt) {
@@ -970,6 +1176,7 @@ const void* pick(Which w, int vpt) {
     case Which::StepReg: PSO_VPT_CASES(k_step_reg)
     case Which::StepTma: PSO_VPT_CASES(k_step_tma)
     case Which::Init: PSO_VPT_CASES(k_init)
+    case Which::GridRes: PSO_VPT_CASES(k_gridres)
     default: PSO_VPT_CASES(k_eval)
   }
 #undef PSO_VPT_CASES
@@ -1133,6 +1340,35 @@ cudaError_t plan_launch(int objective, int d, long long n_local, int sm_count, c
   if (grid > n_local) grid = n_local;
   if (grid < 1) grid = 1;
   cfg->grid = (int)grid;
+
+  // ---- grid-resident path: the whole swarm in the grid's shared memory
+  cfg->gridres = 0;
+  if (h.allow_resident && !cfg->resident && cfg->tma && nvec >= 64) {
+    const void* fn = kernel_for(objective, Which::GridRes, cfg->vpt, &nb);
+    for (int per = 2; per >= 1 && !cfg->gridres; --per) {
+      long long g = (long long)per * sm_count;
+      if (g > n_local) g = n_local;
+      const long long rows = (n_local + g - 1) / g;
+      const size_t smem = row + (size_t)rows * 3 * row + (size_t)rows * 4;
+      if (smem > kSmemPerCtaMax - kStaticReserve || smem * per > kSmemPerSm - per * kStaticReserve)
+        continue;
+      if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) !=
+          cudaSuccess) {
+        cudaGetLastError();
+        continue;
+      }
+      int occ = 0;
+      if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, cfg->compute, smem) != cudaSuccess) {
+        cudaGetLastError();
+        continue;
+      }
+      if ((long long)occ * sm_count < g) continue;  // cooperative: every CTA co-resident
+      cfg->gridres = 1;
+      cfg->gridres_grid = (int)g;
+      cfg->gridres_rows = (int)rows;
+      cfg->gridres_smem = smem;
+    }
+  }
   return cudaSuccess;
 }
 
@@ -1151,6 +1387,16 @@ cudaError_t launch_resident(int objective, const SwarmArgs& a, const LaunchCfg& 
   if (!fn) return cudaErrorInvalidDeviceFunction;
   void* args[] = {const_cast<SwarmArgs*>(&a), &iters};
   return cudaLaunchKernel(fn, dim3(1), dim3(c.resident_threads), args, c.resident_smem, s);
+}
+
+cudaError_t launch_gridres(int objective, const SwarmArgs& a, const LaunchCfg& c, int iters,
+                           cudaStream_t s) {
+  bool nb = false;
+  const void* fn = kernel_for(objective, Which::GridRes, c.vpt, &nb);
+  if (!fn) return cudaErrorInvalidDeviceFunction;
+  void* args[] = {const_cast<SwarmArgs*>(&a), &iters};
+  return cudaLaunchCooperativeKernel(fn, dim3(c.gridres_grid), dim3(c.compute), args,
+                                     c.gridres_smem, s);
 }
 
 cudaError_t launch_init(int objective, const SwarmArgs& a, const LaunchCfg& c, cudaStream_t s) {

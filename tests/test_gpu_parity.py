@@ -359,3 +359,28 @@ def test_resident_path_bitwise_equals_streaming(obj, n, d, monkeypatch):
     info = a.info()
     assert info["launches"] == 3 and info["t"] == 50
     assert info["improvements"] > 0
+
+
+@pytest.mark.parametrize("obj,n,d", [(RASTRIGIN, 1024, 1000), (ROSENBROCK, 300, 1001),
+                                     (GRIEWANK, 70, 2000), (ACKLEY, 9, 4096), (SPHERE, 600, 256)])
+def test_grid_resident_bitwise_equals_streaming(obj, n, d, monkeypatch):
+    """Swarms that fit in the grid's shared memory run whole pso_step calls in
+    one cooperative launch; results are the streaming TMA kernel's bit for bit."""
+    a = gpu_swarm(n, d, obj, seed=41)
+    assert a.info()["resident"] == 2
+    monkeypatch.setenv("PSO_RESIDENT", "0")
+    b = gpu_swarm(n, d, obj, seed=41)
+    assert b.info()["resident"] == 0 and b.info()["tma_pipeline"] == 1
+    a.reset_counters()
+    for k in (1, 5, 14):
+        a.step(k)
+        b.step(k)
+        for x, y in zip(a.get_state()[:4], b.get_state()[:4]):
+            assert_bitwise(x, y, f"grid-resident vs streaming after +{k}")
+        fa, ia, Ga = a.gbest()
+        fb, ib, Gb = b.gbest()
+        assert (fa, ia) == (fb, ib)
+        assert_bitwise(Ga, Gb, "G")
+    info = a.info()
+    assert info["launches"] == 3 and info["t"] == 20
+    assert info["improvements"] > 0
