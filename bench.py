@@ -335,7 +335,8 @@ def run_gpu(args, w):
                                  "grid": info["grid"], "ctas_per_sm": info["ctas_per_sm"],
                                  "tma_pipeline": info["tma_pipeline"],
                                  "stages": info["pipeline_stages"],
-                                 "smem_bytes": info["smem_bytes"]}},
+                                 "smem_bytes": info["smem_bytes"],
+                                 "path": ["streaming", "cta-resident", "grid-resident"][info["resident"]]}},
             "clocks": clk.result, "e2e": e2e, "clocks_e2e": clk_e2e,
             "cpu_baseline": cpu, "gbest": {"fitness": gf, "index": gi},
         }

@@ -596,7 +596,12 @@ pso_status pso_get_info(pso_handle h, pso_info* info) {
   info->pipeline_stages = h->cfg.stages;
   info->smem_bytes = (int32_t)(h->cfg.resident ? h->cfg.resident_smem : h->cfg.smem);
   info->resident = h->cfg.resident ? 1 : (h->cfg.gridres ? 2 : 0);
+  if (h->cfg.resident) {
+    info->threads_per_cta = h->cfg.resident_threads;
+    info->grid = 1;
+  }
   if (h->cfg.gridres) {
+    info->threads_per_cta = h->cfg.compute;
     info->grid = h->cfg.gridres_grid;
     info->smem_bytes = (int32_t)h->cfg.gridres_smem;
   }

@@ -242,7 +242,8 @@ def test_step_splitting_and_determinism():
     assert not np.array_equal(a.get_state()[0], c.step(7).get_state()[0])
 
 
-def test_launch_counter_and_improvements():
+def test_launch_counter_and_improvements(monkeypatch):
+    monkeypatch.setenv("PSO_RESIDENT", "0")  # one streaming launch per iteration
     g = gpu_swarm(1000, 256, SPHERE, seed=3, timing=True)
     g.reset_counters()
     g.step(20)
