@@ -24,8 +24,21 @@ oracle: $(ORACLE)
 $(ORACLE): oracle/pso_oracle.cpp oracle/pso_oracle.h
 	$(CXX) -O3 -std=c++17 -ffp-contract=off -fno-fast-math -fPIC -shared -Wall -o $@ $<
 
-$(LIB): $(CU_SRCS) $(CPP_SRCS) $(HDRS)
-	$(NVCC) $(NVFLAGS) -shared -o $@ $(CU_SRCS) $(CPP_SRCS) -ldl 2> $(PKG)/build.log || (cat $(PKG)/build.log; exit 1)
+OBJDIR   := build/obj
+CU_OBJS  := $(patsubst $(CSRC)/%.cu,$(OBJDIR)/%.o,$(CU_SRCS))
+CPP_OBJS := $(patsubst $(CSRC)/%.cpp,$(OBJDIR)/%.o,$(CPP_SRCS))
+
+$(OBJDIR)/%.o: $(CSRC)/%.cu $(HDRS)
+	@mkdir -p $(OBJDIR)
+	$(NVCC) $(NVFLAGS) -c -o $@ $< 2> $@.log || (cat $@.log; exit 1)
+
+$(OBJDIR)/%.o: $(CSRC)/%.cpp $(HDRS)
+	@mkdir -p $(OBJDIR)
+	$(NVCC) $(NVFLAGS) -c -o $@ $< 2> $@.log || (cat $@.log; exit 1)
+
+$(LIB): $(CU_OBJS) $(CPP_OBJS)
+	$(NVCC) $(ARCH) -shared -o $@ $^ -ldl
+	cat $(OBJDIR)/*.log > $(PKG)/build.log
 
 clean:
-	rm -f $(LIB) $(ORACLE) $(PKG)/build.log
+	rm -rf $(LIB) $(ORACLE) $(PKG)/build.log $(OBJDIR)

@@ -103,6 +103,11 @@ typedef struct {
   void* stream;    /* cudaStream_t to enqueue on; NULL -> a library-owned stream */
   void* nccl_comm; /* ncclComm_t (see pso_nccl_comm_init); NULL -> single GPU */
   uint32_t flags;  /* PSO_FLAG_* */
+  const float* bounds; /* NULL, or 4*d host floats [vlo | vhi | xlo | xhi]: per-dimension
+                          velocity bounds (Eq. 5: lower/upper_bound_j) and
+                          domain (x clamp); replaces vmax / lo / hi (which must still be
+                          valid).  Init draws x0 ~ U[xlo_j, xhi_j], v0 ~ U[vlo_j, vhi_j].
+                          Needs finite values, vlo_j <= vhi_j, xlo_j < xhi_j. */
 } pso_opts;
 
 /* Create a swarm of n particles in d dimensions and initialise it (Alg. 1
@@ -150,6 +155,11 @@ pso_status pso_get_state(pso_handle h, float* x, float* v, float* pb, float* pf,
 pso_status pso_set_state(pso_handle h, const float* x, const float* v, const float* pb,
                          const float* pf, uint64_t t);
 
+/* Replace the per-dimension bounds (same layout as pso_opts.bounds) of a
+ * handle created with bounds; applies to the following iterations.
+ * PSO_ERR_UNSUPPORTED for a handle created with scalar bounds.  Synchronous. */
+pso_status pso_set_bounds(pso_handle h, const float* bounds);
+
 /* Information and counters. */
 typedef struct {
   int64_t n, n_local, row_begin; /* global size, local rows, first global row */
@@ -164,6 +174,7 @@ typedef struct {
                                     2: swarm held in the whole grid's shared memory
                                     (cooperative launch); 1 and 2 run a whole
                                     pso_step call in one launch (single GPU only) */
+  int32_t bounds;                /* 1: per-dimension bounds in use */
   float vmax;
   uint64_t t;                    /* iterations done */
   uint64_t launches;             /* kernels launched by this handle so far */

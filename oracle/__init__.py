@@ -29,7 +29,7 @@ class _Params(C.Structure):
         ("n", C.c_int64), ("d", C.c_int32), ("objective", C.c_int32),
         ("w", C.c_float), ("c1", C.c_float), ("c2", C.c_float),
         ("lo", C.c_float), ("hi", C.c_float), ("vmax", C.c_float),
-        ("seed", C.c_uint64),
+        ("seed", C.c_uint64), ("bounds", C.c_void_p),
     ]
 
 
@@ -141,13 +141,18 @@ class OracleSwarm:
     """
 
     def __init__(self, n, d, w, c1, c2, lo, hi, objective, seed, vmax=0.0,
-                 nshards=1, row_begin=0, nrows=None, create=True):
+                 nshards=1, row_begin=0, nrows=None, create=True, bounds=None):
         self.p = _Params()
         self.p.n, self.p.d, self.p.objective = int(n), int(d), int(objective)
         self.p.w, self.p.c1, self.p.c2 = w, c1, c2
         self.p.lo, self.p.hi = lo, hi
         self.p.vmax = vmax if vmax > 0 else default_vmax(lo, hi)
         self.p.seed = int(seed) & 0xFFFFFFFFFFFFFFFF
+        # per-dimension [vlo | vhi | xlo | xhi] (NEXT-2); kept alive with the swarm
+        self.bounds = None
+        if bounds is not None:
+            self.bounds = np.ascontiguousarray(bounds, dtype=np.float32).reshape(4 * int(d))
+            self.p.bounds = self.bounds.ctypes.data
         self.n, self.d, self.nshards = int(n), int(d), int(nshards)
         nrows = self.n - row_begin if nrows is None else int(nrows)
         self.row_begin, self.nrows = int(row_begin), nrows

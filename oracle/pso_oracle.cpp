@@ -126,14 +126,26 @@ double objective(int32_t obj, const float* x, int32_t d) {
 // Eq. 2 and the domain clamp (reading 2).  Fixed fp32 order:
 //   a = w*v; b = (c1*r1)*(pb-x); c = (c2*r2)*(g-x); v' = (a+b)+c
 // ---------------------------------------------------------------------------
-inline void move_element(const orc_params* p, float r1, float r2, float pb, float g,
-                         float* x, float* v) {
+// Bounds of dimension j: Eq. 5's lower/upper velocity bound and the domain.
+struct Bounds {
+  float vlo, vhi, xlo, xhi;
+};
+inline Bounds bounds_of(const orc_params* p, int32_t j) {
+  if (p->bounds) {
+    const int32_t d = p->d;
+    return Bounds{p->bounds[j], p->bounds[d + j], p->bounds[2 * d + j], p->bounds[3 * d + j]};
+  }
+  return Bounds{-p->vmax, p->vmax, p->lo, p->hi};
+}
+
+inline void move_element(const orc_params* p, const Bounds& bd, float r1, float r2, float pb,
+                         float g, float* x, float* v) {
   float a = p->w * *v;
   float b = (p->c1 * r1) * (pb - *x);
   float c = (p->c2 * r2) * (g - *x);
   float vn = (a + b) + c;
-  vn = std::fmin(std::fmax(vn, -p->vmax), p->vmax);   // Eq. 5
-  float xn = std::fmin(std::fmax(*x + vn, p->lo), p->hi);  // Eq. 2 + clamp
+  vn = std::fmin(std::fmax(vn, bd.vlo), bd.vhi);            // Eq. 5
+  float xn = std::fmin(std::fmax(*x + vn, bd.xlo), bd.xhi);  // Eq. 2 + clamp
   *v = vn;
   *x = xn;
 }
@@ -146,7 +158,7 @@ void row_step(const orc_params* p, uint32_t t, const float* G, uint32_t gi,
   for (int32_t j = 0; j < d; ++j) {
     float r1 = uniform(word(p->seed, ORC_TAG_R1, t, gi, (uint32_t)j));
     float r2 = uniform(word(p->seed, ORC_TAG_R2, t, gi, (uint32_t)j));
-    move_element(p, r1, r2, pb[j], G[j], &x[j], &v[j]);
+    move_element(p, bounds_of(p, j), r1, r2, pb[j], G[j], &x[j], &v[j]);
   }
   float fi = (float)objective(p->objective, x, d);
   *f = fi;
@@ -217,8 +229,6 @@ float orc_default_vmax(float lo, float hi) {
 void orc_init_local(const orc_params* p, orc_state* s, float* cand_f, int64_t* cand_i,
                     float* cand_row) {
   const int32_t d = p->d;
-  const float span = p->hi - p->lo;
-  const float two_vmax = 2.0f * p->vmax;
   bool have = false;
   float bf = 0.0f;
   int64_t bi = 0;
@@ -227,10 +237,11 @@ void orc_init_local(const orc_params* p, orc_state* s, float* cand_f, int64_t* c
     float* x = s->X + r * d;
     float* v = s->V + r * d;
     for (int32_t j = 0; j < d; ++j) {  // Alg. 1 line 2, reading 4
+      const Bounds bd = bounds_of(p, j);
       float ux = uniform(word(p->seed, ORC_TAG_X0, 0, (uint32_t)gi, (uint32_t)j));
       float uv = uniform(word(p->seed, ORC_TAG_V0, 0, (uint32_t)gi, (uint32_t)j));
-      x[j] = std::fmin(std::fmax(p->lo + span * ux, p->lo), p->hi);
-      v[j] = (-p->vmax) + two_vmax * uv;
+      x[j] = std::fmin(std::fmax(bd.xlo + (bd.xhi - bd.xlo) * ux, bd.xlo), bd.xhi);
+      v[j] = bd.vlo + (bd.vhi - bd.vlo) * uv;
     }
     float fi = (float)objective(p->objective, x, d);
     s->f[r] = fi;

@@ -55,6 +55,8 @@ typedef struct {
   float lo, hi;       /* domain */
   float vmax;         /* velocity bound (Eq. 5), symmetric |v| <= vmax; reading 3 */
   uint64_t seed;      /* Philox key */
+  const float* bounds; /* NULL, or 4*d floats [vlo | vhi | xlo | xhi] per dimension
+                          (Eq. 5 per-dimension reading, NEXT-2); replaces vmax/lo/hi */
 } orc_params;
 
 /* Caller-owned state of one shard: global rows [row_begin, row_begin+nrows).

@@ -49,7 +49,7 @@ class Swarm:
 
     def __init__(self, n: int, d: int, w: float, c1: float, c2: float, lo: float, hi: float,
                  objective: int, seed: int, *, vmax: float = 0.0, device: int = -1,
-                 stream=None, nccl_comm=None, timing: bool = False):
+                 stream=None, nccl_comm=None, timing: bool = False, bounds=None):
         L = lib()
         opts = pso_opts()
         opts.vmax = float(vmax)
@@ -58,6 +58,9 @@ class Swarm:
             opts.stream = int(getattr(stream, "cuda_stream", stream))
         opts.nccl_comm = nccl_comm
         opts.flags = PSO_FLAG_TIMING if timing else 0
+        if bounds is not None:  # per-dimension [vlo | vhi | xlo | xhi], 4 x d
+            bounds = np.ascontiguousarray(bounds, dtype=np.float32).reshape(4 * int(d))
+            opts.bounds = bounds.ctypes.data
         self._h = C.c_void_p()
         check(L.pso_create_ex(C.byref(self._h), int(n), int(d), float(w), float(c1), float(c2),
                               float(lo), float(hi), int(objective), int(seed) & (2**64 - 1),
@@ -133,6 +136,11 @@ class Swarm:
                 raise ValueError(f"state shape {tuple(a.shape)} != {shape}")
         check(lib().pso_set_state(self._h, _ptr(X), _ptr(V), _ptr(PB), _ptr(pf), int(t)),
               "pso_set_state")
+        return self
+
+    def set_bounds(self, bounds) -> "Swarm":
+        b = np.ascontiguousarray(bounds, dtype=np.float32).reshape(4 * self.d)
+        check(lib().pso_set_bounds(self._h, C.c_void_p(b.ctypes.data)), "pso_set_bounds")
         return self
 
     def info(self) -> dict:

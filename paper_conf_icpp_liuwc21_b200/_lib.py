@@ -22,7 +22,7 @@ PSO_D_MAX = 8192
 # every symbol include/fastpso.h declares
 EXPORTS = (
     "pso_create", "pso_create_ex", "pso_step", "pso_synchronize", "pso_get_gbest",
-    "pso_get_state", "pso_set_state", "pso_get_info", "pso_reset_counters", "pso_destroy",
+    "pso_get_state", "pso_set_state", "pso_set_bounds", "pso_get_info", "pso_reset_counters", "pso_destroy",
     "pso_status_string", "pso_last_error", "pso_objective_registered",
     "pso_nccl_get_unique_id", "pso_nccl_comm_init", "pso_nccl_comm_destroy",
     "pso_debug_philox", "pso_debug_objective",
@@ -31,7 +31,7 @@ EXPORTS = (
 
 class pso_opts(C.Structure):
     _fields_ = [("vmax", C.c_float), ("device", C.c_int32), ("stream", C.c_void_p),
-                ("nccl_comm", C.c_void_p), ("flags", C.c_uint32)]
+                ("nccl_comm", C.c_void_p), ("flags", C.c_uint32), ("bounds", C.c_void_p)]
 
 
 class pso_info(C.Structure):
@@ -40,7 +40,8 @@ class pso_info(C.Structure):
         ("d", C.c_int32), ("pitch", C.c_int32), ("rank", C.c_int32), ("world", C.c_int32),
         ("threads_per_cta", C.c_int32), ("vec_per_thread", C.c_int32), ("grid", C.c_int32),
         ("ctas_per_sm", C.c_int32), ("tma_pipeline", C.c_int32), ("pipeline_stages", C.c_int32),
-        ("smem_bytes", C.c_int32), ("resident", C.c_int32), ("vmax", C.c_float), ("t", C.c_uint64),
+        ("smem_bytes", C.c_int32), ("resident", C.c_int32), ("bounds", C.c_int32),
+        ("vmax", C.c_float), ("t", C.c_uint64),
         ("launches", C.c_uint64), ("improvements", C.c_uint64),
         ("step_kernel_ms", C.c_double), ("step_kernel_count", C.c_uint64),
         ("arena_bytes", C.c_size_t),
@@ -80,6 +81,7 @@ def lib() -> C.CDLL:
     L.pso_get_state.argtypes = [H, C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p, u64p]
     L.pso_set_state.argtypes = [H, C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p, C.c_uint64]
     L.pso_get_info.argtypes = [H, C.POINTER(pso_info)]
+    L.pso_set_bounds.argtypes = [H, C.c_void_p]
     L.pso_reset_counters.argtypes = [H]
     L.pso_destroy.argtypes = [H]
     L.pso_destroy.restype = None

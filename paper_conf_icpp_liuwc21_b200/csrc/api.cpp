@@ -247,6 +247,30 @@ pso_status next_event(pso_swarm* h, pso_swarm::Timed** out, uint64_t steps) {
   return PSO_OK;
 }
 
+// Per-dimension bounds [vlo | vhi | xlo | xhi] (4 x d host floats): finite,
+// vlo_j <= vhi_j, xlo_j < xhi_j.
+pso_status check_bounds(const float* b, int32_t d) {
+  for (int32_t j = 0; j < d; ++j) {
+    const float vlo = b[j], vhi = b[d + j], xlo = b[2 * d + j], xhi = b[3 * d + j];
+    if (!std::isfinite(vlo) || !std::isfinite(vhi) || !std::isfinite(xlo) || !std::isfinite(xhi))
+      return fail(PSO_ERR_INVALID, "bounds of dim %d are not finite", j);
+    if (!(vlo <= vhi)) return fail(PSO_ERR_INVALID, "vlo > vhi at dim %d", j);
+    if (!(xlo < xhi)) return fail(PSO_ERR_INVALID, "xlo >= xhi at dim %d", j);
+  }
+  return PSO_OK;
+}
+
+// Copy host bounds (dense d) into the pitched device table (padding 0).
+pso_status upload_bounds(pso_swarm* h, const float* b) {
+  std::vector<float> tab((size_t)4 * h->pitch, 0.f);
+  for (int k = 0; k < 4; ++k)
+    std::memcpy(&tab[(size_t)k * h->pitch], b + (size_t)k * h->d, sizeof(float) * (size_t)h->d);
+  PSO_CUDA(h, cudaMemcpyAsync(const_cast<float*>(h->args.bounds), tab.data(), tab.size() * 4,
+                              cudaMemcpyHostToDevice, h->stream));
+  PSO_CUDA(h, cudaStreamSynchronize(h->stream));
+  return PSO_OK;
+}
+
 float decode_fitness(unsigned long long key) {
   uint32_t o = (uint32_t)(key >> 32);
   uint32_t u = (o & 0x80000000u) ? (o & 0x7FFFFFFFu) : ~o;
@@ -308,6 +332,10 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
   if (!objective_registered(objective))
     return fail(PSO_ERR_INVALID, "objective %d is not registered", objective);
   if (o.flags & ~(uint32_t)PSO_FLAG_TIMING) return fail(PSO_ERR_INVALID, "unknown flags 0x%x", o.flags);
+  if (o.bounds) {
+    pso_status bs = check_bounds(o.bounds, d);
+    if (bs != PSO_OK) return bs;
+  }
 
   pso_swarm* h = new (std::nothrow) pso_swarm();
   if (!h) return fail(PSO_ERR_NOMEM, "host allocation failed");
@@ -384,6 +412,7 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
   {
     const char* v = std::getenv("PSO_RESIDENT");
     hints.allow_resident = !h->xchg && hints.kernel == -1 && !(v && !std::strcmp(v, "0"));
+    hints.bounds = o.bounds != nullptr;
   }
   {
     cudaError_t e = plan_launch(objective, d, h->n_local > 0 ? h->n_local : 1, h->sm_count,
@@ -397,11 +426,12 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
   const size_t pfb = align_up(rows * 4, 256);
   const size_t gb = align_up((size_t)h->pitch * 4, 256);
   const size_t ctlb = align_up(sizeof(DevCtl), 256);
+  const size_t boundb = o.bounds ? align_up(4 * (size_t)h->pitch * 4, 256) : 0;
   const size_t rec = align_up(record_bytes(h->pitch), 256);
   const size_t candb = h->cfg.gridres ? align_up(2 * (size_t)h->cfg.gridres_grid * h->pitch * 4, 256) : 0;
   const size_t sendb = h->xchg ? rec : 0;
   const size_t recvb = h->xchg ? (size_t)h->world * record_bytes(h->pitch) : 0;
-  h->arena_bytes = 3 * mat + pfb + gb + ctlb + candb + sendb + align_up(recvb, 256);
+  h->arena_bytes = 3 * mat + pfb + gb + ctlb + boundb + candb + sendb + align_up(recvb, 256);
   {
     cudaError_t e = cudaMalloc(&h->arena, h->arena_bytes);
     if (e == cudaErrorMemoryAllocation) {
@@ -418,6 +448,7 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
   A.pf = (float*)p; p += pfb;
   A.G = (float*)p; p += gb;
   A.ctl = (DevCtl*)p; p += ctlb;
+  A.bounds = o.bounds ? (const float*)p : nullptr; p += boundb;
   A.cand = h->cfg.gridres ? (float*)p : nullptr; p += candb;
   A.send = h->xchg ? p : nullptr; p += sendb;
   A.recv = h->xchg ? p : nullptr;
@@ -441,6 +472,7 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
   }
   pso_status st = reset_ctl(h, 0);
   if (st != PSO_OK) return bail(st);
+  if (o.bounds && (st = upload_bounds(h, o.bounds)) != PSO_OK) return bail(st);
 
   // ---- Alg. 1 lines 1-3 + first evaluation and best update
   if (h->n_local > 0) {
@@ -570,6 +602,18 @@ pso_status pso_set_state(pso_handle h, const float* x, const float* v, const flo
   return PSO_OK;
 }
 
+pso_status pso_set_bounds(pso_handle h, const float* bounds) {
+  pso_status st = check_handle(h);
+  if (st != PSO_OK) return st;
+  if (!bounds) return fail(PSO_ERR_INVALID, "bounds is NULL");
+  if (!h->args.bounds)
+    return fail(PSO_ERR_UNSUPPORTED, "handle was created without per-dimension bounds");
+  if ((st = check_bounds(bounds, h->d)) != PSO_OK) return st;
+  if ((st = use_device(h)) != PSO_OK) return st;
+  if ((st = sync_and_check(h)) != PSO_OK) return st;
+  return upload_bounds(h, bounds);
+}
+
 pso_status pso_get_info(pso_handle h, pso_info* info) {
   if (!h) return fail(PSO_ERR_INVALID, "NULL handle");
   if (!info) return fail(PSO_ERR_INVALID, "info is NULL");
@@ -596,6 +640,7 @@ pso_status pso_get_info(pso_handle h, pso_info* info) {
   info->pipeline_stages = h->cfg.stages;
   info->smem_bytes = (int32_t)(h->cfg.resident ? h->cfg.resident_smem : h->cfg.smem);
   info->resident = h->cfg.resident ? 1 : (h->cfg.gridres ? 2 : 0);
+  info->bounds = h->args.bounds ? 1 : 0;
   if (h->cfg.resident) {
     info->threads_per_cta = h->cfg.resident_threads;
     info->grid = 1;

@@ -32,6 +32,7 @@ struct SwarmArgs {
   float* pf;  // n_local
   float* G;   // pitch (gbest position)
   float* cand;                // grid-resident kernel: [2][grid][pitch] candidate rows
+  const float* bounds;        // per-dimension bounds [vlo | vhi | xlo | xhi] (4 x pitch), or null
   unsigned char* send;        // world > 1: this rank's exchange record
   const unsigned char* recv;  // world > 1: world records after the all-gather
   DevCtl* ctl;
@@ -61,6 +62,7 @@ struct LaunchCfg {
   int resident_threads = 0;
   size_t resident_smem = 0;
   size_t init_smem = 0;
+  int bounds = 0;     // kernels instantiated with per-dimension bounds
 };
 
 // Tuning overrides (0 / -1 = automatic): PSO_VPT, PSO_KERNEL=reg|tma, PSO_STAGES, PSO_CTAS.
@@ -70,7 +72,21 @@ struct PlanHints {
   int stages = 0;
   int ctas = 0;     // max CTAs per SM for the TMA pipeline (0: auto = 2)
   bool allow_resident = false;  // single-GPU tiny swarms (PSO_RESIDENT=0 disables)
+  bool bounds = false;          // per-dimension bounds tables are in use
 };
+
+// Kernel entry points of one objective functor: [VPT index 1,2,4,8][per-dim bounds].
+struct KernelTable {
+  bool neighbor;
+  const void* step_reg[4][2];
+  const void* step_tma[4][2];
+  const void* gridres[4][2];
+  const void* resident[2];
+  const void* init[4];
+  const void* eval[4];
+};
+// The table of a registered objective id, or null (obj_*.cu).
+const KernelTable* kernel_table(int objective);
 
 bool objective_registered(int objective);
 // Choose the CTA shape for d and size the persistent grid for n_local rows.

@@ -1,0 +1,347 @@
+// swarm_host.cu — launch planning and dispatch of the fused kernels, and the
+// objective-independent kernels (gbest rebest after set_state, multi-GPU select).
+#include "swarm_kernels.cuh"
+
+namespace fastpso {
+namespace {
+
+// ---------------------------------------------------------- rebest kernel
+// After set_state: pf NaN -> +inf, gbest = lowest index attaining min pf.
+struct NoObj {
+  static constexpr int kAcc = 1;
+};
+__global__ void __launch_bounds__(256) k_rebest(const SwarmArgs a, unsigned t) {
+  __shared__ unsigned long long s_best[8];
+  __shared__ RowSmem<NoObj> sm;
+  const int tid = threadIdx.x, nthr = blockDim.x;
+  unsigned long long best = ~0ull;
+  for (long long r = blockIdx.x * (long long)blockDim.x + threadIdx.x; r < a.n_local;
+       r += (long long)gridDim.x * blockDim.x) {
+    float f = a.pf[r];
+    if (f != f) {
+      f = __int_as_float(0x7f800000);
+      a.pf[r] = f;
+    }
+    const unsigned long long k = pack_key(f, (uint32_t)(a.row_begin + r));
+    best = k < best ? k : best;
+  }
+#pragma unroll
+  for (int off = 16; off > 0; off >>= 1) {
+    const unsigned long long o = __shfl_xor_sync(kFull, best, off);
+    best = o < best ? o : best;
+  }
+  if ((tid & 31) == 0) s_best[tid >> 5] = best;
+  __syncthreads();
+  if (tid == 0)
+    for (int w = 1; w < (nthr >> 5); ++w) best = s_best[w] < best ? s_best[w] : best;
+  if (cta_finish<NoObj>(a, sm, tid == 0 ? best : ~0ull, 0, tid, nthr))
+    gbest_epilogue<NoObj>(a, sm, t, tid, nthr);
+}
+
+// ---------------------------------------------------------- select kernel
+// world > 1, after ncclAllGather of the records: the global candidate is the
+// minimum key over ranks (keys carry global indices, so ties resolve to the
+// lowest global index, as one GPU would).  Every rank computes the same bits.
+__global__ void __launch_bounds__(128) k_select(const SwarmArgs a) {
+  __shared__ unsigned long long s_min;
+  __shared__ int s_src;
+  const size_t rec = record_bytes(a.nvec * 4);
+  if (threadIdx.x < 32) {
+    unsigned long long best = ~0ull;
+    int src = -1;
+    for (int r = threadIdx.x; r < a.world; r += 32) {
+      const unsigned long long k =
+          *reinterpret_cast<const unsigned long long*>(a.recv + (size_t)r * rec);
+      if (k < best) {
+        best = k;
+        src = r;
+      }
+    }
+#pragma unroll
+    for (int off = 16; off > 0; off >>= 1) {
+      const unsigned long long o = __shfl_xor_sync(kFull, best, off);
+      const int os = __shfl_xor_sync(kFull, src, off);
+      if (o < best || (o == best && os >= 0 && (src < 0 || os < src))) {
+        best = o;
+        src = os;
+      }
+    }
+    if (threadIdx.x == 0) {
+      s_min = best;
+      s_src = src;
+    }
+  }
+  __syncthreads();
+  const unsigned long long cur = a.ctl->key_cur;
+  const bool take = s_src >= 0 && s_min < cur;
+  if (take) {
+    const float4* row = reinterpret_cast<const float4*>(a.recv + (size_t)s_src * rec + 16);
+    float4* G4 = reinterpret_cast<float4*>(a.G);
+    for (int q = threadIdx.x; q < a.nvec; q += blockDim.x) G4[q] = row[q];
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    if (take) a.ctl->key_cur = s_min;
+    a.ctl->key_acc = take ? s_min : cur;
+  }
+}
+
+// ---------------------------------------------------------- dispatch
+enum class Which { StepReg, StepTma, Init, Eval, GridRes };
+
+int vpt_index(int vpt) { return vpt == 1 ? 0 : vpt == 2 ? 1 : vpt == 4 ? 2 : 3; }
+
+const void* kernel_for(int objective, Which w, int vpt, bool bounds, bool* neighbor) {
+  const KernelTable* t = kernel_table(objective);
+  if (!t) return nullptr;
+  *neighbor = t->neighbor;
+  const int i = vpt_index(vpt), b = bounds ? 1 : 0;
+  switch (w) {
+    case Which::StepReg: return t->step_reg[i][b];
+    case Which::StepTma: return t->step_tma[i][b];
+    case Which::GridRes: return t->gridres[i][b];
+    case Which::Init: return t->init[i];
+    default: return t->eval[i];
+  }
+}
+
+const void* resident_kernel_for(int objective, bool bounds) {
+  const KernelTable* t = kernel_table(objective);
+  return t ? t->resident[bounds ? 1 : 0] : nullptr;
+}
+
+// CTA shape for a row of nvec float4: the smallest VPT in {1,2,4,8} whose
+// thread count fits 256, threads rounded up to a warp multiple.
+void shape_for(int nvec, int vpt_override, int* vpt, int* threads) {
+  static const int kVpts[] = {1, 2, 4, 8};
+  int v = 8;
+  for (int c : kVpts) {
+    if ((nvec + c - 1) / c <= kMaxThreads) {
+      v = c;
+      break;
+    }
+  }
+  if (vpt_override == 1 || vpt_override == 2 || vpt_override == 4 || vpt_override == 8) {
+    if ((nvec + vpt_override - 1) / vpt_override <= kMaxThreads) v = vpt_override;
+  }
+  const int t = (nvec + v - 1) / v;
+  *vpt = v;
+  *threads = ((t + 31) / 32) * 32;
+}
+
+constexpr size_t kSmemPerSm = 228 * 1024;       // B200 unified L1/shared per SM
+constexpr size_t kSmemPerCtaMax = 227 * 1024;   // opt-in maximum per CTA
+constexpr size_t kStaticReserve = 2048;         // static shared + per-CTA reservation
+constexpr long long kResidentElems = 8192;      // resident path: n d <= this
+
+}  // namespace
+
+bool objective_registered(int objective) {
+  bool nb;
+  return kernel_for(objective, Which::Init, 1, false, &nb) != nullptr;
+}
+
+cudaError_t plan_launch(int objective, int d, long long n_local, int sm_count, const PlanHints& h,
+                        LaunchCfg* cfg) {
+  const int nvec = (d + 3) / 4;
+  shape_for(nvec, h.vpt, &cfg->vpt, &cfg->compute);
+  bool nb = false;
+  if (!kernel_for(objective, Which::Init, cfg->vpt, false, &nb)) return cudaErrorInvalidDeviceFunction;
+  const size_t row = (size_t)nvec * 16;
+  const size_t btab = h.bounds ? 4 * row : 0;  // per-dimension bounds table in shared memory
+  cfg->bounds = h.bounds ? 1 : 0;
+  const size_t first = nb ? (size_t)nvec * 4 : 0;
+  cfg->init_smem = first;
+  cudaError_t e;
+
+  // ---- resident single-CTA path for tiny swarms (single GPU only)
+  cfg->resident = 0;
+  if (h.allow_resident && nvec <= 32 && n_local * nvec * 4 <= kResidentElems) {
+    const size_t smem =
+        (size_t)n_local * nvec * 16 * 3 + (size_t)nvec * 16 + btab + (size_t)n_local * 4;
+    const void* fn = resident_kernel_for(objective, h.bounds);
+    if (smem <= kSmemPerCtaMax - kStaticReserve &&
+        cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) ==
+            cudaSuccess) {
+      int gs = 1;
+      while (gs < nvec) gs <<= 1;
+      const long long rpw = 32 / gs;
+      long long warps = (n_local + rpw - 1) / rpw;
+      if (warps > 32) warps = 32;
+      cfg->resident = 1;
+      cfg->resident_threads = 32 * (int)(warps < 1 ? 1 : warps);
+      cfg->resident_smem = smem;
+    }
+    cudaGetLastError();
+  }
+
+  // ---- TMA pipeline: rows of >= 256 dims unless forced otherwise
+  bool tma = h.kernel == 1 || (h.kernel == -1 && nvec >= 64);
+  if (tma) {
+    const void* fn = kernel_for(objective, Which::StepTma, cfg->vpt, h.bounds, &nb);
+    const int threads = cfg->compute + 64;  // + producer warp + finaliser warp
+    // CTAs per SM the registers allow, capped at 2; the ring fills the rest.
+    int by_regs = 0;
+    if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&by_regs, fn, threads, 0)) != cudaSuccess)
+      return e;
+    const int cap = (h.ctas >= 1 && h.ctas <= 8) ? h.ctas : 2;
+    int ctas = by_regs < 1 ? 1 : (by_regs > cap ? cap : by_regs);
+    // The most CTAs per SM (<= cap) that still keep >= 3 rows in flight per
+    // CTA; two rows only if nothing else fits (measured: 2-stage rings leave
+    // HBM idle between rows, 3-4 stages saturate it).
+    auto stages_for = [&](int c) -> int {
+      size_t budget = kSmemPerSm / c - kStaticReserve;
+      if (budget > kSmemPerCtaMax - kStaticReserve) budget = kSmemPerCtaMax - kStaticReserve;
+      return budget > row + btab ? (int)((budget - row - btab) / (3 * row)) : 0;
+    };
+    int stages = 0;
+    int c = ctas;
+    for (; c >= 1; --c)
+      if (stages_for(c) >= 3) break;
+    if (c >= 1) {
+      ctas = c;
+    } else {
+      for (c = ctas; c >= 1 && stages_for(c) < 2; --c) {
+      }
+      ctas = c < 1 ? 1 : c;
+    }
+    stages = stages_for(ctas);
+    if (h.stages >= 2 && h.stages <= kMaxStages) stages = stages < h.stages ? stages : h.stages;
+    if (stages > kMaxStages) stages = kMaxStages;
+    if (stages >= 2) {
+      const size_t smem = row + btab + (size_t)stages * 3 * row;
+      if ((e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem)) !=
+          cudaSuccess)
+        return e;
+      int per_sm = 0;
+      if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, threads, smem)) !=
+          cudaSuccess)
+        return e;
+      if (per_sm >= 1) {
+        cfg->tma = 1;
+        cfg->stages = stages;
+        cfg->threads = threads;
+        cfg->smem = smem;
+        cfg->ctas_per_sm = per_sm;
+      } else {
+        tma = false;
+      }
+    } else {
+      tma = false;
+    }
+  }
+  if (!tma) {
+    const void* fn = kernel_for(objective, Which::StepReg, cfg->vpt, h.bounds, &nb);
+    cfg->tma = 0;
+    cfg->stages = 0;
+    cfg->threads = cfg->compute;
+    cfg->smem = row + first;
+    int per_sm = 0;
+    if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, cfg->threads, cfg->smem)) !=
+        cudaSuccess)
+      return e;
+    cfg->ctas_per_sm = per_sm < 1 ? 1 : per_sm;
+  }
+  long long grid = (long long)cfg->ctas_per_sm * sm_count;
+  if (grid > n_local) grid = n_local;
+  if (grid < 1) grid = 1;
+  cfg->grid = (int)grid;
+
+  // ---- grid-resident path: the whole swarm in the grid's shared memory
+  cfg->gridres = 0;
+  if (h.allow_resident && !cfg->resident && cfg->tma && nvec >= 64) {
+    const void* fn = kernel_for(objective, Which::GridRes, cfg->vpt, h.bounds, &nb);
+    for (int per = 2; per >= 1 && !cfg->gridres; --per) {
+      long long g = (long long)per * sm_count;
+      if (g > n_local) g = n_local;
+      const long long rows = (n_local + g - 1) / g;
+      const size_t smem = row + btab + (size_t)rows * 3 * row + (size_t)rows * 4;
+      if (smem > kSmemPerCtaMax - kStaticReserve || smem * per > kSmemPerSm - per * kStaticReserve)
+        continue;
+      if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) !=
+          cudaSuccess) {
+        cudaGetLastError();
+        continue;
+      }
+      int occ = 0;
+      if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, cfg->compute, smem) != cudaSuccess) {
+        cudaGetLastError();
+        continue;
+      }
+      if ((long long)occ * sm_count < g) continue;  // cooperative: every CTA co-resident
+      cfg->gridres = 1;
+      cfg->gridres_grid = (int)g;
+      cfg->gridres_rows = (int)rows;
+      cfg->gridres_smem = smem;
+    }
+  }
+  return cudaSuccess;
+}
+
+cudaError_t launch_step(int objective, const SwarmArgs& a, const LaunchCfg& c, cudaStream_t s) {
+  bool nb = false;
+  const void* fn = kernel_for(objective, c.tma ? Which::StepTma : Which::StepReg, c.vpt, c.bounds != 0, &nb);
+  if (!fn) return cudaErrorInvalidDeviceFunction;
+  int stages = c.stages;
+  void* args[] = {const_cast<SwarmArgs*>(&a), &stages};
+  return cudaLaunchKernel(fn, dim3(c.grid), dim3(c.threads), args, c.smem, s);
+}
+
+cudaError_t launch_resident(int objective, const SwarmArgs& a, const LaunchCfg& c, int iters,
+                            cudaStream_t s) {
+  const void* fn = resident_kernel_for(objective, c.bounds != 0);
+  if (!fn) return cudaErrorInvalidDeviceFunction;
+  void* args[] = {const_cast<SwarmArgs*>(&a), &iters};
+  return cudaLaunchKernel(fn, dim3(1), dim3(c.resident_threads), args, c.resident_smem, s);
+}
+
+cudaError_t launch_gridres(int objective, const SwarmArgs& a, const LaunchCfg& c, int iters,
+                           cudaStream_t s) {
+  bool nb = false;
+  const void* fn = kernel_for(objective, Which::GridRes, c.vpt, c.bounds != 0, &nb);
+  if (!fn) return cudaErrorInvalidDeviceFunction;
+  void* args[] = {const_cast<SwarmArgs*>(&a), &iters};
+  return cudaLaunchCooperativeKernel(fn, dim3(c.gridres_grid), dim3(c.compute), args,
+                                     c.gridres_smem, s);
+}
+
+cudaError_t launch_init(int objective, const SwarmArgs& a, const LaunchCfg& c, cudaStream_t s) {
+  bool nb = false;
+  const void* fn = kernel_for(objective, Which::Init, c.vpt, false, &nb);
+  if (!fn) return cudaErrorInvalidDeviceFunction;
+  long long grid = a.n_local < 4LL * 148 * 2 ? a.n_local : 4LL * 148 * 2;
+  if (grid < 1) grid = 1;
+  void* args[] = {const_cast<SwarmArgs*>(&a)};
+  return cudaLaunchKernel(fn, dim3((unsigned)grid), dim3(c.compute), args, c.init_smem, s);
+}
+
+cudaError_t launch_rebest(const SwarmArgs& a, unsigned t, cudaStream_t s) {
+  long long blocks = (a.n_local + 255) / 256;
+  if (blocks > 1024) blocks = 1024;
+  if (blocks < 1) blocks = 1;
+  k_rebest<<<(unsigned)blocks, 256, 0, s>>>(a, t);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_select(const SwarmArgs& a, cudaStream_t s) {
+  k_select<<<1, 128, 0, s>>>(a);
+  return cudaGetLastError();
+}
+
+cudaError_t debug_objective(int objective, const float* X_dev, long long m, int d, int pitch,
+                            float* out_dev, int sm_count, cudaStream_t s) {
+  const int nvec = pitch / 4;
+  int vpt, threads;
+  shape_for(nvec, 0, &vpt, &threads);
+  bool nb = false;
+  const void* fn = kernel_for(objective, Which::Eval, vpt, false, &nb);
+  if (!fn) return cudaErrorInvalidDeviceFunction;
+  long long grid = m < (long long)sm_count * 4 ? m : (long long)sm_count * 4;
+  if (grid < 1) grid = 1;
+  void* args[] = {(void*)&X_dev, (void*)&m, (void*)&d, (void*)&nvec, (void*)&out_dev};
+  return cudaLaunchKernel(fn, dim3((unsigned)grid), dim3(threads), args, nb ? (size_t)nvec * 4 : 0,
+                          s);
+}
+
+}  // namespace fastpso
+

@@ -1,4 +1,8 @@
-// swarm_kernels.cu — the fused FastPSO iteration for sm_100a.
+// swarm_kernels.cuh — the fused FastPSO iteration for sm_100a (kernel templates).
+//
+// Instantiated once per objective functor in obj_*.cu (parallel build); the
+// host side (planning, launches, the gbest rebest/select kernels) is
+// swarm_host.cu.
 //
 // One kernel per iteration replaces the paper's five phases (Fig. 5, P:L561-567:
 // init / eval / pbest / gbest / swarm) and its materialised random matrices.
@@ -26,6 +30,7 @@
 //               parallelism is the ring depth, independent of registers.
 //   k_step_reg  (short rows): every thread loads its float4s with 128-bit
 //               LDGs; many rows per SM in flight through occupancy.
+#pragma once
 #include <cuda_runtime.h>
 
 #include <cstdint>
@@ -154,6 +159,41 @@ __device__ __forceinline__ void move1(const MoveParams& m, float& x, float& v, f
   v = vn;
 }
 
+// Eq. 1 with per-dimension bounds (NEXT-2 reading of Eq. 5):
+// v' = clamp(v', vlo_j, vhi_j), x' = clamp(x + v', xlo_j, xhi_j).  With the
+// scalar bounds (vlo = -vmax, vhi = vmax, xlo = lo, xhi = hi) this is move1.
+__device__ __forceinline__ void move1b(const MoveParams& m, float& x, float& v, float pb, float g,
+                                       float m1, float m2, float vlo, float vhi, float xlo,
+                                       float xhi) {
+  const float a = __fmul_rn(m.w, v);
+  const float b = __fmul_rn(__fmul_rn(m.c1s, m1), __fsub_rn(pb, x));
+  const float c = __fmul_rn(__fmul_rn(m.c2s, m2), __fsub_rn(g, x));
+  float vn = __fadd_rn(__fadd_rn(a, b), c);
+  vn = fminf(fmaxf(vn, vlo), vhi);
+  x = fminf(fmaxf(__fadd_rn(x, vn), xlo), xhi);
+  v = vn;
+}
+
+// Update one float4 (dims 4q..4q+3).  kB: bounds per dimension from the
+// shared-memory table sB = [vlo | vhi | xlo | xhi] (nvec float4 each).
+template <bool kB>
+__device__ __forceinline__ void move4(const MoveParams& m, float4& x, float4& v, const float4& pb,
+                                      const float4& g, const float4& r1, const float4& r2,
+                                      const float4* sB, int nvec, int q) {
+  if constexpr (kB) {
+    const float4 vlo = sB[q], vhi = sB[nvec + q], xlo = sB[2 * nvec + q], xhi = sB[3 * nvec + q];
+    move1b(m, x.x, v.x, pb.x, g.x, r1.x, r2.x, vlo.x, vhi.x, xlo.x, xhi.x);
+    move1b(m, x.y, v.y, pb.y, g.y, r1.y, r2.y, vlo.y, vhi.y, xlo.y, xhi.y);
+    move1b(m, x.z, v.z, pb.z, g.z, r1.z, r2.z, vlo.z, vhi.z, xlo.z, xhi.z);
+    move1b(m, x.w, v.w, pb.w, g.w, r1.w, r2.w, vlo.w, vhi.w, xlo.w, xhi.w);
+  } else {
+    move1(m, x.x, v.x, pb.x, g.x, r1.x, r2.x);
+    move1(m, x.y, v.y, pb.y, g.y, r1.y, r2.y);
+    move1(m, x.z, v.z, pb.z, g.z, r1.z, r2.z);
+    move1(m, x.w, v.w, pb.w, g.w, r1.w, r2.w);
+  }
+}
+
 // --- CTA reduction of the functor accumulators -----------------------------
 template <class Obj>
 __device__ __forceinline__ void warp_combine(float* a) {
@@ -254,10 +294,11 @@ __device__ __forceinline__ void map_row(float* acc, const float4 (&x)[VPT], floa
 // registers (k_step_reg) or from the shared-memory stage (k_step_tma);
 // release() runs once every operand has been read.  x' stays in registers
 // (xn) until the pbest decision.  Returns f; `improved` is CTA-uniform.
-template <class Obj, int VPT, class Src, class Release>
+template <class Obj, int VPT, bool kB, class Src, class Release>
 __device__ __forceinline__ float process_row(const SwarmArgs& a, const MoveParams& mp,
                                              PhiloxKey key, uint32_t t, uint32_t gi, long long r,
                                              Src&& src, Release&& release, const float4* sG,
+                                             const float4* sB,
                                              float* sFirst, RowSmem<Obj>& sm, int tid, int nthr,
                                              float pf_old, bool& improved) {
   const int nvec = a.nvec, d = a.d;
@@ -274,10 +315,7 @@ __device__ __forceinline__ float process_row(const SwarmArgs& a, const MoveParam
       const float4 g = sG[q];
       const float4 r1 = raw24x4(key, kTagR1, t, gi, (uint32_t)q);
       const float4 r2 = raw24x4(key, kTagR2, t, gi, (uint32_t)q);
-      move1(mp, x.x, v.x, pb.x, g.x, r1.x, r2.x);
-      move1(mp, x.y, v.y, pb.y, g.y, r1.y, r2.y);
-      move1(mp, x.z, v.z, pb.z, g.z, r1.z, r2.z);
-      move1(mp, x.w, v.w, pb.w, g.w, r1.w, r2.w);
+      move4<kB>(mp, x, v, pb, g, r1, r2, sB, nvec, q);
       if ((d & 3) && q == nvec - 1) {  // keep the row padding at zero
         const int j = 4 * q;
         if (j + 1 >= d) x.y = v.y = 0.f;
@@ -408,19 +446,22 @@ __device__ __forceinline__ void row_bookkeeping(const SwarmArgs& a, long long r,
 }
 
 // ------------------------------------------------- step kernel: registers
-template <class Obj, int VPT>
+template <class Obj, int VPT, bool kB>
 __global__ void __launch_bounds__(kMaxThreads, (VPT >= 8) ? 1 : 2)
     k_step_reg(const SwarmArgs a, int /*stages: unused, same signature as k_step_tma*/) {
   extern __shared__ __align__(128) unsigned char dsmem[];
   float4* sG = reinterpret_cast<float4*>(dsmem);
-  float* sFirst = reinterpret_cast<float*>(sG + a.nvec);
+  float4* sB = sG + a.nvec;  // kB: [vlo | vhi | xlo | xhi]
+  float* sFirst = reinterpret_cast<float*>(sB + (kB ? 4 * a.nvec : 0));
   __shared__ RowSmem<Obj> sm;
   const int tid = threadIdx.x, nthr = blockDim.x;
   if (tid == 0) {
+    const unsigned row_bytes = (unsigned)a.nvec * 16u;
     mbar_init(&sm.gbar, 1);
     mbar_fence_init();
-    mbar_expect_tx(&sm.gbar, (unsigned)a.nvec * 16u);
-    bulk_g2s(sG, a.G, (unsigned)a.nvec * 16u, &sm.gbar);
+    mbar_expect_tx(&sm.gbar, row_bytes * (kB ? 5u : 1u));
+    bulk_g2s(sG, a.G, row_bytes, &sm.gbar);
+    if (kB) bulk_g2s(sB, a.bounds, 4u * row_bytes, &sm.gbar);
   }
   __syncthreads();
   const uint32_t t = a.ctl->t + 1u;
@@ -449,14 +490,14 @@ __global__ void __launch_bounds__(kMaxThreads, (VPT >= 8) ? 1 : 2)
     }
     const float pf_old = (tid == 0) ? a.pf[r] : 0.f;
     bool improved;
-    const float f = process_row<Obj, VPT>(
+    const float f = process_row<Obj, VPT, kB>(
         a, mp, key, t, gi, r,
         [&](int s, int, float4& xo, float4& vo, float4& po) {
           xo = x[s];
           vo = v[s];
           po = pb[s];
         },
-        [] {}, sG, sFirst, sm, tid, nthr, pf_old, improved);
+        [] {}, sG, sB, sFirst, sm, tid, nthr, pf_old, improved);
     if (tid == 0) row_bookkeeping(a, r, gi, f, improved, inc_ord, best, nimp);
   }
   if (cta_finish<Obj>(a, sm, best, nimp, tid, nthr)) gbest_epilogue<Obj>(a, sm, t, tid, nthr);
@@ -477,7 +518,7 @@ __global__ void __launch_bounds__(kMaxThreads, (VPT >= 8) ? 1 : 2)
 //                 bulk stores have read it (wait_group.read).
 // Barriers per stage: full (1 arrival + tx bytes), done (W arrivals), empty (1).
 // Shared memory: [G: nvec float4][stages x {x, v, pb}: nvec float4 each].
-template <class Obj, int VPT>
+template <class Obj, int VPT, bool kB>
 __global__ void __launch_bounds__(kMaxThreads + 64, 2)
     k_step_tma(const SwarmArgs a, int stages) {
   extern __shared__ __align__(128) unsigned char dsmem[];
@@ -485,7 +526,8 @@ __global__ void __launch_bounds__(kMaxThreads + 64, 2)
   const int nthr = (int)blockDim.x - 64;  // compute threads
   const int nwarps = nthr >> 5;
   float4* sG = reinterpret_cast<float4*>(dsmem);
-  float4* ring = sG + nvec;
+  float4* sB = sG + nvec;  // kB: [vlo | vhi | xlo | xhi]
+  float4* ring = sB + (kB ? 4 * nvec : 0);
   __shared__ float red[kMaxStages][(kMaxThreads / 32) * 2];
   __shared__ unsigned long long full[kMaxStages], empty[kMaxStages], done[kMaxStages], gbar;
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
@@ -504,8 +546,9 @@ __global__ void __launch_bounds__(kMaxThreads + 64, 2)
 
   if (warp == nwarps) {  // ---------------- producer
     if (lane == 0) {
-      mbar_expect_tx(&gbar, row_bytes);
+      mbar_expect_tx(&gbar, row_bytes * (kB ? 5u : 1u));
       bulk_g2s(sG, a.G, row_bytes, &gbar);
+      if (kB) bulk_g2s(sB, a.bounds, 4u * row_bytes, &gbar);
       int s = 0;
       unsigned ph = 0;
       int k = 0;
@@ -604,10 +647,7 @@ __global__ void __launch_bounds__(kMaxThreads + 64, 2)
         const float4 g = sG[q];
         const float4 r1 = raw24x4(key, kTagR1, t, gi, (uint32_t)q);
         const float4 r2 = raw24x4(key, kTagR2, t, gi, (uint32_t)q);
-        move1(mp, x.x, v.x, pb.x, g.x, r1.x, r2.x);
-        move1(mp, x.y, v.y, pb.y, g.y, r1.y, r2.y);
-        move1(mp, x.z, v.z, pb.z, g.z, r1.z, r2.z);
-        move1(mp, x.w, v.w, pb.w, g.w, r1.w, r2.w);
+        move4<kB>(mp, x, v, pb, g, r1, r2, sB, nvec, q);
         if ((d & 3) && q == nvec - 1) {  // keep the row padding at zero
           const int jj = 4 * q;
           if (jj + 1 >= d) x.y = v.y = 0.f;
@@ -652,7 +692,7 @@ __global__ void __launch_bounds__(kMaxThreads + 64, 2)
 // k_step_reg's one-warp shape produces for these rows (its wider butterfly
 // steps only add the identities of idle lanes), so fitness, decisions and
 // state are bitwise those of the streaming kernels.
-template <class Obj>
+template <class Obj, bool kB>
 __global__ void __launch_bounds__(1024, 1) k_resident(const SwarmArgs a, int iters) {
   extern __shared__ __align__(16) unsigned char dsmem[];
   const int nvec = a.nvec, d = a.d;
@@ -662,7 +702,8 @@ __global__ void __launch_bounds__(1024, 1) k_resident(const SwarmArgs a, int ite
   float4* sV = sX + cells;
   float4* sP = sV + cells;
   float4* sG = sP + cells;
-  float* spf = reinterpret_cast<float*>(sG + nvec);
+  float4* sB = sG + nvec;  // kB: [vlo | vhi | xlo | xhi]
+  float* spf = reinterpret_cast<float*>(sB + (kB ? 4 * nvec : 0));
   __shared__ unsigned long long s_acc;
   __shared__ unsigned s_imp;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, nwarps = blockDim.x >> 5;
@@ -680,6 +721,9 @@ __global__ void __launch_bounds__(1024, 1) k_resident(const SwarmArgs a, int ite
     sP[i] = P4[i];
   }
   for (int i = tid; i < nvec; i += blockDim.x) sG[i] = reinterpret_cast<const float4*>(a.G)[i];
+  if (kB)
+    for (int i = tid; i < 4 * nvec; i += blockDim.x)
+      sB[i] = reinterpret_cast<const float4*>(a.bounds)[i];
   for (int i = tid; i < n; i += blockDim.x) spf[i] = a.pf[i];
   const unsigned long long cur0 = a.ctl->key_cur;
   const uint32_t t0 = a.ctl->t;
@@ -709,10 +753,7 @@ __global__ void __launch_bounds__(1024, 1) k_resident(const SwarmArgs a, int ite
         x = sX[c];
         const float4 r1 = raw24x4(key, kTagR1, t, gi, (uint32_t)sub);
         const float4 r2 = raw24x4(key, kTagR2, t, gi, (uint32_t)sub);
-        move1(mp, x.x, v.x, pb.x, g.x, r1.x, r2.x);
-        move1(mp, x.y, v.y, pb.y, g.y, r1.y, r2.y);
-        move1(mp, x.z, v.z, pb.z, g.z, r1.z, r2.z);
-        move1(mp, x.w, v.w, pb.w, g.w, r1.w, r2.w);
+        move4<kB>(mp, x, v, pb, g, r1, r2, sB, nvec, sub);
         if ((d & 3) && sub == nvec - 1) {
           const int jj = 4 * sub;
           if (jj + 1 >= d) x.y = v.y = 0.f;
@@ -807,7 +848,7 @@ __device__ __forceinline__ unsigned ld_acquire_u32(const unsigned* p) {
   return v;
 }
 
-template <class Obj, int VPT>
+template <class Obj, int VPT, bool kB>
 __global__ void __launch_bounds__(kMaxThreads, 1) k_gridres(const SwarmArgs a, int iters) {
   extern __shared__ __align__(16) unsigned char dsmem[];
   const int nvec = a.nvec, d = a.d;
@@ -817,7 +858,8 @@ __global__ void __launch_bounds__(kMaxThreads, 1) k_gridres(const SwarmArgs a, i
   const long long n = a.n_local;
   const int myrows = (int)((n - b + grid - 1) / grid);  // rows b, b+grid, ...
   float4* sG = reinterpret_cast<float4*>(dsmem);
-  float4* sRows = sG + nvec;  // [myrows][3][nvec]
+  float4* sB = sG + nvec;                          // kB: [vlo | vhi | xlo | xhi]
+  float4* sRows = sB + (kB ? 4 * nvec : 0);        // [myrows][3][nvec]
   float* spf = reinterpret_cast<float*>(sRows + (size_t)myrows * 3 * nvec);
   __shared__ float red[(kMaxThreads / 32) * 2];
   __shared__ float s_f;
@@ -840,6 +882,8 @@ __global__ void __launch_bounds__(kMaxThreads, 1) k_gridres(const SwarmArgs a, i
     if (tid == 0) spf[k] = a.pf[r];
   }
   for (int q = tid; q < nvec; q += nthr) sG[q] = reinterpret_cast<const float4*>(a.G)[q];
+  if (kB)
+    for (int q = tid; q < 4 * nvec; q += nthr) sB[q] = reinterpret_cast<const float4*>(a.bounds)[q];
   const unsigned long long cur0 = a.ctl->key_cur;
   const uint32_t t0 = a.ctl->t;
   __syncthreads();
@@ -869,10 +913,7 @@ __global__ void __launch_bounds__(kMaxThreads, 1) k_gridres(const SwarmArgs a, i
           const float4 g = sG[q];
           const float4 r1 = raw24x4(key, kTagR1, t, gi, (uint32_t)q);
           const float4 r2 = raw24x4(key, kTagR2, t, gi, (uint32_t)q);
-          move1(mp, x.x, v.x, pb.x, g.x, r1.x, r2.x);
-          move1(mp, x.y, v.y, pb.y, g.y, r1.y, r2.y);
-          move1(mp, x.z, v.z, pb.z, g.z, r1.z, r2.z);
-          move1(mp, x.w, v.w, pb.w, g.w, r1.w, r2.w);
+          move4<kB>(mp, x, v, pb, g, r1, r2, sB, nvec, q);
           if ((d & 3) && q == nvec - 1) {
             const int jj = 4 * q;
             if (jj + 1 >= d) x.y = v.y = 0.f;
@@ -1007,8 +1048,7 @@ __global__ void __launch_bounds__(kMaxThreads, (VPT >= 8) ? 1 : 2)
   const int tid = threadIdx.x, nthr = blockDim.x;
   const PhiloxKey key{a.seed_lo, a.seed_hi};
   const int nvec = a.nvec, d = a.d;
-  const float span = __fsub_rn(a.hi, a.lo);
-  const float two_vmax = __fmul_rn(2.f, a.vmax);
+  const float4* B4 = reinterpret_cast<const float4*>(a.bounds);  // null: scalar bounds
   const uint32_t inc_ord = (uint32_t)(a.ctl->key_cur >> 32);
   unsigned long long best = ~0ull;
   for (long long r = blockIdx.x; r < a.n_local; r += gridDim.x) {
@@ -1025,11 +1065,26 @@ __global__ void __launch_bounds__(kMaxThreads, (VPT >= 8) ? 1 : 2)
         const float4 uv = uniforms4(key, kTagV0, 0u, gi, (uint32_t)q);
         float xs[4] = {ux.x, ux.y, ux.z, ux.w};
         float vs[4] = {uv.x, uv.y, uv.z, uv.w};
+        float4 vlo4 = make_float4(-a.vmax, -a.vmax, -a.vmax, -a.vmax);
+        float4 vhi4 = make_float4(a.vmax, a.vmax, a.vmax, a.vmax);
+        float4 xlo4 = make_float4(a.lo, a.lo, a.lo, a.lo), xhi4 = make_float4(a.hi, a.hi, a.hi, a.hi);
+        if (B4) {
+          vlo4 = B4[q];
+          vhi4 = B4[nvec + q];
+          xlo4 = B4[2 * nvec + q];
+          xhi4 = B4[3 * nvec + q];
+        }
+        const float vlo[4] = {vlo4.x, vlo4.y, vlo4.z, vlo4.w};
+        const float vhi[4] = {vhi4.x, vhi4.y, vhi4.z, vhi4.w};
+        const float xlo[4] = {xlo4.x, xlo4.y, xlo4.z, xlo4.w};
+        const float xhi[4] = {xhi4.x, xhi4.y, xhi4.z, xhi4.w};
 #pragma unroll
-        for (int e = 0; e < 4; ++e) {
+        for (int e = 0; e < 4; ++e) {  // x0 = clamp(lo + (hi - lo) U), v0 = vlo + (vhi - vlo) U
           const bool pad = 4 * q + e >= d;
-          xs[e] = pad ? 0.f : fminf(fmaxf(__fadd_rn(a.lo, __fmul_rn(span, xs[e])), a.lo), a.hi);
-          vs[e] = pad ? 0.f : __fadd_rn(-a.vmax, __fmul_rn(two_vmax, vs[e]));
+          const float span = __fsub_rn(xhi[e], xlo[e]);
+          const float vspan = __fsub_rn(vhi[e], vlo[e]);
+          xs[e] = pad ? 0.f : fminf(fmaxf(__fadd_rn(xlo[e], __fmul_rn(span, xs[e])), xlo[e]), xhi[e]);
+          vs[e] = pad ? 0.f : __fadd_rn(vlo[e], __fmul_rn(vspan, vs[e]));
         }
         x[s] = make_float4(xs[0], xs[1], xs[2], xs[3]);
         st_stream(Xr + q, x[s]);
@@ -1052,87 +1107,6 @@ __global__ void __launch_bounds__(kMaxThreads, (VPT >= 8) ? 1 : 2)
     }
   }
   if (cta_finish<Obj>(a, sm, best, 0, tid, nthr)) gbest_epilogue<Obj>(a, sm, 0u, tid, nthr);
-}
-
-// ---------------------------------------------------------- rebest kernel
-// After set_state: pf NaN -> +inf, gbest = lowest index attaining min pf.
-struct NoObj {
-  static constexpr int kAcc = 1;
-};
-__global__ void __launch_bounds__(256) k_rebest(const SwarmArgs a, unsigned t) {
-  __shared__ unsigned long long s_best[8];
-  __shared__ RowSmem<NoObj> sm;
-  const int tid = threadIdx.x, nthr = blockDim.x;
-  unsigned long long best = ~0ull;
-  for (long long r = blockIdx.x * (long long)blockDim.x + threadIdx.x; r < a.n_local;
-       r += (long long)gridDim.x * blockDim.x) {
-    float f = a.pf[r];
-    if (f != f) {
-      f = __int_as_float(0x7f800000);
-      a.pf[r] = f;
-    }
-    const unsigned long long k = pack_key(f, (uint32_t)(a.row_begin + r));
-    best = k < best ? k : best;
-  }
-#pragma unroll
-  for (int off = 16; off > 0; off >>= 1) {
-    const unsigned long long o = __shfl_xor_sync(kFull, best, off);
-    best = o < best ? o : best;
-  }
-  if ((tid & 31) == 0) s_best[tid >> 5] = best;
-  __syncthreads();
-  if (tid == 0)
-    for (int w = 1; w < (nthr >> 5); ++w) best = s_best[w] < best ? s_best[w] : best;
-  if (cta_finish<NoObj>(a, sm, tid == 0 ? best : ~0ull, 0, tid, nthr))
-    gbest_epilogue<NoObj>(a, sm, t, tid, nthr);
-}
-
-// ---------------------------------------------------------- select kernel
-// world > 1, after ncclAllGather of the records: the global candidate is the
-// minimum key over ranks (keys carry global indices, so ties resolve to the
-// lowest global index, as one GPU would).  Every rank computes the same bits.
-__global__ void __launch_bounds__(128) k_select(const SwarmArgs a) {
-  __shared__ unsigned long long s_min;
-  __shared__ int s_src;
-  const size_t rec = record_bytes(a.nvec * 4);
-  if (threadIdx.x < 32) {
-    unsigned long long best = ~0ull;
-    int src = -1;
-    for (int r = threadIdx.x; r < a.world; r += 32) {
-      const unsigned long long k =
-          *reinterpret_cast<const unsigned long long*>(a.recv + (size_t)r * rec);
-      if (k < best) {
-        best = k;
-        src = r;
-      }
-    }
-#pragma unroll
-    for (int off = 16; off > 0; off >>= 1) {
-      const unsigned long long o = __shfl_xor_sync(kFull, best, off);
-      const int os = __shfl_xor_sync(kFull, src, off);
-      if (o < best || (o == best && os >= 0 && (src < 0 || os < src))) {
-        best = o;
-        src = os;
-      }
-    }
-    if (threadIdx.x == 0) {
-      s_min = best;
-      s_src = src;
-    }
-  }
-  __syncthreads();
-  const unsigned long long cur = a.ctl->key_cur;
-  const bool take = s_src >= 0 && s_min < cur;
-  if (take) {
-    const float4* row = reinterpret_cast<const float4*>(a.recv + (size_t)s_src * rec + 16);
-    float4* G4 = reinterpret_cast<float4*>(a.G);
-    for (int q = threadIdx.x; q < a.nvec; q += blockDim.x) G4[q] = row[q];
-  }
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    if (take) a.ctl->key_cur = s_min;
-    a.ctl->key_acc = take ? s_min : cur;
-  }
 }
 
 // ---------------------------------------------------------- debug: objective
@@ -1160,281 +1134,32 @@ __global__ void __launch_bounds__(kMaxThreads) k_eval(const float* X, long long 
   }
 }
 
-// ---------------------------------------------------------- dispatch
-enum class Which { StepReg, StepTma, Init, Eval, GridRes };
 
 template <class Obj>
-const void* pick(Which w, int vpt) {
-#define PSO_VPT_CASES(KERNEL)                          \
-  switch (vpt) {                                       \
-    case 1: return (const void*)KERNEL<Obj, 1>;        \
-    case 2: return (const void*)KERNEL<Obj, 2>;        \
-    case 4: return (const void*)KERNEL<Obj, 4>;        \
-    default: return (const void*)KERNEL<Obj, 8>;       \
-  }
-  switch (w) {
-    case Which::StepReg: PSO_VPT_CASES(k_step_reg)
-    case Which::StepTma: PSO_VPT_CASES(k_step_tma)
-    case Which::Init: PSO_VPT_CASES(k_init)
-    case Which::GridRes: PSO_VPT_CASES(k_gridres)
-    default: PSO_VPT_CASES(k_eval)
-  }
-#undef PSO_VPT_CASES
+KernelTable make_kernel_table() {
+  KernelTable t{};
+  t.neighbor = Obj::kNeighbor;
+#define PSO_T(ARR, KER, V, I)                     \
+  t.ARR[I][0] = (const void*)KER<Obj, V, false>; \
+  t.ARR[I][1] = (const void*)KER<Obj, V, true>;
+#define PSO_ALLV(ARR, KER) PSO_T(ARR, KER, 1, 0) PSO_T(ARR, KER, 2, 1) PSO_T(ARR, KER, 4, 2) PSO_T(ARR, KER, 8, 3)
+  PSO_ALLV(step_reg, k_step_reg)
+  PSO_ALLV(step_tma, k_step_tma)
+  PSO_ALLV(gridres, k_gridres)
+#undef PSO_ALLV
+#undef PSO_T
+  t.resident[0] = (const void*)k_resident<Obj, false>;
+  t.resident[1] = (const void*)k_resident<Obj, true>;
+  t.init[0] = (const void*)k_init<Obj, 1>;
+  t.init[1] = (const void*)k_init<Obj, 2>;
+  t.init[2] = (const void*)k_init<Obj, 4>;
+  t.init[3] = (const void*)k_init<Obj, 8>;
+  t.eval[0] = (const void*)k_eval<Obj, 1>;
+  t.eval[1] = (const void*)k_eval<Obj, 2>;
+  t.eval[2] = (const void*)k_eval<Obj, 4>;
+  t.eval[3] = (const void*)k_eval<Obj, 8>;
+  return t;
 }
-
-const void* resident_kernel_for(int objective) {
-#define PSO_CASE(ID, F) \
-  case ID:              \
-    return (const void*)k_resident<F>;
-  switch (objective) {
-    PSO_ALL_OBJECTIVES(PSO_CASE)
-    default:
-      return nullptr;
-  }
-#undef PSO_CASE
-}
-
-const void* kernel_for(int objective, Which w, int vpt, bool* neighbor) {
-#define PSO_CASE(ID, F)                      \
-  case ID:                                   \
-    *neighbor = F::kNeighbor;                \
-    return pick<F>(w, vpt);
-  switch (objective) {
-    PSO_ALL_OBJECTIVES(PSO_CASE)
-    default:
-      return nullptr;
-  }
-#undef PSO_CASE
-}
-
-// CTA shape for a row of nvec float4: the smallest VPT in {1,2,4,8} whose
-// thread count fits 256, threads rounded up to a warp multiple.
-void shape_for(int nvec, int vpt_override, int* vpt, int* threads) {
-  static const int kVpts[] = {1, 2, 4, 8};
-  int v = 8;
-  for (int c : kVpts) {
-    if ((nvec + c - 1) / c <= kMaxThreads) {
-      v = c;
-      break;
-    }
-  }
-  if (vpt_override == 1 || vpt_override == 2 || vpt_override == 4 || vpt_override == 8) {
-    if ((nvec + vpt_override - 1) / vpt_override <= kMaxThreads) v = vpt_override;
-  }
-  const int t = (nvec + v - 1) / v;
-  *vpt = v;
-  *threads = ((t + 31) / 32) * 32;
-}
-
-constexpr size_t kSmemPerSm = 228 * 1024;       // B200 unified L1/shared per SM
-constexpr size_t kSmemPerCtaMax = 227 * 1024;   // opt-in maximum per CTA
-constexpr size_t kStaticReserve = 2048;         // static shared + per-CTA reservation
-constexpr long long kResidentElems = 8192;      // resident path: n d <= this
 
 }  // namespace
-
-bool objective_registered(int objective) {
-  bool nb;
-  return kernel_for(objective, Which::Init, 1, &nb) != nullptr;
-}
-
-cudaError_t plan_launch(int objective, int d, long long n_local, int sm_count, const PlanHints& h,
-                        LaunchCfg* cfg) {
-  const int nvec = (d + 3) / 4;
-  shape_for(nvec, h.vpt, &cfg->vpt, &cfg->compute);
-  bool nb = false;
-  if (!kernel_for(objective, Which::Init, cfg->vpt, &nb)) return cudaErrorInvalidDeviceFunction;
-  const size_t row = (size_t)nvec * 16;
-  const size_t first = nb ? (size_t)nvec * 4 : 0;
-  cfg->init_smem = first;
-  cudaError_t e;
-
-  // ---- resident single-CTA path for tiny swarms (single GPU only)
-  cfg->resident = 0;
-  if (h.allow_resident && nvec <= 32 && n_local * nvec * 4 <= kResidentElems) {
-    const size_t smem = (size_t)n_local * nvec * 16 * 3 + (size_t)nvec * 16 + (size_t)n_local * 4;
-    const void* fn = resident_kernel_for(objective);
-    if (smem <= kSmemPerCtaMax - kStaticReserve &&
-        cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) ==
-            cudaSuccess) {
-      int gs = 1;
-      while (gs < nvec) gs <<= 1;
-      const long long rpw = 32 / gs;
-      long long warps = (n_local + rpw - 1) / rpw;
-      if (warps > 32) warps = 32;
-      cfg->resident = 1;
-      cfg->resident_threads = 32 * (int)(warps < 1 ? 1 : warps);
-      cfg->resident_smem = smem;
-    }
-    cudaGetLastError();
-  }
-
-  // ---- TMA pipeline: rows of >= 256 dims unless forced otherwise
-  bool tma = h.kernel == 1 || (h.kernel == -1 && nvec >= 64);
-  if (tma) {
-    const void* fn = kernel_for(objective, Which::StepTma, cfg->vpt, &nb);
-    const int threads = cfg->compute + 64;  // + producer warp + finaliser warp
-    // CTAs per SM the registers allow, capped at 2; the ring fills the rest.
-    int by_regs = 0;
-    if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&by_regs, fn, threads, 0)) != cudaSuccess)
-      return e;
-    const int cap = (h.ctas >= 1 && h.ctas <= 8) ? h.ctas : 2;
-    int ctas = by_regs < 1 ? 1 : (by_regs > cap ? cap : by_regs);
-    // The most CTAs per SM (<= cap) that still keep >= 3 rows in flight per
-    // CTA; two rows only if nothing else fits (measured: 2-stage rings leave
-    // HBM idle between rows, 3-4 stages saturate it).
-    auto stages_for = [&](int c) -> int {
-      size_t budget = kSmemPerSm / c - kStaticReserve;
-      if (budget > kSmemPerCtaMax - kStaticReserve) budget = kSmemPerCtaMax - kStaticReserve;
-      return budget > row ? (int)((budget - row) / (3 * row)) : 0;
-    };
-    int stages = 0;
-    int c = ctas;
-    for (; c >= 1; --c)
-      if (stages_for(c) >= 3) break;
-    if (c >= 1) {
-      ctas = c;
-    } else {
-      for (c = ctas; c >= 1 && stages_for(c) < 2; --c) {
-      }
-      ctas = c < 1 ? 1 : c;
-    }
-    stages = stages_for(ctas);
-    if (h.stages >= 2 && h.stages <= kMaxStages) stages = stages < h.stages ? stages : h.stages;
-    if (stages > kMaxStages) stages = kMaxStages;
-    if (stages >= 2) {
-      const size_t smem = row + (size_t)stages * 3 * row;
-      if ((e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem)) !=
-          cudaSuccess)
-        return e;
-      int per_sm = 0;
-      if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, threads, smem)) !=
-          cudaSuccess)
-        return e;
-      if (per_sm >= 1) {
-        cfg->tma = 1;
-        cfg->stages = stages;
-        cfg->threads = threads;
-        cfg->smem = smem;
-        cfg->ctas_per_sm = per_sm;
-      } else {
-        tma = false;
-      }
-    } else {
-      tma = false;
-    }
-  }
-  if (!tma) {
-    const void* fn = kernel_for(objective, Which::StepReg, cfg->vpt, &nb);
-    cfg->tma = 0;
-    cfg->stages = 0;
-    cfg->threads = cfg->compute;
-    cfg->smem = row + first;
-    int per_sm = 0;
-    if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, cfg->threads, cfg->smem)) !=
-        cudaSuccess)
-      return e;
-    cfg->ctas_per_sm = per_sm < 1 ? 1 : per_sm;
-  }
-  long long grid = (long long)cfg->ctas_per_sm * sm_count;
-  if (grid > n_local) grid = n_local;
-  if (grid < 1) grid = 1;
-  cfg->grid = (int)grid;
-
-  // ---- grid-resident path: the whole swarm in the grid's shared memory
-  cfg->gridres = 0;
-  if (h.allow_resident && !cfg->resident && cfg->tma && nvec >= 64) {
-    const void* fn = kernel_for(objective, Which::GridRes, cfg->vpt, &nb);
-    for (int per = 2; per >= 1 && !cfg->gridres; --per) {
-      long long g = (long long)per * sm_count;
-      if (g > n_local) g = n_local;
-      const long long rows = (n_local + g - 1) / g;
-      const size_t smem = row + (size_t)rows * 3 * row + (size_t)rows * 4;
-      if (smem > kSmemPerCtaMax - kStaticReserve || smem * per > kSmemPerSm - per * kStaticReserve)
-        continue;
-      if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) !=
-          cudaSuccess) {
-        cudaGetLastError();
-        continue;
-      }
-      int occ = 0;
-      if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, cfg->compute, smem) != cudaSuccess) {
-        cudaGetLastError();
-        continue;
-      }
-      if ((long long)occ * sm_count < g) continue;  // cooperative: every CTA co-resident
-      cfg->gridres = 1;
-      cfg->gridres_grid = (int)g;
-      cfg->gridres_rows = (int)rows;
-      cfg->gridres_smem = smem;
-    }
-  }
-  return cudaSuccess;
-}
-
-cudaError_t launch_step(int objective, const SwarmArgs& a, const LaunchCfg& c, cudaStream_t s) {
-  bool nb = false;
-  const void* fn = kernel_for(objective, c.tma ? Which::StepTma : Which::StepReg, c.vpt, &nb);
-  if (!fn) return cudaErrorInvalidDeviceFunction;
-  int stages = c.stages;
-  void* args[] = {const_cast<SwarmArgs*>(&a), &stages};
-  return cudaLaunchKernel(fn, dim3(c.grid), dim3(c.threads), args, c.smem, s);
-}
-
-cudaError_t launch_resident(int objective, const SwarmArgs& a, const LaunchCfg& c, int iters,
-                            cudaStream_t s) {
-  const void* fn = resident_kernel_for(objective);
-  if (!fn) return cudaErrorInvalidDeviceFunction;
-  void* args[] = {const_cast<SwarmArgs*>(&a), &iters};
-  return cudaLaunchKernel(fn, dim3(1), dim3(c.resident_threads), args, c.resident_smem, s);
-}
-
-cudaError_t launch_gridres(int objective, const SwarmArgs& a, const LaunchCfg& c, int iters,
-                           cudaStream_t s) {
-  bool nb = false;
-  const void* fn = kernel_for(objective, Which::GridRes, c.vpt, &nb);
-  if (!fn) return cudaErrorInvalidDeviceFunction;
-  void* args[] = {const_cast<SwarmArgs*>(&a), &iters};
-  return cudaLaunchCooperativeKernel(fn, dim3(c.gridres_grid), dim3(c.compute), args,
-                                     c.gridres_smem, s);
-}
-
-cudaError_t launch_init(int objective, const SwarmArgs& a, const LaunchCfg& c, cudaStream_t s) {
-  bool nb = false;
-  const void* fn = kernel_for(objective, Which::Init, c.vpt, &nb);
-  if (!fn) return cudaErrorInvalidDeviceFunction;
-  long long grid = a.n_local < 4LL * 148 * 2 ? a.n_local : 4LL * 148 * 2;
-  if (grid < 1) grid = 1;
-  void* args[] = {const_cast<SwarmArgs*>(&a)};
-  return cudaLaunchKernel(fn, dim3((unsigned)grid), dim3(c.compute), args, c.init_smem, s);
-}
-
-cudaError_t launch_rebest(const SwarmArgs& a, unsigned t, cudaStream_t s) {
-  long long blocks = (a.n_local + 255) / 256;
-  if (blocks > 1024) blocks = 1024;
-  if (blocks < 1) blocks = 1;
-  k_rebest<<<(unsigned)blocks, 256, 0, s>>>(a, t);
-  return cudaGetLastError();
-}
-
-cudaError_t launch_select(const SwarmArgs& a, cudaStream_t s) {
-  k_select<<<1, 128, 0, s>>>(a);
-  return cudaGetLastError();
-}
-
-cudaError_t debug_objective(int objective, const float* X_dev, long long m, int d, int pitch,
-                            float* out_dev, int sm_count, cudaStream_t s) {
-  const int nvec = pitch / 4;
-  int vpt, threads;
-  shape_for(nvec, 0, &vpt, &threads);
-  bool nb = false;
-  const void* fn = kernel_for(objective, Which::Eval, vpt, &nb);
-  if (!fn) return cudaErrorInvalidDeviceFunction;
-  long long grid = m < (long long)sm_count * 4 ? m : (long long)sm_count * 4;
-  if (grid < 1) grid = 1;
-  void* args[] = {(void*)&X_dev, (void*)&m, (void*)&d, (void*)&nvec, (void*)&out_dev};
-  return cudaLaunchKernel(fn, dim3((unsigned)grid), dim3(threads), args, nb ? (size_t)nvec * 4 : 0,
-                          s);
-}
-
 }  // namespace fastpso

@@ -118,3 +118,19 @@ def test_product_path_fails_loudly_without_library(monkeypatch, tmp_path):
     monkeypatch.setattr(_lib, "_lib", None)
     with pytest.raises(ImportError):
         _lib.lib()
+
+
+def test_bounds_validation_without_gpu():
+    import numpy as np
+    o = _lib.pso_opts()
+    o.device = -1
+    b = np.zeros(4 * 10, np.float32)
+    b[10:20] = 1.0   # vhi
+    b[20:30] = -1.0  # xlo
+    b[30:40] = 1.0   # xhi
+    b[25] = 2.0      # xlo > xhi at dim 5
+    o.bounds = b.ctypes.data
+    assert _create(opts=o)[0] == 1
+    b[25] = -1.0
+    b[3] = np.nan
+    assert _create(opts=o)[0] == 1

@@ -385,3 +385,58 @@ def test_grid_resident_bitwise_equals_streaming(obj, n, d, monkeypatch):
     info = a.info()
     assert info["launches"] == 3 and info["t"] == 20
     assert info["improvements"] > 0
+
+
+# ------------------------------------------------------------------ per-dimension bounds (NEXT-2)
+def _dim_bounds(d, seed):
+    rng = np.random.default_rng(seed)
+    xlo = rng.uniform(-5, -0.5, d).astype(np.float32)
+    xhi = (xlo + rng.uniform(0.5, 6, d)).astype(np.float32)
+    vhi = rng.uniform(0.05, 2, d).astype(np.float32)
+    vlo = (-rng.uniform(0.05, 2, d)).astype(np.float32)
+    return np.stack([vlo, vhi, xlo, xhi])
+
+
+@pytest.mark.parametrize("path", ["auto", "reg", "tma", "streaming"])
+@pytest.mark.parametrize("obj,n,d", [(SPHERE, 32, 10), (RASTRIGIN, 300, 1000), (ROSENBROCK, 70, 2001),
+                                     (GRIEWANK, 257, 13), (ACKLEY, 9, 4096)])
+def test_per_dim_bounds_match_oracle(path, obj, n, d, monkeypatch):
+    if path in ("reg", "tma"):
+        monkeypatch.setenv("PSO_KERNEL", path)
+    elif path == "streaming":
+        monkeypatch.setenv("PSO_RESIDENT", "0")
+    b = _dim_bounds(d, n + d)
+    lo, hi = DOMAINS[obj]
+    g = fp.Swarm(n, d, 0.9, 2.0, 2.0, lo, hi, obj, 13, device=0, bounds=b)
+    assert g.info()["bounds"] == 1
+    c = orc.OracleSwarm(n, d, 0.9, 2.0, 2.0, lo, hi, obj, 13, bounds=b)
+    X, V, PB, pf, _ = g.get_state()
+    assert_bitwise(X, c.X, "X0")
+    assert_bitwise(V, c.V, "V0")
+    for _ in range(3):
+        X, V, PB, pf, t = g.get_state()
+        c.set_state(X, V, PB, pf, t=t)
+        g.step(1)
+        c.step(1)
+        X2, V2, _, pf2, _ = g.get_state()
+        assert_bitwise(X2, c.X, "X")
+        assert_bitwise(V2, c.V, "V")
+        assert (X2 >= b[2]).all() and (X2 <= b[3]).all()
+        assert (V2 >= b[0]).all() and (V2 <= b[1]).all()
+    b2 = _dim_bounds(d, 99)
+    g.set_bounds(b2)
+    g.step(2)
+    X3, V3, _, _, _ = g.get_state()
+    assert (V3 >= b2[0]).all() and (V3 <= b2[1]).all()
+
+
+def test_set_bounds_requires_bounds_handle():
+    g = gpu_swarm(10, 10, SPHERE)
+    with pytest.raises(fp.PsoError) as e:
+        g.set_bounds(_dim_bounds(10, 1))
+    assert e.value.status == 5
+    with pytest.raises(fp.PsoError) as e:
+        bad = _dim_bounds(10, 1)
+        bad[0, 3] = 5.0  # vlo > vhi
+        gpu_swarm(10, 10, SPHERE, bounds=bad)
+    assert e.value.status == 1

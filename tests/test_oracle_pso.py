@@ -280,3 +280,57 @@ def test_table2_plausibility(golden_dir):
         lo_band = min(v[k] for v in ref.values()) / 10.0
         hi_band = max(v[k] for v in ref.values()) * 10.0
         assert lo_band < got < hi_band, (k, got)
+
+
+# --------------------------------------------------- per-dimension bounds (NEXT-2)
+def _bounds(d, seed=0):
+    rng = np.random.default_rng(seed)
+    xlo = rng.uniform(-5, -0.5, d).astype(np.float32)
+    xhi = (xlo + rng.uniform(0.5, 6, d)).astype(np.float32)
+    vhi = rng.uniform(0.05, 2, d).astype(np.float32)
+    vlo = (-rng.uniform(0.05, 2, d)).astype(np.float32)
+    return np.stack([vlo, vhi, xlo, xhi])
+
+
+def test_per_dim_bounds_equal_to_scalars_is_the_scalar_run():
+    d = 9
+    b = np.array([[-0.7] * d, [0.7] * d, [-3.0] * d, [2.5] * d], np.float32)
+    s = orc.OracleSwarm(20, d, 0.9, 2, 2, -3.0, 2.5, orc.RASTRIGIN, 4, vmax=0.7)
+    t = orc.OracleSwarm(20, d, 0.9, 2, 2, -3.0, 2.5, orc.RASTRIGIN, 4, vmax=0.7, bounds=b)
+    assert_same(snapshot(s), snapshot(t))
+    s.step(30)
+    t.step(30)
+    assert_same(snapshot(s), snapshot(t))
+
+
+def test_per_dim_bounds_invariants_and_saturation():
+    d = 11
+    b = _bounds(d, 1)
+    s = orc.OracleSwarm(64, d, 0.9, 2, 2, -5, 5, orc.SPHERE, 5, bounds=b)
+    assert (s.X >= b[2]).all() and (s.X <= b[3]).all()
+    assert (s.V >= b[0]).all() and (s.V <= b[1]).all()
+    for j in range(d):  # init is uniform on each dimension's own interval
+        assert stats.kstest((s.X[:, j] - b[2, j]) / (b[3, j] - b[2, j]), "uniform").pvalue > 1e-4
+    for _ in range(20):
+        s.step(1)
+        assert (s.X >= b[2]).all() and (s.X <= b[3]).all()
+        assert (s.V >= b[0]).all() and (s.V <= b[1]).all()
+    # huge c1: most velocities sit exactly on their own dimension's bound
+    h = orc.OracleSwarm(64, d, 0.0, 1e4, 0.0, -5, 5, orc.SPHERE, 6, bounds=b)
+    X, V, PB, pf = random_state(64, d, -0.5, 0.5, 0.1, 17, pf_mode="zero")
+    h.set_state(X, V, PB, pf, t=0)
+    h.step(1)
+    on_bound = (h.V == b[0][None, :]) | (h.V == b[1][None, :])
+    assert on_bound.mean() > 0.9
+
+
+def test_one_sided_velocity_bound_makes_positions_monotone():
+    # Eq. 5 with lower_bound = 0: no particle can move backwards in any dimension
+    d = 6
+    b = np.array([[0.0] * d, [0.5] * d, [-5.0] * d, [5.0] * d], np.float32)
+    s = orc.OracleSwarm(32, d, 0.9, 2, 2, -5, 5, orc.RASTRIGIN, 8, bounds=b)
+    prev = s.X.copy()
+    for _ in range(25):
+        s.step(1)
+        assert (s.X >= prev).all()
+        prev = s.X.copy()
