@@ -235,7 +235,7 @@ cudaError_t plan_launch(int objective, int d, long long n_local, int sm_count, c
     cfg->tma = 0;
     cfg->stages = 0;
     cfg->threads = cfg->compute;
-    cfg->smem = row + first;
+    cfg->smem = row + btab + first;
     int per_sm = 0;
     if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, cfg->threads, cfg->smem)) !=
         cudaSuccess)
