@@ -236,6 +236,9 @@ cudaError_t plan_launch(int objective, int d, long long n_local, int sm_count, c
     cfg->stages = 0;
     cfg->threads = cfg->compute;
     cfg->smem = row + btab + first;
+    if ((e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                  (int)cfg->smem)) != cudaSuccess)
+      return e;
     int per_sm = 0;
     if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, cfg->threads, cfg->smem)) !=
         cudaSuccess)
