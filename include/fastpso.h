@@ -53,7 +53,8 @@ extern "C" {
 
 #define FASTPSO_VERSION_MAJOR 0
 #define FASTPSO_VERSION_MINOR 1
-#define PSO_D_MAX 8192 /* max dimension held per fused row (one CTA per row) */
+#define PSO_D_MAX 65536 /* max dimension: <= 8192 one CTA per row; above, a thread-block
+                          cluster of up to 16 CTAs per row (column blocks) */
 
 typedef struct pso_swarm* pso_handle; /* opaque; owns all device memory */
 
@@ -175,6 +176,8 @@ typedef struct {
                                     (cooperative launch); 1 and 2 run a whole
                                     pso_step call in one launch (single GPU only) */
   int32_t bounds;                /* 1: per-dimension bounds in use */
+  int32_t cluster;               /* > 0: each row is split in column blocks over a
+                                    thread-block cluster of this many CTAs (d > 8192) */
   float vmax;
   uint64_t t;                    /* iterations done */
   uint64_t launches;             /* kernels launched by this handle so far */

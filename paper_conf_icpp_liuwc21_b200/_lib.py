@@ -17,7 +17,7 @@ PSO_ERR_NCCL, PSO_ERR_UNSUPPORTED, PSO_ERR_POISONED = 4, 5, 6
 PSO_OBJ_SPHERE, PSO_OBJ_RASTRIGIN, PSO_OBJ_ROSENBROCK = 1, 2, 3
 PSO_OBJ_GRIEWANK, PSO_OBJ_ACKLEY, PSO_OBJ_EASOM, PSO_OBJ_CUSTOM_BASE = 4, 5, 6, 64
 PSO_FLAG_TIMING = 1
-PSO_D_MAX = 8192
+PSO_D_MAX = 65536
 
 # every symbol include/fastpso.h declares
 EXPORTS = (
@@ -40,7 +40,7 @@ class pso_info(C.Structure):
         ("d", C.c_int32), ("pitch", C.c_int32), ("rank", C.c_int32), ("world", C.c_int32),
         ("threads_per_cta", C.c_int32), ("vec_per_thread", C.c_int32), ("grid", C.c_int32),
         ("ctas_per_sm", C.c_int32), ("tma_pipeline", C.c_int32), ("pipeline_stages", C.c_int32),
-        ("smem_bytes", C.c_int32), ("resident", C.c_int32), ("bounds", C.c_int32),
+        ("smem_bytes", C.c_int32), ("resident", C.c_int32), ("bounds", C.c_int32), ("cluster", C.c_int32),
         ("vmax", C.c_float), ("t", C.c_uint64),
         ("launches", C.c_uint64), ("improvements", C.c_uint64),
         ("step_kernel_ms", C.c_double), ("step_kernel_count", C.c_uint64),

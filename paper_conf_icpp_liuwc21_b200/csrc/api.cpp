@@ -405,6 +405,7 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
   if (const char* v = std::getenv("PSO_VPT")) hints.vpt = std::atoi(v);
   if (const char* v = std::getenv("PSO_STAGES")) hints.stages = std::atoi(v);
   if (const char* v = std::getenv("PSO_CTAS")) hints.ctas = std::atoi(v);
+  if (const char* v = std::getenv("PSO_CLUSTER")) hints.cluster = std::atoi(v);
   if (const char* v = std::getenv("PSO_KERNEL")) {
     if (!std::strcmp(v, "reg")) hints.kernel = 0;
     if (!std::strcmp(v, "tma")) hints.kernel = 1;
@@ -641,6 +642,7 @@ pso_status pso_get_info(pso_handle h, pso_info* info) {
   info->smem_bytes = (int32_t)(h->cfg.resident ? h->cfg.resident_smem : h->cfg.smem);
   info->resident = h->cfg.resident ? 1 : (h->cfg.gridres ? 2 : 0);
   info->bounds = h->args.bounds ? 1 : 0;
+  info->cluster = h->cfg.cluster;
   if (h->cfg.resident) {
     info->threads_per_cta = h->cfg.resident_threads;
     info->grid = 1;

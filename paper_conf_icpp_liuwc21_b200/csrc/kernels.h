@@ -56,6 +56,10 @@ struct LaunchCfg {
   size_t smem = 0;    // dynamic shared memory bytes of the step kernel
   int resident = 0;   // 1: tiny swarm, whole pso_step in one single-CTA launch
   int gridres = 0;    // 1: swarm held in the grid's shared memory (cooperative launch)
+  int cluster = 0;    // > 0: rows split across a thread-block cluster of this many CTAs
+  int chunk = 0;      // float4 per CTA block in the cluster path
+  int init_threads = 0;
+  int init_vpt = 1;
   int gridres_grid = 0;
   int gridres_rows = 0;     // max rows per CTA
   size_t gridres_smem = 0;
@@ -73,6 +77,7 @@ struct PlanHints {
   int ctas = 0;     // max CTAs per SM for the TMA pipeline (0: auto = 2)
   bool allow_resident = false;  // single-GPU tiny swarms (PSO_RESIDENT=0 disables)
   bool bounds = false;          // per-dimension bounds tables are in use
+  int cluster = 0;              // force the cluster path with this many CTAs (PSO_CLUSTER)
 };
 
 // Kernel entry points of one objective functor: [VPT index 1,2,4,8][per-dim bounds].
@@ -81,6 +86,7 @@ struct KernelTable {
   const void* step_reg[4][2];
   const void* step_tma[4][2];
   const void* gridres[4][2];
+  const void* step_cluster[4][2];
   const void* resident[2];
   const void* init[4];
   const void* eval[4];

@@ -105,11 +105,6 @@ const void* kernel_for(int objective, Which w, int vpt, bool bounds, bool* neigh
   }
 }
 
-const void* resident_kernel_for(int objective, bool bounds) {
-  const KernelTable* t = kernel_table(objective);
-  return t ? t->resident[bounds ? 1 : 0] : nullptr;
-}
-
 // CTA shape for a row of nvec float4: the smallest VPT in {1,2,4,8} whose
 // thread count fits 256, threads rounded up to a warp multiple.
 void shape_for(int nvec, int vpt_override, int* vpt, int* threads) {
@@ -141,25 +136,101 @@ bool objective_registered(int objective) {
   return kernel_for(objective, Which::Init, 1, false, &nb) != nullptr;
 }
 
+namespace {
+
+// Ring depth for stages of `stage_bytes` next to `fixed` bytes, at `ctas` CTAs per SM.
+int ring_stages(size_t fixed, size_t stage_bytes, int ctas) {
+  size_t budget = kSmemPerSm / ctas - kStaticReserve;
+  if (budget > kSmemPerCtaMax - kStaticReserve) budget = kSmemPerCtaMax - kStaticReserve;
+  return budget > fixed ? (int)((budget - fixed) / stage_bytes) : 0;
+}
+
+// Cluster path (NEXT-3): rows of more than 2048 float4 (d > 8192), or forced.
+cudaError_t plan_cluster(const KernelTable* t, int nvec, long long n_local, const PlanHints& h,
+                         LaunchCfg* cfg) {
+  int C = h.cluster > 0 ? h.cluster : 2;
+  if (h.cluster <= 0)
+    while (C < 16 && (nvec + C - 1) / C > 1024) C *= 2;
+  const int chunk = (nvec + C - 1) / C;
+  if (C < 2 || C > 16 || (C & (C - 1)) || chunk > 2048) return cudaErrorInvalidConfiguration;
+  int vpt, compute;
+  shape_for(chunk, h.vpt, &vpt, &compute);
+  const void* fn = t->step_cluster[vpt_index(vpt)][h.bounds ? 1 : 0];
+  const size_t crow = (size_t)chunk * 16, btab = h.bounds ? 4 * crow : 0;
+  int stages = ring_stages(crow + btab, 3 * crow, 1);
+  if (h.stages >= 2 && h.stages < stages) stages = h.stages;
+  if (stages > kMaxStages) stages = kMaxStages;
+  if (stages < 2) return cudaErrorInvalidConfiguration;
+  const size_t smem = crow + btab + (size_t)stages * 3 * crow;
+  cudaError_t e;
+  if (C > 8 &&
+      (e = cudaFuncSetAttribute(fn, cudaFuncAttributeNonPortableClusterSizeAllowed, 1)) != cudaSuccess)
+    return e;
+  if ((e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem)) !=
+      cudaSuccess)
+    return e;
+  cudaLaunchConfig_t lc{};
+  lc.gridDim = dim3(C);
+  lc.blockDim = dim3(compute + 64);
+  lc.dynamicSmemBytes = smem;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeClusterDimension;
+  attr[0].val.clusterDim.x = C;
+  attr[0].val.clusterDim.y = 1;
+  attr[0].val.clusterDim.z = 1;
+  lc.attrs = attr;
+  lc.numAttrs = 1;
+  int ncl = 0;
+  if ((e = cudaOccupancyMaxActiveClusters(&ncl, fn, &lc)) != cudaSuccess) return e;
+  if (ncl < 1) return cudaErrorInvalidConfiguration;
+  long long clusters = ncl < n_local ? ncl : n_local;
+  cfg->cluster = C;
+  cfg->chunk = chunk;
+  cfg->vpt = vpt;
+  cfg->compute = compute;
+  cfg->threads = compute + 64;
+  cfg->tma = 1;
+  cfg->stages = stages;
+  cfg->smem = smem;
+  cfg->grid = (int)(clusters * C);
+  cfg->ctas_per_sm = 1;
+  return cudaSuccess;
+}
+
+}  // namespace
+
 cudaError_t plan_launch(int objective, int d, long long n_local, int sm_count, const PlanHints& h,
                         LaunchCfg* cfg) {
+  const KernelTable* tab = kernel_table(objective);
+  if (!tab) return cudaErrorInvalidDeviceFunction;
+  const bool nb = tab->neighbor;
   const int nvec = (d + 3) / 4;
-  shape_for(nvec, h.vpt, &cfg->vpt, &cfg->compute);
-  bool nb = false;
-  if (!kernel_for(objective, Which::Init, cfg->vpt, false, &nb)) return cudaErrorInvalidDeviceFunction;
   const size_t row = (size_t)nvec * 16;
   const size_t btab = h.bounds ? 4 * row : 0;  // per-dimension bounds table in shared memory
-  cfg->bounds = h.bounds ? 1 : 0;
   const size_t first = nb ? (size_t)nvec * 4 : 0;
-  cfg->init_smem = first;
+  cfg->bounds = h.bounds ? 1 : 0;
+  cfg->init_smem = 0;
+  cfg->resident = cfg->gridres = cfg->cluster = 0;
   cudaError_t e;
 
+  // init kernel: one CTA per row, looping over the row's float4s
+  {
+    int iv, it;
+    shape_for(nvec <= 2048 ? nvec : 2048, 0, &iv, &it);
+    cfg->init_vpt = iv;
+    cfg->init_threads = it;
+  }
+
+  // ---- wide rows: thread-block cluster per row
+  if (nvec > 2048 || h.cluster > 0) return plan_cluster(tab, nvec, n_local, h, cfg);
+  shape_for(nvec, h.vpt, &cfg->vpt, &cfg->compute);
+  const int vi = vpt_index(cfg->vpt), bi = h.bounds ? 1 : 0;
+
   // ---- resident single-CTA path for tiny swarms (single GPU only)
-  cfg->resident = 0;
   if (h.allow_resident && nvec <= 32 && n_local * nvec * 4 <= kResidentElems) {
     const size_t smem =
         (size_t)n_local * nvec * 16 * 3 + (size_t)nvec * 16 + btab + (size_t)n_local * 4;
-    const void* fn = resident_kernel_for(objective, h.bounds);
+    const void* fn = tab->resident[bi];
     if (smem <= kSmemPerCtaMax - kStaticReserve &&
         cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) ==
             cudaSuccess) {
@@ -175,10 +246,10 @@ cudaError_t plan_launch(int objective, int d, long long n_local, int sm_count, c
     cudaGetLastError();
   }
 
-  // ---- TMA pipeline: rows of >= 256 dims unless forced otherwise
+  // ---- streaming kernels: TMA pipeline for rows of >= 256 dims unless forced
   bool tma = h.kernel == 1 || (h.kernel == -1 && nvec >= 64);
   if (tma) {
-    const void* fn = kernel_for(objective, Which::StepTma, cfg->vpt, h.bounds, &nb);
+    const void* fn = tab->step_tma[vi][bi];
     const int threads = cfg->compute + 64;  // + producer warp + finaliser warp
     // CTAs per SM the registers allow, capped at 2; the ring fills the rest.
     int by_regs = 0;
@@ -189,25 +260,20 @@ cudaError_t plan_launch(int objective, int d, long long n_local, int sm_count, c
     // The most CTAs per SM (<= cap) that still keep >= 3 rows in flight per
     // CTA; two rows only if nothing else fits (measured: 2-stage rings leave
     // HBM idle between rows, 3-4 stages saturate it).
-    auto stages_for = [&](int c) -> int {
-      size_t budget = kSmemPerSm / c - kStaticReserve;
-      if (budget > kSmemPerCtaMax - kStaticReserve) budget = kSmemPerCtaMax - kStaticReserve;
-      return budget > row + btab ? (int)((budget - row - btab) / (3 * row)) : 0;
-    };
-    int stages = 0;
     int c = ctas;
     for (; c >= 1; --c)
-      if (stages_for(c) >= 3) break;
+      if (ring_stages(row + btab, 3 * row, c) >= 3) break;
     if (c >= 1) {
       ctas = c;
     } else {
-      for (c = ctas; c >= 1 && stages_for(c) < 2; --c) {
+      for (c = ctas; c >= 1 && ring_stages(row + btab, 3 * row, c) < 2; --c) {
       }
       ctas = c < 1 ? 1 : c;
     }
-    stages = stages_for(ctas);
+    int stages = ring_stages(row + btab, 3 * row, ctas);
     if (h.stages >= 2 && h.stages <= kMaxStages) stages = stages < h.stages ? stages : h.stages;
     if (stages > kMaxStages) stages = kMaxStages;
+    tma = false;
     if (stages >= 2) {
       const size_t smem = row + btab + (size_t)stages * 3 * row;
       if ((e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem)) !=
@@ -218,20 +284,17 @@ cudaError_t plan_launch(int objective, int d, long long n_local, int sm_count, c
           cudaSuccess)
         return e;
       if (per_sm >= 1) {
+        tma = true;
         cfg->tma = 1;
         cfg->stages = stages;
         cfg->threads = threads;
         cfg->smem = smem;
         cfg->ctas_per_sm = per_sm;
-      } else {
-        tma = false;
       }
-    } else {
-      tma = false;
     }
   }
   if (!tma) {
-    const void* fn = kernel_for(objective, Which::StepReg, cfg->vpt, h.bounds, &nb);
+    const void* fn = tab->step_reg[vi][bi];
     cfg->tma = 0;
     cfg->stages = 0;
     cfg->threads = cfg->compute;
@@ -251,9 +314,8 @@ cudaError_t plan_launch(int objective, int d, long long n_local, int sm_count, c
   cfg->grid = (int)grid;
 
   // ---- grid-resident path: the whole swarm in the grid's shared memory
-  cfg->gridres = 0;
   if (h.allow_resident && !cfg->resident && cfg->tma && nvec >= 64) {
-    const void* fn = kernel_for(objective, Which::GridRes, cfg->vpt, h.bounds, &nb);
+    const void* fn = tab->gridres[vi][bi];
     for (int per = 2; per >= 1 && !cfg->gridres; --per) {
       long long g = (long long)per * sm_count;
       if (g > n_local) g = n_local;
@@ -282,40 +344,58 @@ cudaError_t plan_launch(int objective, int d, long long n_local, int sm_count, c
 }
 
 cudaError_t launch_step(int objective, const SwarmArgs& a, const LaunchCfg& c, cudaStream_t s) {
-  bool nb = false;
-  const void* fn = kernel_for(objective, c.tma ? Which::StepTma : Which::StepReg, c.vpt, c.bounds != 0, &nb);
-  if (!fn) return cudaErrorInvalidDeviceFunction;
+  const KernelTable* t = kernel_table(objective);
+  if (!t) return cudaErrorInvalidDeviceFunction;
+  const int vi = vpt_index(c.vpt), bi = c.bounds ? 1 : 0;
   int stages = c.stages;
+  if (c.cluster) {
+    int C = c.cluster, chunk = c.chunk;
+    void* args[] = {const_cast<SwarmArgs*>(&a), &stages, &C, &chunk};
+    cudaLaunchConfig_t lc{};
+    lc.gridDim = dim3(c.grid);
+    lc.blockDim = dim3(c.threads);
+    lc.dynamicSmemBytes = c.smem;
+    lc.stream = s;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeClusterDimension;
+    attr[0].val.clusterDim.x = C;
+    attr[0].val.clusterDim.y = 1;
+    attr[0].val.clusterDim.z = 1;
+    lc.attrs = attr;
+    lc.numAttrs = 1;
+    return cudaLaunchKernelExC(&lc, t->step_cluster[vi][bi], args);
+  }
+  const void* fn = c.tma ? t->step_tma[vi][bi] : t->step_reg[vi][bi];
   void* args[] = {const_cast<SwarmArgs*>(&a), &stages};
   return cudaLaunchKernel(fn, dim3(c.grid), dim3(c.threads), args, c.smem, s);
 }
 
 cudaError_t launch_resident(int objective, const SwarmArgs& a, const LaunchCfg& c, int iters,
                             cudaStream_t s) {
-  const void* fn = resident_kernel_for(objective, c.bounds != 0);
-  if (!fn) return cudaErrorInvalidDeviceFunction;
+  const KernelTable* t = kernel_table(objective);
+  if (!t) return cudaErrorInvalidDeviceFunction;
   void* args[] = {const_cast<SwarmArgs*>(&a), &iters};
-  return cudaLaunchKernel(fn, dim3(1), dim3(c.resident_threads), args, c.resident_smem, s);
+  return cudaLaunchKernel(t->resident[c.bounds ? 1 : 0], dim3(1), dim3(c.resident_threads), args,
+                          c.resident_smem, s);
 }
 
 cudaError_t launch_gridres(int objective, const SwarmArgs& a, const LaunchCfg& c, int iters,
                            cudaStream_t s) {
-  bool nb = false;
-  const void* fn = kernel_for(objective, Which::GridRes, c.vpt, c.bounds != 0, &nb);
-  if (!fn) return cudaErrorInvalidDeviceFunction;
+  const KernelTable* t = kernel_table(objective);
+  if (!t) return cudaErrorInvalidDeviceFunction;
   void* args[] = {const_cast<SwarmArgs*>(&a), &iters};
-  return cudaLaunchCooperativeKernel(fn, dim3(c.gridres_grid), dim3(c.compute), args,
-                                     c.gridres_smem, s);
+  return cudaLaunchCooperativeKernel(t->gridres[vpt_index(c.vpt)][c.bounds ? 1 : 0],
+                                     dim3(c.gridres_grid), dim3(c.compute), args, c.gridres_smem, s);
 }
 
 cudaError_t launch_init(int objective, const SwarmArgs& a, const LaunchCfg& c, cudaStream_t s) {
-  bool nb = false;
-  const void* fn = kernel_for(objective, Which::Init, c.vpt, false, &nb);
-  if (!fn) return cudaErrorInvalidDeviceFunction;
+  const KernelTable* t = kernel_table(objective);
+  if (!t) return cudaErrorInvalidDeviceFunction;
   long long grid = a.n_local < 4LL * 148 * 2 ? a.n_local : 4LL * 148 * 2;
   if (grid < 1) grid = 1;
   void* args[] = {const_cast<SwarmArgs*>(&a)};
-  return cudaLaunchKernel(fn, dim3((unsigned)grid), dim3(c.compute), args, c.init_smem, s);
+  return cudaLaunchKernel(t->init[vpt_index(c.init_vpt)], dim3((unsigned)grid),
+                          dim3(c.init_threads), args, 0, s);
 }
 
 cudaError_t launch_rebest(const SwarmArgs& a, unsigned t, cudaStream_t s) {
@@ -335,15 +415,14 @@ cudaError_t debug_objective(int objective, const float* X_dev, long long m, int 
                             float* out_dev, int sm_count, cudaStream_t s) {
   const int nvec = pitch / 4;
   int vpt, threads;
-  shape_for(nvec, 0, &vpt, &threads);
+  shape_for(nvec <= 2048 ? nvec : 2048, 0, &vpt, &threads);
   bool nb = false;
   const void* fn = kernel_for(objective, Which::Eval, vpt, false, &nb);
   if (!fn) return cudaErrorInvalidDeviceFunction;
   long long grid = m < (long long)sm_count * 4 ? m : (long long)sm_count * 4;
   if (grid < 1) grid = 1;
   void* args[] = {(void*)&X_dev, (void*)&m, (void*)&d, (void*)&nvec, (void*)&out_dev};
-  return cudaLaunchKernel(fn, dim3((unsigned)grid), dim3(threads), args, nb ? (size_t)nvec * 4 : 0,
-                          s);
+  return cudaLaunchKernel(fn, dim3((unsigned)grid), dim3(threads), args, 0, s);
 }
 
 }  // namespace fastpso

@@ -136,6 +136,41 @@ __device__ __forceinline__ void fence_proxy_async_global() {
   asm volatile("fence.proxy.async.global;" ::: "memory");
 }
 
+// --- thread-block clusters: DSMEM stores and remote mbarrier arrivals -----
+__device__ __forceinline__ uint32_t cluster_rank() {
+  uint32_t r;
+  asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+  return r;
+}
+__device__ __forceinline__ void cluster_sync_all() {
+  asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::
+                   : "memory");
+}
+// Address of `p` (this CTA's shared memory) in the shared window of CTA `rank`.
+__device__ __forceinline__ uint32_t map_to_rank(const void* p, uint32_t rank) {
+  uint32_t r;
+  asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(smem_addr(p)), "r"(rank));
+  return r;
+}
+__device__ __forceinline__ void st_cluster_f32(uint32_t addr, float v) {
+  asm volatile("st.shared::cluster.f32 [%0], %1;" ::"r"(addr), "f"(v) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_remote(uint32_t bar_addr) {
+  asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(bar_addr)
+               : "memory");
+}
+__device__ __forceinline__ void mbar_wait_cluster(unsigned long long* bar, unsigned phase) {
+  asm volatile(
+      "{\n"
+      ".reg .pred p;\n"
+      "WAITC_%=:\n"
+      "mbarrier.try_wait.parity.acquire.cluster.shared::cta.b64 p, [%0], %1;\n"
+      "@!p bra WAITC_%=;\n"
+      "}\n" ::"r"(smem_addr(bar)),
+      "r"(phase)
+      : "memory");
+}
+
 // --- Eq. 1, 5, 2 on one element, fixed fp32 order, no contraction --------
 // The oracle computes b = (c1 * r1) * (pb - x) with r1 = m 2^-24 (m the 24-bit
 // Philox integer).  Here c1s = c1 2^-24 is folded once per kernel, and
@@ -682,6 +717,248 @@ __global__ void __launch_bounds__(kMaxThreads + 64, 2)
   }
 }
 
+// ------------------------------------------------- step kernel: cluster (wide rows)
+// NEXT-3 within one GPU (the paper's "tile matrix" split, applied to a
+// row): a thread-block cluster of C CTAs owns a row at a time, CTA k the
+// column block [k chunk, (k+1) chunk) of float4s.  Each CTA is a k_step_tma
+// pipeline on its block (producer / compute / finaliser warps, bulk copies of
+// the block of x, v, pb, G and bounds).  Per row the C finalisers publish
+// their block partial (and, for neighbour functors, the block's first and
+// last x') into CTA 0's shared memory (DSMEM stores + remote mbarrier
+// arrivals); CTA 0 combines the blocks in rank order, adds the terms that
+// straddle block boundaries, decides the pbest update and sends the decision
+// back to every CTA, which then bulk-stores its block of x', v' (and pb).
+template <class Obj, int VPT, bool kB>
+__global__ void __launch_bounds__(kMaxThreads + 64, 1)
+    k_step_cluster(const SwarmArgs a, int stages, int C, int chunk) {
+  extern __shared__ __align__(128) unsigned char dsmem[];
+  constexpr int kSlot = Obj::kAcc + 2;  // partial accumulators, first x', last x'
+  const int nvec = a.nvec, d = a.d;
+  const int nthr = (int)blockDim.x - 64;
+  const int nwarps = nthr >> 5;
+  const int crank = (int)cluster_rank();
+  const int cid = blockIdx.x / C, ncl = gridDim.x / C;
+  const int q0 = crank * chunk;
+  const int cnt = max(0, min(chunk, nvec - q0));  // float4s of this CTA's block
+  const bool row_tail = q0 + cnt < nvec;            // a later block follows
+  float4* sG = reinterpret_cast<float4*>(dsmem);
+  float4* sB = sG + chunk;
+  float4* ring = sB + (kB ? 4 * chunk : 0);
+  __shared__ float red[kMaxStages][(kMaxThreads / 32) * 2];
+  __shared__ float parts[kMaxStages][16 * kSlot];  // CTA 0: block partials by rank
+  __shared__ float dec[kMaxStages][2];             // every CTA: {improved, f}
+  __shared__ unsigned long long full[kMaxStages], empty[kMaxStages], done[kMaxStages];
+  __shared__ unsigned long long pbar[kMaxStages], dbar[kMaxStages], gbar;
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  if (tid == 0) {
+    mbar_init(&gbar, 1);
+    for (int s = 0; s < stages; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&done[s], (unsigned)nwarps);
+      mbar_init(&empty[s], 1);
+      mbar_init(&pbar[s], (unsigned)C);
+      mbar_init(&dbar[s], 1);
+    }
+    mbar_fence_init();
+  }
+  __syncthreads();
+  cluster_sync_all();  // every CTA's barriers exist before any remote arrival
+  const uint32_t t = a.ctl->t + 1u;
+  const unsigned blk_bytes = (unsigned)cnt * 16u;
+
+  if (warp == nwarps) {  // ---------------- producer
+    if (lane == 0) {
+      mbar_expect_tx(&gbar, blk_bytes * (kB ? 5u : 1u));
+      if (cnt > 0) {
+        bulk_g2s(sG, a.G + (size_t)q0 * 4, blk_bytes, &gbar);
+        if (kB)
+          for (int k = 0; k < 4; ++k)
+            bulk_g2s(sB + k * chunk, a.bounds + ((size_t)k * nvec + q0) * 4, blk_bytes, &gbar);
+      }
+      int s = 0;
+      unsigned ph = 0;
+      int k = 0;
+      for (long long r = cid; r < a.n_local; r += ncl, ++k) {
+        if (k >= stages) mbar_wait(&empty[s], ph ^ 1u);
+        float4* st = ring + (size_t)s * 3 * chunk;
+        mbar_expect_tx(&full[s], 3u * blk_bytes);
+        if (cnt > 0) {
+          const size_t off = ((size_t)r * nvec + q0) * 4;
+          bulk_g2s(st, a.X + off, blk_bytes, &full[s]);
+          bulk_g2s(st + chunk, a.V + off, blk_bytes, &full[s]);
+          bulk_g2s(st + 2 * chunk, a.PB + off, blk_bytes, &full[s]);
+        }
+        if (++s == stages) {
+          s = 0;
+          ph ^= 1u;
+        }
+      }
+    }
+    return;
+  }
+
+  if (warp == nwarps + 1) {  // ---------------- finaliser
+    __shared__ int s_last;
+    if (lane == 0) {
+      const uint32_t inc_ord = (uint32_t)(a.ctl->key_cur >> 32);
+      unsigned long long best = ~0ull;
+      unsigned nimp = 0;
+      int s = 0, prev = -1;
+      unsigned ph = 0;
+      for (long long r = cid; r < a.n_local; r += ncl) {
+        const uint32_t gi = (uint32_t)(a.row_begin + r);
+        const float pf_old = crank == 0 ? a.pf[r] : 0.f;
+        mbar_wait(&done[s], ph);
+        float c[Obj::kAcc];
+        Obj::init(c);
+        for (int w = 0; w < nwarps; ++w) {
+          float b[Obj::kAcc];
+#pragma unroll
+          for (int j = 0; j < Obj::kAcc; ++j) b[j] = red[s][w * Obj::kAcc + j];
+          Obj::combine(c, b);
+        }
+        const float4* st = ring + (size_t)s * 3 * chunk;
+        // publish {partial, first x', last x'} to CTA 0
+        const uint32_t slot = map_to_rank(&parts[s][crank * kSlot], 0);
+#pragma unroll
+        for (int j = 0; j < Obj::kAcc; ++j) st_cluster_f32(slot + 4u * j, c[j]);
+        if (Obj::kNeighbor && cnt > 0) {
+          st_cluster_f32(slot + 4u * Obj::kAcc, st[0].x);
+          st_cluster_f32(slot + 4u * (Obj::kAcc + 1), st[cnt - 1].w);
+        }
+        mbar_arrive_remote(map_to_rank(&pbar[s], 0));
+        if (crank == 0) {  // combine blocks in rank order, decide, broadcast
+          mbar_wait_cluster(&pbar[s], ph);
+          float tot[Obj::kAcc];
+          Obj::init(tot);
+          for (int k = 0; k < C; ++k) {
+            Obj::combine(tot, &parts[s][k * kSlot]);
+            const int qk = k * chunk, ck = min(chunk, nvec - qk);
+            if (Obj::kNeighbor && k + 1 < C && ck > 0 && qk + ck < nvec) {
+              float bterm[Obj::kAcc];
+              Obj::init(bterm);
+              const int jl = 4 * (qk + ck) - 1;  // last dim of block k
+              Obj::map(bterm, parts[s][k * kSlot + Obj::kAcc + 1], parts[s][(k + 1) * kSlot + Obj::kAcc],
+                       jl, d);
+              Obj::combine(tot, bterm);
+            }
+          }
+          const float f = Obj::finalize(tot, d);
+          const float imp = (f < pf_old) ? 1.f : 0.f;  // strict; NaN never improves
+          for (int k = 0; k < C; ++k) {
+            st_cluster_f32(map_to_rank(&dec[s][0], k), imp);
+            st_cluster_f32(map_to_rank(&dec[s][1], k), f);
+            mbar_arrive_remote(map_to_rank(&dbar[s], k));
+          }
+          if (imp != 0.f) {
+            a.pf[r] = f;
+            ++nimp;
+          }
+          if (f == f && ord_f32(f) < inc_ord) {  // strictly below gf
+            const unsigned long long key = pack_key(f, gi);
+            best = key < best ? key : best;
+          }
+        }
+        mbar_wait_cluster(&dbar[s], ph);
+        const bool improved = dec[s][0] != 0.f;
+        if (cnt > 0) {
+          const size_t off = ((size_t)r * nvec + q0) * 4;
+          bulk_s2g(a.X + off, st, blk_bytes);
+          bulk_s2g(a.V + off, st + chunk, blk_bytes);
+          if (improved) bulk_s2g(a.PB + off, st, blk_bytes);
+        }
+        bulk_commit();
+        if (prev >= 0) {
+          bulk_wait_read<1>();
+          mbar_arrive(&empty[prev]);
+        }
+        prev = s;
+        if (++s == stages) {
+          s = 0;
+          ph ^= 1u;
+        }
+      }
+      bulk_wait_all();
+      fence_proxy_async_global();
+      if (best != ~0ull) atomicMin(&a.ctl->key_acc, best);
+      if (nimp) atomicAdd(&a.ctl->improvements, (unsigned long long)nimp);
+      __threadfence();
+      s_last = (atomicAdd(&a.ctl->done, 1u) == gridDim.x - 1) ? 1 : 0;
+    }
+    __syncwarp();
+    if (s_last) warp_gbest_epilogue(a, t, lane);
+    return;
+  }
+
+  // ---------------- compute warps
+  const PhiloxKey key{a.seed_lo, a.seed_hi};
+  const MoveParams mp = move_params(a);
+  mbar_wait(&gbar, 0);
+  int s = 0;
+  unsigned ph = 0;
+  for (long long r = cid; r < a.n_local; r += ncl) {
+    const uint32_t gi = (uint32_t)(a.row_begin + r);
+    float4* st = ring + (size_t)s * 3 * chunk;
+    mbar_wait(&full[s], ph);
+    float acc[Obj::kAcc];
+    Obj::init(acc);
+#pragma unroll(VPT <= 2 ? VPT : 2)
+    for (int j = 0; j < VPT; ++j) {
+      const int ql = tid + j * nthr;
+      if (ql < cnt) {
+        const int q = q0 + ql;
+        float4 x = st[ql], v = st[chunk + ql];
+        const float4 pb = st[2 * chunk + ql];
+        const float4 g = sG[ql];
+        const float4 r1 = raw24x4(key, kTagR1, t, gi, (uint32_t)q);
+        const float4 r2 = raw24x4(key, kTagR2, t, gi, (uint32_t)q);
+        move4<kB>(mp, x, v, pb, g, r1, r2, sB, chunk, ql);
+        if ((d & 3) && q == nvec - 1) {
+          const int jj = 4 * q;
+          if (jj + 1 >= d) x.y = v.y = 0.f;
+          if (jj + 2 >= d) x.z = v.z = 0.f;
+          if (jj + 3 >= d) x.w = v.w = 0.f;
+        }
+        st[ql] = x;
+        st[chunk + ql] = v;
+        if constexpr (!Obj::kNeighbor) map4<Obj>(acc, x, 0.f, 4 * q, d);
+      }
+    }
+    if constexpr (Obj::kNeighbor) {
+      team_sync(nthr);  // every x' of the block is in the stage
+#pragma unroll(VPT <= 2 ? VPT : 2)
+      for (int j = 0; j < VPT; ++j) {
+        const int ql = tid + j * nthr;
+        if (ql < cnt) {
+          const int q = q0 + ql;
+          const float4 x = st[ql];
+          if (ql + 1 < cnt) {
+            map4<Obj>(acc, x, st[ql + 1].x, 4 * q, d);
+          } else if (!row_tail) {
+            map4<Obj>(acc, x, 0.f, 4 * q, d);  // the row's last float4
+          } else {  // x_{j+1} of the last dim lives in the next block: CTA 0 adds it
+            Obj::map(acc, x.x, x.y, 4 * q, d);
+            Obj::map(acc, x.y, x.z, 4 * q + 1, d);
+            Obj::map(acc, x.z, x.w, 4 * q + 2, d);
+          }
+        }
+      }
+    }
+    warp_combine<Obj>(acc);
+    if (lane == 0) {
+#pragma unroll
+      for (int j = 0; j < Obj::kAcc; ++j) red[s][warp * Obj::kAcc + j] = acc[j];
+    }
+    fence_proxy_async_shared();
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&done[s]);
+    if (++s == stages) {
+      s = 0;
+      ph ^= 1u;
+    }
+  }
+}
+
 // ------------------------------------------------- resident kernel (small swarms)
 // NEXT-1 latency path: for tiny swarms (d <= 128, n d <= 8192)
 // one CTA keeps X, V, PB, pf and G in shared memory for all `iters`
@@ -1036,19 +1313,53 @@ __global__ void __launch_bounds__(kMaxThreads, 1) k_gridres(const SwarmArgs a, i
 }
 
 // ------------------------------------------------------------ init kernel
-// Alg. 1 lines 1-3 (Sec 3.1): x0 = clamp(lo + span U, lo, hi), v0 = -vmax +
-// 2 vmax U from the X0 / V0 streams at t = 0; f = F(x0); pf = f (NaN -> +inf);
-// PB = x0; every row is a gbest candidate (key_cur = ~0 on entry).
+// Alg. 1 lines 1-3 (Sec 3.1): x0 = clamp(xlo + (xhi - xlo) U, xlo, xhi), v0 =
+// vlo + (vhi - vlo) U from the X0 / V0 streams at t = 0 (scalar bounds: xlo =
+// lo, xhi = hi, vlo = -vmax, vhi = vmax); f = F(x0); pf = f (NaN -> +inf);
+// PB = x0; every row is a gbest candidate (key_cur = ~0 on entry).  Thread t
+// handles float4 t, t + nthr, ... of a row (any d; the same accumulation
+// order as the register kernels); a neighbour functor's x_{j+1} across a
+// float4 boundary is recomputed from its Philox word.
+__device__ __forceinline__ void init_float4(const SwarmArgs& a, PhiloxKey key, uint32_t gi, int q,
+                                            float4& xo, float4& vo) {
+  const int nvec = a.nvec, d = a.d;
+  const float4* B4 = reinterpret_cast<const float4*>(a.bounds);  // null: scalar bounds
+  const float4 ux = uniforms4(key, kTagX0, 0u, gi, (uint32_t)q);
+  const float4 uv = uniforms4(key, kTagV0, 0u, gi, (uint32_t)q);
+  float xs[4] = {ux.x, ux.y, ux.z, ux.w};
+  float vs[4] = {uv.x, uv.y, uv.z, uv.w};
+  float4 vlo4 = make_float4(-a.vmax, -a.vmax, -a.vmax, -a.vmax);
+  float4 vhi4 = make_float4(a.vmax, a.vmax, a.vmax, a.vmax);
+  float4 xlo4 = make_float4(a.lo, a.lo, a.lo, a.lo), xhi4 = make_float4(a.hi, a.hi, a.hi, a.hi);
+  if (B4) {
+    vlo4 = B4[q];
+    vhi4 = B4[nvec + q];
+    xlo4 = B4[2 * nvec + q];
+    xhi4 = B4[3 * nvec + q];
+  }
+  const float vlo[4] = {vlo4.x, vlo4.y, vlo4.z, vlo4.w};
+  const float vhi[4] = {vhi4.x, vhi4.y, vhi4.z, vhi4.w};
+  const float xlo[4] = {xlo4.x, xlo4.y, xlo4.z, xlo4.w};
+  const float xhi[4] = {xhi4.x, xhi4.y, xhi4.z, xhi4.w};
+#pragma unroll
+  for (int e = 0; e < 4; ++e) {
+    const bool pad = 4 * q + e >= d;
+    const float span = __fsub_rn(xhi[e], xlo[e]);
+    const float vspan = __fsub_rn(vhi[e], vlo[e]);
+    xs[e] = pad ? 0.f : fminf(fmaxf(__fadd_rn(xlo[e], __fmul_rn(span, xs[e])), xlo[e]), xhi[e]);
+    vs[e] = pad ? 0.f : __fadd_rn(vlo[e], __fmul_rn(vspan, vs[e]));
+  }
+  xo = make_float4(xs[0], xs[1], xs[2], xs[3]);
+  vo = make_float4(vs[0], vs[1], vs[2], vs[3]);
+}
+
 template <class Obj, int VPT>
 __global__ void __launch_bounds__(kMaxThreads, (VPT >= 8) ? 1 : 2)
     k_init(const SwarmArgs a) {
-  extern __shared__ __align__(128) unsigned char dsmem[];
-  float* sFirst = reinterpret_cast<float*>(dsmem);
   __shared__ RowSmem<Obj> sm;
   const int tid = threadIdx.x, nthr = blockDim.x;
   const PhiloxKey key{a.seed_lo, a.seed_hi};
   const int nvec = a.nvec, d = a.d;
-  const float4* B4 = reinterpret_cast<const float4*>(a.bounds);  // null: scalar bounds
   const uint32_t inc_ord = (uint32_t)(a.ctl->key_cur >> 32);
   unsigned long long best = ~0ull;
   for (long long r = blockIdx.x; r < a.n_local; r += gridDim.x) {
@@ -1056,45 +1367,24 @@ __global__ void __launch_bounds__(kMaxThreads, (VPT >= 8) ? 1 : 2)
     float4* Xr = reinterpret_cast<float4*>(a.X) + r * nvec;
     float4* Vr = reinterpret_cast<float4*>(a.V) + r * nvec;
     float4* Pr = reinterpret_cast<float4*>(a.PB) + r * nvec;
-    float4 x[VPT];
-#pragma unroll
-    for (int s = 0; s < VPT; ++s) {
-      const int q = tid + s * nthr;
-      if (q < nvec) {
-        const float4 ux = uniforms4(key, kTagX0, 0u, gi, (uint32_t)q);
-        const float4 uv = uniforms4(key, kTagV0, 0u, gi, (uint32_t)q);
-        float xs[4] = {ux.x, ux.y, ux.z, ux.w};
-        float vs[4] = {uv.x, uv.y, uv.z, uv.w};
-        float4 vlo4 = make_float4(-a.vmax, -a.vmax, -a.vmax, -a.vmax);
-        float4 vhi4 = make_float4(a.vmax, a.vmax, a.vmax, a.vmax);
-        float4 xlo4 = make_float4(a.lo, a.lo, a.lo, a.lo), xhi4 = make_float4(a.hi, a.hi, a.hi, a.hi);
-        if (B4) {
-          vlo4 = B4[q];
-          vhi4 = B4[nvec + q];
-          xlo4 = B4[2 * nvec + q];
-          xhi4 = B4[3 * nvec + q];
-        }
-        const float vlo[4] = {vlo4.x, vlo4.y, vlo4.z, vlo4.w};
-        const float vhi[4] = {vhi4.x, vhi4.y, vhi4.z, vhi4.w};
-        const float xlo[4] = {xlo4.x, xlo4.y, xlo4.z, xlo4.w};
-        const float xhi[4] = {xhi4.x, xhi4.y, xhi4.z, xhi4.w};
-#pragma unroll
-        for (int e = 0; e < 4; ++e) {  // x0 = clamp(lo + (hi - lo) U), v0 = vlo + (vhi - vlo) U
-          const bool pad = 4 * q + e >= d;
-          const float span = __fsub_rn(xhi[e], xlo[e]);
-          const float vspan = __fsub_rn(vhi[e], vlo[e]);
-          xs[e] = pad ? 0.f : fminf(fmaxf(__fadd_rn(xlo[e], __fmul_rn(span, xs[e])), xlo[e]), xhi[e]);
-          vs[e] = pad ? 0.f : __fadd_rn(vlo[e], __fmul_rn(vspan, vs[e]));
-        }
-        x[s] = make_float4(xs[0], xs[1], xs[2], xs[3]);
-        st_stream(Xr + q, x[s]);
-        st_stream(Vr + q, make_float4(vs[0], vs[1], vs[2], vs[3]));
-        st_stream(Pr + q, x[s]);
-      }
-    }
     float acc[Obj::kAcc];
     Obj::init(acc);
-    map_row<Obj, VPT>(acc, x, sFirst, nvec, d, tid, nthr);
+    for (int q = tid; q < nvec; q += nthr) {
+      float4 x, v;
+      init_float4(a, key, gi, q, x, v);
+      st_stream(Xr + q, x);
+      st_stream(Vr + q, v);
+      st_stream(Pr + q, x);
+      float nx = 0.f;
+      if constexpr (Obj::kNeighbor) {
+        if (q + 1 < nvec) {
+          float4 xn, vn;
+          init_float4(a, key, gi, q + 1, xn, vn);
+          nx = xn.x;
+        }
+      }
+      map4<Obj>(acc, x, nx, 4 * q, d);
+    }
     bool improved;
     float f = cta_fitness<Obj>(acc, sm, d, 0.f, improved, tid, nthr);
     if (tid == 0) {
@@ -1110,30 +1400,26 @@ __global__ void __launch_bounds__(kMaxThreads, (VPT >= 8) ? 1 : 2)
 }
 
 // ---------------------------------------------------------- debug: objective
+// The functor + CTA reduction on given rows (any d; thread t maps float4 t,
+// t + nthr, ...).
 template <class Obj, int VPT>
 __global__ void __launch_bounds__(kMaxThreads) k_eval(const float* X, long long m, int d,
                                                       int nvec, float* out) {
-  extern __shared__ __align__(128) unsigned char dsmem[];
-  float* sFirst = reinterpret_cast<float*>(dsmem);
   __shared__ RowSmem<Obj> sm;
   const int tid = threadIdx.x, nthr = blockDim.x;
   for (long long r = blockIdx.x; r < m; r += gridDim.x) {
     const float4* Xr = reinterpret_cast<const float4*>(X) + r * nvec;
-    float4 x[VPT];
-#pragma unroll
-    for (int s = 0; s < VPT; ++s) {
-      const int q = tid + s * nthr;
-      if (q < nvec) x[s] = Xr[q];
-    }
     float acc[Obj::kAcc];
     Obj::init(acc);
-    map_row<Obj, VPT>(acc, x, sFirst, nvec, d, tid, nthr);
+    for (int q = tid; q < nvec; q += nthr) {
+      const float nx = (Obj::kNeighbor && q + 1 < nvec) ? Xr[q + 1].x : 0.f;
+      map4<Obj>(acc, Xr[q], nx, 4 * q, d);
+    }
     bool improved;
     const float f = cta_fitness<Obj>(acc, sm, d, 0.f, improved, tid, nthr);
     if (tid == 0) out[r] = f;
   }
 }
-
 
 template <class Obj>
 KernelTable make_kernel_table() {
@@ -1146,6 +1432,7 @@ KernelTable make_kernel_table() {
   PSO_ALLV(step_reg, k_step_reg)
   PSO_ALLV(step_tma, k_step_tma)
   PSO_ALLV(gridres, k_gridres)
+  PSO_ALLV(step_cluster, k_step_cluster)
 #undef PSO_ALLV
 #undef PSO_T
   t.resident[0] = (const void*)k_resident<Obj, false>;

@@ -58,7 +58,7 @@ def _create(n=10, d=10, w=0.9, c1=2.0, c2=2.0, lo=-1.0, hi=1.0, obj=1, seed=1, o
 
 
 @pytest.mark.parametrize("kw,status", [
-    (dict(n=0), 1), (dict(n=2**32), 1), (dict(d=0), 1), (dict(d=8193), 5),
+    (dict(n=0), 1), (dict(n=2**32), 1), (dict(d=0), 1), (dict(d=65537), 5),
     (dict(lo=1.0, hi=1.0), 1), (dict(lo=2.0, hi=1.0), 1), (dict(hi=float("inf")), 1),
     (dict(w=float("nan")), 1), (dict(c1=float("inf")), 1), (dict(obj=0), 1), (dict(obj=63), 1),
 ])

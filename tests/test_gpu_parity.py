@@ -258,7 +258,7 @@ def test_errors_do_not_abort():
         gpu_swarm(0, 10, SPHERE)
     assert e.value.status == 1
     with pytest.raises(fp.PsoError) as e:
-        gpu_swarm(10, 10000, SPHERE)
+        gpu_swarm(10, 70000, SPHERE)
     assert e.value.status == 5
     g = gpu_swarm(10, 10, SPHERE)
     with pytest.raises(fp.PsoError):
@@ -440,3 +440,57 @@ def test_set_bounds_requires_bounds_handle():
         bad[0, 3] = 5.0  # vlo > vhi
         gpu_swarm(10, 10, SPHERE, bounds=bad)
     assert e.value.status == 1
+
+
+# ------------------------------------------------------------------ wide rows (NEXT-3)
+WIDE = [(5, 8193), (3, 10000), (4, 16384), (2, 65536)]
+
+
+@pytest.mark.parametrize("obj", [SPHERE, RASTRIGIN, ROSENBROCK, GRIEWANK, ACKLEY])
+@pytest.mark.parametrize("n,d", WIDE)
+def test_wide_rows_cluster_path(obj, n, d):
+    """d > 8192: each row is split in column blocks over a thread-block cluster
+    (DSMEM partials, CTA 0 decides); init bit-exact, one step bit-exact in X/V."""
+    g = gpu_swarm(n, d, obj, seed=d + obj)
+    assert g.info()["cluster"] >= 2
+    c = cpu_swarm(n, d, obj, seed=d + obj)
+    X, V, PB, pf, _ = g.get_state()
+    assert_bitwise(X, c.X, "X0")
+    assert_bitwise(V, c.V, "V0")
+    assert_fitness_close(obj, c.X, pf, c.pf, "pf0")
+    _step_and_compare(obj, n, d, seed=5000 + d, pf_mode="mixed", t0=2)
+    _step_and_compare(obj, n, d, seed=5100 + d, pf_mode="inf", t0=0)
+
+
+@pytest.mark.parametrize("C", [2, 4, 8, 16])
+@pytest.mark.parametrize("obj,n,d", [(RASTRIGIN, 40, 1000), (ROSENBROCK, 33, 2001),
+                                     (GRIEWANK, 20, 999), (ACKLEY, 17, 4096)])
+def test_forced_cluster_split_matches_oracle(C, obj, n, d, monkeypatch):
+    monkeypatch.setenv("PSO_CLUSTER", str(C))
+    g, _ = _step_and_compare(obj, n, d, seed=6000 + C + d, pf_mode="mixed", t0=7)
+    assert g.info()["cluster"] == C
+    # several iterations: invariants and G == PB[gi]
+    lo, hi = DOMAINS[obj]
+    g.step(5)
+    X, V, PB, pf, _ = g.get_state()
+    gf, gi, G = g.gbest()
+    assert (X >= np.float32(lo)).all() and (X <= np.float32(hi)).all()
+    assert gf == pf.min() and gi == int(np.argmin(pf))
+    assert_bitwise(G, PB[gi], "G == PB[gi]")
+
+
+def test_wide_rows_with_bounds_and_lockstep(monkeypatch):
+    n, d, obj = 6, 12000, ROSENBROCK
+    b = _dim_bounds(d, 3)
+    lo, hi = DOMAINS[obj]
+    g = fp.Swarm(n, d, 0.9, 2.0, 2.0, lo, hi, obj, 21, device=0, bounds=b)
+    c = orc.OracleSwarm(n, d, 0.9, 2.0, 2.0, lo, hi, obj, 21, bounds=b)
+    for _ in range(4):
+        X, V, PB, pf, t = g.get_state()
+        c.set_state(X, V, PB, pf, t=t)
+        g.step(1)
+        c.step(1)
+        X2, V2, _, pf2, _ = g.get_state()
+        assert_bitwise(X2, c.X, "X")
+        assert_bitwise(V2, c.V, "V")
+        assert_fitness_close(obj, c.PB, pf2, c.pf, "pf")
