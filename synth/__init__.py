@@ -76,6 +76,9 @@ WORKLOADS = {
     # north_star target: >= 70% of HBM bandwidth on Rastrigin 100k x 2000 at 1 GPU
     "NS": Workload("northstar-rastrigin-100000x2000", RASTRIGIN, 100_000, 2000, 500,
                    gpus=(1, 2, 4, 8)),
+    # NEXT-3: rows wider than one CTA (d > 8192), split over a thread-block cluster
+    "W64K": Workload("wide-rastrigin-4096x65536", RASTRIGIN, 4096, 65536, 200),
+    "W16K": Workload("wide-griewank-16384x16384", GRIEWANK, 16384, 16384, 200),
     # the paper's own default experiment, for the Table 2 plausibility band
     "PAPER": Workload("paper-default-5000x200", SPHERE, 5000, 200, 2000),
 }
