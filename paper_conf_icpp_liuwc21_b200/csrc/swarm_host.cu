@@ -107,17 +107,17 @@ const void* kernel_for(int objective, Which w, int vpt, bool bounds, bool* neigh
 
 // CTA shape for a row of nvec float4: the smallest VPT in {1,2,4,8} whose
 // thread count fits 256, threads rounded up to a warp multiple.
-void shape_for(int nvec, int vpt_override, int* vpt, int* threads) {
+void shape_for(int nvec, int vpt_override, int* vpt, int* threads, int max_threads = kMaxThreads) {
   static const int kVpts[] = {1, 2, 4, 8};
   int v = 8;
   for (int c : kVpts) {
-    if ((nvec + c - 1) / c <= kMaxThreads) {
+    if ((nvec + c - 1) / c <= max_threads) {
       v = c;
       break;
     }
   }
   if (vpt_override == 1 || vpt_override == 2 || vpt_override == 4 || vpt_override == 8) {
-    if ((nvec + vpt_override - 1) / vpt_override <= kMaxThreads) v = vpt_override;
+    if ((nvec + vpt_override - 1) / vpt_override <= max_threads) v = vpt_override;
   }
   const int t = (nvec + v - 1) / v;
   *vpt = v;
@@ -154,7 +154,7 @@ cudaError_t plan_cluster(const KernelTable* t, int nvec, long long n_local, cons
   const int chunk = (nvec + C - 1) / C;
   if (C < 2 || C > 16 || (C & (C - 1)) || chunk > 2048) return cudaErrorInvalidConfiguration;
   int vpt, compute;
-  shape_for(chunk, h.vpt, &vpt, &compute);
+  shape_for(chunk, h.vpt, &vpt, &compute, kMaxThreadsCluster);
   const void* fn = t->step_cluster[vpt_index(vpt)][h.bounds ? 1 : 0];
   const size_t crow = (size_t)chunk * 16, btab = h.bounds ? 4 * crow : 0;
   int stages = ring_stages(crow + btab, 3 * crow, 1);

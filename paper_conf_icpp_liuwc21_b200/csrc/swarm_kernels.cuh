@@ -42,7 +42,8 @@
 namespace fastpso {
 namespace {
 
-constexpr int kMaxThreads = 256;  // compute threads per CTA
+constexpr int kMaxThreads = 256;         // compute threads per CTA
+constexpr int kMaxThreadsCluster = 512;  // compute threads per CTA of the cluster kernel
 constexpr int kMaxStages = 8;
 constexpr unsigned kFull = 0xFFFFFFFFu;
 
@@ -729,7 +730,7 @@ __global__ void __launch_bounds__(kMaxThreads + 64, 2)
 // straddle block boundaries, decides the pbest update and sends the decision
 // back to every CTA, which then bulk-stores its block of x', v' (and pb).
 template <class Obj, int VPT, bool kB>
-__global__ void __launch_bounds__(kMaxThreads + 64, 1)
+__global__ void __launch_bounds__(kMaxThreadsCluster + 64, 1)
     k_step_cluster(const SwarmArgs a, int stages, int C, int chunk) {
   extern __shared__ __align__(128) unsigned char dsmem[];
   constexpr int kSlot = Obj::kAcc + 2;  // partial accumulators, first x', last x'
@@ -744,7 +745,7 @@ __global__ void __launch_bounds__(kMaxThreads + 64, 1)
   float4* sG = reinterpret_cast<float4*>(dsmem);
   float4* sB = sG + chunk;
   float4* ring = sB + (kB ? 4 * chunk : 0);
-  __shared__ float red[kMaxStages][(kMaxThreads / 32) * 2];
+  __shared__ float red[kMaxStages][(kMaxThreadsCluster / 32) * 2];
   __shared__ float parts[kMaxStages][16 * kSlot];  // CTA 0: block partials by rank
   __shared__ float dec[kMaxStages][2];             // every CTA: {improved, f}
   __shared__ unsigned long long full[kMaxStages], empty[kMaxStages], done[kMaxStages];
