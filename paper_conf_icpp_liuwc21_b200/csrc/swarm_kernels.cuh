@@ -156,6 +156,19 @@ __device__ __forceinline__ uint32_t map_to_rank(const void* p, uint32_t rank) {
 __device__ __forceinline__ void st_cluster_f32(uint32_t addr, float v) {
   asm volatile("st.shared::cluster.f32 [%0], %1;" ::"r"(addr), "f"(v) : "memory");
 }
+// Store into another CTA's shared memory and signal its mbarrier (complete_tx).
+__device__ __forceinline__ void st_async_v4(uint32_t addr, float4 v, uint32_t bar_addr) {
+  asm volatile(
+      "st.async.shared::cluster.mbarrier::complete_tx::bytes.v4.f32 [%0], {%1, %2, %3, %4}, [%5];" ::"r"(addr),
+      "f"(v.x), "f"(v.y), "f"(v.z), "f"(v.w), "r"(bar_addr)
+      : "memory");
+}
+__device__ __forceinline__ void st_async_v2(uint32_t addr, float2 v, uint32_t bar_addr) {
+  asm volatile(
+      "st.async.shared::cluster.mbarrier::complete_tx::bytes.v2.f32 [%0], {%1, %2}, [%3];" ::"r"(addr),
+      "f"(v.x), "f"(v.y), "r"(bar_addr)
+      : "memory");
+}
 __device__ __forceinline__ void mbar_arrive_remote(uint32_t bar_addr) {
   asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(bar_addr)
                : "memory");
@@ -746,8 +759,10 @@ __global__ void __launch_bounds__(kMaxThreadsCluster + 64, 1)
   float4* sB = sG + chunk;
   float4* ring = sB + (kB ? 4 * chunk : 0);
   __shared__ float red[kMaxStages][(kMaxThreadsCluster / 32) * 2];
-  __shared__ float parts[kMaxStages][16 * kSlot];  // CTA 0: block partials by rank
-  __shared__ float dec[kMaxStages][2];             // every CTA: {improved, f}
+  // CTA 0: per rank {acc0, acc1, first x', last x'}; every CTA: {improved, f}.
+  // Both arrive by st.async, which signals the receiver's mbarrier (complete_tx).
+  __shared__ __align__(16) float4 parts[kMaxStages][16];
+  __shared__ __align__(8) float2 dec[kMaxStages];
   __shared__ unsigned long long full[kMaxStages], empty[kMaxStages], done[kMaxStages];
   __shared__ unsigned long long pbar[kMaxStages], dbar[kMaxStages], gbar;
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
@@ -757,7 +772,7 @@ __global__ void __launch_bounds__(kMaxThreadsCluster + 64, 1)
       mbar_init(&full[s], 1);
       mbar_init(&done[s], (unsigned)nwarps);
       mbar_init(&empty[s], 1);
-      mbar_init(&pbar[s], (unsigned)C);
+      mbar_init(&pbar[s], 1);
       mbar_init(&dbar[s], 1);
     }
     mbar_fence_init();
@@ -819,38 +834,38 @@ __global__ void __launch_bounds__(kMaxThreadsCluster + 64, 1)
           Obj::combine(c, b);
         }
         const float4* st = ring + (size_t)s * 3 * chunk;
-        // publish {partial, first x', last x'} to CTA 0
-        const uint32_t slot = map_to_rank(&parts[s][crank * kSlot], 0);
-#pragma unroll
-        for (int j = 0; j < Obj::kAcc; ++j) st_cluster_f32(slot + 4u * j, c[j]);
-        if (Obj::kNeighbor && cnt > 0) {
-          st_cluster_f32(slot + 4u * Obj::kAcc, st[0].x);
-          st_cluster_f32(slot + 4u * (Obj::kAcc + 1), st[cnt - 1].w);
+        // publish {partial, first x', last x'} to CTA 0 (one 16-byte st.async)
+        {
+          float4 msg = make_float4(c[0], Obj::kAcc > 1 ? c[Obj::kAcc - 1] : 0.f, 0.f, 0.f);
+          if (Obj::kNeighbor && cnt > 0) {
+            msg.z = st[0].x;
+            msg.w = st[cnt - 1].w;
+          }
+          st_async_v4(map_to_rank(&parts[s][crank], 0), msg, map_to_rank(&pbar[s], 0));
         }
-        mbar_arrive_remote(map_to_rank(&pbar[s], 0));
+        mbar_expect_tx(&dbar[s], 8u);  // this CTA's decision message
         if (crank == 0) {  // combine blocks in rank order, decide, broadcast
+          mbar_expect_tx(&pbar[s], 16u * (unsigned)C);
           mbar_wait_cluster(&pbar[s], ph);
           float tot[Obj::kAcc];
           Obj::init(tot);
           for (int k = 0; k < C; ++k) {
-            Obj::combine(tot, &parts[s][k * kSlot]);
+            const float4 pk = parts[s][k];
+            float ck_acc[2] = {pk.x, pk.y};
+            Obj::combine(tot, ck_acc);
             const int qk = k * chunk, ck = min(chunk, nvec - qk);
             if (Obj::kNeighbor && k + 1 < C && ck > 0 && qk + ck < nvec) {
               float bterm[Obj::kAcc];
               Obj::init(bterm);
               const int jl = 4 * (qk + ck) - 1;  // last dim of block k
-              Obj::map(bterm, parts[s][k * kSlot + Obj::kAcc + 1], parts[s][(k + 1) * kSlot + Obj::kAcc],
-                       jl, d);
+              Obj::map(bterm, pk.w, parts[s][k + 1].z, jl, d);
               Obj::combine(tot, bterm);
             }
           }
           const float f = Obj::finalize(tot, d);
           const float imp = (f < pf_old) ? 1.f : 0.f;  // strict; NaN never improves
-          for (int k = 0; k < C; ++k) {
-            st_cluster_f32(map_to_rank(&dec[s][0], k), imp);
-            st_cluster_f32(map_to_rank(&dec[s][1], k), f);
-            mbar_arrive_remote(map_to_rank(&dbar[s], k));
-          }
+          for (int k = 0; k < C; ++k)
+            st_async_v2(map_to_rank(&dec[s], k), make_float2(imp, f), map_to_rank(&dbar[s], k));
           if (imp != 0.f) {
             a.pf[r] = f;
             ++nimp;
@@ -861,7 +876,7 @@ __global__ void __launch_bounds__(kMaxThreadsCluster + 64, 1)
           }
         }
         mbar_wait_cluster(&dbar[s], ph);
-        const bool improved = dec[s][0] != 0.f;
+        const bool improved = dec[s].x != 0.f;
         if (cnt > 0) {
           const size_t off = ((size_t)r * nvec + q0) * 4;
           bulk_s2g(a.X + off, st, blk_bytes);
