@@ -126,7 +126,7 @@ void shape_for(int nvec, int vpt_override, int* vpt, int* threads, int max_threa
 
 constexpr size_t kSmemPerSm = 228 * 1024;       // B200 unified L1/shared per SM
 constexpr size_t kSmemPerCtaMax = 227 * 1024;   // opt-in maximum per CTA
-constexpr size_t kStaticReserve = 2048;         // static shared + per-CTA reservation
+constexpr size_t kStaticReserve = 4096;         // static shared (<= 3 KB) + per-CTA reservation
 constexpr long long kResidentElems = 8192;      // resident path: n d <= this
 
 }  // namespace
