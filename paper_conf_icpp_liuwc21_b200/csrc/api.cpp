@@ -418,6 +418,10 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
   {
     cudaError_t e = plan_launch(objective, d, h->n_local > 0 ? h->n_local : 1, h->sm_count,
                                 hints, &h->cfg);
+    if (e == cudaErrorInvalidConfiguration) {
+      cudaGetLastError();
+      return bail(fail(PSO_ERR_UNSUPPORTED, "no launch shape fits d=%d with the requested hints", d));
+    }
     if (e != cudaSuccess) return bail(cuda_fail(nullptr, e, "plan_launch"));
   }
 
