@@ -164,7 +164,11 @@ pso_status use_device(pso_swarm* h) {
   return PSO_OK;
 }
 
-pso_status exchange(pso_swarm* h) {
+// All-gather the records of iteration t (one per rank: its best candidate key
+// and row) into recv[t & 1].  The next step kernel merges them in its
+// prologue; `fold` additionally runs the select kernel so key_cur / G are
+// final for the host (end of create, set_state and every pso_step call).
+pso_status exchange(pso_swarm* h, uint64_t t, bool fold) {
   if (!h->xchg) return PSO_OK;
   NcclApi* a = nccl();
   if (!a) {
@@ -172,14 +176,16 @@ pso_status exchange(pso_swarm* h) {
     return fail(PSO_ERR_NCCL, "NCCL unavailable");
   }
   const size_t rec = record_bytes(h->pitch);
-  ncclResult_t r = a->AllGather(h->args.send, const_cast<unsigned char*>(h->args.recv), rec,
-                                kNcclUint8, h->comm, h->stream);
+  unsigned char* dst = const_cast<unsigned char*>(h->args.recv) + (t & 1) * (size_t)h->world * rec;
+  ncclResult_t r = a->AllGather(h->args.send, dst, rec, kNcclUint8, h->comm, h->stream);
   if (r != 0) {
     h->poisoned = true;
     return fail(PSO_ERR_NCCL, "ncclAllGather: %s", nccl_str(r));
   }
-  PSO_CUDA(h, launch_select(h->args, h->stream));
-  ++h->launches;
+  if (fold) {
+    PSO_CUDA(h, launch_select(h->args, (unsigned)t, h->stream));
+    ++h->launches;
+  }
   return PSO_OK;
 }
 
@@ -435,7 +441,7 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
   const size_t rec = align_up(record_bytes(h->pitch), 256);
   const size_t candb = h->cfg.gridres ? align_up(2 * (size_t)h->cfg.gridres_grid * h->pitch * 4, 256) : 0;
   const size_t sendb = h->xchg ? rec : 0;
-  const size_t recvb = h->xchg ? (size_t)h->world * record_bytes(h->pitch) : 0;
+  const size_t recvb = h->xchg ? 2 * (size_t)h->world * record_bytes(h->pitch) : 0;
   h->arena_bytes = 3 * mat + pfb + gb + ctlb + boundb + candb + sendb + align_up(recvb, 256);
   {
     cudaError_t e = cudaMalloc(&h->arena, h->arena_bytes);
@@ -490,7 +496,7 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
     cudaError_t e = cudaMemcpyAsync(A.send, none, 16, cudaMemcpyHostToDevice, h->stream);
     if (e != cudaSuccess) return bail(cuda_fail(nullptr, e, "cudaMemcpyAsync"));
   }
-  if ((st = exchange(h)) != PSO_OK) return bail(st);
+  if ((st = exchange(h, 0, true)) != PSO_OK) return bail(st);
   if ((st = sync_and_check(h)) != PSO_OK) return bail(st);
   h->t = 0;
   *out = h;
@@ -530,7 +536,7 @@ pso_status pso_step(pso_handle h, int64_t iters) {
       ++h->launches;
       if (ev) PSO_CUDA(h, cudaEventRecord(ev->stop, h->stream));
     }
-    if ((st = exchange(h)) != PSO_OK) return st;
+    if ((st = exchange(h, h->t + (uint64_t)it + 1, it + 1 == iters)) != PSO_OK) return st;
   }
   h->t += (uint64_t)iters;
   return PSO_OK;
@@ -601,7 +607,7 @@ pso_status pso_set_state(pso_handle h, const float* x, const float* v, const flo
     unsigned long long none[2] = {~0ull, 0ull};
     PSO_CUDA(h, cudaMemcpyAsync(h->args.send, none, 16, cudaMemcpyHostToDevice, h->stream));
   }
-  if ((st = exchange(h)) != PSO_OK) return st;
+  if ((st = exchange(h, t, true)) != PSO_OK) return st;
   if ((st = sync_and_check(h)) != PSO_OK) return st;
   h->t = t;
   return PSO_OK;

@@ -34,7 +34,7 @@ struct SwarmArgs {
   float* cand;                // grid-resident kernel: [2][grid][pitch] candidate rows
   const float* bounds;        // per-dimension bounds [vlo | vhi | xlo | xhi] (4 x pitch), or null
   unsigned char* send;        // world > 1: this rank's exchange record
-  const unsigned char* recv;  // world > 1: world records after the all-gather
+  const unsigned char* recv;  // exchange: [2 iteration parities][world] records after the all-gather
   DevCtl* ctl;
   long long n_local;
   long long row_begin;
@@ -105,7 +105,7 @@ cudaError_t launch_resident(int objective, const SwarmArgs& a, const LaunchCfg& 
 cudaError_t launch_gridres(int objective, const SwarmArgs& a, const LaunchCfg& c, int iters,
                            cudaStream_t s);
 cudaError_t launch_rebest(const SwarmArgs& a, unsigned t, cudaStream_t s);
-cudaError_t launch_select(const SwarmArgs& a, cudaStream_t s);
+cudaError_t launch_select(const SwarmArgs& a, unsigned t, cudaStream_t s);
 
 cudaError_t debug_philox(unsigned long long seed, unsigned tag, unsigned t, unsigned i,
                          unsigned j0, long long m, unsigned* out_dev, int use_curand,

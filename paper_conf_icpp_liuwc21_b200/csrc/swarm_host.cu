@@ -39,51 +39,28 @@ __global__ void __launch_bounds__(256) k_rebest(const SwarmArgs a, unsigned t) {
 }
 
 // ---------------------------------------------------------- select kernel
-// world > 1, after ncclAllGather of the records: the global candidate is the
-// minimum key over ranks (keys carry global indices, so ties resolve to the
-// lowest global index, as one GPU would).  Every rank computes the same bits.
-__global__ void __launch_bounds__(128) k_select(const SwarmArgs a) {
-  __shared__ unsigned long long s_min;
+// Exchange mode: fold the records of iteration t (after the all-gather) into
+// key_cur / G — the same merge a step kernel's prologue performs, run once at
+// the end of create / set_state / each pso_step call so the host reads the
+// final gbest.  Idempotent (the next step's prologue merges the same records
+// again and finds nothing better).  Every rank computes the same bits.
+__global__ void __launch_bounds__(128) k_select(const SwarmArgs a, unsigned t) {
+  __shared__ unsigned long long s_best;
   __shared__ int s_src;
-  const size_t rec = record_bytes(a.nvec * 4);
-  if (threadIdx.x < 32) {
-    unsigned long long best = ~0ull;
-    int src = -1;
-    for (int r = threadIdx.x; r < a.world; r += 32) {
-      const unsigned long long k =
-          *reinterpret_cast<const unsigned long long*>(a.recv + (size_t)r * rec);
-      if (k < best) {
-        best = k;
-        src = r;
-      }
-    }
-#pragma unroll
-    for (int off = 16; off > 0; off >>= 1) {
-      const unsigned long long o = __shfl_xor_sync(kFull, best, off);
-      const int os = __shfl_xor_sync(kFull, src, off);
-      if (o < best || (o == best && os >= 0 && (src < 0 || os < src))) {
-        best = o;
-        src = os;
-      }
-    }
-    if (threadIdx.x == 0) {
-      s_min = best;
-      s_src = src;
-    }
+  if (threadIdx.x == 0) {
+    int src;
+    s_best = exchange_merge(a, t, &src);
+    s_src = src;
   }
   __syncthreads();
-  const unsigned long long cur = a.ctl->key_cur;
-  const bool take = s_src >= 0 && s_min < cur;
-  if (take) {
-    const float4* row = reinterpret_cast<const float4*>(a.recv + (size_t)s_src * rec + 16);
+  const int src = s_src;
+  if (src >= 0) {
+    const float4* row = reinterpret_cast<const float4*>(merged_gbest_row(a, t, src));
     float4* G4 = reinterpret_cast<float4*>(a.G);
     for (int q = threadIdx.x; q < a.nvec; q += blockDim.x) G4[q] = row[q];
   }
   __syncthreads();
-  if (threadIdx.x == 0) {
-    if (take) a.ctl->key_cur = s_min;
-    a.ctl->key_acc = take ? s_min : cur;
-  }
+  if (threadIdx.x == 0 && src >= 0) a.ctl->key_cur = s_best;
 }
 
 // ---------------------------------------------------------- dispatch
@@ -406,8 +383,8 @@ cudaError_t launch_rebest(const SwarmArgs& a, unsigned t, cudaStream_t s) {
   return cudaGetLastError();
 }
 
-cudaError_t launch_select(const SwarmArgs& a, cudaStream_t s) {
-  k_select<<<1, 128, 0, s>>>(a);
+cudaError_t launch_select(const SwarmArgs& a, unsigned t, cudaStream_t s) {
+  k_select<<<1, 128, 0, s>>>(a, t);
   return cudaGetLastError();
 }
 

@@ -262,8 +262,10 @@ struct RowSmem {
   float f;
   int improved;
   int last;
-  unsigned long long gbar;  // gbest staging barrier
-  unsigned long long acc, cur;
+  unsigned long long gbar;      // gbest staging barrier
+  unsigned long long acc, cur;  // epilogue scratch (adjacent: sh[0], sh[1])
+  unsigned long long inc;       // exchange: merged incumbent of the previous iteration
+  int src;                      // exchange: rank whose record won (-1: none)
 };
 
 // Reduce a[] over the nthr compute threads (fixed order: lanes by
@@ -391,76 +393,105 @@ __device__ __forceinline__ float process_row(const SwarmArgs& a, const MoveParam
   return f;
 }
 
-// Last-CTA epilogue: publish the iteration's gbest.  world == 1: copy PB[gi]
-// into G and advance the incumbent key.  world > 1: write the local candidate
-// record (key, PB row) for the all-gather; the select kernel finishes.
-template <class Obj>
-__device__ __forceinline__ void gbest_epilogue(const SwarmArgs& a, RowSmem<Obj>& sm, uint32_t t,
-                                               int tid, int nthr) {
-  if (tid == 0) {
-    __threadfence();
-    sm.acc = *(volatile unsigned long long*)&a.ctl->key_acc;
-    sm.cur = a.ctl->key_cur;
-  }
-  team_sync(nthr);
-  const unsigned long long acc = sm.acc, cur = sm.cur;
-  const bool have = acc < cur;
-  const float4* src = nullptr;
-  if (have)
-    src = reinterpret_cast<const float4*>(a.PB) + ((long long)(uint32_t)acc - a.row_begin) * a.nvec;
-  if (!a.exchange) {
-    if (have) {
-      float4* G4 = reinterpret_cast<float4*>(a.G);
-      for (int q = tid; q < a.nvec; q += nthr) G4[q] = __ldcg(src + q);
-    }
-    if (tid == 0) {
-      if (have) a.ctl->key_cur = acc;
-      a.ctl->t = t;
-      a.ctl->done = 0;
-    }
-  } else {
-    unsigned long long* hdr = reinterpret_cast<unsigned long long*>(a.send);
-    float4* row = reinterpret_cast<float4*>(a.send + 16);
-    if (have)
-      for (int q = tid; q < a.nvec; q += nthr) row[q] = __ldcg(src + q);
-    if (tid == 0) {
-      hdr[0] = have ? acc : ~0ull;
-      hdr[1] = 0;
-      a.ctl->t = t;
-      a.ctl->done = 0;
+// --- gbest exchange (world > 1, or forced): records of iteration t live in
+// recv[t & 1][rank] = {u64 key, u64 tag, pitch floats}.  The step kernel of
+// iteration t + 1 merges them in its prologue (the incumbent for its strict
+// filter and the G it stages); its last CTA commits that merge to key_cur / G
+// and publishes the new local candidate.
+__device__ __forceinline__ const unsigned char* records(const SwarmArgs& a, uint32_t t) {
+  return a.recv + (size_t)(t & 1u) * a.world * record_bytes(a.nvec * 4);
+}
+// Minimum of the incumbent and the records of iteration prev_t; *src = the
+// winning rank, or -1 when nothing beat the incumbent.  One thread.
+__device__ __forceinline__ unsigned long long exchange_merge(const SwarmArgs& a, uint32_t prev_t,
+                                                             int* src) {
+  const size_t rec = record_bytes(a.nvec * 4);
+  const unsigned char* base = records(a, prev_t);
+  unsigned long long best = *(volatile unsigned long long*)&a.ctl->key_cur;
+  int s = -1;
+  for (int r = 0; r < a.world; ++r) {
+    const unsigned long long k = *reinterpret_cast<const unsigned long long*>(base + (size_t)r * rec);
+    if (k < best) {
+      best = k;
+      s = r;
     }
   }
+  *src = s;
+  return best;
+}
+__device__ __forceinline__ const float* merged_gbest_row(const SwarmArgs& a, uint32_t prev_t, int src) {
+  return src < 0 ? a.G
+                 : reinterpret_cast<const float*>(records(a, prev_t) +
+                                                  (size_t)src * record_bytes(a.nvec * 4) + 16);
 }
 
-// The same epilogue run by one warp (the TMA kernel's finaliser warp).
-__device__ __forceinline__ void warp_gbest_epilogue(const SwarmArgs& a, uint32_t t, int lane) {
-  unsigned long long acc = 0, cur = 0;
-  if (lane == 0) {
+// Last-CTA epilogue of iteration t, run by `nthr` threads (tid 0 leads;
+// `sync` orders them; `sh` is 2 words of shared scratch).
+//   single GPU: copy PB[gi] into G and advance the incumbent key.
+//   exchange:   commit the prologue's merge (inc from rank `src`) to key_cur /
+//               G, then write the local candidate record (strictly below inc)
+//               for the all-gather, tagged with t; reset the accumulator.
+template <class SyncF>
+__device__ __forceinline__ void epilogue_core(const SwarmArgs& a, uint32_t t, unsigned long long inc,
+                                              int src, unsigned long long* sh, int tid, int nthr,
+                                              SyncF sync) {
+  if (tid == 0) {
     __threadfence();
-    acc = *(volatile unsigned long long*)&a.ctl->key_acc;
-    cur = a.ctl->key_cur;
+    sh[0] = *(volatile unsigned long long*)&a.ctl->key_acc;
+    sh[1] = a.ctl->key_cur;
   }
-  acc = __shfl_sync(kFull, acc, 0);
-  cur = __shfl_sync(kFull, cur, 0);
-  const bool have = acc < cur;
-  const float4* src = nullptr;
-  if (have)
-    src = reinterpret_cast<const float4*>(a.PB) + ((long long)(uint32_t)acc - a.row_begin) * a.nvec;
-  float4* dst = !a.exchange ? reinterpret_cast<float4*>(a.G) : reinterpret_cast<float4*>(a.send + 16);
-  if (have)
-    for (int q = lane; q < a.nvec; q += 32) dst[q] = __ldcg(src + q);
-  __syncwarp();
-  if (lane == 0) {
-    if (!a.exchange) {
-      if (have) a.ctl->key_cur = acc;
-    } else {
-      unsigned long long* hdr = reinterpret_cast<unsigned long long*>(a.send);
-      hdr[0] = have ? acc : ~0ull;
-      hdr[1] = 0;
+  sync();
+  const unsigned long long acc = sh[0], cur = sh[1];
+  float4* G4 = reinterpret_cast<float4*>(a.G);
+  if (!a.exchange) {
+    const bool have = acc < cur;
+    if (have) {
+      const float4* pb = reinterpret_cast<const float4*>(a.PB) +
+                         ((long long)(uint32_t)acc - a.row_begin) * a.nvec;
+      for (int q = tid; q < a.nvec; q += nthr) G4[q] = __ldcg(pb + q);
     }
+    if (tid == 0) {
+      if (have) a.ctl->key_cur = acc;
+      a.ctl->t = t;
+      a.ctl->done = 0;
+    }
+    return;
+  }
+  const bool merged = src >= 0 && inc < cur;
+  if (merged) {
+    const float4* w = reinterpret_cast<const float4*>(merged_gbest_row(a, t - 1u, src));
+    for (int q = tid; q < a.nvec; q += nthr) G4[q] = __ldcg(w + q);
+  }
+  const bool have = acc != ~0ull;
+  if (have) {
+    const float4* pb = reinterpret_cast<const float4*>(a.PB) +
+                       ((long long)(uint32_t)acc - a.row_begin) * a.nvec;
+    float4* row = reinterpret_cast<float4*>(a.send + 16);
+    for (int q = tid; q < a.nvec; q += nthr) row[q] = __ldcg(pb + q);
+  }
+  if (tid == 0) {
+    unsigned long long* hdr = reinterpret_cast<unsigned long long*>(a.send);
+    hdr[0] = have ? acc : ~0ull;
+    hdr[1] = t;
+    if (merged) a.ctl->key_cur = inc;
+    a.ctl->key_acc = ~0ull;
     a.ctl->t = t;
     a.ctl->done = 0;
   }
+}
+
+template <class Obj>
+__device__ __forceinline__ void gbest_epilogue(const SwarmArgs& a, RowSmem<Obj>& sm, uint32_t t,
+                                               int tid, int nthr, unsigned long long inc = ~0ull,
+                                               int src = -1) {
+  epilogue_core(a, t, inc, src, &sm.acc, tid, nthr, [&] { team_sync(nthr); });
+}
+
+// The same epilogue run by one warp (the finaliser warp of the TMA kernels).
+__device__ __forceinline__ void warp_gbest_epilogue(const SwarmArgs& a, uint32_t t, int lane,
+                                                    unsigned long long inc = ~0ull, int src = -1) {
+  __shared__ unsigned long long sh[2];
+  epilogue_core(a, t, inc, src, sh, lane, 32, [] { __syncwarp(); });
 }
 
 // Publish this CTA's candidate and improvement count; true in the last CTA
@@ -504,17 +535,24 @@ __global__ void __launch_bounds__(kMaxThreads, (VPT >= 8) ? 1 : 2)
   float* sFirst = reinterpret_cast<float*>(sB + (kB ? 4 * a.nvec : 0));
   __shared__ RowSmem<Obj> sm;
   const int tid = threadIdx.x, nthr = blockDim.x;
+  const uint32_t t = a.ctl->t + 1u;
   if (tid == 0) {
     const unsigned row_bytes = (unsigned)a.nvec * 16u;
+    const float* gsrc = a.G;
+    sm.src = -1;
+    sm.inc = a.ctl->key_cur;
+    if (a.exchange) {  // merge the previous iteration's records (the all-gather)
+      sm.inc = exchange_merge(a, t - 1u, &sm.src);
+      gsrc = merged_gbest_row(a, t - 1u, sm.src);
+    }
     mbar_init(&sm.gbar, 1);
     mbar_fence_init();
     mbar_expect_tx(&sm.gbar, row_bytes * (kB ? 5u : 1u));
-    bulk_g2s(sG, a.G, row_bytes, &sm.gbar);
+    bulk_g2s(sG, gsrc, row_bytes, &sm.gbar);
     if (kB) bulk_g2s(sB, a.bounds, 4u * row_bytes, &sm.gbar);
   }
   __syncthreads();
-  const uint32_t t = a.ctl->t + 1u;
-  const uint32_t inc_ord = (uint32_t)(a.ctl->key_cur >> 32);
+  const uint32_t inc_ord = (uint32_t)(sm.inc >> 32);
   const PhiloxKey key{a.seed_lo, a.seed_hi};
   const MoveParams mp = move_params(a);
   const int nvec = a.nvec;
@@ -549,7 +587,8 @@ __global__ void __launch_bounds__(kMaxThreads, (VPT >= 8) ? 1 : 2)
         [] {}, sG, sB, sFirst, sm, tid, nthr, pf_old, improved);
     if (tid == 0) row_bookkeeping(a, r, gi, f, improved, inc_ord, best, nimp);
   }
-  if (cta_finish<Obj>(a, sm, best, nimp, tid, nthr)) gbest_epilogue<Obj>(a, sm, t, tid, nthr);
+  if (cta_finish<Obj>(a, sm, best, nimp, tid, nthr))
+    gbest_epilogue<Obj>(a, sm, t, tid, nthr, sm.inc, sm.src);
 }
 
 // ------------------------------------------------- step kernel: TMA pipeline
@@ -579,6 +618,8 @@ __global__ void __launch_bounds__(kMaxThreads + 64, 2)
   float4* ring = sB + (kB ? 4 * nvec : 0);
   __shared__ float red[kMaxStages][(kMaxThreads / 32) * 2];
   __shared__ unsigned long long full[kMaxStages], empty[kMaxStages], done[kMaxStages], gbar;
+  __shared__ unsigned long long s_inc;  // incumbent of this iteration (after the exchange merge)
+  __shared__ int s_src;
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   if (tid == 0) {
     mbar_init(&gbar, 1);
@@ -595,8 +636,17 @@ __global__ void __launch_bounds__(kMaxThreads + 64, 2)
 
   if (warp == nwarps) {  // ---------------- producer
     if (lane == 0) {
-      mbar_expect_tx(&gbar, row_bytes * (kB ? 5u : 1u));
-      bulk_g2s(sG, a.G, row_bytes, &gbar);
+      const float* gsrc = a.G;
+      s_src = -1;
+      s_inc = a.ctl->key_cur;
+      if (a.exchange) {  // merge the previous iteration's records (the all-gather)
+        int src;
+        s_inc = exchange_merge(a, t - 1u, &src);
+        s_src = src;
+        gsrc = merged_gbest_row(a, t - 1u, src);
+      }
+      mbar_expect_tx(&gbar, row_bytes * (kB ? 5u : 1u));  // releases s_inc / s_src too
+      bulk_g2s(sG, gsrc, row_bytes, &gbar);
       if (kB) bulk_g2s(sB, a.bounds, 4u * row_bytes, &gbar);
       int s = 0;
       unsigned ph = 0;
@@ -620,7 +670,8 @@ __global__ void __launch_bounds__(kMaxThreads + 64, 2)
   if (warp == nwarps + 1) {  // ---------------- finaliser
     __shared__ int s_last;
     if (lane == 0) {
-      const uint32_t inc_ord = (uint32_t)(a.ctl->key_cur >> 32);
+      mbar_wait(&gbar, 0);
+      const uint32_t inc_ord = (uint32_t)(s_inc >> 32);
       unsigned long long best = ~0ull;
       unsigned nimp = 0;
       int s = 0, prev = -1;
@@ -670,7 +721,7 @@ __global__ void __launch_bounds__(kMaxThreads + 64, 2)
       s_last = (atomicAdd(&a.ctl->done, 1u) == gridDim.x - 1) ? 1 : 0;
     }
     __syncwarp();
-    if (s_last) warp_gbest_epilogue(a, t, lane);
+    if (s_last) warp_gbest_epilogue(a, t, lane, s_inc, s_src);
     return;
   }
 
@@ -765,6 +816,8 @@ __global__ void __launch_bounds__(kMaxThreadsCluster + 64, 1)
   __shared__ __align__(8) float2 dec[kMaxStages];
   __shared__ unsigned long long full[kMaxStages], empty[kMaxStages], done[kMaxStages];
   __shared__ unsigned long long pbar[kMaxStages], dbar[kMaxStages], gbar;
+  __shared__ unsigned long long s_inc;  // incumbent of this iteration (after the exchange merge)
+  __shared__ int s_src;
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   if (tid == 0) {
     mbar_init(&gbar, 1);
@@ -784,9 +837,18 @@ __global__ void __launch_bounds__(kMaxThreadsCluster + 64, 1)
 
   if (warp == nwarps) {  // ---------------- producer
     if (lane == 0) {
-      mbar_expect_tx(&gbar, blk_bytes * (kB ? 5u : 1u));
+      const float* gsrc = a.G;
+      s_src = -1;
+      s_inc = a.ctl->key_cur;
+      if (a.exchange) {  // merge the previous iteration's records (the all-gather)
+        int src;
+        s_inc = exchange_merge(a, t - 1u, &src);
+        s_src = src;
+        gsrc = merged_gbest_row(a, t - 1u, src);
+      }
+      mbar_expect_tx(&gbar, blk_bytes * (kB ? 5u : 1u));  // releases s_inc / s_src too
       if (cnt > 0) {
-        bulk_g2s(sG, a.G + (size_t)q0 * 4, blk_bytes, &gbar);
+        bulk_g2s(sG, gsrc + (size_t)q0 * 4, blk_bytes, &gbar);
         if (kB)
           for (int k = 0; k < 4; ++k)
             bulk_g2s(sB + k * chunk, a.bounds + ((size_t)k * nvec + q0) * 4, blk_bytes, &gbar);
@@ -816,7 +878,8 @@ __global__ void __launch_bounds__(kMaxThreadsCluster + 64, 1)
   if (warp == nwarps + 1) {  // ---------------- finaliser
     __shared__ int s_last;
     if (lane == 0) {
-      const uint32_t inc_ord = (uint32_t)(a.ctl->key_cur >> 32);
+      mbar_wait(&gbar, 0);
+      const uint32_t inc_ord = (uint32_t)(s_inc >> 32);
       unsigned long long best = ~0ull;
       unsigned nimp = 0;
       int s = 0, prev = -1;
@@ -902,7 +965,7 @@ __global__ void __launch_bounds__(kMaxThreadsCluster + 64, 1)
       s_last = (atomicAdd(&a.ctl->done, 1u) == gridDim.x - 1) ? 1 : 0;
     }
     __syncwarp();
-    if (s_last) warp_gbest_epilogue(a, t, lane);
+    if (s_last) warp_gbest_epilogue(a, t, lane, s_inc, s_src);
     return;
   }
 
