@@ -207,6 +207,20 @@ pso_status pso_nccl_comm_init(void** comm, int32_t nranks, const void* id128, in
                               int32_t device);
 pso_status pso_nccl_comm_destroy(void* comm);
 
+/* --- NVLink peer exchange (the fused alternative to the all-gather) -------- *
+ * After pso_create_ex with a communicator, every rank may switch its handle to
+ * exchange gbest records by direct NVLink stores: the last CTA of each step
+ * kernel writes its record (key, candidate row) into recv[t & 1][rank] of
+ * every rank and releases a per-record iteration tag; the next step kernel's
+ * prologue acquires the tags and merges.  No collective call per iteration.
+ * Protocol (collective): each rank calls pso_p2p_handle, the 64-byte CUDA IPC
+ * handles and offsets are all-gathered out of band (e.g. torch.distributed),
+ * then every rank calls pso_p2p_connect with the world arrays in rank order.
+ * A peer that stops delivering makes the waiting kernels trap after 60 s. */
+pso_status pso_p2p_handle(pso_handle h, void* ipc_handle /* 64 bytes */, uint64_t* offset);
+pso_status pso_p2p_connect(pso_handle h, const void* ipc_handles /* world x 64 bytes */,
+                           const uint64_t* offsets /* world */);
+
 /* --- Device-side primitives exposed for parity tests ---------------------- */
 /* out[k] = word(tag, t, i, j0 + k) computed on the device (k < m), with the
  * library's Philox (use_curand = 0) or with curand_Philox4x32_10 (1).

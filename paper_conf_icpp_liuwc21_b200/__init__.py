@@ -143,6 +143,20 @@ class Swarm:
         check(lib().pso_set_bounds(self._h, C.c_void_p(b.ctypes.data)), "pso_set_bounds")
         return self
 
+    def p2p_handle(self) -> tuple[bytes, int]:
+        """(64-byte CUDA IPC handle of the arena, offset of the receive buffer)."""
+        buf = C.create_string_buffer(64)
+        off = C.c_uint64()
+        check(lib().pso_p2p_handle(self._h, buf, C.byref(off)), "pso_p2p_handle")
+        return buf.raw, int(off.value)
+
+    def p2p_connect(self, handles, offsets) -> "Swarm":
+        """Switch to the NVLink peer exchange (handles/offsets of every rank, in rank order)."""
+        blob = C.create_string_buffer(b"".join(bytes(h) for h in handles), 64 * len(handles))
+        offs = (C.c_uint64 * len(offsets))(*[int(o) for o in offsets])
+        check(lib().pso_p2p_connect(self._h, blob, offs), "pso_p2p_connect")
+        return self
+
     def info(self) -> dict:
         inf = pso_info()
         check(lib().pso_get_info(self._h, C.byref(inf)), "pso_get_info")

@@ -136,6 +136,9 @@ struct pso_swarm {
   size_t events_used = 0;
   double timed_ms = 0;
   uint64_t timed_count = 0;
+  // NVLink peer exchange (pso_p2p_connect)
+  std::vector<void*> ipc_opened;
+  void* peers_dev = nullptr;
 };
 
 namespace {
@@ -176,6 +179,13 @@ pso_status exchange(pso_swarm* h, uint64_t t, bool fold) {
     return fail(PSO_ERR_NCCL, "NCCL unavailable");
   }
   const size_t rec = record_bytes(h->pitch);
+  if (h->args.p2p) {  // records travel by NVLink peer stores inside the kernels
+    if (fold) {
+      PSO_CUDA(h, launch_select(h->args, (unsigned)t, h->stream));
+      ++h->launches;
+    }
+    return PSO_OK;
+  }
   unsigned char* dst = const_cast<unsigned char*>(h->args.recv) + (t & 1) * (size_t)h->world * rec;
   ncclResult_t r = a->AllGather(h->args.send, dst, rec, kNcclUint8, h->comm, h->stream);
   if (r != 0) {
@@ -468,6 +478,7 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
   A.d = d;
   A.nvec = h->pitch / 4;
   A.world = h->world;
+  A.rank = h->rank;
   A.exchange = h->xchg ? 1 : 0;
   A.w = w; A.c1 = c1; A.c2 = c2; A.lo = lo; A.hi = hi; A.vmax = h->vmax;
   A.seed_lo = (unsigned)seed;
@@ -478,6 +489,8 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
     if (e != cudaSuccess) return bail(cuda_fail(nullptr, e, "cudaMemsetAsync"));
     if (h->xchg) {
       e = cudaMemsetAsync(A.send, 0, sendb, h->stream);
+      if (e == cudaSuccess)  // record tags that no iteration matches until written
+        e = cudaMemsetAsync(const_cast<unsigned char*>(A.recv), 0xFF, recvb, h->stream);
       if (e != cudaSuccess) return bail(cuda_fail(nullptr, e, "cudaMemsetAsync"));
     }
   }
@@ -625,6 +638,48 @@ pso_status pso_set_bounds(pso_handle h, const float* bounds) {
   return upload_bounds(h, bounds);
 }
 
+pso_status pso_p2p_handle(pso_handle h, void* ipc_handle, uint64_t* offset) {
+  pso_status st = check_handle(h);
+  if (st != PSO_OK) return st;
+  if (!ipc_handle || !offset) return fail(PSO_ERR_INVALID, "ipc_handle/offset is NULL");
+  if (!h->xchg) return fail(PSO_ERR_UNSUPPORTED, "handle has no exchange (no NCCL communicator)");
+  if ((st = use_device(h)) != PSO_OK) return st;
+  cudaIpcMemHandle_t mh;
+  PSO_CUDA(h, cudaIpcGetMemHandle(&mh, h->arena));
+  std::memcpy(ipc_handle, &mh, sizeof(mh));
+  *offset = (uint64_t)((const unsigned char*)h->args.recv - (const unsigned char*)h->arena);
+  return PSO_OK;
+}
+
+pso_status pso_p2p_connect(pso_handle h, const void* ipc_handles, const uint64_t* offsets) {
+  pso_status st = check_handle(h);
+  if (st != PSO_OK) return st;
+  if (!ipc_handles || !offsets) return fail(PSO_ERR_INVALID, "ipc_handles/offsets is NULL");
+  if (!h->xchg) return fail(PSO_ERR_UNSUPPORTED, "handle has no exchange (no NCCL communicator)");
+  if (h->args.p2p) return fail(PSO_ERR_INVALID, "already connected");
+  if ((st = use_device(h)) != PSO_OK) return st;
+  if ((st = sync_and_check(h)) != PSO_OK) return st;
+  std::vector<unsigned char*> peers((size_t)h->world);
+  for (int r = 0; r < h->world; ++r) {
+    if (r == h->rank) {  // our own receive buffer
+      peers[r] = const_cast<unsigned char*>(h->args.recv);
+      continue;
+    }
+    cudaIpcMemHandle_t mh;
+    std::memcpy(&mh, (const unsigned char*)ipc_handles + (size_t)r * sizeof(mh), sizeof(mh));
+    void* base = nullptr;
+    PSO_CUDA(h, cudaIpcOpenMemHandle(&base, mh, cudaIpcMemLazyEnablePeerAccess));
+    h->ipc_opened.push_back(base);
+    peers[r] = (unsigned char*)base + offsets[r];
+  }
+  PSO_CUDA(h, cudaMalloc(&h->peers_dev, sizeof(unsigned char*) * peers.size()));
+  PSO_CUDA(h, cudaMemcpy(h->peers_dev, peers.data(), sizeof(unsigned char*) * peers.size(),
+                         cudaMemcpyHostToDevice));
+  h->args.peers = (unsigned char* const*)h->peers_dev;
+  h->args.p2p = 1;
+  return PSO_OK;
+}
+
 pso_status pso_get_info(pso_handle h, pso_info* info) {
   if (!h) return fail(PSO_ERR_INVALID, "NULL handle");
   if (!info) return fail(PSO_ERR_INVALID, "info is NULL");
@@ -694,6 +749,8 @@ void pso_destroy(pso_handle h) {
     cudaEventDestroy(e.start);
     cudaEventDestroy(e.stop);
   }
+  for (void* p : h->ipc_opened) cudaIpcCloseMemHandle(p);
+  if (h->peers_dev) cudaFree(h->peers_dev);
   if (h->arena) cudaFree(h->arena);
   if (h->own_stream && h->stream) cudaStreamDestroy(h->stream);
   cudaGetLastError();

@@ -40,7 +40,10 @@ struct SwarmArgs {
   long long row_begin;
   int d, nvec;                // nvec = pitch / 4
   int world;
+  int rank;
   int exchange;               // 1: publish (key, row) records for the all-gather + select
+  int p2p;                    // exchange over NVLink peer stores instead of NCCL
+  unsigned char* const* peers;  // p2p: device array, world pointers to every rank's recv
   float w, c1, c2, lo, hi, vmax;
   unsigned int seed_lo, seed_hi;
 };

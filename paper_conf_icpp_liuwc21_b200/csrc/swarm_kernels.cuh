@@ -401,10 +401,45 @@ __device__ __forceinline__ float process_row(const SwarmArgs& a, const MoveParam
 __device__ __forceinline__ const unsigned char* records(const SwarmArgs& a, uint32_t t) {
   return a.recv + (size_t)(t & 1u) * a.world * record_bytes(a.nvec * 4);
 }
+// --- NVLink peer exchange (p2p): every rank stores its record of iteration
+// t straight into recv[t & 1][rank] of every peer (CUDA-IPC-mapped), then the
+// record's tag with release semantics at system scope; readers acquire the
+// tags.  No collective call and no host involvement per iteration.
+__device__ __forceinline__ unsigned long long ld_acquire_sys_u64(const void* p) {
+  unsigned long long v;
+  asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release_sys_u64(void* p, unsigned long long v) {
+  asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ unsigned long long globaltimer_ns() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+// Wait until every rank's record of iteration t has landed (one thread).  A
+// peer that never delivers (a crashed rank) traps after 60 s instead of
+// hanging the GPU.
+__device__ __forceinline__ void wait_records(const SwarmArgs& a, uint32_t t) {
+  const size_t rec = record_bytes(a.nvec * 4);
+  const unsigned char* base = records(a, t);
+  const unsigned long long t0 = globaltimer_ns();
+  for (int r = 0; r < a.world; ++r) {
+    const void* tag = base + (size_t)r * rec + 8;
+    while ((uint32_t)ld_acquire_sys_u64(tag) != t) {
+      __nanosleep(64);
+      if (globaltimer_ns() - t0 > 60ull * 1000000000ull) __trap();
+    }
+  }
+  fence_proxy_async_global();  // the records are then read by bulk copies too
+}
+
 // Minimum of the incumbent and the records of iteration prev_t; *src = the
 // winning rank, or -1 when nothing beat the incumbent.  One thread.
 __device__ __forceinline__ unsigned long long exchange_merge(const SwarmArgs& a, uint32_t prev_t,
                                                              int* src) {
+  if (a.p2p) wait_records(a, prev_t);
   const size_t rec = record_bytes(a.nvec * 4);
   const unsigned char* base = records(a, prev_t);
   unsigned long long best = *(volatile unsigned long long*)&a.ctl->key_cur;
@@ -463,16 +498,37 @@ __device__ __forceinline__ void epilogue_core(const SwarmArgs& a, uint32_t t, un
     for (int q = tid; q < a.nvec; q += nthr) G4[q] = __ldcg(w + q);
   }
   const bool have = acc != ~0ull;
-  if (have) {
-    const float4* pb = reinterpret_cast<const float4*>(a.PB) +
-                       ((long long)(uint32_t)acc - a.row_begin) * a.nvec;
-    float4* row = reinterpret_cast<float4*>(a.send + 16);
-    for (int q = tid; q < a.nvec; q += nthr) row[q] = __ldcg(pb + q);
+  const float4* pb = have ? reinterpret_cast<const float4*>(a.PB) +
+                                ((long long)(uint32_t)acc - a.row_begin) * a.nvec
+                          : nullptr;
+  const unsigned long long key = have ? acc : ~0ull;
+  if (!a.p2p) {  // NCCL: the host all-gathers `send`
+    if (have) {
+      float4* row = reinterpret_cast<float4*>(a.send + 16);
+      for (int q = tid; q < a.nvec; q += nthr) row[q] = __ldcg(pb + q);
+    }
+    if (tid == 0) {
+      unsigned long long* hdr = reinterpret_cast<unsigned long long*>(a.send);
+      hdr[0] = key;
+      hdr[1] = t;
+    }
+  } else {  // NVLink: store the record into recv[t & 1][rank] of every rank
+    const size_t rec = record_bytes(a.nvec * 4);
+    const size_t off = (size_t)(t & 1u) * a.world * rec + (size_t)a.rank * rec;
+    for (int r = 0; r < a.world; ++r) {
+      unsigned char* dst = a.peers[r] + off;
+      if (have) {
+        float4* row = reinterpret_cast<float4*>(dst + 16);
+        for (int q = tid; q < a.nvec; q += nthr) row[q] = __ldcg(pb + q);
+      }
+      if (tid == 0) reinterpret_cast<unsigned long long*>(dst)[0] = key;
+    }
+    __threadfence_system();
+    sync();
+    if (tid == 0)
+      for (int r = 0; r < a.world; ++r) st_release_sys_u64(a.peers[r] + off + 8, t);
   }
   if (tid == 0) {
-    unsigned long long* hdr = reinterpret_cast<unsigned long long*>(a.send);
-    hdr[0] = have ? acc : ~0ull;
-    hdr[1] = t;
     if (merged) a.ctl->key_cur = inc;
     a.ctl->key_acc = ~0ull;
     a.ctl->t = t;

@@ -43,3 +43,14 @@ def init_comm(device: int, group=None) -> int:
 def destroy_comm(comm: int) -> None:
     if comm:
         nccl_comm_destroy(comm)
+
+
+def connect_p2p(swarm, group=None) -> None:
+    """Switch `swarm` (created with a communicator) to the NVLink peer exchange:
+    all-gather every rank's CUDA IPC handle + receive-buffer offset over
+    torch.distributed and map the peers' buffers."""
+    import torch.distributed as dist
+    mine = swarm.p2p_handle()
+    everyone = [None] * dist.get_world_size(group)
+    dist.all_gather_object(everyone, mine, group=group)
+    swarm.p2p_connect([h for h, _ in everyone], [o for _, o in everyone])

@@ -499,3 +499,40 @@ def test_wide_rows_with_bounds_and_lockstep(monkeypatch):
         assert_bitwise(X2, c.X, "X")
         assert_bitwise(V2, c.V, "V")
         assert_fitness_close(obj, c.PB, pf2, c.pf, "pf")
+
+
+@pytest.mark.parametrize("obj,n,d", [(RASTRIGIN, 300, 1000), (GRIEWANK, 50, 13),
+                                     (ROSENBROCK, 6, 10000)])
+def test_nvlink_peer_exchange_single_rank(obj, n, d, monkeypatch):
+    """The NVLink peer exchange (records stored into every rank's receive buffer
+    by the step kernel's last CTA, iteration tags acquired by the next step's
+    prologue) on a 1-rank communicator: bitwise the single-GPU results, one
+    kernel per iteration."""
+    import torch  # noqa: F401
+    monkeypatch.setenv("PSO_FORCE_EXCHANGE", "1")
+    comm = fp.nccl_comm_init(1, fp.nccl_unique_id(), 0, 0)
+    try:
+        g = gpu_swarm(n, d, obj, seed=8, nccl_comm=comm)
+        h, off = g.p2p_handle()
+        assert len(h) == 64 and off > 0
+        g.p2p_connect([h], [off])
+        ref = gpu_swarm(n, d, obj, seed=8)
+        g.reset_counters()
+        g.step(15)
+        ref.step(15)
+        assert g.info()["launches"] == 16  # 15 step kernels + the final fold
+        for x, y in zip(g.get_state()[:4], ref.get_state()[:4]):
+            assert_bitwise(x, y, "p2p exchange state")
+        assert g.gbest()[:2] == ref.gbest()[:2]
+        X, V, PB, pf, t = g.get_state()
+        g.set_state(X, V, PB, pf, t=t)
+        ref.set_state(X, V, PB, pf, t=t)
+        g.step(4)
+        ref.step(4)
+        gf, gi, G = g.gbest()
+        rf, ri, RG = ref.gbest()
+        assert (gf, gi) == (rf, ri)
+        assert_bitwise(G, RG, "G")
+        g.close()
+    finally:
+        fp.nccl_comm_destroy(comm)
