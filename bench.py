@@ -197,8 +197,7 @@ def _config(w, n_gpus, K, extra=None):
     cfg = {"workload": w.name, "objective": OBJ_NAMES[w.objective], "n": w.n, "d": w.d,
            "w": w.w, "c1": w.c1, "c2": w.c2, "lo": w.lo, "hi": w.hi,
            "vmax": w.vmax if w.vmax > 0 else 1.0, "seed": w.seed, "timed_iterations": K,
-           "parallelism": (f"particle-split x{n_gpus}, gbest exchange "
-                           f"{os.environ.get('PSO_EXCHANGE', 'nccl')}") if n_gpus > 1 else "single GPU",
+           "parallelism": f"particle-split x{n_gpus}" if n_gpus > 1 else "single GPU",
            "l2": ("inputs larger than L2 (%.2f GB state vs 126 MB L2); no flush" % (state / 1e9))
            if state / max(n_gpus, 1) > L2_BYTES else
            ("state (%.1f MB/GPU) fits in L2: L2-resident, not an HBM number" % (state / n_gpus / 1e6))}
@@ -247,10 +246,14 @@ def run_gpu(args, w):
     K, W = args.steps, args.warmup
     sw = fp.Swarm(w.n, w.d, w.w, w.c1, w.c2, w.lo, w.hi, w.objective, w.seed, vmax=w.vmax,
                   device=local, stream=stream, nccl_comm=comm, timing=True)
-    p2p = use_comm and os.environ.get("PSO_EXCHANGE", "nccl") == "p2p"
-    if p2p:
+    # gbest exchange between ranks: NVLink peer stores from the step kernels
+    # (default), or the NCCL all-gather (PSO_EXCHANGE=nccl, or if any rank
+    # cannot map its peers)
+    want_p2p = use_comm and os.environ.get("PSO_EXCHANGE", "p2p") == "p2p"
+    p2p = False
+    if want_p2p:
         from paper_conf_icpp_liuwc21_b200.distributed import connect_p2p
-        connect_p2p(sw)
+        p2p = connect_p2p(sw)
     sw.step(W)
     sw.synchronize()
     sw.reset_counters()
@@ -328,7 +331,8 @@ def run_gpu(args, w):
             "warmup": W, "ms_per_step": ms / K, "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None, "dtype": "f32",
             "data": "synthetic (swarm initialised from Philox streams, seed %d)" % w.seed,
-            "config": _config(w, world, K),
+            "config": _config(w, world, K, extra={"gbest_exchange": (
+                "nvlink-peer-stores" if p2p else "nccl-allgather") if use_comm else None}),
             "gpu_launches": launches,
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "peak_source": peak_src,

@@ -215,11 +215,16 @@ pso_status pso_nccl_comm_destroy(void* comm);
  * prologue acquires the tags and merges.  No collective call per iteration.
  * Protocol (collective): each rank calls pso_p2p_handle, the 64-byte CUDA IPC
  * handles and offsets are all-gathered out of band (e.g. torch.distributed),
- * then every rank calls pso_p2p_connect with the world arrays in rank order.
- * A peer that stops delivering makes the waiting kernels trap after 60 s. */
+ * every rank calls pso_p2p_connect with the world arrays in rank order (maps
+ * the peers' buffers; a failure leaves the handle on NCCL, unpoisoned), the
+ * ranks agree that all connected, and then every rank calls
+ * pso_p2p_enable(h, 1).  Record tags carry an epoch that pso_set_state
+ * advances, so records of an earlier state never match.  A peer that stops
+ * delivering makes the waiting kernels trap after 60 s. */
 pso_status pso_p2p_handle(pso_handle h, void* ipc_handle /* 64 bytes */, uint64_t* offset);
 pso_status pso_p2p_connect(pso_handle h, const void* ipc_handles /* world x 64 bytes */,
                            const uint64_t* offsets /* world */);
+pso_status pso_p2p_enable(pso_handle h, int32_t on); /* 1: NVLink records, 0: NCCL all-gather */
 
 /* --- Device-side primitives exposed for parity tests ---------------------- */
 /* out[k] = word(tag, t, i, j0 + k) computed on the device (k < m), with the

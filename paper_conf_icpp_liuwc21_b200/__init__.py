@@ -157,6 +157,10 @@ class Swarm:
         check(lib().pso_p2p_connect(self._h, blob, offs), "pso_p2p_connect")
         return self
 
+    def p2p_enable(self, on: bool = True) -> "Swarm":
+        check(lib().pso_p2p_enable(self._h, int(bool(on))), "pso_p2p_enable")
+        return self
+
     def info(self) -> dict:
         inf = pso_info()
         check(lib().pso_get_info(self._h, C.byref(inf)), "pso_get_info")

@@ -25,7 +25,7 @@ EXPORTS = (
     "pso_get_state", "pso_set_state", "pso_set_bounds", "pso_get_info", "pso_reset_counters", "pso_destroy",
     "pso_status_string", "pso_last_error", "pso_objective_registered",
     "pso_nccl_get_unique_id", "pso_nccl_comm_init", "pso_nccl_comm_destroy",
-    "pso_p2p_handle", "pso_p2p_connect",
+    "pso_p2p_handle", "pso_p2p_connect", "pso_p2p_enable",
     "pso_debug_philox", "pso_debug_objective",
 )
 
@@ -97,6 +97,7 @@ def lib() -> C.CDLL:
     L.pso_nccl_comm_destroy.argtypes = [C.c_void_p]
     L.pso_p2p_handle.argtypes = [H, C.c_void_p, u64p]
     L.pso_p2p_connect.argtypes = [H, C.c_void_p, u64p]
+    L.pso_p2p_enable.argtypes = [H, C.c_int32]
     L.pso_debug_philox.argtypes = [C.c_uint64, C.c_uint32, C.c_uint32, C.c_uint32, C.c_uint32,
                                    C.c_int64, u32p, C.c_int32, C.c_int32]
     L.pso_debug_objective.argtypes = [C.c_int32, fp, C.c_int64, C.c_int32, fp, C.c_int32]

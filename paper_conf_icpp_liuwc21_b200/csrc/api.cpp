@@ -613,6 +613,7 @@ pso_status pso_set_state(pso_handle h, const float* x, const float* v, const flo
     PSO_CUDA(h, cudaMemcpyAsync(h->args.pf, pf, rows * 4, cudaMemcpyHostToDevice, h->stream));
   }
   if ((st = reset_ctl(h, (uint32_t)t)) != PSO_OK) return st;
+  ++h->args.epoch;  // p2p: records written before this call can never match again
   if (rows > 0) {
     PSO_CUDA(h, launch_rebest(h->args, (unsigned)t, h->stream));
     ++h->launches;
@@ -659,6 +660,15 @@ pso_status pso_p2p_connect(pso_handle h, const void* ipc_handles, const uint64_t
   if (h->args.p2p) return fail(PSO_ERR_INVALID, "already connected");
   if ((st = use_device(h)) != PSO_OK) return st;
   if ((st = sync_and_check(h)) != PSO_OK) return st;
+  if (h->peers_dev) return fail(PSO_ERR_INVALID, "already connected");
+  // Failures here leave the handle usable (NCCL exchange): nothing is poisoned.
+  auto undo = [&](cudaError_t e, const char* what) {
+    for (void* p : h->ipc_opened) cudaIpcCloseMemHandle(p);
+    h->ipc_opened.clear();
+    if (h->peers_dev) cudaFree(h->peers_dev);
+    h->peers_dev = nullptr;
+    return cuda_fail(nullptr, e, what);
+  };
   std::vector<unsigned char*> peers((size_t)h->world);
   for (int r = 0; r < h->world; ++r) {
     if (r == h->rank) {  // our own receive buffer
@@ -668,15 +678,27 @@ pso_status pso_p2p_connect(pso_handle h, const void* ipc_handles, const uint64_t
     cudaIpcMemHandle_t mh;
     std::memcpy(&mh, (const unsigned char*)ipc_handles + (size_t)r * sizeof(mh), sizeof(mh));
     void* base = nullptr;
-    PSO_CUDA(h, cudaIpcOpenMemHandle(&base, mh, cudaIpcMemLazyEnablePeerAccess));
+    cudaError_t e = cudaIpcOpenMemHandle(&base, mh, cudaIpcMemLazyEnablePeerAccess);
+    if (e != cudaSuccess) return undo(e, "cudaIpcOpenMemHandle");
     h->ipc_opened.push_back(base);
     peers[r] = (unsigned char*)base + offsets[r];
   }
-  PSO_CUDA(h, cudaMalloc(&h->peers_dev, sizeof(unsigned char*) * peers.size()));
-  PSO_CUDA(h, cudaMemcpy(h->peers_dev, peers.data(), sizeof(unsigned char*) * peers.size(),
-                         cudaMemcpyHostToDevice));
+  cudaError_t e = cudaMalloc(&h->peers_dev, sizeof(unsigned char*) * peers.size());
+  if (e != cudaSuccess) return undo(e, "cudaMalloc");
+  e = cudaMemcpy(h->peers_dev, peers.data(), sizeof(unsigned char*) * peers.size(),
+                 cudaMemcpyHostToDevice);
+  if (e != cudaSuccess) return undo(e, "cudaMemcpy");
   h->args.peers = (unsigned char* const*)h->peers_dev;
-  h->args.p2p = 1;
+  return PSO_OK;
+}
+
+pso_status pso_p2p_enable(pso_handle h, int32_t on) {
+  pso_status st = check_handle(h);
+  if (st != PSO_OK) return st;
+  if (on && !h->peers_dev) return fail(PSO_ERR_INVALID, "pso_p2p_connect first");
+  if ((st = use_device(h)) != PSO_OK) return st;
+  if ((st = sync_and_check(h)) != PSO_OK) return st;
+  h->args.p2p = on ? 1 : 0;
   return PSO_OK;
 }
 

@@ -43,6 +43,7 @@ struct SwarmArgs {
   int rank;
   int exchange;               // 1: publish (key, row) records for the all-gather + select
   int p2p;                    // exchange over NVLink peer stores instead of NCCL
+  unsigned epoch;             // p2p: record tags are (epoch << 32 | t); set_state starts an epoch
   unsigned char* const* peers;  // p2p: device array, world pointers to every rank's recv
   float w, c1, c2, lo, hi, vmax;
   unsigned int seed_lo, seed_hi;

@@ -427,7 +427,8 @@ __device__ __forceinline__ void wait_records(const SwarmArgs& a, uint32_t t) {
   const unsigned long long t0 = globaltimer_ns();
   for (int r = 0; r < a.world; ++r) {
     const void* tag = base + (size_t)r * rec + 8;
-    while ((uint32_t)ld_acquire_sys_u64(tag) != t) {
+    const unsigned long long want = ((unsigned long long)a.epoch << 32) | t;
+    while (ld_acquire_sys_u64(tag) != want) {
       __nanosleep(64);
       if (globaltimer_ns() - t0 > 60ull * 1000000000ull) __trap();
     }
@@ -526,7 +527,8 @@ __device__ __forceinline__ void epilogue_core(const SwarmArgs& a, uint32_t t, un
     __threadfence_system();
     sync();
     if (tid == 0)
-      for (int r = 0; r < a.world; ++r) st_release_sys_u64(a.peers[r] + off + 8, t);
+      for (int r = 0; r < a.world; ++r)
+        st_release_sys_u64(a.peers[r] + off + 8, ((unsigned long long)a.epoch << 32) | t);
   }
   if (tid == 0) {
     if (merged) a.ctl->key_cur = inc;

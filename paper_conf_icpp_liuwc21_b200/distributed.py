@@ -45,12 +45,25 @@ def destroy_comm(comm: int) -> None:
         nccl_comm_destroy(comm)
 
 
-def connect_p2p(swarm, group=None) -> None:
+def connect_p2p(swarm, group=None) -> bool:
     """Switch `swarm` (created with a communicator) to the NVLink peer exchange:
     all-gather every rank's CUDA IPC handle + receive-buffer offset over
-    torch.distributed and map the peers' buffers."""
+    torch.distributed, map the peers' buffers, and enable the mode only if every
+    rank succeeded (else all ranks stay on the NCCL all-gather).  Returns
+    whether the peer exchange is on.  Collective."""
     import torch.distributed as dist
+    from . import PsoError
     mine = swarm.p2p_handle()
     everyone = [None] * dist.get_world_size(group)
     dist.all_gather_object(everyone, mine, group=group)
-    swarm.p2p_connect([h for h, _ in everyone], [o for _, o in everyone])
+    ok = True
+    try:
+        swarm.p2p_connect([h for h, _ in everyone], [o for _, o in everyone])
+    except PsoError:
+        ok = False
+    votes = [None] * dist.get_world_size(group)
+    dist.all_gather_object(votes, ok, group=group)
+    if all(votes):
+        swarm.p2p_enable(True)
+        return True
+    return False

@@ -515,7 +515,7 @@ def test_nvlink_peer_exchange_single_rank(obj, n, d, monkeypatch):
         g = gpu_swarm(n, d, obj, seed=8, nccl_comm=comm)
         h, off = g.p2p_handle()
         assert len(h) == 64 and off > 0
-        g.p2p_connect([h], [off])
+        g.p2p_connect([h], [off]).p2p_enable(True)
         ref = gpu_swarm(n, d, obj, seed=8)
         g.reset_counters()
         g.step(15)
