@@ -661,6 +661,8 @@ pso_status pso_p2p_connect(pso_handle h, const void* ipc_handles, const uint64_t
   if ((st = use_device(h)) != PSO_OK) return st;
   if ((st = sync_and_check(h)) != PSO_OK) return st;
   if (h->peers_dev) return fail(PSO_ERR_INVALID, "already connected");
+  if (h->n_local == 0)  // records are written by step kernels; an empty shard runs none
+    return fail(PSO_ERR_UNSUPPORTED, "rank owns no particles: use the NCCL exchange");
   // Failures here leave the handle usable (NCCL exchange): nothing is poisoned.
   auto undo = [&](cudaError_t e, const char* what) {
     for (void* p : h->ipc_opened) cudaIpcCloseMemHandle(p);
