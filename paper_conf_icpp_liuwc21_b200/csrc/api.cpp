@@ -448,11 +448,16 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
   const size_t gb = align_up((size_t)h->pitch * 4, 256);
   const size_t ctlb = align_up(sizeof(DevCtl), 256);
   const size_t boundb = o.bounds ? align_up(4 * (size_t)h->pitch * 4, 256) : 0;
+  // lazy pbest rows on the TMA pipelines (step kernels that skip PB when PB == X)
+  const char* lz = std::getenv("PSO_LAZY_PB");
+  const bool lazy = h->cfg.tma && !h->cfg.resident && !h->cfg.gridres && !(lz && *lz == '0');
+  const size_t pbxb = lazy ? align_up(rows, 256) : 0;
   const size_t rec = align_up(record_bytes(h->pitch), 256);
   const size_t candb = h->cfg.gridres ? align_up(2 * (size_t)h->cfg.gridres_grid * h->pitch * 4, 256) : 0;
   const size_t sendb = h->xchg ? rec : 0;
   const size_t recvb = h->xchg ? 2 * (size_t)h->world * record_bytes(h->pitch) : 0;
-  h->arena_bytes = 3 * mat + pfb + gb + ctlb + boundb + candb + sendb + align_up(recvb, 256);
+  h->arena_bytes =
+      3 * mat + pfb + gb + ctlb + boundb + pbxb + candb + sendb + align_up(recvb, 256);
   {
     cudaError_t e = cudaMalloc(&h->arena, h->arena_bytes);
     if (e == cudaErrorMemoryAllocation) {
@@ -470,6 +475,8 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
   A.G = (float*)p; p += gb;
   A.ctl = (DevCtl*)p; p += ctlb;
   A.bounds = o.bounds ? (const float*)p : nullptr; p += boundb;
+  A.pbx = lazy ? p : nullptr; p += pbxb;
+  A.lazy_pb = lazy ? 1 : 0;
   A.cand = h->cfg.gridres ? (float*)p : nullptr; p += candb;
   A.send = h->xchg ? p : nullptr; p += sendb;
   A.recv = h->xchg ? p : nullptr;
@@ -583,7 +590,13 @@ pso_status pso_get_state(pso_handle h, float* x, float* v, float* pb, float* pf,
   if (rows > 0) {
     if (x) PSO_CUDA(h, cudaMemcpy2DAsync(x, w, h->args.X, sp, w, rows, cudaMemcpyDeviceToHost, h->stream));
     if (v) PSO_CUDA(h, cudaMemcpy2DAsync(v, w, h->args.V, sp, w, rows, cudaMemcpyDeviceToHost, h->stream));
-    if (pb) PSO_CUDA(h, cudaMemcpy2DAsync(pb, w, h->args.PB, sp, w, rows, cudaMemcpyDeviceToHost, h->stream));
+    if (pb) {
+      if (h->args.lazy_pb) {  // write out the deferred pbest rows (PB == X) first
+        PSO_CUDA(h, launch_materialize_pb(h->args, h->stream));
+        ++h->launches;
+      }
+      PSO_CUDA(h, cudaMemcpy2DAsync(pb, w, h->args.PB, sp, w, rows, cudaMemcpyDeviceToHost, h->stream));
+    }
     if (pf) PSO_CUDA(h, cudaMemcpyAsync(pf, h->args.pf, rows * 4, cudaMemcpyDeviceToHost, h->stream));
   }
   if ((st = sync_and_check(h)) != PSO_OK) return st;
@@ -611,6 +624,7 @@ pso_status pso_set_state(pso_handle h, const float* x, const float* v, const flo
     PSO_CUDA(h, cudaMemcpy2DAsync(h->args.V, sp, v, w, w, rows, cudaMemcpyHostToDevice, h->stream));
     PSO_CUDA(h, cudaMemcpy2DAsync(h->args.PB, sp, pb, w, w, rows, cudaMemcpyHostToDevice, h->stream));
     PSO_CUDA(h, cudaMemcpyAsync(h->args.pf, pf, rows * 4, cudaMemcpyHostToDevice, h->stream));
+    if (h->args.lazy_pb) PSO_CUDA(h, cudaMemsetAsync(h->args.pbx, 0, rows, h->stream));
   }
   if ((st = reset_ctl(h, (uint32_t)t)) != PSO_OK) return st;
   ++h->args.epoch;  // p2p: records written before this call can never match again

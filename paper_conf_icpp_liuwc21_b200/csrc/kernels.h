@@ -33,6 +33,8 @@ struct SwarmArgs {
   float* G;   // pitch (gbest position)
   float* cand;                // grid-resident kernel: [2][grid][pitch] candidate rows
   const float* bounds;        // per-dimension bounds [vlo | vhi | xlo | xhi] (4 x pitch), or null
+  unsigned char* pbx;         // lazy pbest: 1 = the row's PB equals its X (PB not stored)
+  int lazy_pb;
   unsigned char* send;        // world > 1: this rank's exchange record
   const unsigned char* recv;  // exchange: [2 iteration parities][world] records after the all-gather
   DevCtl* ctl;
@@ -110,6 +112,8 @@ cudaError_t launch_gridres(int objective, const SwarmArgs& a, const LaunchCfg& c
                            cudaStream_t s);
 cudaError_t launch_rebest(const SwarmArgs& a, unsigned t, cudaStream_t s);
 cudaError_t launch_select(const SwarmArgs& a, unsigned t, cudaStream_t s);
+// lazy pbest: copy X -> PB for flagged rows and clear the flags (host reads)
+cudaError_t launch_materialize_pb(const SwarmArgs& a, cudaStream_t s);
 
 cudaError_t debug_philox(unsigned long long seed, unsigned tag, unsigned t, unsigned i,
                          unsigned j0, long long m, unsigned* out_dev, int use_curand,

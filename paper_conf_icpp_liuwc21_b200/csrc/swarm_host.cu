@@ -35,7 +35,7 @@ __global__ void __launch_bounds__(256) k_rebest(const SwarmArgs a, unsigned t) {
   if (tid == 0)
     for (int w = 1; w < (nthr >> 5); ++w) best = s_best[w] < best ? s_best[w] : best;
   if (cta_finish<NoObj>(a, sm, tid == 0 ? best : ~0ull, 0, tid, nthr))
-    gbest_epilogue<NoObj>(a, sm, t, tid, nthr);
+    gbest_epilogue<NoObj>(a, sm, t, tid, nthr, ~0ull, -1, a.PB);  // pbest rows given by the host
 }
 
 // ---------------------------------------------------------- select kernel
@@ -61,6 +61,22 @@ __global__ void __launch_bounds__(128) k_select(const SwarmArgs a, unsigned t) {
   }
   __syncthreads();
   if (threadIdx.x == 0 && src >= 0) a.ctl->key_cur = s_best;
+}
+
+// ---------------------------------------------------------- materialize PB
+// Lazy pbest rows (PB == X, not stored): one warp per flagged row copies X -> PB.
+__global__ void __launch_bounds__(256) k_materialize_pb(const SwarmArgs a) {
+  const int lane = threadIdx.x & 31;
+  const long long warps = (long long)gridDim.x * (blockDim.x >> 5);
+  for (long long r = blockIdx.x * (long long)(blockDim.x >> 5) + (threadIdx.x >> 5); r < a.n_local;
+       r += warps) {
+    if (!a.pbx[r]) continue;
+    const float4* x = reinterpret_cast<const float4*>(a.X) + r * a.nvec;
+    float4* pb = reinterpret_cast<float4*>(a.PB) + r * a.nvec;
+    for (int q = lane; q < a.nvec; q += 32) pb[q] = x[q];
+    __syncwarp();
+    if (lane == 0) a.pbx[r] = 0;
+  }
 }
 
 // ---------------------------------------------------------- dispatch
@@ -380,6 +396,14 @@ cudaError_t launch_rebest(const SwarmArgs& a, unsigned t, cudaStream_t s) {
   if (blocks > 1024) blocks = 1024;
   if (blocks < 1) blocks = 1;
   k_rebest<<<(unsigned)blocks, 256, 0, s>>>(a, t);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_materialize_pb(const SwarmArgs& a, cudaStream_t s) {
+  if (!a.lazy_pb || a.n_local < 1) return cudaSuccess;
+  long long blocks = (a.n_local + 7) / 8;
+  if (blocks > 2048) blocks = 2048;
+  k_materialize_pb<<<(unsigned)blocks, 256, 0, s>>>(a);
   return cudaGetLastError();
 }
 

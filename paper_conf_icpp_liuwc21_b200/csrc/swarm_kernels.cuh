@@ -470,10 +470,12 @@ __device__ __forceinline__ const float* merged_gbest_row(const SwarmArgs& a, uin
 //   exchange:   commit the prologue's merge (inc from rank `src`) to key_cur /
 //               G, then write the local candidate record (strictly below inc)
 //               for the all-gather, tagged with t; reset the accumulator.
+// `rows` holds the winning candidate's position: X for the step and init
+// kernels (a candidate improved, so its x' is its pbest), PB for rebest.
 template <class SyncF>
 __device__ __forceinline__ void epilogue_core(const SwarmArgs& a, uint32_t t, unsigned long long inc,
                                               int src, unsigned long long* sh, int tid, int nthr,
-                                              SyncF sync) {
+                                              SyncF sync, const float* rows) {
   if (tid == 0) {
     __threadfence();
     sh[0] = *(volatile unsigned long long*)&a.ctl->key_acc;
@@ -485,7 +487,7 @@ __device__ __forceinline__ void epilogue_core(const SwarmArgs& a, uint32_t t, un
   if (!a.exchange) {
     const bool have = acc < cur;
     if (have) {
-      const float4* pb = reinterpret_cast<const float4*>(a.PB) +
+      const float4* pb = reinterpret_cast<const float4*>(rows) +
                          ((long long)(uint32_t)acc - a.row_begin) * a.nvec;
       for (int q = tid; q < a.nvec; q += nthr) G4[q] = __ldcg(pb + q);
     }
@@ -502,7 +504,7 @@ __device__ __forceinline__ void epilogue_core(const SwarmArgs& a, uint32_t t, un
     for (int q = tid; q < a.nvec; q += nthr) G4[q] = __ldcg(w + q);
   }
   const bool have = acc != ~0ull;
-  const float4* pb = have ? reinterpret_cast<const float4*>(a.PB) +
+  const float4* pb = have ? reinterpret_cast<const float4*>(rows) +
                                 ((long long)(uint32_t)acc - a.row_begin) * a.nvec
                           : nullptr;
   const unsigned long long key = have ? acc : ~0ull;
@@ -544,15 +546,15 @@ __device__ __forceinline__ void epilogue_core(const SwarmArgs& a, uint32_t t, un
 template <class Obj>
 __device__ __forceinline__ void gbest_epilogue(const SwarmArgs& a, RowSmem<Obj>& sm, uint32_t t,
                                                int tid, int nthr, unsigned long long inc = ~0ull,
-                                               int src = -1) {
-  epilogue_core(a, t, inc, src, &sm.acc, tid, nthr, [&] { team_sync(nthr); });
+                                               int src = -1, const float* rows = nullptr) {
+  epilogue_core(a, t, inc, src, &sm.acc, tid, nthr, [&] { team_sync(nthr); }, rows ? rows : a.X);
 }
 
 // The same epilogue run by one warp (the finaliser warp of the TMA kernels).
 __device__ __forceinline__ void warp_gbest_epilogue(const SwarmArgs& a, uint32_t t, int lane,
                                                     unsigned long long inc = ~0ull, int src = -1) {
   __shared__ unsigned long long sh[2];
-  epilogue_core(a, t, inc, src, sh, lane, 32, [] { __syncwarp(); });
+  epilogue_core(a, t, inc, src, sh, lane, 32, [] { __syncwarp(); }, a.X);
 }
 
 // Publish this CTA's candidate and improvement count; true in the last CTA
@@ -681,6 +683,7 @@ __global__ void __launch_bounds__(kMaxThreads + 64, 2)
   __shared__ unsigned long long full[kMaxStages], empty[kMaxStages], done[kMaxStages], gbar;
   __shared__ unsigned long long s_inc;  // incumbent of this iteration (after the exchange merge)
   __shared__ int s_src;
+  __shared__ int sflag[kMaxStages];     // lazy pbest: the stage's row had PB == X (pb not loaded)
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   if (tid == 0) {
     mbar_init(&gbar, 1);
@@ -712,13 +715,18 @@ __global__ void __launch_bounds__(kMaxThreads + 64, 2)
       int s = 0;
       unsigned ph = 0;
       int k = 0;
+      // lazy pbest: rows whose PB equals X skip the pb load (flag prefetched one row ahead)
+      int fl_next = (a.lazy_pb && blockIdx.x < a.n_local) ? a.pbx[blockIdx.x] : 0;
       for (long long r = blockIdx.x; r < a.n_local; r += gridDim.x, ++k) {
+        const int fl = fl_next;
+        if (a.lazy_pb && r + gridDim.x < a.n_local) fl_next = a.pbx[r + gridDim.x];
         if (k >= stages) mbar_wait(&empty[s], ph ^ 1u);
         float4* st = ring + (size_t)s * 3 * nvec;
-        mbar_expect_tx(&full[s], 3u * row_bytes);
+        sflag[s] = fl;
+        mbar_expect_tx(&full[s], (fl ? 2u : 3u) * row_bytes);  // releases sflag[s] too
         bulk_g2s(st, a.X + (size_t)r * 4 * nvec, row_bytes, &full[s]);
         bulk_g2s(st + nvec, a.V + (size_t)r * 4 * nvec, row_bytes, &full[s]);
-        bulk_g2s(st + 2 * nvec, a.PB + (size_t)r * 4 * nvec, row_bytes, &full[s]);
+        if (!fl) bulk_g2s(st + 2 * nvec, a.PB + (size_t)r * 4 * nvec, row_bytes, &full[s]);
         if (++s == stages) {
           s = 0;
           ph ^= 1u;
@@ -752,10 +760,18 @@ __global__ void __launch_bounds__(kMaxThreads + 64, 2)
         const float f = Obj::finalize(c, d);
         const float4* st = ring + (size_t)s * 3 * nvec;
         const size_t off = (size_t)r * 4 * nvec;
-        bulk_s2g(a.X + off, st, row_bytes);
+        const int fl = sflag[s];
+        const float4* xnew = fl ? st + 2 * nvec : st;  // where the compute warps put x'
+        const bool improved = f < pf_old;  // Alg. 1 line 7: strict; NaN never improves
+        bulk_s2g(a.X + off, xnew, row_bytes);
         bulk_s2g(a.V + off, st + nvec, row_bytes);
-        if (f < pf_old) {  // Alg. 1 line 7: strict; NaN never improves
-          bulk_s2g(a.PB + off, st, row_bytes);
+        if (!a.lazy_pb) {
+          if (improved) bulk_s2g(a.PB + off, st, row_bytes);
+        } else {  // PB == X after an improvement: defer the copy until the row stops improving
+          if (fl && !improved) bulk_s2g(a.PB + off, st, row_bytes);  // st holds the old x
+          if ((int)improved != fl) a.pbx[r] = improved ? 1 : 0;
+        }
+        if (improved) {
           a.pf[r] = f;
           ++nimp;
         }
@@ -796,6 +812,10 @@ __global__ void __launch_bounds__(kMaxThreads + 64, 2)
     const uint32_t gi = (uint32_t)(a.row_begin + r);
     float4* st = ring + (size_t)s * 3 * nvec;
     mbar_wait(&full[s], ph);
+    // lazy pbest row (PB == X): pb is the loaded x, and x' goes to the pb slot
+    // so the old x stays available for a deferred PB store
+    const int fl = sflag[s];
+    float4* xdst = fl ? st + 2 * nvec : st;
     float acc[Obj::kAcc];
     Obj::init(acc);
     // VPT <= 2: fully unrolled for ILP; larger VPT: pairs, to bound registers.
@@ -804,7 +824,7 @@ __global__ void __launch_bounds__(kMaxThreads + 64, 2)
       const int q = tid + j * nthr;
       if (q < nvec) {
         float4 x = st[q], v = st[nvec + q];
-        const float4 pb = st[2 * nvec + q];
+        const float4 pb = fl ? x : st[2 * nvec + q];
         const float4 g = sG[q];
         const float4 r1 = raw24x4(key, kTagR1, t, gi, (uint32_t)q);
         const float4 r2 = raw24x4(key, kTagR2, t, gi, (uint32_t)q);
@@ -815,7 +835,7 @@ __global__ void __launch_bounds__(kMaxThreads + 64, 2)
           if (jj + 2 >= d) x.z = v.z = 0.f;
           if (jj + 3 >= d) x.w = v.w = 0.f;
         }
-        st[q] = x;
+        xdst[q] = x;
         st[nvec + q] = v;
         if constexpr (!Obj::kNeighbor) map4<Obj>(acc, x, 0.f, 4 * q, d);
       }
@@ -825,7 +845,7 @@ __global__ void __launch_bounds__(kMaxThreads + 64, 2)
 #pragma unroll(VPT <= 2 ? VPT : 2)
       for (int j = 0; j < VPT; ++j) {
         const int q = tid + j * nthr;
-        if (q < nvec) map4<Obj>(acc, st[q], (q + 1 < nvec) ? st[q + 1].x : 0.f, 4 * q, d);
+        if (q < nvec) map4<Obj>(acc, xdst[q], (q + 1 < nvec) ? xdst[q + 1].x : 0.f, 4 * q, d);
       }
     }
     warp_combine<Obj>(acc);
@@ -879,6 +899,7 @@ __global__ void __launch_bounds__(kMaxThreadsCluster + 64, 1)
   __shared__ unsigned long long pbar[kMaxStages], dbar[kMaxStages], gbar;
   __shared__ unsigned long long s_inc;  // incumbent of this iteration (after the exchange merge)
   __shared__ int s_src;
+  __shared__ int sflag[kMaxStages];     // lazy pbest: the stage's row had PB == X
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   if (tid == 0) {
     mbar_init(&gbar, 1);
@@ -917,15 +938,19 @@ __global__ void __launch_bounds__(kMaxThreadsCluster + 64, 1)
       int s = 0;
       unsigned ph = 0;
       int k = 0;
+      int fl_next = (a.lazy_pb && cid < a.n_local) ? a.pbx[cid] : 0;
       for (long long r = cid; r < a.n_local; r += ncl, ++k) {
+        const int fl = fl_next;
+        if (a.lazy_pb && r + ncl < a.n_local) fl_next = a.pbx[r + ncl];
         if (k >= stages) mbar_wait(&empty[s], ph ^ 1u);
         float4* st = ring + (size_t)s * 3 * chunk;
-        mbar_expect_tx(&full[s], 3u * blk_bytes);
+        sflag[s] = fl;
+        mbar_expect_tx(&full[s], (fl ? 2u : 3u) * blk_bytes);
         if (cnt > 0) {
           const size_t off = ((size_t)r * nvec + q0) * 4;
           bulk_g2s(st, a.X + off, blk_bytes, &full[s]);
           bulk_g2s(st + chunk, a.V + off, blk_bytes, &full[s]);
-          bulk_g2s(st + 2 * chunk, a.PB + off, blk_bytes, &full[s]);
+          if (!fl) bulk_g2s(st + 2 * chunk, a.PB + off, blk_bytes, &full[s]);
         }
         if (++s == stages) {
           s = 0;
@@ -958,12 +983,14 @@ __global__ void __launch_bounds__(kMaxThreadsCluster + 64, 1)
           Obj::combine(c, b);
         }
         const float4* st = ring + (size_t)s * 3 * chunk;
+        const int fl = sflag[s];
+        const float4* xnew = fl ? st + 2 * chunk : st;  // where the compute warps put x'
         // publish {partial, first x', last x'} to CTA 0 (one 16-byte st.async)
         {
           float4 msg = make_float4(c[0], Obj::kAcc > 1 ? c[Obj::kAcc - 1] : 0.f, 0.f, 0.f);
           if (Obj::kNeighbor && cnt > 0) {
-            msg.z = st[0].x;
-            msg.w = st[cnt - 1].w;
+            msg.z = xnew[0].x;
+            msg.w = xnew[cnt - 1].w;
           }
           st_async_v4(map_to_rank(&parts[s][crank], 0), msg, map_to_rank(&pbar[s], 0));
         }
@@ -994,6 +1021,7 @@ __global__ void __launch_bounds__(kMaxThreadsCluster + 64, 1)
             a.pf[r] = f;
             ++nimp;
           }
+          if (a.lazy_pb && (int)(imp != 0.f) != fl) a.pbx[r] = imp != 0.f ? 1 : 0;
           if (f == f && ord_f32(f) < inc_ord) {  // strictly below gf
             const unsigned long long key = pack_key(f, gi);
             best = key < best ? key : best;
@@ -1003,9 +1031,13 @@ __global__ void __launch_bounds__(kMaxThreadsCluster + 64, 1)
         const bool improved = dec[s].x != 0.f;
         if (cnt > 0) {
           const size_t off = ((size_t)r * nvec + q0) * 4;
-          bulk_s2g(a.X + off, st, blk_bytes);
+          bulk_s2g(a.X + off, xnew, blk_bytes);
           bulk_s2g(a.V + off, st + chunk, blk_bytes);
-          if (improved) bulk_s2g(a.PB + off, st, blk_bytes);
+          if (!a.lazy_pb) {
+            if (improved) bulk_s2g(a.PB + off, st, blk_bytes);
+          } else if (fl && !improved) {
+            bulk_s2g(a.PB + off, st, blk_bytes);  // deferred copy of the old x
+          }
         }
         bulk_commit();
         if (prev >= 0) {
@@ -1040,6 +1072,8 @@ __global__ void __launch_bounds__(kMaxThreadsCluster + 64, 1)
     const uint32_t gi = (uint32_t)(a.row_begin + r);
     float4* st = ring + (size_t)s * 3 * chunk;
     mbar_wait(&full[s], ph);
+    const int fl = sflag[s];
+    float4* xdst = fl ? st + 2 * chunk : st;
     float acc[Obj::kAcc];
     Obj::init(acc);
 #pragma unroll(VPT <= 2 ? VPT : 2)
@@ -1048,7 +1082,7 @@ __global__ void __launch_bounds__(kMaxThreadsCluster + 64, 1)
       if (ql < cnt) {
         const int q = q0 + ql;
         float4 x = st[ql], v = st[chunk + ql];
-        const float4 pb = st[2 * chunk + ql];
+        const float4 pb = fl ? x : st[2 * chunk + ql];
         const float4 g = sG[ql];
         const float4 r1 = raw24x4(key, kTagR1, t, gi, (uint32_t)q);
         const float4 r2 = raw24x4(key, kTagR2, t, gi, (uint32_t)q);
@@ -1059,7 +1093,7 @@ __global__ void __launch_bounds__(kMaxThreadsCluster + 64, 1)
           if (jj + 2 >= d) x.z = v.z = 0.f;
           if (jj + 3 >= d) x.w = v.w = 0.f;
         }
-        st[ql] = x;
+        xdst[ql] = x;
         st[chunk + ql] = v;
         if constexpr (!Obj::kNeighbor) map4<Obj>(acc, x, 0.f, 4 * q, d);
       }
@@ -1071,9 +1105,9 @@ __global__ void __launch_bounds__(kMaxThreadsCluster + 64, 1)
         const int ql = tid + j * nthr;
         if (ql < cnt) {
           const int q = q0 + ql;
-          const float4 x = st[ql];
+          const float4 x = xdst[ql];
           if (ql + 1 < cnt) {
-            map4<Obj>(acc, x, st[ql + 1].x, 4 * q, d);
+            map4<Obj>(acc, x, xdst[ql + 1].x, 4 * q, d);
           } else if (!row_tail) {
             map4<Obj>(acc, x, 0.f, 4 * q, d);  // the row's last float4
           } else {  // x_{j+1} of the last dim lives in the next block: CTA 0 adds it
@@ -1514,7 +1548,7 @@ __global__ void __launch_bounds__(kMaxThreads, (VPT >= 8) ? 1 : 2)
       init_float4(a, key, gi, q, x, v);
       st_stream(Xr + q, x);
       st_stream(Vr + q, v);
-      st_stream(Pr + q, x);
+      if (!a.lazy_pb) st_stream(Pr + q, x);  // lazy pbest: PB == X is recorded in pbx
       float nx = 0.f;
       if constexpr (Obj::kNeighbor) {
         if (q + 1 < nvec) {
@@ -1530,6 +1564,7 @@ __global__ void __launch_bounds__(kMaxThreads, (VPT >= 8) ? 1 : 2)
     if (tid == 0) {
       if (f != f) f = __int_as_float(0x7f800000);  // reading 11: NaN -> +inf
       a.pf[r] = f;
+      if (a.lazy_pb) a.pbx[r] = 1;
       if (ord_f32(f) < inc_ord) {
         const unsigned long long k = pack_key(f, gi);
         best = k < best ? k : best;
