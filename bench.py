@@ -277,8 +277,15 @@ def run_gpu(args, w):
     total_updates = w.n * w.d * K
     value = total_updates / (ms / 1e3)
     rho = improvements / max(n_local * K, 1)
-    # algorithmic bytes per launch of the step kernel
-    bytes_per_update = 20.0 + 4.0 * rho
+    # algorithmic bytes per launch of the step kernel: x, v read and
+    # written every row; pbest rows read / written only where the kernel must
+    # (pb_loads / pb_stores counted in-kernel: with lazy pbest rows a row whose
+    # pbest equals x skips both); pf read + written on improvement
+    pbl = info["pb_loads"] / max(n_local * K, 1)
+    pbs = info["pb_stores"] / max(n_local * K, 1)
+    if info["resident"]:  # state held in shared memory: no per-iteration row traffic counted
+        pbl, pbs = 1.0, rho
+    bytes_per_update = 16.0 + 4.0 * pbl + 4.0 * pbs
     alg_bytes = n_local * w.d * bytes_per_update + n_local * (4.0 + 4.0 * rho)
     achieved = alg_bytes / (kern_ms / 1e3) / 1e9
     peak, peak_src = hbm_peak()
@@ -340,6 +347,8 @@ def run_gpu(args, w):
                          "kernel": "k_step (fused move+eval+pbest+gbest)",
                          "kernel_avg_us": kern_ms * 1e3,
                          "bytes_per_update": bytes_per_update, "rho": rho,
+                         "pb_load_frac": pbl, "pb_store_frac": pbs,
+                         "lazy_pbest": bool(info["lazy_pb"]),
                          "alg_bytes_per_launch": alg_bytes,
                          "l2_resident": state_per_gpu <= L2_BYTES,
                          "cta": {"threads": info["threads_per_cta"], "vpt": info["vec_per_thread"],

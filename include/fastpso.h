@@ -182,6 +182,9 @@ typedef struct {
   uint64_t t;                    /* iterations done */
   uint64_t launches;             /* kernels launched by this handle so far */
   uint64_t improvements;         /* pbest improvements (rows) so far, all steps */
+  uint64_t pb_loads;             /* streaming kernels: pbest rows read from memory */
+  uint64_t pb_stores;            /* streaming kernels: pbest rows written to memory */
+  int32_t lazy_pb;               /* 1: rows whose pbest equals x skip the pb load/store */
   double step_kernel_ms;         /* PSO_FLAG_TIMING: summed step-kernel time */
   uint64_t step_kernel_count;    /* PSO_FLAG_TIMING: step kernels timed */
   size_t arena_bytes;            /* device bytes owned by the handle */

@@ -44,6 +44,7 @@ class pso_info(C.Structure):
         ("smem_bytes", C.c_int32), ("resident", C.c_int32), ("bounds", C.c_int32), ("cluster", C.c_int32),
         ("vmax", C.c_float), ("t", C.c_uint64),
         ("launches", C.c_uint64), ("improvements", C.c_uint64),
+        ("pb_loads", C.c_uint64), ("pb_stores", C.c_uint64), ("lazy_pb", C.c_int32),
         ("step_kernel_ms", C.c_double), ("step_kernel_count", C.c_uint64),
         ("arena_bytes", C.c_size_t),
     ]

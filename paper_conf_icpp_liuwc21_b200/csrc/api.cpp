@@ -759,6 +759,9 @@ pso_status pso_get_info(pso_handle h, pso_info* info) {
   info->t = h->t;
   info->launches = h->launches;
   info->improvements = c.improvements;
+  info->pb_loads = c.pb_loads;
+  info->pb_stores = c.pb_stores;
+  info->lazy_pb = h->args.lazy_pb;
   info->step_kernel_ms = h->timed_ms;
   info->step_kernel_count = h->timed_count;
   info->arena_bytes = h->arena_bytes;
@@ -774,8 +777,9 @@ pso_status pso_reset_counters(pso_handle h) {
   h->timed_ms = 0;
   h->timed_count = 0;
   h->events_used = 0;
-  unsigned long long zero = 0;
-  PSO_CUDA(h, cudaMemcpy(&h->args.ctl->improvements, &zero, 8, cudaMemcpyHostToDevice));
+  unsigned long long zero[2] = {0, 0};
+  PSO_CUDA(h, cudaMemcpy(&h->args.ctl->improvements, zero, 8, cudaMemcpyHostToDevice));
+  PSO_CUDA(h, cudaMemcpy(&h->args.ctl->pb_loads, zero, 16, cudaMemcpyHostToDevice));
   return PSO_OK;
 }
 

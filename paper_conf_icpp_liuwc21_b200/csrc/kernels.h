@@ -17,9 +17,11 @@ struct DevCtl {
   unsigned int t;                   // iterations done (low 32 bits; Philox ctr[2])
   unsigned long long key_par[2];    // grid-resident kernel: per-iteration-parity accumulators
   unsigned int bar_count, bar_gen;  // grid-resident kernel: grid barrier
-  unsigned long long pad;
+  unsigned long long pb_loads;      // streaming kernels: pbest rows read from HBM
+  unsigned long long pb_stores;     // streaming kernels: pbest rows written to HBM
+  unsigned long long pad[7];
 };
-static_assert(sizeof(DevCtl) == 64, "DevCtl is one 64-byte block");
+static_assert(sizeof(DevCtl) == 128, "DevCtl is two 64-byte blocks");
 
 // Exchange record for world > 1: the local candidate key and its PB row.
 // Layout: [u64 key][u64 pad][pitch floats].

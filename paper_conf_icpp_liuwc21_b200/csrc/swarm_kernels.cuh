@@ -650,6 +650,11 @@ __global__ void __launch_bounds__(kMaxThreads, (VPT >= 8) ? 1 : 2)
         [] {}, sG, sB, sFirst, sm, tid, nthr, pf_old, improved);
     if (tid == 0) row_bookkeeping(a, r, gi, f, improved, inc_ord, best, nimp);
   }
+  if (tid == 0) {  // traffic counters: every pbest row read, improved ones written
+    const long long rows = (a.n_local - blockIdx.x + gridDim.x - 1) / gridDim.x;
+    if (rows > 0) atomicAdd(&a.ctl->pb_loads, (unsigned long long)rows);
+    if (nimp) atomicAdd(&a.ctl->pb_stores, (unsigned long long)nimp);
+  }
   if (cta_finish<Obj>(a, sm, best, nimp, tid, nthr))
     gbest_epilogue<Obj>(a, sm, t, tid, nthr, sm.inc, sm.src);
 }
@@ -742,7 +747,7 @@ __global__ void __launch_bounds__(kMaxThreads + 64, 2)
       mbar_wait(&gbar, 0);
       const uint32_t inc_ord = (uint32_t)(s_inc >> 32);
       unsigned long long best = ~0ull;
-      unsigned nimp = 0;
+      unsigned nimp = 0, n_pbl = 0, n_pbs = 0;
       int s = 0, prev = -1;
       unsigned ph = 0;
       for (long long r = blockIdx.x; r < a.n_local; r += gridDim.x) {
@@ -765,10 +770,17 @@ __global__ void __launch_bounds__(kMaxThreads + 64, 2)
         const bool improved = f < pf_old;  // Alg. 1 line 7: strict; NaN never improves
         bulk_s2g(a.X + off, xnew, row_bytes);
         bulk_s2g(a.V + off, st + nvec, row_bytes);
+        n_pbl += fl ? 0u : 1u;
         if (!a.lazy_pb) {
-          if (improved) bulk_s2g(a.PB + off, st, row_bytes);
+          if (improved) {
+            bulk_s2g(a.PB + off, st, row_bytes);
+            ++n_pbs;
+          }
         } else {  // PB == X after an improvement: defer the copy until the row stops improving
-          if (fl && !improved) bulk_s2g(a.PB + off, st, row_bytes);  // st holds the old x
+          if (fl && !improved) {
+            bulk_s2g(a.PB + off, st, row_bytes);  // st holds the old x
+            ++n_pbs;
+          }
           if ((int)improved != fl) a.pbx[r] = improved ? 1 : 0;
         }
         if (improved) {
@@ -794,6 +806,8 @@ __global__ void __launch_bounds__(kMaxThreads + 64, 2)
       fence_proxy_async_global();
       if (best != ~0ull) atomicMin(&a.ctl->key_acc, best);
       if (nimp) atomicAdd(&a.ctl->improvements, (unsigned long long)nimp);
+      if (n_pbl) atomicAdd(&a.ctl->pb_loads, (unsigned long long)n_pbl);
+      if (n_pbs) atomicAdd(&a.ctl->pb_stores, (unsigned long long)n_pbs);
       __threadfence();
       s_last = (atomicAdd(&a.ctl->done, 1u) == gridDim.x - 1) ? 1 : 0;
     }
@@ -967,7 +981,7 @@ __global__ void __launch_bounds__(kMaxThreadsCluster + 64, 1)
       mbar_wait(&gbar, 0);
       const uint32_t inc_ord = (uint32_t)(s_inc >> 32);
       unsigned long long best = ~0ull;
-      unsigned nimp = 0;
+      unsigned nimp = 0, n_pbl = 0, n_pbs = 0;
       int s = 0, prev = -1;
       unsigned ph = 0;
       for (long long r = cid; r < a.n_local; r += ncl) {
@@ -1022,6 +1036,8 @@ __global__ void __launch_bounds__(kMaxThreadsCluster + 64, 1)
             ++nimp;
           }
           if (a.lazy_pb && (int)(imp != 0.f) != fl) a.pbx[r] = imp != 0.f ? 1 : 0;
+          n_pbl += fl ? 0u : 1u;
+          n_pbs += (a.lazy_pb ? (fl && imp == 0.f) : (imp != 0.f)) ? 1u : 0u;
           if (f == f && ord_f32(f) < inc_ord) {  // strictly below gf
             const unsigned long long key = pack_key(f, gi);
             best = key < best ? key : best;
@@ -1054,6 +1070,8 @@ __global__ void __launch_bounds__(kMaxThreadsCluster + 64, 1)
       fence_proxy_async_global();
       if (best != ~0ull) atomicMin(&a.ctl->key_acc, best);
       if (nimp) atomicAdd(&a.ctl->improvements, (unsigned long long)nimp);
+      if (n_pbl) atomicAdd(&a.ctl->pb_loads, (unsigned long long)n_pbl);
+      if (n_pbs) atomicAdd(&a.ctl->pb_stores, (unsigned long long)n_pbs);
       __threadfence();
       s_last = (atomicAdd(&a.ctl->done, 1u) == gridDim.x - 1) ? 1 : 0;
     }

@@ -536,3 +536,32 @@ def test_nvlink_peer_exchange_single_rank(obj, n, d, monkeypatch):
         g.close()
     finally:
         fp.nccl_comm_destroy(comm)
+
+
+# ------------------------------------------------------------------ lazy pbest rows
+@pytest.mark.parametrize("obj,n,d", [(GRIEWANK, 300, 2000), (RASTRIGIN, 301, 1000),
+                                     (ROSENBROCK, 5, 12000)])
+def test_lazy_pbest_rows_lockstep(obj, n, d, monkeypatch):
+    """Streaming TMA / cluster kernels keep a row's pbest implicit while it equals
+    x (no pb load, no pb store) and write it when the row stops improving.  Over
+    several iterations with both transitions, PB (materialised by get_state),
+    pf and X/V equal the oracle's and the eager kernel's bit for bit."""
+    monkeypatch.setenv("PSO_RESIDENT", "0")
+    g = gpu_swarm(n, d, obj, seed=77)
+    assert g.info()["lazy_pb"] == 1
+    monkeypatch.setenv("PSO_LAZY_PB", "0")
+    e = gpu_swarm(n, d, obj, seed=77)
+    assert e.info()["lazy_pb"] == 0
+    c = cpu_swarm(n, d, obj, seed=77)
+    for k in (1, 1, 3, 1, 6):
+        g.step(k)
+        e.step(k)
+        c.step(k)
+        gs, es = g.get_state(), e.get_state()
+        for x, y, nm in zip(gs[:4], es[:4], "X V PB pf".split()):
+            assert_bitwise(x, y, f"lazy vs eager {nm}")
+        assert_bitwise(gs[0], c.X, "X vs oracle")
+        assert_bitwise(gs[2], c.PB, "PB vs oracle")
+        assert g.gbest()[:2] == e.gbest()[:2]
+    info = g.info()
+    assert info["pb_loads"] < e.info()["pb_loads"]  # flagged rows skipped their pb load
