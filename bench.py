@@ -45,6 +45,8 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=15.0,
                     help="CPU budget of the cpu_baseline oracle sample")
+    ap.add_argument("--ref-seconds", type=float, default=150.0,
+                    help="CPU budget of the whole --impl reference run (warm-up + timed steps)")
     return ap.parse_args()
 
 
@@ -170,7 +172,7 @@ def run_reference(args, w):
     if rank != 0:
         return 0
     K, W = args.steps, args.warmup
-    budget = 150.0  # whole --steps K --warmup W run
+    budget = args.ref_seconds  # whole --steps K --warmup W run
     s, rows, _ = oracle_sample(w, budget / max(K + W, 1), steps_hint=1)
     s.step(W)
     t0 = time.perf_counter()
