@@ -92,8 +92,10 @@ enum {
 
 /* Option flags. */
 enum {
-  PSO_FLAG_TIMING = 1 /* record CUDA events around every step kernel launch;
-                         totals are reported by pso_get_info */
+  PSO_FLAG_TIMING = 1,     /* record CUDA events around every step kernel launch;
+                              totals are reported by pso_get_info */
+  PSO_FLAG_DEFER_INIT = 2  /* allocate and plan only; pso_init runs Alg. 1 lines 1-3
+                              (lets ranks connect the NVLink exchange first) */
 };
 
 /* Options; a zero-initialised struct means "defaults". */
@@ -104,6 +106,9 @@ typedef struct {
   void* stream;    /* cudaStream_t to enqueue on; NULL -> a library-owned stream */
   void* nccl_comm; /* ncclComm_t (see pso_nccl_comm_init); NULL -> single GPU */
   uint32_t flags;  /* PSO_FLAG_* */
+  int32_t world, rank; /* without nccl_comm: world > 1 ranks that exchange only over
+                          NVLink (needs PSO_FLAG_DEFER_INIT: create, p2p connect +
+                          enable, then pso_init); ignored with a communicator */
   const float* bounds; /* NULL, or 4*d host floats [vlo | vhi | xlo | xhi]: per-dimension
                           velocity bounds (Eq. 5: lower/upper_bound_j) and
                           domain (x clamp); replaces vmax / lo / hi (which must still be
@@ -130,6 +135,12 @@ pso_status pso_create(pso_handle* out, int64_t n, int32_t d, float w, float c1, 
 pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c1, float c2,
                          float lo, float hi, int32_t objective, uint64_t seed,
                          const pso_opts* opts);
+
+/* Run the deferred initialisation of a handle created with PSO_FLAG_DEFER_INIT
+ * (Alg. 1 lines 1-3 + the first evaluation and gbest).  Collective.  Every
+ * other call except pso_set_state, pso_get_info, the p2p calls and destroy
+ * needs an initialised swarm (else PSO_ERR_INVALID). */
+pso_status pso_init(pso_handle h);
 
 /* Enqueue iters >= 0 iterations; each is one fused kernel: move (Eq. 1, 5,
  * 2), evaluate (Sec 3.2), pbest (Sec 3.3, strict <) and gbest (strict <,

@@ -16,12 +16,12 @@ PSO_OK, PSO_ERR_INVALID, PSO_ERR_NOMEM, PSO_ERR_CUDA = 0, 1, 2, 3
 PSO_ERR_NCCL, PSO_ERR_UNSUPPORTED, PSO_ERR_POISONED = 4, 5, 6
 PSO_OBJ_SPHERE, PSO_OBJ_RASTRIGIN, PSO_OBJ_ROSENBROCK = 1, 2, 3
 PSO_OBJ_GRIEWANK, PSO_OBJ_ACKLEY, PSO_OBJ_EASOM, PSO_OBJ_CUSTOM_BASE = 4, 5, 6, 64
-PSO_FLAG_TIMING = 1
+PSO_FLAG_TIMING, PSO_FLAG_DEFER_INIT = 1, 2
 PSO_D_MAX = 65536
 
 # every symbol include/fastpso.h declares
 EXPORTS = (
-    "pso_create", "pso_create_ex", "pso_step", "pso_synchronize", "pso_get_gbest",
+    "pso_create", "pso_create_ex", "pso_init", "pso_step", "pso_synchronize", "pso_get_gbest",
     "pso_get_state", "pso_set_state", "pso_set_bounds", "pso_get_info", "pso_reset_counters", "pso_destroy",
     "pso_status_string", "pso_last_error", "pso_objective_registered",
     "pso_nccl_get_unique_id", "pso_nccl_comm_init", "pso_nccl_comm_destroy",
@@ -32,7 +32,8 @@ EXPORTS = (
 
 class pso_opts(C.Structure):
     _fields_ = [("vmax", C.c_float), ("device", C.c_int32), ("stream", C.c_void_p),
-                ("nccl_comm", C.c_void_p), ("flags", C.c_uint32), ("bounds", C.c_void_p)]
+                ("nccl_comm", C.c_void_p), ("flags", C.c_uint32), ("world", C.c_int32),
+                ("rank", C.c_int32), ("bounds", C.c_void_p)]
 
 
 class pso_info(C.Structure):
@@ -78,6 +79,7 @@ def lib() -> C.CDLL:
                              C.c_float, C.c_float, C.c_int32, C.c_uint64]
     L.pso_create_ex.argtypes = L.pso_create.argtypes + [C.POINTER(pso_opts)]
     L.pso_step.argtypes = [H, C.c_int64]
+    L.pso_init.argtypes = [H]
     L.pso_synchronize.argtypes = [H]
     L.pso_get_gbest.argtypes = [H, fp, i64p, C.c_void_p]
     L.pso_get_state.argtypes = [H, C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p, u64p]

@@ -136,6 +136,7 @@ struct pso_swarm {
   size_t events_used = 0;
   double timed_ms = 0;
   uint64_t timed_count = 0;
+  bool inited = false;  // pso_init done (or state set)
   // NVLink peer exchange (pso_p2p_connect)
   std::vector<void*> ipc_opened;
   void* peers_dev = nullptr;
@@ -161,6 +162,14 @@ pso_status check_handle(pso_swarm* h) {
   return PSO_OK;
 }
 
+// Calls that read or advance the swarm need it initialised (pso_init / set_state).
+pso_status check_ready(pso_swarm* h) {
+  pso_status st = check_handle(h);
+  if (st != PSO_OK) return st;
+  if (!h->inited) return fail(PSO_ERR_INVALID, "swarm not initialised: call pso_init (deferred init)");
+  return PSO_OK;
+}
+
 // Make the handle's device current for this call.
 pso_status use_device(pso_swarm* h) {
   PSO_CUDA(h, cudaSetDevice(h->device));
@@ -173,11 +182,6 @@ pso_status use_device(pso_swarm* h) {
 // final for the host (end of create, set_state and every pso_step call).
 pso_status exchange(pso_swarm* h, uint64_t t, bool fold) {
   if (!h->xchg) return PSO_OK;
-  NcclApi* a = nccl();
-  if (!a) {
-    h->poisoned = true;
-    return fail(PSO_ERR_NCCL, "NCCL unavailable");
-  }
   const size_t rec = record_bytes(h->pitch);
   if (h->args.p2p) {  // records travel by NVLink peer stores inside the kernels
     if (fold) {
@@ -185,6 +189,15 @@ pso_status exchange(pso_swarm* h, uint64_t t, bool fold) {
       ++h->launches;
     }
     return PSO_OK;
+  }
+  if (!h->comm) {
+    h->poisoned = true;
+    return fail(PSO_ERR_INVALID, "no communicator: enable the NVLink exchange before this call");
+  }
+  NcclApi* a = nccl();
+  if (!a) {
+    h->poisoned = true;
+    return fail(PSO_ERR_NCCL, "NCCL unavailable");
   }
   unsigned char* dst = const_cast<unsigned char*>(h->args.recv) + (t & 1) * (size_t)h->world * rec;
   ncclResult_t r = a->AllGather(h->args.send, dst, rec, kNcclUint8, h->comm, h->stream);
@@ -202,7 +215,7 @@ pso_status exchange(pso_swarm* h, uint64_t t, bool fold) {
 pso_status sync_and_check(pso_swarm* h) {
   cudaError_t e = cudaStreamSynchronize(h->stream);
   if (e != cudaSuccess) return cuda_fail(h, e, "cudaStreamSynchronize");
-  if (h->world > 1) {
+  if (h->comm) {
     NcclApi* a = nccl();
     ncclResult_t ar = 0;
     if (a && a->CommGetAsyncError(h->comm, &ar) == 0 && ar != 0) {
@@ -287,6 +300,21 @@ pso_status upload_bounds(pso_swarm* h, const float* b) {
   return PSO_OK;
 }
 
+// Alg. 1 lines 1-3 + the first evaluation and best update (and, with an
+// exchange, the first gbest exchange).
+pso_status run_init(pso_swarm* h) {
+  if (h->n_local > 0) {
+    PSO_CUDA(h, launch_init(h->objective, h->args, h->cfg, h->stream));
+    ++h->launches;
+  }
+  pso_status st = exchange(h, 0, true);
+  if (st != PSO_OK) return st;
+  if ((st = sync_and_check(h)) != PSO_OK) return st;
+  h->t = 0;
+  h->inited = true;
+  return PSO_OK;
+}
+
 float decode_fitness(unsigned long long key) {
   uint32_t o = (uint32_t)(key >> 32);
   uint32_t u = (o & 0x80000000u) ? (o & 0x7FFFFFFFu) : ~o;
@@ -347,7 +375,8 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
   if (!(o.vmax == o.vmax) || std::isinf(o.vmax)) return fail(PSO_ERR_INVALID, "vmax must be finite");
   if (!objective_registered(objective))
     return fail(PSO_ERR_INVALID, "objective %d is not registered", objective);
-  if (o.flags & ~(uint32_t)PSO_FLAG_TIMING) return fail(PSO_ERR_INVALID, "unknown flags 0x%x", o.flags);
+  if (o.flags & ~(uint32_t)(PSO_FLAG_TIMING | PSO_FLAG_DEFER_INIT))
+    return fail(PSO_ERR_INVALID, "unknown flags 0x%x", o.flags);
   if (o.bounds) {
     pso_status bs = check_bounds(o.bounds, d);
     if (bs != PSO_OK) return bs;
@@ -412,6 +441,15 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
     h->rank = rk;
     const char* fx = std::getenv("PSO_FORCE_EXCHANGE");
     h->xchg = cnt > 1 || (fx && *fx && *fx != '0');
+  } else if (o.world > 1) {  // ranks without a communicator: NVLink exchange only
+    if (o.rank < 0 || o.rank >= o.world)
+      return bail(fail(PSO_ERR_INVALID, "rank %d outside [0, %d)", o.rank, o.world));
+    if (!(o.flags & PSO_FLAG_DEFER_INIT))
+      return bail(fail(PSO_ERR_INVALID, "world > 1 without a communicator needs PSO_FLAG_DEFER_INIT "
+                                        "(connect the NVLink exchange, then pso_init)"));
+    h->world = o.world;
+    h->rank = o.rank;
+    h->xchg = true;
   }
   h->row_begin = (n * h->rank) / h->world;
   h->n_local = (n * (h->rank + 1)) / h->world - h->row_begin;
@@ -505,26 +543,26 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
   if (st != PSO_OK) return bail(st);
   if (o.bounds && (st = upload_bounds(h, o.bounds)) != PSO_OK) return bail(st);
 
-  // ---- Alg. 1 lines 1-3 + first evaluation and best update
-  if (h->n_local > 0) {
-    cudaError_t e = launch_init(objective, A, h->cfg, h->stream);
-    if (e != cudaSuccess) return bail(cuda_fail(nullptr, e, "launch_init"));
-    ++h->launches;
-  } else if (h->xchg) {
-    // empty shard: contribute "no candidate"
+  if (h->n_local == 0 && h->xchg) {  // empty shard: contribute "no candidate"
     unsigned long long none[2] = {~0ull, 0ull};
     cudaError_t e = cudaMemcpyAsync(A.send, none, 16, cudaMemcpyHostToDevice, h->stream);
     if (e != cudaSuccess) return bail(cuda_fail(nullptr, e, "cudaMemcpyAsync"));
   }
-  if ((st = exchange(h, 0, true)) != PSO_OK) return bail(st);
-  if ((st = sync_and_check(h)) != PSO_OK) return bail(st);
-  h->t = 0;
+  if (!(o.flags & PSO_FLAG_DEFER_INIT) && (st = run_init(h)) != PSO_OK) return bail(st);
   *out = h;
   return PSO_OK;
 }
 
-pso_status pso_step(pso_handle h, int64_t iters) {
+pso_status pso_init(pso_handle h) {
   pso_status st = check_handle(h);
+  if (st != PSO_OK) return st;
+  if (h->inited) return fail(PSO_ERR_INVALID, "already initialised");
+  if ((st = use_device(h)) != PSO_OK) return st;
+  return run_init(h);
+}
+
+pso_status pso_step(pso_handle h, int64_t iters) {
+  pso_status st = check_ready(h);
   if (st != PSO_OK) return st;
   if (iters < 0) return fail(PSO_ERR_INVALID, "iters=%lld < 0", (long long)iters);
   if (iters == 0) return PSO_OK;
@@ -570,7 +608,7 @@ pso_status pso_synchronize(pso_handle h) {
 }
 
 pso_status pso_get_gbest(pso_handle h, float* fitness, int64_t* index, float* pos) {
-  pso_status st = check_handle(h);
+  pso_status st = check_ready(h);
   if (st != PSO_OK) return st;
   if ((st = use_device(h)) != PSO_OK) return st;
   unsigned long long key = 0;
@@ -583,7 +621,7 @@ pso_status pso_get_gbest(pso_handle h, float* fitness, int64_t* index, float* po
 }
 
 pso_status pso_get_state(pso_handle h, float* x, float* v, float* pb, float* pf, uint64_t* t) {
-  pso_status st = check_handle(h);
+  pso_status st = check_ready(h);
   if (st != PSO_OK) return st;
   if ((st = use_device(h)) != PSO_OK) return st;
   const size_t w = (size_t)h->d * 4, sp = (size_t)h->pitch * 4, rows = (size_t)h->n_local;
@@ -638,6 +676,7 @@ pso_status pso_set_state(pso_handle h, const float* x, const float* v, const flo
   if ((st = exchange(h, t, true)) != PSO_OK) return st;
   if ((st = sync_and_check(h)) != PSO_OK) return st;
   h->t = t;
+  h->inited = true;
   return PSO_OK;
 }
 

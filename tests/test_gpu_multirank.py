@@ -1,0 +1,79 @@
+"""Two ranks of the particle split as two processes on ONE GPU, with
+the NVLink peer exchange (CUDA IPC mappings between the processes): every
+iteration each rank's step kernel stores its gbest record into both ranks'
+receive buffers and the next step kernel acquires both tags — the real
+multi-rank protocol (parity double-buffering, epoch tags, merge order), not a
+1-rank stand-in.  Results must equal a single-process run bit for bit."""
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+import paper_conf_icpp_liuwc21_b200 as fp
+from synth import DOMAINS, GRIEWANK, RASTRIGIN, ROSENBROCK, row_range
+
+pytestmark = pytest.mark.gpu
+
+
+def _free_port():
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        return s.getsockname()[1]
+
+
+def _worker(rank, world, port, n, d, obj, steps, out_dir):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    from paper_conf_icpp_liuwc21_b200.distributed import connect_p2p
+    lo, hi = DOMAINS[obj]
+    s = fp.Swarm(n, d, 0.9, 2.0, 2.0, lo, hi, obj, 4242, device=0, world=world, rank=rank,
+                 defer_init=True)
+    assert connect_p2p(s)
+    s.init()
+    for k in steps:
+        s.step(k)
+    X, V, PB, pf, t = s.get_state()
+    f, i, G = s.gbest()
+    # set_state starts a new epoch: records of the previous state must never match
+    s.set_state(X, V, PB, pf, t=t)
+    s.step(2)
+    X2, V2, PB2, pf2, t2 = s.get_state()
+    f2, i2, G2 = s.gbest()
+    np.savez(os.path.join(out_dir, f"r{rank}.npz"), X=X, V=V, PB=PB, pf=pf, G=G, f=f, i=i, t=t,
+             X2=X2, PB2=PB2, pf2=pf2, G2=G2, f2=f2, i2=i2, launches=s.info()["launches"])
+    s.close()
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("obj,n,d", [(RASTRIGIN, 300, 1000), (GRIEWANK, 41, 13),
+                                     (ROSENBROCK, 6, 10000)])
+def test_two_processes_nvlink_exchange_matches_single_gpu(tmp_path, obj, n, d):
+    steps = (1, 4, 3)
+    mp.spawn(_worker, args=(2, _free_port(), n, d, obj, steps, str(tmp_path)), nprocs=2,
+             join=True)
+    lo, hi = DOMAINS[obj]
+    ref = fp.Swarm(n, d, 0.9, 2.0, 2.0, lo, hi, obj, 4242, device=0)
+    for k in steps:
+        ref.step(k)
+    RX, RV, RPB, Rpf, Rt = ref.get_state()
+    rf, ri, RG = ref.gbest()
+    ref.set_state(RX, RV, RPB, Rpf, t=Rt)
+    ref.step(2)
+    RX2, _, RPB2, Rpf2, _ = ref.get_state()
+    rf2, ri2, RG2 = ref.gbest()
+    for r in range(2):
+        z = np.load(tmp_path / f"r{r}.npz")
+        b, e = row_range(n, r, 2)
+        for name, full in (("X", RX), ("V", RV), ("PB", RPB), ("pf", Rpf), ("X2", RX2),
+                           ("PB2", RPB2), ("pf2", Rpf2)):
+            assert np.array_equal(z[name].view(np.uint32), full[b:e].view(np.uint32)), (r, name)
+        assert int(z["t"]) == Rt
+        assert (float(z["f"]), int(z["i"])) == (rf, ri)
+        assert (float(z["f2"]), int(z["i2"])) == (rf2, ri2)
+        assert np.array_equal(z["G"].view(np.uint32), RG.view(np.uint32))
+        assert np.array_equal(z["G2"].view(np.uint32), RG2.view(np.uint32))
