@@ -1,4 +1,4 @@
-"""Two ranks of the particle split as two processes on ONE GPU, with
+"""Ranks of the particle split as 2-4 processes on ONE GPU, with
 the NVLink peer exchange (CUDA IPC mappings between the processes): every
 iteration each rank's step kernel stores its gbest record into both ranks'
 receive buffers and the next step kernel acquires both tags — the real
@@ -50,11 +50,12 @@ def _worker(rank, world, port, n, d, obj, steps, out_dir):
     dist.destroy_process_group()
 
 
-@pytest.mark.parametrize("obj,n,d", [(RASTRIGIN, 300, 1000), (GRIEWANK, 41, 13),
-                                     (ROSENBROCK, 6, 10000)])
-def test_two_processes_nvlink_exchange_matches_single_gpu(tmp_path, obj, n, d):
+@pytest.mark.parametrize("world,obj,n,d", [(2, RASTRIGIN, 300, 1000), (2, GRIEWANK, 41, 13),
+                                           (2, ROSENBROCK, 6, 10000), (3, RASTRIGIN, 7, 2000),
+                                           (4, GRIEWANK, 9, 999)])
+def test_processes_nvlink_exchange_matches_single_gpu(tmp_path, world, obj, n, d):
     steps = (1, 4, 3)
-    mp.spawn(_worker, args=(2, _free_port(), n, d, obj, steps, str(tmp_path)), nprocs=2,
+    mp.spawn(_worker, args=(world, _free_port(), n, d, obj, steps, str(tmp_path)), nprocs=world,
              join=True)
     lo, hi = DOMAINS[obj]
     ref = fp.Swarm(n, d, 0.9, 2.0, 2.0, lo, hi, obj, 4242, device=0)
@@ -66,9 +67,9 @@ def test_two_processes_nvlink_exchange_matches_single_gpu(tmp_path, obj, n, d):
     ref.step(2)
     RX2, _, RPB2, Rpf2, _ = ref.get_state()
     rf2, ri2, RG2 = ref.gbest()
-    for r in range(2):
+    for r in range(world):
         z = np.load(tmp_path / f"r{r}.npz")
-        b, e = row_range(n, r, 2)
+        b, e = row_range(n, r, world)
         for name, full in (("X", RX), ("V", RV), ("PB", RPB), ("pf", Rpf), ("X2", RX2),
                            ("PB2", RPB2), ("pf2", Rpf2)):
             assert np.array_equal(z[name].view(np.uint32), full[b:e].view(np.uint32)), (r, name)
