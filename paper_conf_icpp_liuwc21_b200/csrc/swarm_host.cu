@@ -150,7 +150,8 @@ cudaError_t plan_cluster(const KernelTable* t, int nvec, long long n_local, cons
   shape_for(chunk, h.vpt, &vpt, &compute, kMaxThreadsCluster);
   const void* fn = t->step_cluster[vpt_index(vpt)][h.bounds ? 1 : 0];
   const size_t crow = (size_t)chunk * 16, btab = h.bounds ? 4 * crow : 0;
-  int stages = ring_stages(crow + btab, 3 * crow, 1);
+  const int per_sm = (h.ctas >= 1 && h.ctas <= 4) ? h.ctas : 1;  // CTAs per SM to size the ring for
+  int stages = ring_stages(crow + btab, 3 * crow, per_sm);
   if (h.stages >= 2 && h.stages < stages) stages = h.stages;
   if (stages > kMaxStages) stages = kMaxStages;
   if (stages < 2) return cudaErrorInvalidConfiguration;
