@@ -94,8 +94,16 @@ enum {
 enum {
   PSO_FLAG_TIMING = 1,     /* record CUDA events around every step kernel launch;
                               totals are reported by pso_get_info */
-  PSO_FLAG_DEFER_INIT = 2  /* allocate and plan only; pso_init runs Alg. 1 lines 1-3
+  PSO_FLAG_DEFER_INIT = 2,  /* allocate and plan only; pso_init runs Alg. 1 lines 1-3
                               (lets ranks connect the NVLink exchange first) */
+  PSO_FLAG_ASYNC_GBEST = 4  /* NEXT-4, "updated in an asynchronous manner": each
+                              rank's step kernel adopts its own candidates at once and
+                              merges its peers' records one iteration late, so no rank
+                              waits for the iteration its peers are in.  Deterministic
+                              for a given world size, but results depend on it; with
+                              world = 1 identical to the synchronous mode.
+                              pso_get_gbest returns the global view folded from every
+                              rank's records at the end of the last pso_step call. */
 };
 
 /* Options; a zero-initialised struct means "defaults". */

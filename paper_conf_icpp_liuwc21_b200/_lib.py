@@ -16,7 +16,7 @@ PSO_OK, PSO_ERR_INVALID, PSO_ERR_NOMEM, PSO_ERR_CUDA = 0, 1, 2, 3
 PSO_ERR_NCCL, PSO_ERR_UNSUPPORTED, PSO_ERR_POISONED = 4, 5, 6
 PSO_OBJ_SPHERE, PSO_OBJ_RASTRIGIN, PSO_OBJ_ROSENBROCK = 1, 2, 3
 PSO_OBJ_GRIEWANK, PSO_OBJ_ACKLEY, PSO_OBJ_EASOM, PSO_OBJ_CUSTOM_BASE = 4, 5, 6, 64
-PSO_FLAG_TIMING, PSO_FLAG_DEFER_INIT = 1, 2
+PSO_FLAG_TIMING, PSO_FLAG_DEFER_INIT, PSO_FLAG_ASYNC_GBEST = 1, 2, 4
 PSO_D_MAX = 65536
 
 # every symbol include/fastpso.h declares

@@ -180,12 +180,12 @@ pso_status use_device(pso_swarm* h) {
 // and row) into recv[t & 1].  The next step kernel merges them in its
 // prologue; `fold` additionally runs the select kernel so key_cur / G are
 // final for the host (end of create, set_state and every pso_step call).
-pso_status exchange(pso_swarm* h, uint64_t t, bool fold) {
+pso_status exchange(pso_swarm* h, uint64_t t, bool fold, bool into_local) {
   if (!h->xchg) return PSO_OK;
   const size_t rec = record_bytes(h->pitch);
   if (h->args.p2p) {  // records travel by NVLink peer stores inside the kernels
     if (fold) {
-      PSO_CUDA(h, launch_select(h->args, (unsigned)t, h->stream));
+      PSO_CUDA(h, launch_select(h->args, (unsigned)t, into_local, h->stream));
       ++h->launches;
     }
     return PSO_OK;
@@ -199,14 +199,14 @@ pso_status exchange(pso_swarm* h, uint64_t t, bool fold) {
     h->poisoned = true;
     return fail(PSO_ERR_NCCL, "NCCL unavailable");
   }
-  unsigned char* dst = const_cast<unsigned char*>(h->args.recv) + (t & 1) * (size_t)h->world * rec;
+  unsigned char* dst = const_cast<unsigned char*>(h->args.recv) + (t & 3) * (size_t)h->world * rec;
   ncclResult_t r = a->AllGather(h->args.send, dst, rec, kNcclUint8, h->comm, h->stream);
   if (r != 0) {
     h->poisoned = true;
     return fail(PSO_ERR_NCCL, "ncclAllGather: %s", nccl_str(r));
   }
   if (fold) {
-    PSO_CUDA(h, launch_select(h->args, (unsigned)t, h->stream));
+    PSO_CUDA(h, launch_select(h->args, (unsigned)t, into_local, h->stream));
     ++h->launches;
   }
   return PSO_OK;
@@ -307,7 +307,7 @@ pso_status run_init(pso_swarm* h) {
     PSO_CUDA(h, launch_init(h->objective, h->args, h->cfg, h->stream));
     ++h->launches;
   }
-  pso_status st = exchange(h, 0, true);
+  pso_status st = exchange(h, 0, true, true);
   if (st != PSO_OK) return st;
   if ((st = sync_and_check(h)) != PSO_OK) return st;
   h->t = 0;
@@ -375,7 +375,7 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
   if (!(o.vmax == o.vmax) || std::isinf(o.vmax)) return fail(PSO_ERR_INVALID, "vmax must be finite");
   if (!objective_registered(objective))
     return fail(PSO_ERR_INVALID, "objective %d is not registered", objective);
-  if (o.flags & ~(uint32_t)(PSO_FLAG_TIMING | PSO_FLAG_DEFER_INIT))
+  if (o.flags & ~(uint32_t)(PSO_FLAG_TIMING | PSO_FLAG_DEFER_INIT | PSO_FLAG_ASYNC_GBEST))
     return fail(PSO_ERR_INVALID, "unknown flags 0x%x", o.flags);
   if (o.bounds) {
     pso_status bs = check_bounds(o.bounds, d);
@@ -493,7 +493,9 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
   const size_t rec = align_up(record_bytes(h->pitch), 256);
   const size_t candb = h->cfg.gridres ? align_up(2 * (size_t)h->cfg.gridres_grid * h->pitch * 4, 256) : 0;
   const size_t sendb = h->xchg ? rec : 0;
-  const size_t recvb = h->xchg ? 2 * (size_t)h->world * record_bytes(h->pitch) : 0;
+  const size_t recvb = h->xchg ? 4 * (size_t)h->world * record_bytes(h->pitch) : 0;
+  const bool async = (o.flags & PSO_FLAG_ASYNC_GBEST) != 0 && h->xchg;  // needs an exchange
+  const size_t viewb = async ? gb : 0;  // the host's global gbest view
   h->arena_bytes =
       3 * mat + pfb + gb + ctlb + boundb + pbxb + candb + sendb + align_up(recvb, 256);
   {
@@ -516,6 +518,8 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
   A.pbx = lazy ? p : nullptr; p += pbxb;
   A.lazy_pb = lazy ? 1 : 0;
   A.cand = h->cfg.gridres ? (float*)p : nullptr; p += candb;
+  A.G_view = async ? (float*)p : nullptr; p += viewb;
+  A.async_gbest = async ? 1 : 0;
   A.send = h->xchg ? p : nullptr; p += sendb;
   A.recv = h->xchg ? p : nullptr;
   A.n_local = h->n_local;
@@ -594,7 +598,7 @@ pso_status pso_step(pso_handle h, int64_t iters) {
       ++h->launches;
       if (ev) PSO_CUDA(h, cudaEventRecord(ev->stop, h->stream));
     }
-    if ((st = exchange(h, h->t + (uint64_t)it + 1, it + 1 == iters)) != PSO_OK) return st;
+    if ((st = exchange(h, h->t + (uint64_t)it + 1, it + 1 == iters, false)) != PSO_OK) return st;
   }
   h->t += (uint64_t)iters;
   return PSO_OK;
@@ -612,8 +616,12 @@ pso_status pso_get_gbest(pso_handle h, float* fitness, int64_t* index, float* po
   if (st != PSO_OK) return st;
   if ((st = use_device(h)) != PSO_OK) return st;
   unsigned long long key = 0;
-  PSO_CUDA(h, cudaMemcpyAsync(&key, &h->args.ctl->key_cur, 8, cudaMemcpyDeviceToHost, h->stream));
-  if (pos) PSO_CUDA(h, cudaMemcpyAsync(pos, h->args.G, (size_t)h->d * 4, cudaMemcpyDeviceToHost, h->stream));
+  // asynchronous gbest: the view folded at the end of the last call (every rank's records)
+  const bool view = h->args.async_gbest != 0;
+  const unsigned long long* ksrc = view ? &h->args.ctl->key_view : &h->args.ctl->key_cur;
+  const float* gsrc = view ? h->args.G_view : h->args.G;
+  PSO_CUDA(h, cudaMemcpyAsync(&key, ksrc, 8, cudaMemcpyDeviceToHost, h->stream));
+  if (pos) PSO_CUDA(h, cudaMemcpyAsync(pos, gsrc, (size_t)h->d * 4, cudaMemcpyDeviceToHost, h->stream));
   if ((st = sync_and_check(h)) != PSO_OK) return st;
   if (fitness) *fitness = decode_fitness(key);
   if (index) *index = (int64_t)(uint32_t)key;
@@ -673,7 +681,7 @@ pso_status pso_set_state(pso_handle h, const float* x, const float* v, const flo
     unsigned long long none[2] = {~0ull, 0ull};
     PSO_CUDA(h, cudaMemcpyAsync(h->args.send, none, 16, cudaMemcpyHostToDevice, h->stream));
   }
-  if ((st = exchange(h, t, true)) != PSO_OK) return st;
+  if ((st = exchange(h, t, true, true)) != PSO_OK) return st;
   if ((st = sync_and_check(h)) != PSO_OK) return st;
   h->t = t;
   h->inited = true;

@@ -19,7 +19,8 @@ struct DevCtl {
   unsigned int bar_count, bar_gen;  // grid-resident kernel: grid barrier
   unsigned long long pb_loads;      // streaming kernels: pbest rows read from HBM
   unsigned long long pb_stores;     // streaming kernels: pbest rows written to HBM
-  unsigned long long pad[7];
+  unsigned long long key_view;      // async: global gbest key folded for the host
+  unsigned long long pad[6];
 };
 static_assert(sizeof(DevCtl) == 128, "DevCtl is two 64-byte blocks");
 
@@ -47,6 +48,8 @@ struct SwarmArgs {
   int rank;
   int exchange;               // 1: publish (key, row) records for the all-gather + select
   int p2p;                    // exchange over NVLink peer stores instead of NCCL
+  int async_gbest;            // NEXT-4: merge peers' records with a one-iteration lag
+  float* G_view;              // async: the host's global gbest view (pitch floats)
   unsigned epoch;             // p2p: record tags are (epoch << 32 | t); set_state starts an epoch
   unsigned char* const* peers;  // p2p: device array, world pointers to every rank's recv
   float w, c1, c2, lo, hi, vmax;
@@ -113,7 +116,9 @@ cudaError_t launch_resident(int objective, const SwarmArgs& a, const LaunchCfg& 
 cudaError_t launch_gridres(int objective, const SwarmArgs& a, const LaunchCfg& c, int iters,
                            cudaStream_t s);
 cudaError_t launch_rebest(const SwarmArgs& a, unsigned t, cudaStream_t s);
-cudaError_t launch_select(const SwarmArgs& a, unsigned t, cudaStream_t s);
+// Fold the records of iteration t (and, asynchronous, of t - 1) for the host;
+// into_local: also into the kernels' incumbent (create / set_state).
+cudaError_t launch_select(const SwarmArgs& a, unsigned t, bool into_local, cudaStream_t s);
 // lazy pbest: copy X -> PB for flagged rows and clear the flags (host reads)
 cudaError_t launch_materialize_pb(const SwarmArgs& a, cudaStream_t s);
 

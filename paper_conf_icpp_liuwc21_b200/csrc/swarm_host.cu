@@ -39,28 +39,55 @@ __global__ void __launch_bounds__(256) k_rebest(const SwarmArgs a, unsigned t) {
 }
 
 // ---------------------------------------------------------- select kernel
-// Exchange mode: fold the records of iteration t (after the all-gather) into
-// key_cur / G — the same merge a step kernel's prologue performs, run once at
-// the end of create / set_state / each pso_step call so the host reads the
-// final gbest.  Idempotent (the next step's prologue merges the same records
-// again and finds nothing better).  Every rank computes the same bits.
-__global__ void __launch_bounds__(128) k_select(const SwarmArgs a, unsigned t) {
+// Exchange mode: fold records for the host.  Synchronous, or at create /
+// set_state (into_local): the records of iteration t go into key_cur / G —
+// the merge a step kernel's prologue performs, so the next prologue finds
+// nothing new (idempotent).  Asynchronous at the end of a pso_step call: the
+// records of t - 1 and t are folded into the host's view (key_view / G_view)
+// only, leaving the kernels' lagged incumbents untouched, so step(a); step(b)
+// is still step(a + b).  Candidates are records strictly better than the
+// incumbent (Alg. 1 line 10); the lowest key wins.  Every rank computes the
+// same bits.
+__global__ void __launch_bounds__(128) k_select(const SwarmArgs a, unsigned t, int into_local) {
   __shared__ unsigned long long s_best;
-  __shared__ int s_src;
+  __shared__ const float* s_row;
+  const bool view_only = a.async_gbest && !into_local;
   if (threadIdx.x == 0) {
-    int src;
-    s_best = exchange_merge(a, t, &src);
-    s_src = src;
+    const unsigned long long cur = a.ctl->key_cur;
+    unsigned long long best = cur;
+    const float* row = nullptr;
+    const size_t rec = record_bytes(a.nvec * 4);
+    const int n_it = (view_only && t >= 1u) ? 2 : 1;
+    for (int k = n_it - 1; k >= 0; --k) {
+      const unsigned it = t - (unsigned)k;
+      if (a.p2p) wait_records(a, it);
+      const unsigned char* base = records(a, it);
+      for (int r = 0; r < a.world; ++r) {
+        const unsigned long long key =
+            *reinterpret_cast<const unsigned long long*>(base + (size_t)r * rec);
+        if ((key >> 32) < (cur >> 32) && key < best) {
+          best = key;
+          row = reinterpret_cast<const float*>(base + (size_t)r * rec + 16);
+        }
+      }
+    }
+    s_best = best;
+    s_row = row;
   }
   __syncthreads();
-  const int src = s_src;
-  if (src >= 0) {
-    const float4* row = reinterpret_cast<const float4*>(merged_gbest_row(a, t, src));
-    float4* G4 = reinterpret_cast<float4*>(a.G);
-    for (int q = threadIdx.x; q < a.nvec; q += blockDim.x) G4[q] = row[q];
+  const float4* row = reinterpret_cast<const float4*>(s_row);
+  float4* dst = reinterpret_cast<float4*>(view_only ? a.G_view : a.G);
+  const float4* G4 = reinterpret_cast<const float4*>(a.G);
+  for (int q = threadIdx.x; q < a.nvec; q += blockDim.x) {
+    const float4 v = row ? row[q] : G4[q];
+    dst[q] = v;
+    if (!view_only && a.G_view) reinterpret_cast<float4*>(a.G_view)[q] = v;
   }
   __syncthreads();
-  if (threadIdx.x == 0 && src >= 0) a.ctl->key_cur = s_best;
+  if (threadIdx.x == 0) {
+    if (!view_only) a.ctl->key_cur = s_best;
+    a.ctl->key_view = s_best;
+  }
 }
 
 // ---------------------------------------------------------- materialize PB
@@ -408,8 +435,8 @@ cudaError_t launch_materialize_pb(const SwarmArgs& a, cudaStream_t s) {
   return cudaGetLastError();
 }
 
-cudaError_t launch_select(const SwarmArgs& a, unsigned t, cudaStream_t s) {
-  k_select<<<1, 128, 0, s>>>(a, t);
+cudaError_t launch_select(const SwarmArgs& a, unsigned t, bool into_local, cudaStream_t s) {
+  k_select<<<1, 128, 0, s>>>(a, t, into_local ? 1 : 0);
   return cudaGetLastError();
 }
 

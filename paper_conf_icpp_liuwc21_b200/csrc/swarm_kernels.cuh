@@ -401,8 +401,16 @@ __device__ __forceinline__ float process_row(const SwarmArgs& a, const MoveParam
 // iteration t + 1 merges them in its prologue (the incumbent for its strict
 // filter and the G it stages); its last CTA commits that merge to key_cur / G
 // and publishes the new local candidate.
+// Records are kept for 4 iterations (slot t & 3): the asynchronous mode reads
+// iteration t - 2 while a peer that is one iteration ahead writes t + 1.
 __device__ __forceinline__ const unsigned char* records(const SwarmArgs& a, uint32_t t) {
-  return a.recv + (size_t)(t & 1u) * a.world * record_bytes(a.nvec * 4);
+  return a.recv + (size_t)(t & 3u) * a.world * record_bytes(a.nvec * 4);
+}
+// The iteration whose records the step kernel of iteration t merges:
+// synchronous t - 1; asynchronous (NEXT-4, "updated in an asynchronous
+// manner") t - 2, so a rank never waits for the iteration its peers are in.
+__device__ __forceinline__ uint32_t merge_iter(const SwarmArgs& a, uint32_t t) {
+  return a.async_gbest ? (t >= 2u ? t - 2u : 0u) : t - 1u;
 }
 // --- NVLink peer exchange (p2p): every rank stores its record of iteration
 // t straight into recv[t & 1][rank] of every peer (CUDA-IPC-mapped), then the
@@ -446,11 +454,14 @@ __device__ __forceinline__ unsigned long long exchange_merge(const SwarmArgs& a,
   if (a.p2p) wait_records(a, prev_t);
   const size_t rec = record_bytes(a.nvec * 4);
   const unsigned char* base = records(a, prev_t);
-  unsigned long long best = *(volatile unsigned long long*)&a.ctl->key_cur;
+  const unsigned long long cur = *(volatile unsigned long long*)&a.ctl->key_cur;
+  unsigned long long best = cur;
   int s = -1;
   for (int r = 0; r < a.world; ++r) {
     const unsigned long long k = *reinterpret_cast<const unsigned long long*>(base + (size_t)r * rec);
-    if (k < best) {
+    // strictly better fitness than the incumbent (Alg. 1 line 10), then the
+    // lowest key: in the synchronous mode every record already satisfies it
+    if ((k >> 32) < (cur >> 32) && k < best) {
       best = k;
       s = r;
     }
@@ -499,11 +510,20 @@ __device__ __forceinline__ void epilogue_core(const SwarmArgs& a, uint32_t t, un
     return;
   }
   const bool merged = src >= 0 && inc < cur;
-  if (merged) {
-    const float4* w = reinterpret_cast<const float4*>(merged_gbest_row(a, t - 1u, src));
+  const bool have = acc != ~0ull;
+  // asynchronous: this rank's candidate becomes its incumbent at once (it is
+  // strictly below the merged incumbent); synchronous: every rank adopts it
+  // through the next merge
+  const bool local = a.async_gbest && have;
+  if (merged && !local) {
+    const float4* w = reinterpret_cast<const float4*>(merged_gbest_row(a, merge_iter(a, t), src));
     for (int q = tid; q < a.nvec; q += nthr) G4[q] = __ldcg(w + q);
   }
-  const bool have = acc != ~0ull;
+  if (local) {
+    const float4* w = reinterpret_cast<const float4*>(rows) +
+                      ((long long)(uint32_t)acc - a.row_begin) * a.nvec;
+    for (int q = tid; q < a.nvec; q += nthr) G4[q] = __ldcg(w + q);
+  }
   const float4* pb = have ? reinterpret_cast<const float4*>(rows) +
                                 ((long long)(uint32_t)acc - a.row_begin) * a.nvec
                           : nullptr;
@@ -520,7 +540,7 @@ __device__ __forceinline__ void epilogue_core(const SwarmArgs& a, uint32_t t, un
     }
   } else {  // NVLink: store the record into recv[t & 1][rank] of every rank
     const size_t rec = record_bytes(a.nvec * 4);
-    const size_t off = (size_t)(t & 1u) * a.world * rec + (size_t)a.rank * rec;
+    const size_t off = (size_t)(t & 3u) * a.world * rec + (size_t)a.rank * rec;
     for (int r = 0; r < a.world; ++r) {
       unsigned char* dst = a.peers[r] + off;
       if (have) {
@@ -536,7 +556,10 @@ __device__ __forceinline__ void epilogue_core(const SwarmArgs& a, uint32_t t, un
         st_release_sys_u64(a.peers[r] + off + 8, ((unsigned long long)a.epoch << 32) | t);
   }
   if (tid == 0) {
-    if (merged) a.ctl->key_cur = inc;
+    if (local)
+      a.ctl->key_cur = acc;
+    else if (merged)
+      a.ctl->key_cur = inc;
     a.ctl->key_acc = ~0ull;
     a.ctl->t = t;
     a.ctl->done = 0;
@@ -605,8 +628,8 @@ __global__ void __launch_bounds__(kMaxThreads, (VPT >= 8) ? 1 : 2)
     sm.src = -1;
     sm.inc = a.ctl->key_cur;
     if (a.exchange) {  // merge the previous iteration's records (the all-gather)
-      sm.inc = exchange_merge(a, t - 1u, &sm.src);
-      gsrc = merged_gbest_row(a, t - 1u, sm.src);
+      sm.inc = exchange_merge(a, merge_iter(a, t), &sm.src);
+      gsrc = merged_gbest_row(a, merge_iter(a, t), sm.src);
     }
     mbar_init(&sm.gbar, 1);
     mbar_fence_init();
@@ -710,9 +733,9 @@ __global__ void __launch_bounds__(kMaxThreads + 64, 2)
       s_inc = a.ctl->key_cur;
       if (a.exchange) {  // merge the previous iteration's records (the all-gather)
         int src;
-        s_inc = exchange_merge(a, t - 1u, &src);
+        s_inc = exchange_merge(a, merge_iter(a, t), &src);
         s_src = src;
-        gsrc = merged_gbest_row(a, t - 1u, src);
+        gsrc = merged_gbest_row(a, merge_iter(a, t), src);
       }
       mbar_expect_tx(&gbar, row_bytes * (kB ? 5u : 1u));  // releases s_inc / s_src too
       bulk_g2s(sG, gsrc, row_bytes, &gbar);
@@ -938,9 +961,9 @@ __global__ void __launch_bounds__(kMaxThreadsCluster + 64, 1)
       s_inc = a.ctl->key_cur;
       if (a.exchange) {  // merge the previous iteration's records (the all-gather)
         int src;
-        s_inc = exchange_merge(a, t - 1u, &src);
+        s_inc = exchange_merge(a, merge_iter(a, t), &src);
         s_src = src;
-        gsrc = merged_gbest_row(a, t - 1u, src);
+        gsrc = merged_gbest_row(a, merge_iter(a, t), src);
       }
       mbar_expect_tx(&gbar, blk_bytes * (kB ? 5u : 1u));  // releases s_inc / s_src too
       if (cnt > 0) {

@@ -78,3 +78,56 @@ def test_processes_nvlink_exchange_matches_single_gpu(tmp_path, world, obj, n, d
         assert (float(z["f2"]), int(z["i2"])) == (rf2, ri2)
         assert np.array_equal(z["G"].view(np.uint32), RG.view(np.uint32))
         assert np.array_equal(z["G2"].view(np.uint32), RG2.view(np.uint32))
+
+
+def _async_worker(rank, world, port, n, d, obj, steps, out_dir):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    from paper_conf_icpp_liuwc21_b200.distributed import connect_p2p
+    lo, hi = DOMAINS[obj]
+    s = fp.Swarm(n, d, 0.9, 2.0, 2.0, lo, hi, obj, 777, device=0, world=world, rank=rank,
+                 defer_init=True, async_gbest=True)
+    assert connect_p2p(s)
+    s.init()
+    views = []
+    for k in steps:
+        s.step(k)
+        views.append(s.gbest()[:2])
+    X, V, PB, pf, t = s.get_state()
+    f, i, G = s.gbest()
+    np.savez(os.path.join(out_dir, f"a{rank}.npz"), X=X, V=V, PB=PB, pf=pf, G=G, t=t,
+             views=np.array(views, dtype=np.float64))
+    s.close()
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world,obj,n,d", [(2, RASTRIGIN, 40, 300), (3, GRIEWANK, 30, 13),
+                                           (2, ROSENBROCK, 4, 9000)])
+def test_async_split_matches_the_async_oracle(tmp_path, world, obj, n, d):
+    """NEXT-4: each rank adopts its own candidates at once and its peers' one
+    iteration late (merging records of t - 2 over NVLink).  Per-rank state and
+    the host view equal the oracle's asynchronous split model."""
+    from oracle.async_model import AsyncSplitSwarm
+    from pso_testutil import assert_bitwise, assert_fitness_close
+    steps = (2, 3, 4)
+    mp.spawn(_async_worker, args=(world, _free_port(), n, d, obj, steps, str(tmp_path)),
+             nprocs=world, join=True)
+    lo, hi = DOMAINS[obj]
+    model = AsyncSplitSwarm(n, d, 0.9, 2.0, 2.0, lo, hi, obj, 777, k=world)
+    views = []
+    for k in steps:
+        model.step(k)
+        views.append(model.view(0)[:2])
+    for r in range(world):
+        z = np.load(tmp_path / f"a{r}.npz")
+        X, V, PB, pf, t = model.state(r)
+        assert int(z["t"]) == t
+        assert_bitwise(z["X"], X, f"X rank {r}")
+        assert_bitwise(z["V"], V, f"V rank {r}")
+        assert_bitwise(z["PB"], PB, f"PB rank {r}")
+        assert_fitness_close(obj, PB, z["pf"], pf, f"pf rank {r}")
+        for (gf, gi), (mf, mi) in zip(z["views"], views):
+            assert int(gi) == mi
+            assert abs(gf - mf) <= 1e-5 * abs(mf) + 1e-6

@@ -565,3 +565,25 @@ def test_lazy_pbest_rows_lockstep(obj, n, d, monkeypatch):
         assert g.gbest()[:2] == e.gbest()[:2]
     info = g.info()
     assert info["pb_loads"] < e.info()["pb_loads"]  # flagged rows skipped their pb load
+
+
+def test_async_gbest_single_rank_is_synchronous(monkeypatch):
+    """With one rank the asynchronous split has nobody to lag behind: bitwise
+    the synchronous single-GPU run."""
+    import torch  # noqa: F401
+    monkeypatch.setenv("PSO_FORCE_EXCHANGE", "1")
+    comm = fp.nccl_comm_init(1, fp.nccl_unique_id(), 0, 0)
+    try:
+        lo, hi = DOMAINS[RASTRIGIN]
+        g = fp.Swarm(300, 1000, 0.9, 2.0, 2.0, lo, hi, RASTRIGIN, 9, device=0, nccl_comm=comm,
+                     async_gbest=True)
+        ref = gpu_swarm(300, 1000, RASTRIGIN, seed=9)
+        for k in (1, 6, 3):
+            g.step(k)
+            ref.step(k)
+            assert g.gbest()[:2] == ref.gbest()[:2]
+        for x, y in zip(g.get_state()[:4], ref.get_state()[:4]):
+            assert_bitwise(x, y, "async 1-rank state")
+        g.close()
+    finally:
+        fp.nccl_comm_destroy(comm)

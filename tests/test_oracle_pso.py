@@ -334,3 +334,61 @@ def test_one_sided_velocity_bound_makes_positions_monotone():
         s.step(1)
         assert (s.X >= prev).all()
         prev = s.X.copy()
+
+
+# --------------------------------------------------- asynchronous split (NEXT-4)
+def test_async_model_one_shard_is_the_synchronous_run():
+    from oracle.async_model import AsyncSplitSwarm
+    a = AsyncSplitSwarm(24, 9, 0.9, 2, 2, -5.12, 5.12, orc.RASTRIGIN, 3, k=1)
+    s = make(n=24, d=9, obj=orc.RASTRIGIN, seed=3)
+    for k in (1, 5, 9):
+        a.step(k)
+        s.step(k)
+        X, V, PB, pf, t = a.state(0)
+        assert np.array_equal(X, s.X) and np.array_equal(V, s.V) and np.array_equal(PB, s.PB)
+        assert a.view()[:2] == (s.gf, s.gi)
+
+
+def test_async_model_adopts_peer_records_two_iterations_late():
+    """Shard 1 holds a planted particle at the optimum; shard 0's particles can
+    only learn it through the lagged merge: with w = c1 = 0 (pure social term)
+    and a crafted start, shard 0 still moves towards its own incumbent at
+    iterations 1-2 and towards the planted point from iteration 3 on."""
+    from oracle.async_model import AsyncSplitSwarm
+    n, d = 4, 3
+    a = AsyncSplitSwarm(n, d, 0.0, 0.0, 2.0, -5.0, 5.0, orc.SPHERE, 11, k=2, vmax=100.0)
+    # global best after init is some row; plant a better point in shard 1 at t = 1
+    sh0, sh1 = a.shards
+    X1 = sh1.X.copy()
+    X1[:] = 0.25
+    sh1.X[...] = X1
+    sh1.V[...] = 0.0
+    inc0 = sh0.G.copy()
+    a.step(1)
+    # iteration 1: shard 1 found f(0.25..)-ish; shard 0 used the old incumbent
+    rec1 = a.records[1][1]
+    assert rec1[0]  # shard 1 published a strictly better row
+    assert not np.array_equal(inc0, rec1[3])
+    a.step(1)  # iteration 2 merges records of iteration 0 only: shard 1's row not yet known
+    assert not np.array_equal(sh0.G, rec1[3])
+    a.step(1)  # iteration 3 merges records of iteration 1: shard 0 adopts it (or better)
+    assert sh0.gf <= rec1[1]
+
+
+@pytest.mark.parametrize("k", [2, 3])
+def test_async_model_invariants_and_view(k):
+    from oracle.async_model import AsyncSplitSwarm
+    a = AsyncSplitSwarm(30, 7, 0.9, 2, 2, -5.12, 5.12, orc.RASTRIGIN, 5, k=k)
+    prev = [s.pf.copy() for s in a.shards]
+    for _ in range(12):
+        a.step(1)
+        for s, p in zip(a.shards, prev):
+            assert (s.pf <= p).all()
+            assert (s.X >= np.float32(-5.12)).all() and (s.X <= np.float32(5.12)).all()
+        prev = [s.pf.copy() for s in a.shards]
+    # the host view is the global best over every shard's pbest
+    allpf = np.concatenate([s.pf for s in a.shards])
+    gf, gi, G = a.view()
+    assert gf == allpf.min() and gi == int(np.argmin(allpf))
+    for r in range(1, k):
+        assert a.view(r)[:2] == (gf, gi)
