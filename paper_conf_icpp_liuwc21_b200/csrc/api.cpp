@@ -497,7 +497,7 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
   const bool async = (o.flags & PSO_FLAG_ASYNC_GBEST) != 0 && h->xchg;  // needs an exchange
   const size_t viewb = async ? gb : 0;  // the host's global gbest view
   h->arena_bytes =
-      3 * mat + pfb + gb + ctlb + boundb + pbxb + candb + sendb + align_up(recvb, 256);
+      3 * mat + pfb + gb + ctlb + boundb + pbxb + candb + viewb + sendb + align_up(recvb, 256);
   {
     cudaError_t e = cudaMalloc(&h->arena, h->arena_bytes);
     if (e == cudaErrorMemoryAllocation) {
