@@ -246,8 +246,12 @@ def run_gpu(args, w):
     stream = torch.cuda.Stream(device=dev)  # the library enqueues on this stream
     torch.cuda.set_stream(stream)
     K, W = args.steps, args.warmup
+    # PSO_GBEST=async: NEXT-4 asynchronous particle split (peers' records one
+    # iteration late); default synchronous (bitwise independent of N)
+    async_gbest = use_comm and os.environ.get("PSO_GBEST", "sync") == "async"
     sw = fp.Swarm(w.n, w.d, w.w, w.c1, w.c2, w.lo, w.hi, w.objective, w.seed, vmax=w.vmax,
-                  device=local, stream=stream, nccl_comm=comm, timing=True)
+                  device=local, stream=stream, nccl_comm=comm, timing=True,
+                  async_gbest=async_gbest)
     # gbest exchange between ranks: NVLink peer stores from the step kernels
     # (default), or the NCCL all-gather (PSO_EXCHANGE=nccl, or if any rank
     # cannot map its peers)
@@ -303,7 +307,7 @@ def run_gpu(args, w):
         _, _, _, _, t_ck = sw.get_state(out=(X, V, PB, pf))  # a host checkpoint of the swarm
         sw.close()
         sw2 = fp.Swarm(w.n, w.d, w.w, w.c1, w.c2, w.lo, w.hi, w.objective, w.seed, vmax=w.vmax,
-                       device=local, stream=stream, nccl_comm=comm)
+                       device=local, stream=stream, nccl_comm=comm, async_gbest=async_gbest)
         if p2p:
             connect_p2p(sw2)
         gpos = torch.empty((w.d,), dtype=torch.float32).pin_memory()
@@ -341,7 +345,8 @@ def run_gpu(args, w):
             "scaling": "strong", "vs_baseline": None, "dtype": "f32",
             "data": "synthetic (swarm initialised from Philox streams, seed %d)" % w.seed,
             "config": _config(w, world, K, extra={"gbest_exchange": (
-                "nvlink-peer-stores" if p2p else "nccl-allgather") if use_comm else None}),
+                "nvlink-peer-stores" if p2p else "nccl-allgather") if use_comm else None,
+                "gbest_mode": ("async" if async_gbest else "sync") if use_comm else None}),
             "gpu_launches": launches,
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "peak_source": peak_src,
