@@ -221,13 +221,22 @@ def run_gpu(args, w):
     local = int(os.environ.get("LOCAL_RANK", "0"))
     if world != args.gpus:
         raise SystemExit(f"--gpus {args.gpus} but WORLD_SIZE={world}")
+    # PSO_SHARE_GPU=1 (harness test only, never a bench number): every rank runs
+    # on GPU 0 -- gloo process group, no NCCL communicator (NCCL refuses two
+    # ranks on one device), the NVLink-peer protocol over CUDA IPC between the
+    # rank processes.  Exercises the N > 1 code path of this script on one GPU.
+    share = world > 1 and os.environ.get("PSO_SHARE_GPU", "0") not in ("", "0")
+    if share:
+        local = 0
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     comm = None
     # PSO_FORCE_EXCHANGE=1 runs the multi-GPU exchange (process group, NCCL
     # communicator, all-gather + select every step) even on one rank.
     use_comm = world > 1 or os.environ.get("PSO_FORCE_EXCHANGE", "0") not in ("", "0")
-    if use_comm:
+    if share:
+        dist.init_process_group("gloo")
+    elif use_comm:
         dist.init_process_group("nccl", device_id=dev)
         comm = init_comm(local)
 
@@ -239,9 +248,30 @@ def run_gpu(args, w):
     def max_over_ranks(x: float) -> float:
         if world == 1:
             return x
-        t = torch.tensor([x], dtype=torch.float64, device=dev)
+        t = torch.tensor([x], dtype=torch.float64, device="cpu" if share else dev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         return float(t.item())
+
+    def make_swarm(**kw):
+        if share:  # communicator-free ranks: world/rank given, init after P2P connect
+            s = fp.Swarm(w.n, w.d, w.w, w.c1, w.c2, w.lo, w.hi, w.objective, w.seed,
+                         vmax=w.vmax, device=local, stream=stream, world=world, rank=rank,
+                         defer_init=True, async_gbest=async_gbest, **kw)
+            from paper_conf_icpp_liuwc21_b200.distributed import connect_p2p
+            if not connect_p2p(s):
+                raise SystemExit("PSO_SHARE_GPU: peer mapping failed")
+            s.init()
+            return s, True
+        s = fp.Swarm(w.n, w.d, w.w, w.c1, w.c2, w.lo, w.hi, w.objective, w.seed, vmax=w.vmax,
+                     device=local, stream=stream, nccl_comm=comm, async_gbest=async_gbest, **kw)
+        # gbest exchange between ranks: NVLink peer stores from the step kernels
+        # (default), or the NCCL all-gather (PSO_EXCHANGE=nccl, or if any rank
+        # cannot map its peers)
+        on = False
+        if use_comm and os.environ.get("PSO_EXCHANGE", "p2p") == "p2p":
+            from paper_conf_icpp_liuwc21_b200.distributed import connect_p2p
+            on = connect_p2p(s)
+        return s, on
 
     stream = torch.cuda.Stream(device=dev)  # the library enqueues on this stream
     torch.cuda.set_stream(stream)
@@ -249,17 +279,7 @@ def run_gpu(args, w):
     # PSO_GBEST=async: NEXT-4 asynchronous particle split (peers' records one
     # iteration late); default synchronous (bitwise independent of N)
     async_gbest = use_comm and os.environ.get("PSO_GBEST", "sync") == "async"
-    sw = fp.Swarm(w.n, w.d, w.w, w.c1, w.c2, w.lo, w.hi, w.objective, w.seed, vmax=w.vmax,
-                  device=local, stream=stream, nccl_comm=comm, timing=True,
-                  async_gbest=async_gbest)
-    # gbest exchange between ranks: NVLink peer stores from the step kernels
-    # (default), or the NCCL all-gather (PSO_EXCHANGE=nccl, or if any rank
-    # cannot map its peers)
-    want_p2p = use_comm and os.environ.get("PSO_EXCHANGE", "p2p") == "p2p"
-    p2p = False
-    if want_p2p:
-        from paper_conf_icpp_liuwc21_b200.distributed import connect_p2p
-        p2p = connect_p2p(sw)
+    sw, p2p = make_swarm(timing=True)
     sw.step(W)
     sw.synchronize()
     sw.reset_counters()
@@ -306,10 +326,7 @@ def run_gpu(args, w):
         pf = torch.empty((n_local,), dtype=torch.float32).pin_memory()
         _, _, _, _, t_ck = sw.get_state(out=(X, V, PB, pf))  # a host checkpoint of the swarm
         sw.close()
-        sw2 = fp.Swarm(w.n, w.d, w.w, w.c1, w.c2, w.lo, w.hi, w.objective, w.seed, vmax=w.vmax,
-                       device=local, stream=stream, nccl_comm=comm, async_gbest=async_gbest)
-        if p2p:
-            connect_p2p(sw2)
+        sw2, _ = make_swarm()
         gpos = torch.empty((w.d,), dtype=torch.float32).pin_memory()
         with ClockSampler(local) as clk2:
             barrier()
@@ -346,7 +363,8 @@ def run_gpu(args, w):
             "data": "synthetic (swarm initialised from Philox streams, seed %d)" % w.seed,
             "config": _config(w, world, K, extra={"gbest_exchange": (
                 "nvlink-peer-stores" if p2p else "nccl-allgather") if use_comm else None,
-                "gbest_mode": ("async" if async_gbest else "sync") if use_comm else None}),
+                "gbest_mode": ("async" if async_gbest else "sync") if use_comm else None,
+                **({"shared_gpu_harness_test": True} if share else {})}),
             "gpu_launches": launches,
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "peak_source": peak_src,

@@ -16,7 +16,8 @@ shards.  Built only from the pinned shard primitives of the C oracle
      record of iteration t.
 
 Initialisation is synchronous (every shard starts from the global best of
-iteration 0).  The host's view after a pso_step call: each shard's gbest merged
+iteration 0), and so is set_state at iteration t0: records then start at t0
+and step t merges those of max(t - 2, t0).  The host's view after a pso_step call: each shard's gbest merged
 with the records of the last two iterations.
 """
 from __future__ import annotations
@@ -39,6 +40,7 @@ class AsyncSplitSwarm:
             self._merge(s, recs, is_init=True)
         self.records = {0: recs}
         self.t = 0
+        self.t_base = 0  # iteration of the last synchronous (re-)selection
 
     def _merge(self, shard, recs, is_init=False):
         has = [bool(r[0]) for r in recs]
@@ -48,7 +50,7 @@ class AsyncSplitSwarm:
     def step(self, iters=1):
         for _ in range(int(iters)):
             t = self.t + 1
-            lagged = self.records[t - 2 if t >= 2 else 0]
+            lagged = self.records[t - 2 if t >= self.t_base + 2 else self.t_base]
             out = []
             for s in self.shards:
                 self._merge(s, lagged)
@@ -61,12 +63,26 @@ class AsyncSplitSwarm:
             self.t = t
         return self
 
+    def set_state(self, states, t):
+        """Restore every shard's (X, V, PB, pf) at iteration t: a synchronous
+        re-selection (each shard's best pbest row, then the global minimum of
+        (f, i) everywhere), after which the lag restarts from t."""
+        recs = []
+        for s, (X, V, PB, pf) in zip(self.shards, states):
+            s.set_state(X, V, PB, pf, t=t)
+            recs.append((s.nrows > 0, s.gf, s.gi, s.G.copy()))
+        for s in self.shards:
+            self._merge(s, recs, is_init=True)
+        self.records = {int(t): recs}
+        self.t = self.t_base = int(t)
+        return self
+
     def view(self, shard=0):
         """(gf, gi, G) the host reads after a pso_step call on `shard`'s rank."""
         s = self.shards[shard]
         gf, gi = s.gf, s.gi
         best = (gf, gi, s.G.copy())
-        cands = [(f, i, row) for it in (self.t - 1, self.t) if it >= 0
+        cands = [(f, i, row) for it in (self.t - 1, self.t) if it >= self.t_base
                  for has, f, i, row in self.records.get(it, []) if has and f < gf]
         if cands:
             f, i, row = min(cands, key=lambda c: (c[0], c[1]))

@@ -236,6 +236,7 @@ pso_status reset_ctl(pso_swarm* h, uint32_t t) {
   c.t = t;
   c.key_par[0] = c.key_par[1] = ~0ull;
   c.bar_count = 0;
+  h->args.t_base = t;  // async merges never reach back past the re-selection
   // improvements are preserved across set_state: read-modify-write
   DevCtl old{};
   PSO_CUDA(h, cudaMemcpyAsync(&old, h->args.ctl, sizeof(DevCtl), cudaMemcpyDeviceToHost, h->stream));

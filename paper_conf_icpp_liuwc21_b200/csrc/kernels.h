@@ -51,6 +51,7 @@ struct SwarmArgs {
   int async_gbest;            // NEXT-4: merge peers' records with a one-iteration lag
   float* G_view;              // async: the host's global gbest view (pitch floats)
   unsigned epoch;             // p2p: record tags are (epoch << 32 | t); set_state starts an epoch
+  unsigned t_base;            // async: iteration of the last create/set_state (records start there)
   unsigned char* const* peers;  // p2p: device array, world pointers to every rank's recv
   float w, c1, c2, lo, hi, vmax;
   unsigned int seed_lo, seed_hi;

@@ -57,7 +57,7 @@ __global__ void __launch_bounds__(128) k_select(const SwarmArgs a, unsigned t, i
     unsigned long long best = cur;
     const float* row = nullptr;
     const size_t rec = record_bytes(a.nvec * 4);
-    const int n_it = (view_only && t >= 1u) ? 2 : 1;
+    const int n_it = (view_only && t >= a.t_base + 1u) ? 2 : 1;  // records start at t_base
     for (int k = n_it - 1; k >= 0; --k) {
       const unsigned it = t - (unsigned)k;
       if (a.p2p) wait_records(a, it);

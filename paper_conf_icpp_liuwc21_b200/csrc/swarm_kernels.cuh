@@ -408,9 +408,11 @@ __device__ __forceinline__ const unsigned char* records(const SwarmArgs& a, uint
 }
 // The iteration whose records the step kernel of iteration t merges:
 // synchronous t - 1; asynchronous (NEXT-4, "updated in an asynchronous
-// manner") t - 2, so a rank never waits for the iteration its peers are in.
+// manner") t - 2, so a rank never waits for the iteration its peers are in --
+// but never before t_base, the iteration of the last synchronous re-selection
+// (create: 0, set_state: its t), the oldest records of the current epoch.
 __device__ __forceinline__ uint32_t merge_iter(const SwarmArgs& a, uint32_t t) {
-  return a.async_gbest ? (t >= 2u ? t - 2u : 0u) : t - 1u;
+  return a.async_gbest ? (t >= a.t_base + 2u ? t - 2u : a.t_base) : t - 1u;
 }
 // --- NVLink peer exchange (p2p): every rank stores its record of iteration
 // t straight into recv[t & 1][rank] of every peer (CUDA-IPC-mapped), then the

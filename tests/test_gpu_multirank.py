@@ -91,7 +91,9 @@ def _async_worker(rank, world, port, n, d, obj, steps, out_dir):
     assert connect_p2p(s)
     s.init()
     views = []
-    for k in steps:
+    for n_call, k in enumerate(steps):
+        if n_call == len(steps) - 1:  # restore mid-run: synchronous re-selection, lag restarts
+            s.set_state(*s.get_state())
         s.step(k)
         views.append(s.gbest()[:2])
     X, V, PB, pf, t = s.get_state()
@@ -107,8 +109,9 @@ def _async_worker(rank, world, port, n, d, obj, steps, out_dir):
                                            (2, ROSENBROCK, 4, 9000)])
 def test_async_split_matches_the_async_oracle(tmp_path, world, obj, n, d):
     """NEXT-4: each rank adopts its own candidates at once and its peers' one
-    iteration late (merging records of t - 2 over NVLink).  Per-rank state and
-    the host view equal the oracle's asynchronous split model."""
+    iteration late (merging records of t - 2 over NVLink); set_state mid-run
+    re-selects synchronously and restarts the lag.  Per-rank state and the host
+    view equal the oracle's asynchronous split model."""
     from oracle.async_model import AsyncSplitSwarm
     from pso_testutil import assert_bitwise, assert_fitness_close
     steps = (2, 3, 4)
@@ -117,7 +120,9 @@ def test_async_split_matches_the_async_oracle(tmp_path, world, obj, n, d):
     lo, hi = DOMAINS[obj]
     model = AsyncSplitSwarm(n, d, 0.9, 2.0, 2.0, lo, hi, obj, 777, k=world)
     views = []
-    for k in steps:
+    for n_call, k in enumerate(steps):
+        if n_call == len(steps) - 1:
+            model.set_state([model.state(r)[:4] for r in range(world)], t=model.t)
         model.step(k)
         views.append(model.view(0)[:2])
     for r in range(world):

@@ -392,3 +392,28 @@ def test_async_model_invariants_and_view(k):
     assert gf == allpf.min() and gi == int(np.argmin(allpf))
     for r in range(1, k):
         assert a.view(r)[:2] == (gf, gi)
+
+
+@pytest.mark.parametrize("k", [1, 3])
+def test_async_model_set_state_is_a_synchronous_reselection(k):
+    """set_state at t0 re-selects the global best everywhere (the lowest
+    (pf, index) over all shards, as a single-swarm rebest finds it) and the lag
+    restarts at t0: with one shard the model equals the synchronous oracle."""
+    from oracle.async_model import AsyncSplitSwarm
+    a = AsyncSplitSwarm(33, 6, 0.9, 2, 2, -5.12, 5.12, orc.GRIEWANK, 8, k=k)
+    a.step(5)
+    states = [a.state(r)[:4] for r in range(k)]
+    full = [np.concatenate([s[m] for s in states]) for m in range(4)]
+    a.set_state([tuple(np.copy(m) for m in s) for s in states], t=5)
+    ref = make(n=33, d=6, obj=orc.GRIEWANK, seed=8).set_state(*full, t=5)
+    for r in range(k):
+        sh = a.shards[r]
+        assert (sh.gf, sh.gi) == (ref.gf, ref.gi) and np.array_equal(sh.G, ref.G)
+    assert a.view()[:2] == (ref.gf, ref.gi)
+    a.step(4)
+    assert a.t == 9
+    if k == 1:
+        ref.step(4)
+        X, V, PB, pf, _ = a.state(0)
+        assert np.array_equal(X, ref.X) and np.array_equal(PB, ref.PB) and np.array_equal(pf, ref.pf)
+        assert a.view()[:2] == (ref.gf, ref.gi)
