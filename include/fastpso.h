@@ -53,8 +53,10 @@ extern "C" {
 
 #define FASTPSO_VERSION_MAJOR 0
 #define FASTPSO_VERSION_MINOR 1
-#define PSO_D_MAX 65536 /* max dimension: <= 8192 one CTA per row; above, a thread-block
-                          cluster of up to 16 CTAs per row (column blocks) */
+#define PSO_D_MAX_ROW 65536 /* max dimension of the row kernels: <= 8192 one CTA per row;
+                              above, a thread-block cluster of up to 16 CTAs per row */
+#define PSO_D_MAX (1 << 24) /* max dimension: above PSO_D_MAX_ROW the column split
+                              (PSO_FLAG_COLUMN_SPLIT) is used on a single GPU */
 
 typedef struct pso_swarm* pso_handle; /* opaque; owns all device memory */
 
@@ -96,7 +98,7 @@ enum {
                               totals are reported by pso_get_info */
   PSO_FLAG_DEFER_INIT = 2,  /* allocate and plan only; pso_init runs Alg. 1 lines 1-3
                               (lets ranks connect the NVLink exchange first) */
-  PSO_FLAG_ASYNC_GBEST = 4  /* NEXT-4, "updated in an asynchronous manner": each
+  PSO_FLAG_ASYNC_GBEST = 4, /* NEXT-4, "updated in an asynchronous manner": each
                               rank's step kernel adopts its own candidates at once and
                               merges its peers' records one iteration late, so no rank
                               waits for the iteration its peers are in.  Deterministic
@@ -104,6 +106,24 @@ enum {
                               world = 1 identical to the synchronous mode.
                               pso_get_gbest returns the global view folded from every
                               rank's records at the end of the last pso_step call. */
+  PSO_FLAG_COLUMN_SPLIT = 8 /* NEXT-3, "tile matrix": every rank holds ALL n
+                              particles but only a block of the columns.  Rows are cut
+                              into column tiles of T = clamp(ceil(nv / 64), 32, 512)
+                              float4 (nv = ceil(d / 4)); rank r owns tiles
+                              [floor(nt r / world), floor(nt (r+1) / world)) of the nt
+                              (dims [col_begin, col_begin + d_local), pso_get_info).
+                              Each iteration: the move of the block + per-tile fitness
+                              partials stored into every rank's partial table over
+                              NVLink; then every rank combines the partials of each row
+                              in tile order, decides pbest / gbest identically, and
+                              keeps its block of G.  The tiling depends on d only, so
+                              results are bitwise the same for every world size.  State calls (get/set_state,
+                              get_gbest) read and write the rank's column block (n x
+                              d_local; pf has all n rows and must be the same on every
+                              rank).  world > 1 needs the NVLink exchange (p2p connect +
+                              enable before pso_init, so PSO_FLAG_DEFER_INIT) and
+                              nt >= world.  Chosen automatically for a single
+                              GPU when d > PSO_D_MAX_ROW.  Not with ASYNC_GBEST. */
 };
 
 /* Options; a zero-initialised struct means "defaults". */
@@ -130,7 +150,9 @@ typedef struct {
  * gbest = the lowest index attaining min f(x0).
  *   out        receives the handle (set to NULL on failure)
  *   n          global swarm size, 1 <= n < 2^32
- *   d          dimension, 1 <= d <= PSO_D_MAX (else PSO_ERR_UNSUPPORTED)
+ *   d          dimension, 1 <= d <= PSO_D_MAX (else PSO_ERR_UNSUPPORTED); a
+ *              particle-split handle (world > 1 without PSO_FLAG_COLUMN_SPLIT)
+ *              needs d <= PSO_D_MAX_ROW
  *   w, c1, c2  Eq. 1 parameters, finite; c1, c2 = 0 or |c| >= 2^-100 (else
  *              PSO_ERR_UNSUPPORTED: the kernel folds the 2^-24 of the uniform
  *              into c, exact only away from the subnormal range)
@@ -207,6 +229,10 @@ typedef struct {
   double step_kernel_ms;         /* PSO_FLAG_TIMING: summed step-kernel time */
   uint64_t step_kernel_count;    /* PSO_FLAG_TIMING: step kernels timed */
   size_t arena_bytes;            /* device bytes owned by the handle */
+  int32_t column_split;          /* 1: PSO_FLAG_COLUMN_SPLIT layout (NEXT-3) */
+  int32_t col_begin, d_local;    /* the rank's column block: dims [col_begin,
+                                    col_begin + d_local) (0, d without the split) */
+  int32_t col_tiles;             /* column split: tiles per row over all ranks */
 } pso_info;
 pso_status pso_get_info(pso_handle h, pso_info* info);
 /* Reset launches / improvements / timing counters. */

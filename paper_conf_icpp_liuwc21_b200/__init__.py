@@ -11,7 +11,8 @@ import ctypes as C
 
 import numpy as np
 
-from ._lib import (EXPORTS, PSO_D_MAX, PSO_FLAG_ASYNC_GBEST, PSO_FLAG_DEFER_INIT, PSO_FLAG_TIMING, PSO_OBJ_ACKLEY, PSO_OBJ_CUSTOM_BASE,
+from ._lib import (EXPORTS, PSO_D_MAX, PSO_D_MAX_ROW, PSO_FLAG_ASYNC_GBEST, PSO_FLAG_COLUMN_SPLIT,
+                   PSO_FLAG_DEFER_INIT, PSO_FLAG_TIMING, PSO_OBJ_ACKLEY, PSO_OBJ_CUSTOM_BASE,
                    PSO_OBJ_EASOM, PSO_OBJ_GRIEWANK, PSO_OBJ_RASTRIGIN, PSO_OBJ_ROSENBROCK,
                    PSO_OBJ_SPHERE, PSO_OK, PsoError, check, last_error, lib, pso_info, pso_opts,
                    status_string)
@@ -21,6 +22,7 @@ __all__ = [
     "debug_philox", "debug_objective", "nccl_unique_id", "nccl_comm_init", "nccl_comm_destroy",
     "PSO_OBJ_SPHERE", "PSO_OBJ_RASTRIGIN", "PSO_OBJ_ROSENBROCK", "PSO_OBJ_GRIEWANK",
     "PSO_OBJ_ACKLEY", "PSO_OBJ_EASOM", "PSO_OBJ_CUSTOM_BASE", "PSO_FLAG_TIMING", "PSO_D_MAX",
+    "PSO_D_MAX_ROW",
     "EXPORTS",
 ]
 
@@ -51,7 +53,7 @@ class Swarm:
                  objective: int, seed: int, *, vmax: float = 0.0, device: int = -1,
                  stream=None, nccl_comm=None, timing: bool = False, bounds=None,
                  world: int = 1, rank: int = 0, defer_init: bool = False,
-                 async_gbest: bool = False):
+                 async_gbest: bool = False, column_split: bool = False):
         L = lib()
         opts = pso_opts()
         opts.vmax = float(vmax)
@@ -60,7 +62,8 @@ class Swarm:
             opts.stream = int(getattr(stream, "cuda_stream", stream))
         opts.nccl_comm = nccl_comm
         opts.flags = ((PSO_FLAG_TIMING if timing else 0) | (PSO_FLAG_DEFER_INIT if defer_init else 0)
-                      | (PSO_FLAG_ASYNC_GBEST if async_gbest else 0))
+                      | (PSO_FLAG_ASYNC_GBEST if async_gbest else 0)
+                      | (PSO_FLAG_COLUMN_SPLIT if column_split else 0))
         opts.world, opts.rank = int(world), int(rank)
         if bounds is not None:  # per-dimension [vlo | vhi | xlo | xhi], 4 x d
             bounds = np.ascontiguousarray(bounds, dtype=np.float32).reshape(4 * int(d))
@@ -73,6 +76,9 @@ class Swarm:
         self.n, self.d = int(n), int(d)
         self.n_local, self.row_begin = info["n_local"], info["row_begin"]
         self.rank, self.world = info["rank"], info["world"]
+        # column split (NEXT-3): state and gbest position cover dims [col_begin, col_begin + d_local)
+        self.column_split = bool(info["column_split"])
+        self.col_begin, self.d_local = info["col_begin"], info["d_local"]
         self.vmax = float(np.float32(info["vmax"]))
 
     # -------------------------------------------------------------- lifecycle
@@ -115,7 +121,7 @@ class Swarm:
         f, i = C.c_float(), C.c_int64()
         buf = None
         if pos:
-            buf = out if out is not None else np.empty(self.d, np.float32)
+            buf = out if out is not None else np.empty(self.d_local, np.float32)
         check(lib().pso_get_gbest(self._h, C.byref(f), C.byref(i), _ptr(buf, writable=True)),
               "pso_get_gbest")
         return float(np.float32(f.value)), int(i.value), buf
@@ -123,7 +129,7 @@ class Swarm:
     def get_state(self, out=None):
         """Rank-local (X, V, PB, pf, t) as dense host arrays — synchronises."""
         if out is None:
-            m, d = self.n_local, self.d
+            m, d = self.n_local, self.d_local
             out = (np.empty((m, d), np.float32), np.empty((m, d), np.float32),
                    np.empty((m, d), np.float32), np.empty(m, np.float32))
         X, V, PB, pf = out
@@ -139,8 +145,9 @@ class Swarm:
                 return a
             return np.ascontiguousarray(a, dtype=np.float32)
         X, V, PB, pf = prep(X), prep(V), prep(PB), prep(pf)
-        for a, shape in ((X, (self.n_local, self.d)), (V, (self.n_local, self.d)),
-                         (PB, (self.n_local, self.d)), (pf, (self.n_local,))):
+        dl = self.d_local
+        for a, shape in ((X, (self.n_local, dl)), (V, (self.n_local, dl)),
+                         (PB, (self.n_local, dl)), (pf, (self.n_local,))):
             if tuple(a.shape) != shape:
                 raise ValueError(f"state shape {tuple(a.shape)} != {shape}")
         check(lib().pso_set_state(self._h, _ptr(X), _ptr(V), _ptr(PB), _ptr(pf), int(t)),

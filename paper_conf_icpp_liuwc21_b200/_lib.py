@@ -16,8 +16,9 @@ PSO_OK, PSO_ERR_INVALID, PSO_ERR_NOMEM, PSO_ERR_CUDA = 0, 1, 2, 3
 PSO_ERR_NCCL, PSO_ERR_UNSUPPORTED, PSO_ERR_POISONED = 4, 5, 6
 PSO_OBJ_SPHERE, PSO_OBJ_RASTRIGIN, PSO_OBJ_ROSENBROCK = 1, 2, 3
 PSO_OBJ_GRIEWANK, PSO_OBJ_ACKLEY, PSO_OBJ_EASOM, PSO_OBJ_CUSTOM_BASE = 4, 5, 6, 64
-PSO_FLAG_TIMING, PSO_FLAG_DEFER_INIT, PSO_FLAG_ASYNC_GBEST = 1, 2, 4
-PSO_D_MAX = 65536
+PSO_FLAG_TIMING, PSO_FLAG_DEFER_INIT, PSO_FLAG_ASYNC_GBEST, PSO_FLAG_COLUMN_SPLIT = 1, 2, 4, 8
+PSO_D_MAX_ROW = 65536
+PSO_D_MAX = 1 << 24
 
 # every symbol include/fastpso.h declares
 EXPORTS = (
@@ -48,6 +49,8 @@ class pso_info(C.Structure):
         ("pb_loads", C.c_uint64), ("pb_stores", C.c_uint64), ("lazy_pb", C.c_int32),
         ("step_kernel_ms", C.c_double), ("step_kernel_count", C.c_uint64),
         ("arena_bytes", C.c_size_t),
+        ("column_split", C.c_int32), ("col_begin", C.c_int32), ("d_local", C.c_int32),
+        ("col_tiles", C.c_int32),
     ]
 
     def as_dict(self):

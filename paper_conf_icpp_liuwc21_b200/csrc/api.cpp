@@ -8,6 +8,7 @@
 #include <cuda_runtime.h>
 #include <dlfcn.h>
 
+#include <algorithm>
 #include <cmath>
 #include <cstdarg>
 #include <cstdio>
@@ -115,6 +116,9 @@ struct pso_swarm {
   // placement
   int device = 0, sm_count = 0, rank = 0, world = 1;
   bool xchg = false;  // run the all-gather + select exchange (world > 1, or forced for testing)
+  // column split (NEXT-3): all n rows, columns [col_begin, col_begin + d_local)
+  bool colsplit = false;
+  int32_t col_begin = 0, d_local = 0;
   cudaStream_t stream = nullptr;
   bool own_stream = false;
   ncclComm_t comm = nullptr;
@@ -181,7 +185,7 @@ pso_status use_device(pso_swarm* h) {
 // prologue; `fold` additionally runs the select kernel so key_cur / G are
 // final for the host (end of create, set_state and every pso_step call).
 pso_status exchange(pso_swarm* h, uint64_t t, bool fold, bool into_local) {
-  if (!h->xchg) return PSO_OK;
+  if (!h->xchg || h->colsplit) return PSO_OK;  // the column split exchanges inside its kernels
   const size_t rec = record_bytes(h->pitch);
   if (h->args.p2p) {  // records travel by NVLink peer stores inside the kernels
     if (fold) {
@@ -293,8 +297,9 @@ pso_status check_bounds(const float* b, int32_t d) {
 // Copy host bounds (dense d) into the pitched device table (padding 0).
 pso_status upload_bounds(pso_swarm* h, const float* b) {
   std::vector<float> tab((size_t)4 * h->pitch, 0.f);
-  for (int k = 0; k < 4; ++k)
-    std::memcpy(&tab[(size_t)k * h->pitch], b + (size_t)k * h->d, sizeof(float) * (size_t)h->d);
+  for (int k = 0; k < 4; ++k)  // the column block [col_begin, col_begin + d_local)
+    std::memcpy(&tab[(size_t)k * h->pitch], b + (size_t)k * h->d + h->col_begin,
+                sizeof(float) * (size_t)h->d_local);
   PSO_CUDA(h, cudaMemcpyAsync(const_cast<float*>(h->args.bounds), tab.data(), tab.size() * 4,
                               cudaMemcpyHostToDevice, h->stream));
   PSO_CUDA(h, cudaStreamSynchronize(h->stream));
@@ -304,6 +309,20 @@ pso_status upload_bounds(pso_swarm* h, const float* b) {
 // Alg. 1 lines 1-3 + the first evaluation and best update (and, with an
 // exchange, the first gbest exchange).
 pso_status run_init(pso_swarm* h) {
+  if (h->colsplit) {
+    if (h->world > 1 && !h->args.p2p) {
+      h->poisoned = true;
+      return fail(PSO_ERR_INVALID, "column split with world > 1: enable the NVLink exchange first");
+    }
+    PSO_CUDA(h, launch_col_step(h->objective, h->args, h->cfg, 1, h->stream));
+    PSO_CUDA(h, launch_col_decide(h->objective, h->args, h->cfg, 1, h->stream));
+    h->launches += 2;
+    pso_status st = sync_and_check(h);
+    if (st != PSO_OK) return st;
+    h->t = 0;
+    h->inited = true;
+    return PSO_OK;
+  }
   if (h->n_local > 0) {
     PSO_CUDA(h, launch_init(h->objective, h->args, h->cfg, h->stream));
     ++h->launches;
@@ -367,6 +386,15 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
   if (n < 1 || n >= (int64_t)1 << 32) return fail(PSO_ERR_INVALID, "n=%lld outside [1, 2^32)", (long long)n);
   if (d < 1) return fail(PSO_ERR_INVALID, "d=%d < 1", d);
   if (d > PSO_D_MAX) return fail(PSO_ERR_UNSUPPORTED, "d=%d > PSO_D_MAX=%d", d, PSO_D_MAX);
+  bool colsplit = (o.flags & PSO_FLAG_COLUMN_SPLIT) != 0;
+  if (d > PSO_D_MAX_ROW && !colsplit) {
+    if (o.nccl_comm || o.world > 1)
+      return fail(PSO_ERR_UNSUPPORTED, "d=%d > PSO_D_MAX_ROW=%d with a particle split: use "
+                  "PSO_FLAG_COLUMN_SPLIT", d, PSO_D_MAX_ROW);
+    colsplit = true;  // one GPU: rows longer than a cluster are tiled
+  }
+  if (colsplit && (o.flags & PSO_FLAG_ASYNC_GBEST))
+    return fail(PSO_ERR_INVALID, "PSO_FLAG_COLUMN_SPLIT excludes PSO_FLAG_ASYNC_GBEST");
   if (!finite(w) || !finite(c1) || !finite(c2))
     return fail(PSO_ERR_INVALID, "w, c1, c2 must be finite");
   if ((c1 != 0.f && std::fabs(c1) < 0x1p-100f) || (c2 != 0.f && std::fabs(c2) < 0x1p-100f))
@@ -376,7 +404,8 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
   if (!(o.vmax == o.vmax) || std::isinf(o.vmax)) return fail(PSO_ERR_INVALID, "vmax must be finite");
   if (!objective_registered(objective))
     return fail(PSO_ERR_INVALID, "objective %d is not registered", objective);
-  if (o.flags & ~(uint32_t)(PSO_FLAG_TIMING | PSO_FLAG_DEFER_INIT | PSO_FLAG_ASYNC_GBEST))
+  if (o.flags & ~(uint32_t)(PSO_FLAG_TIMING | PSO_FLAG_DEFER_INIT | PSO_FLAG_ASYNC_GBEST |
+                            PSO_FLAG_COLUMN_SPLIT))
     return fail(PSO_ERR_INVALID, "unknown flags 0x%x", o.flags);
   if (o.bounds) {
     pso_status bs = check_bounds(o.bounds, d);
@@ -454,6 +483,29 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
   }
   h->row_begin = (n * h->rank) / h->world;
   h->n_local = (n * (h->rank + 1)) / h->world - h->row_begin;
+  h->d_local = d;
+  int col_nvl = 0, col_q0 = 0, col_tile_f4 = 0, col_t0 = 0, col_nt = 0, col_nbt = 0;
+  if (colsplit) {  // every rank: all rows, a block of whole column tiles (kernels.h col_tile)
+    const int nvg = (d + 3) / 4;
+    col_tile_f4 = col_tile(nvg);
+    col_nbt = col_ntiles(nvg);
+    if (col_nbt < h->world)
+      return bail(fail(PSO_ERR_UNSUPPORTED, "column split: %d column tiles < world=%d (d too small)",
+                       col_nbt, h->world));
+    if (h->world > 1 && !(o.flags & PSO_FLAG_DEFER_INIT))
+      return bail(fail(PSO_ERR_INVALID, "column split with world > 1 needs PSO_FLAG_DEFER_INIT "
+                                        "(connect the NVLink exchange, then pso_init)"));
+    h->colsplit = true;
+    h->xchg = h->world > 1;
+    h->row_begin = 0;
+    h->n_local = n;
+    col_rank_tiles(col_nbt, h->world, h->rank, &col_t0, &col_nt);
+    col_q0 = col_t0 * col_tile_f4;
+    col_nvl = std::min((col_t0 + col_nt) * col_tile_f4, nvg) - col_q0;
+    h->col_begin = 4 * col_q0;
+    h->d_local = std::min(4 * (col_q0 + col_nvl), d) - h->col_begin;
+    h->pitch = 4 * col_nvl;
+  }
 
   // ---- launch plan
   PlanHints hints;
@@ -465,12 +517,21 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
     if (!std::strcmp(v, "reg")) hints.kernel = 0;
     if (!std::strcmp(v, "tma")) hints.kernel = 1;
   }
-  {
+  if (colsplit) {
+    cudaError_t e = plan_colsplit(objective, col_tile_f4, col_nt, n, h->sm_count,
+                                  o.bounds != nullptr, &h->cfg);
+    if (e == cudaErrorInvalidConfiguration) {
+      cudaGetLastError();
+      return bail(fail(PSO_ERR_UNSUPPORTED, "no column-split plan for d=%d", d));
+    }
+    if (e != cudaSuccess) return bail(cuda_fail(nullptr, e, "plan_colsplit"));
+  }
+  if (!colsplit) {
     const char* v = std::getenv("PSO_RESIDENT");
     hints.allow_resident = !h->xchg && hints.kernel == -1 && !(v && !std::strcmp(v, "0"));
     hints.bounds = o.bounds != nullptr;
   }
-  {
+  if (!colsplit) {
     cudaError_t e = plan_launch(objective, d, h->n_local > 0 ? h->n_local : 1, h->sm_count,
                                 hints, &h->cfg);
     if (e == cudaErrorInvalidConfiguration) {
@@ -489,12 +550,14 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
   const size_t boundb = o.bounds ? align_up(4 * (size_t)h->pitch * 4, 256) : 0;
   // lazy pbest rows on the TMA pipelines (step kernels that skip PB when PB == X)
   const char* lz = std::getenv("PSO_LAZY_PB");
-  const bool lazy = h->cfg.tma && !h->cfg.resident && !h->cfg.gridres && !(lz && *lz == '0');
+  const bool lazy = colsplit ||  // the column split always defers pbest copies
+                    (h->cfg.tma && !h->cfg.resident && !h->cfg.gridres && !(lz && *lz == '0'));
   const size_t pbxb = lazy ? align_up(rows, 256) : 0;
   const size_t rec = align_up(record_bytes(h->pitch), 256);
   const size_t candb = h->cfg.gridres ? align_up(2 * (size_t)h->cfg.gridres_grid * h->pitch * 4, 256) : 0;
-  const size_t sendb = h->xchg ? rec : 0;
-  const size_t recvb = h->xchg ? 4 * (size_t)h->world * record_bytes(h->pitch) : 0;
+  const size_t sendb = (h->xchg && !colsplit) ? rec : 0;
+  const size_t recvb = colsplit ? col_tag_bytes(h->world) + 2 * rows * (size_t)col_nbt * 16
+                       : h->xchg ? 4 * (size_t)h->world * record_bytes(h->pitch) : 0;
   const bool async = (o.flags & PSO_FLAG_ASYNC_GBEST) != 0 && h->xchg;  // needs an exchange
   const size_t viewb = async ? gb : 0;  // the host's global gbest view
   h->arena_bytes =
@@ -521,15 +584,22 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
   A.cand = h->cfg.gridres ? (float*)p : nullptr; p += candb;
   A.G_view = async ? (float*)p : nullptr; p += viewb;
   A.async_gbest = async ? 1 : 0;
-  A.send = h->xchg ? p : nullptr; p += sendb;
-  A.recv = h->xchg ? p : nullptr;
+  A.send = sendb ? p : nullptr; p += sendb;
+  A.recv = recvb ? p : nullptr;
   A.n_local = h->n_local;
   A.row_begin = h->row_begin;
   A.d = d;
   A.nvec = h->pitch / 4;
   A.world = h->world;
   A.rank = h->rank;
-  A.exchange = h->xchg ? 1 : 0;
+  A.exchange = (h->xchg && !colsplit) ? 1 : 0;
+  A.colsplit = colsplit ? 1 : 0;
+  A.col_q0 = col_q0;
+  A.nvec_glob = (d + 3) / 4;
+  A.col_chunk = h->cfg.chunk;
+  A.col_nb = col_nt;
+  A.col_bbase = col_t0;
+  A.col_nbt = col_nbt;
   A.w = w; A.c1 = c1; A.c2 = c2; A.lo = lo; A.hi = hi; A.vmax = h->vmax;
   A.seed_lo = (unsigned)seed;
   A.seed_hi = (unsigned)(seed >> 32);
@@ -537,18 +607,17 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
   {
     cudaError_t e = cudaMemsetAsync(A.G, 0, gb + ctlb, h->stream);  // G and ctl
     if (e != cudaSuccess) return bail(cuda_fail(nullptr, e, "cudaMemsetAsync"));
-    if (h->xchg) {
-      e = cudaMemsetAsync(A.send, 0, sendb, h->stream);
-      if (e == cudaSuccess)  // record tags that no iteration matches until written
-        e = cudaMemsetAsync(const_cast<unsigned char*>(A.recv), 0xFF, recvb, h->stream);
-      if (e != cudaSuccess) return bail(cuda_fail(nullptr, e, "cudaMemsetAsync"));
-    }
+    if (sendb) e = cudaMemsetAsync(A.send, 0, sendb, h->stream);
+    if (e == cudaSuccess && recvb)  // record tags that no iteration matches until written
+      e = cudaMemsetAsync(const_cast<unsigned char*>(A.recv), 0xFF,
+                          colsplit ? col_tag_bytes(h->world) : recvb, h->stream);
+    if (e != cudaSuccess) return bail(cuda_fail(nullptr, e, "cudaMemsetAsync"));
   }
   pso_status st = reset_ctl(h, 0);
   if (st != PSO_OK) return bail(st);
   if (o.bounds && (st = upload_bounds(h, o.bounds)) != PSO_OK) return bail(st);
 
-  if (h->n_local == 0 && h->xchg) {  // empty shard: contribute "no candidate"
+  if (h->n_local == 0 && h->xchg && !colsplit) {  // empty shard: contribute "no candidate"
     unsigned long long none[2] = {~0ull, 0ull};
     cudaError_t e = cudaMemcpyAsync(A.send, none, 16, cudaMemcpyHostToDevice, h->stream);
     if (e != cudaSuccess) return bail(cuda_fail(nullptr, e, "cudaMemcpyAsync"));
@@ -573,6 +642,19 @@ pso_status pso_step(pso_handle h, int64_t iters) {
   if (iters == 0) return PSO_OK;
   if ((st = use_device(h)) != PSO_OK) return st;
   const bool timing = (h->flags & PSO_FLAG_TIMING) != 0;
+  if (h->colsplit) {  // two kernels per iteration; the partials travel inside them
+    for (int64_t it = 0; it < iters; ++it) {
+      pso_swarm::Timed* ev = nullptr;
+      if (timing && (st = next_event(h, &ev, 1)) != PSO_OK) return st;
+      if (ev) PSO_CUDA(h, cudaEventRecord(ev->start, h->stream));
+      PSO_CUDA(h, launch_col_step(h->objective, h->args, h->cfg, 0, h->stream));
+      if (ev) PSO_CUDA(h, cudaEventRecord(ev->stop, h->stream));
+      PSO_CUDA(h, launch_col_decide(h->objective, h->args, h->cfg, 0, h->stream));
+      h->launches += 2;
+    }
+    h->t += (uint64_t)iters;
+    return PSO_OK;
+  }
   if (h->cfg.resident || h->cfg.gridres) {  // the whole call is one launch
     for (int64_t done = 0; done < iters;) {
       const int chunk = (int)((iters - done) < (1 << 30) ? (iters - done) : (1 << 30));
@@ -622,7 +704,7 @@ pso_status pso_get_gbest(pso_handle h, float* fitness, int64_t* index, float* po
   const unsigned long long* ksrc = view ? &h->args.ctl->key_view : &h->args.ctl->key_cur;
   const float* gsrc = view ? h->args.G_view : h->args.G;
   PSO_CUDA(h, cudaMemcpyAsync(&key, ksrc, 8, cudaMemcpyDeviceToHost, h->stream));
-  if (pos) PSO_CUDA(h, cudaMemcpyAsync(pos, gsrc, (size_t)h->d * 4, cudaMemcpyDeviceToHost, h->stream));
+  if (pos) PSO_CUDA(h, cudaMemcpyAsync(pos, gsrc, (size_t)h->d_local * 4, cudaMemcpyDeviceToHost, h->stream));
   if ((st = sync_and_check(h)) != PSO_OK) return st;
   if (fitness) *fitness = decode_fitness(key);
   if (index) *index = (int64_t)(uint32_t)key;
@@ -633,7 +715,7 @@ pso_status pso_get_state(pso_handle h, float* x, float* v, float* pb, float* pf,
   pso_status st = check_ready(h);
   if (st != PSO_OK) return st;
   if ((st = use_device(h)) != PSO_OK) return st;
-  const size_t w = (size_t)h->d * 4, sp = (size_t)h->pitch * 4, rows = (size_t)h->n_local;
+  const size_t w = (size_t)h->d_local * 4, sp = (size_t)h->pitch * 4, rows = (size_t)h->n_local;
   if (rows > 0) {
     if (x) PSO_CUDA(h, cudaMemcpy2DAsync(x, w, h->args.X, sp, w, rows, cudaMemcpyDeviceToHost, h->stream));
     if (v) PSO_CUDA(h, cudaMemcpy2DAsync(v, w, h->args.V, sp, w, rows, cudaMemcpyDeviceToHost, h->stream));
@@ -659,10 +741,10 @@ pso_status pso_set_state(pso_handle h, const float* x, const float* v, const flo
     return fail(PSO_ERR_INVALID, "set_state needs x, v, pb and pf");
   if (t >= ((uint64_t)1 << 32)) return fail(PSO_ERR_INVALID, "t=%llu >= 2^32", (unsigned long long)t);
   if ((st = use_device(h)) != PSO_OK) return st;
-  const size_t w = (size_t)h->d * 4, sp = (size_t)h->pitch * 4, rows = (size_t)h->n_local;
+  const size_t w = (size_t)h->d_local * 4, sp = (size_t)h->pitch * 4, rows = (size_t)h->n_local;
   if (rows > 0) {
     const size_t mat = rows * sp;
-    if (h->pitch != h->d) {  // zero the row padding
+    if (h->pitch != h->d_local) {  // zero the row padding
       PSO_CUDA(h, cudaMemsetAsync(h->args.X, 0, mat, h->stream));
       PSO_CUDA(h, cudaMemsetAsync(h->args.V, 0, mat, h->stream));
       PSO_CUDA(h, cudaMemsetAsync(h->args.PB, 0, mat, h->stream));
@@ -760,6 +842,8 @@ pso_status pso_p2p_enable(pso_handle h, int32_t on) {
   pso_status st = check_handle(h);
   if (st != PSO_OK) return st;
   if (on && !h->peers_dev) return fail(PSO_ERR_INVALID, "pso_p2p_connect first");
+  if (!on && h->colsplit)
+    return fail(PSO_ERR_UNSUPPORTED, "the column split exchanges only over NVLink");
   if ((st = use_device(h)) != PSO_OK) return st;
   if ((st = sync_and_check(h)) != PSO_OK) return st;
   h->args.p2p = on ? 1 : 0;
@@ -812,6 +896,10 @@ pso_status pso_get_info(pso_handle h, pso_info* info) {
   info->lazy_pb = h->args.lazy_pb;
   info->step_kernel_ms = h->timed_ms;
   info->step_kernel_count = h->timed_count;
+  info->column_split = h->colsplit ? 1 : 0;
+  info->col_begin = h->col_begin;
+  info->d_local = h->d_local;
+  info->col_tiles = h->args.col_nbt;
   info->arena_bytes = h->arena_bytes;
   return PSO_OK;
 }

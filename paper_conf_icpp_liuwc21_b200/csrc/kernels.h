@@ -53,9 +53,46 @@ struct SwarmArgs {
   unsigned epoch;             // p2p: record tags are (epoch << 32 | t); set_state starts an epoch
   unsigned t_base;            // async: iteration of the last create/set_state (records start there)
   unsigned char* const* peers;  // p2p: device array, world pointers to every rank's recv
+  // Column split (NEXT-3, "tile matrix"): this rank holds float4 columns
+  // [col_q0, col_q0 + nvec) of every row (n_local = n); X, V, PB, G, bounds are
+  // that block (pitch 4 nvec).  recv = [2][world] u64 tags, then the partials
+  // [2 parities][n][col_nbt] float4 {acc0, acc1, first x', last x'}.
+  int colsplit;
+  int col_q0;       // first global float4 of the block
+  int nvec_glob;    // float4 of a full row
+  int col_chunk;    // float4 per local tile (a row of the block is col_nb tiles)
+  int col_nb;       // local tiles per row
+  int col_bbase;    // index of this rank's first tile among all ranks' tiles
+  int col_nbt;      // tiles per row over all ranks
   float w, c1, c2, lo, hi, vmax;
   unsigned int seed_lo, seed_hi;
 };
+
+// Column split geometry (host plan and decide kernel).  The tiling depends on
+// d only, never on the world size: rows of nvec = ceil(d / 4) float4 are cut
+// into tiles of T = clamp(ceil(nvec / 64), 32, 512) float4 (the last one
+// ragged), and rank r of `world` owns tiles [floor(nt r / world),
+// floor(nt (r+1) / world)).  The partial of a tile and the combine order over
+// tiles are therefore the same for every world size, so fitness, decisions
+// and state are bitwise independent of it.
+constexpr int kColTileMax = 512, kColTileMin = 32;
+__host__ __device__ inline int col_tile(int nvec) {
+  int t = (nvec + 63) / 64;
+  t = t < kColTileMin ? kColTileMin : (t > kColTileMax ? kColTileMax : t);
+  return t < nvec ? t : nvec;
+}
+__host__ __device__ inline int col_ntiles(int nvec) {
+  const int t = col_tile(nvec);
+  return (nvec + t - 1) / t;
+}
+__host__ __device__ inline void col_rank_tiles(int ntiles, int world, int r, int* t0, int* nt) {
+  const long long b = (long long)ntiles * r / world, e = (long long)ntiles * (r + 1) / world;
+  *t0 = (int)b;
+  *nt = (int)(e - b);
+}
+__host__ __device__ inline size_t col_tag_bytes(int world) {
+  return ((size_t)2 * world * 8 + 255) / 256 * 256;
+}
 
 struct LaunchCfg {
   int vpt = 1;        // float4 per compute thread per row
@@ -79,6 +116,9 @@ struct LaunchCfg {
   size_t resident_smem = 0;
   size_t init_smem = 0;
   int bounds = 0;     // kernels instantiated with per-dimension bounds
+  int colsplit = 0;   // column split: k_col_step + k_col_decide per iteration
+  int col_grid = 0, col_stages = 0, col_decide_grid = 0;
+  size_t col_smem = 0, col_decide_smem = 0;
 };
 
 // Tuning overrides (0 / -1 = automatic): PSO_VPT, PSO_KERNEL=reg|tma, PSO_STAGES, PSO_CTAS.
@@ -102,6 +142,8 @@ struct KernelTable {
   const void* resident[2];
   const void* init[4];
   const void* eval[4];
+  const void* col_step[2];  // [per-dim bounds]
+  const void* col_decide;
 };
 // The table of a registered objective id, or null (obj_*.cu).
 const KernelTable* kernel_table(int objective);
@@ -116,6 +158,14 @@ cudaError_t launch_resident(int objective, const SwarmArgs& a, const LaunchCfg& 
                             cudaStream_t s);
 cudaError_t launch_gridres(int objective, const SwarmArgs& a, const LaunchCfg& c, int iters,
                            cudaStream_t s);
+// Column split (NEXT-3): tile plan for this rank's block, and the two kernels
+// of an iteration (init = 1: Alg. 1 lines 1-3 instead of the move).
+cudaError_t plan_colsplit(int objective, int tile, int tiles_local, long long n, int sm_count,
+                          bool bounds, LaunchCfg* cfg);
+cudaError_t launch_col_step(int objective, const SwarmArgs& a, const LaunchCfg& c, int init,
+                            cudaStream_t s);
+cudaError_t launch_col_decide(int objective, const SwarmArgs& a, const LaunchCfg& c, int init,
+                              cudaStream_t s);
 cudaError_t launch_rebest(const SwarmArgs& a, unsigned t, cudaStream_t s);
 // Fold the records of iteration t (and, asynchronous, of t - 1) for the host;
 // into_local: also into the kernels' incumbent (create / set_state).

@@ -1,0 +1,351 @@
+// swarm_colsplit.cuh — the column split (the
+// paper's second multi-GPU approach: "tile the matrix").  Included by
+// swarm_kernels.cuh inside namespace fastpso::{anon}.
+//
+// Each rank holds a block of whole tiles of EVERY row (kernels.h col_tile);
+// one iteration is two kernels:
+//
+//   k_col_step    the Eq. 1 move of the rank's tiles (a tile = up to kColTile
+//                 float4 of one row), streamed through the same warp-specialised
+//                 TMA ring as k_step_tma (producer warp: bulk copies of x, v, pb
+//                 and the G tile; compute warps: Philox + move + the functor's
+//                 map over the tile; finaliser warp: warp partials -> the tile's
+//                 partial {acc0, acc1, first x', last x'}, bulk stores of x', v').
+//                 The tile partial is stored into the partial table of every
+//                 rank (own memory, and the peers' over NVLink, CUDA-IPC-mapped);
+//                 the last CTA then releases this rank's tag of iteration t.
+//   k_col_decide  acquires every rank's tag, combines a row's tile partials in
+//                 tile order (plus the neighbour terms x_j, x_{j+1} across tile
+//                 borders), finalises f, and takes the pbest decision (Alg. 1
+//                 lines 7-9) and the gbest argmin (lines 10-12) -- every rank
+//                 computes the same bits from the same table, so the decisions
+//                 agree without another exchange.  The last CTA copies the
+//                 winner's x (this rank's block) into G.
+//
+// The pbest copy cannot wait for the decision (x' is stored before f is
+// known), so pbest rows use the lazy form: pbx[r] = 1 records "row r improved
+// in the last decision, its pbest is its current X".  The next k_col_step then
+// uses pb = x and stores the old x into PB (the deferred copy); a row that
+// never improves only reads PB.  Bytes per element: 16 (x, v in and out) + 4
+// (PB read, or PB written after an improvement).
+//
+// Init (init = 1, Alg. 1 lines 1-3): the producer loads nothing; the compute
+// warps draw x0, v0 (Philox X0 / V0 at the global column), the finaliser stores
+// X, V and PB = x0, and k_col_decide sets pf = f (NaN -> +inf) and selects the
+// global best from scratch.
+
+template <class Obj>
+__device__ __forceinline__ float4* col_parts(unsigned char* region, const SwarmArgs& a, int par) {
+  return reinterpret_cast<float4*>(region + col_tag_bytes(a.world)) +
+         (size_t)par * (size_t)a.n_local * (size_t)a.col_nbt;
+}
+
+constexpr int kColCompute = 256;  // compute threads of k_col_step (+ producer + finaliser warps)
+
+template <class Obj, bool kB>
+__global__ void __launch_bounds__(kColCompute + 64, 2)
+    k_col_step(const SwarmArgs a, int init, int stages) {
+  static_assert(Obj::kAcc <= 2, "the tile partial carries two accumulators");
+  extern __shared__ __align__(128) unsigned char dsmem[];
+  constexpr int nthr = kColCompute, nwarps = nthr / 32;
+  constexpr int per = kB ? 8 : 4;  // stage arrays: x, v, pb, g [, vlo, vhi, xlo, xhi]
+  const int chunk = a.col_chunk, nb = a.col_nb, nvl = a.nvec, d = a.d;
+  float4* ring = reinterpret_cast<float4*>(dsmem);
+  __shared__ float red[kMaxStages][nwarps * 2];
+  __shared__ unsigned long long full[kMaxStages], empty[kMaxStages], done[kMaxStages];
+  __shared__ int sflag[kMaxStages];
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  if (tid == 0) {
+    for (int s = 0; s < stages; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&done[s], (unsigned)nwarps);
+      mbar_init(&empty[s], 1);
+    }
+    mbar_fence_init();
+  }
+  __syncthreads();
+  const uint32_t t = init ? 0u : a.ctl->t + 1u;
+  const long long items = a.n_local * (long long)nb;
+
+  if (warp == nwarps) {  // ---------------- producer
+    if (lane == 0) {
+      int s = 0;
+      unsigned ph = 0;
+      long long i = 0;
+      for (long long k = blockIdx.x; k < items; k += gridDim.x, ++i) {
+        const long long r = k / nb;
+        const int q0 = (int)(k - r * nb) * chunk;
+        const int cnt = min(chunk, nvl - q0);
+        const unsigned bytes = (unsigned)cnt * 16u;
+        if (i >= stages) mbar_wait(&empty[s], ph ^ 1u);
+        float4* st = ring + (size_t)s * per * chunk;
+        if (init) {
+          sflag[s] = 0;
+          mbar_arrive(&full[s]);
+        } else {
+          const int fl = a.pbx[r];
+          sflag[s] = fl;
+          mbar_expect_tx(&full[s], bytes * ((fl ? 3u : 4u) + (kB ? 4u : 0u)));
+          const size_t off = ((size_t)r * nvl + q0) * 4;
+          bulk_g2s(st, a.X + off, bytes, &full[s]);
+          bulk_g2s(st + chunk, a.V + off, bytes, &full[s]);
+          if (!fl) bulk_g2s(st + 2 * chunk, a.PB + off, bytes, &full[s]);
+          bulk_g2s(st + 3 * chunk, a.G + (size_t)q0 * 4, bytes, &full[s]);
+          if (kB)
+            for (int m = 0; m < 4; ++m)
+              bulk_g2s(st + (4 + m) * chunk, a.bounds + ((size_t)m * nvl + q0) * 4, bytes, &full[s]);
+        }
+        if (++s == stages) {
+          s = 0;
+          ph ^= 1u;
+        }
+      }
+    }
+    return;
+  }
+
+  if (warp == nwarps + 1) {  // ---------------- finaliser
+    if (lane == 0) {
+      const int par = (int)(t & 1u);
+      unsigned n_pbl = 0, n_pbs = 0;
+      int s = 0, prev = -1;
+      unsigned ph = 0;
+      for (long long k = blockIdx.x; k < items; k += gridDim.x) {
+        const long long r = k / nb;
+        const int b = (int)(k - r * nb);
+        const int q0 = b * chunk;
+        const int cnt = min(chunk, nvl - q0);
+        const unsigned bytes = (unsigned)cnt * 16u;
+        mbar_wait(&done[s], ph);
+        float c[Obj::kAcc];
+        Obj::init(c);
+        for (int w = 0; w < nwarps; ++w) {
+          float bw[Obj::kAcc];
+#pragma unroll
+          for (int j = 0; j < Obj::kAcc; ++j) bw[j] = red[s][w * Obj::kAcc + j];
+          Obj::combine(c, bw);
+        }
+        const float4* st = ring + (size_t)s * per * chunk;
+        const int fl = sflag[s];
+        const float4* xnew = fl ? st + 2 * chunk : st;  // where the compute warps put x'
+        const float4 msg =
+            make_float4(c[0], Obj::kAcc > 1 ? c[Obj::kAcc - 1] : 0.f, xnew[0].x, xnew[cnt - 1].w);
+        const size_t pidx = (size_t)r * a.col_nbt + (size_t)(a.col_bbase + b);
+        if (a.world > 1) {
+          for (int q = 0; q < a.world; ++q) col_parts<Obj>(a.peers[q], a, par)[pidx] = msg;
+        } else {
+          col_parts<Obj>(const_cast<unsigned char*>(a.recv), a, par)[pidx] = msg;
+        }
+        const size_t off = ((size_t)r * nvl + q0) * 4;
+        bulk_s2g(a.X + off, xnew, bytes);
+        bulk_s2g(a.V + off, st + chunk, bytes);
+        if (init || fl) bulk_s2g(a.PB + off, st, bytes);  // x0, or the deferred pbest (old x)
+        if (b == 0 && !init) {  // per row: PB read, or PB written
+          n_pbl += fl ? 0u : 1u;
+          n_pbs += fl ? 1u : 0u;
+        }
+        bulk_commit();
+        if (prev >= 0) {
+          bulk_wait_read<1>();
+          mbar_arrive(&empty[prev]);
+        }
+        prev = s;
+        if (++s == stages) {
+          s = 0;
+          ph ^= 1u;
+        }
+      }
+      bulk_wait_all();
+      fence_proxy_async_global();
+      if (n_pbl) atomicAdd(&a.ctl->pb_loads, (unsigned long long)n_pbl);
+      if (n_pbs) atomicAdd(&a.ctl->pb_stores, (unsigned long long)n_pbs);
+      __threadfence_system();  // this CTA's partials (local and peer stores) before the ticket
+      if (atomicAdd(&a.ctl->done, 1u) == gridDim.x - 1) {
+        __threadfence_system();
+        a.ctl->done = 0;
+        if (a.world > 1) {
+          const unsigned long long tag = ((unsigned long long)a.epoch << 32) | t;
+          for (int q = 0; q < a.world; ++q)
+            st_release_sys_u64(a.peers[q] + ((size_t)par * a.world + a.rank) * 8, tag);
+        }
+      }
+    }
+    return;
+  }
+
+  // ---------------- compute warps
+  const PhiloxKey key{a.seed_lo, a.seed_hi};
+  const MoveParams mp = move_params(a);
+  const float4* B4 = reinterpret_cast<const float4*>(a.bounds);
+  int s = 0;
+  unsigned ph = 0;
+  for (long long k = blockIdx.x; k < items; k += gridDim.x) {
+    const long long r = k / nb;
+    const int q0 = (int)(k - r * nb) * chunk;
+    const int cnt = min(chunk, nvl - q0);
+    const uint32_t gi = (uint32_t)(a.row_begin + r);
+    float4* st = ring + (size_t)s * per * chunk;
+    mbar_wait(&full[s], ph);
+    const int fl = sflag[s];
+    float4* xdst = fl ? st + 2 * chunk : st;  // keep the old x for the deferred pbest copy
+    float acc[Obj::kAcc];
+    Obj::init(acc);
+    for (int ql = tid; ql < cnt; ql += nthr) {
+      const int qg = a.col_q0 + q0 + ql;  // global float4: Philox counter, functor index
+      float4 x, v;
+      if (init) {
+        init_float4_at(a, key, gi, qg, B4, nvl, q0 + ql, x, v);
+      } else {
+        x = st[ql];
+        v = st[chunk + ql];
+        const float4 pb = fl ? x : st[2 * chunk + ql];
+        const float4 g = st[3 * chunk + ql];
+        const float4 r1 = raw24x4(key, kTagR1, t, gi, (uint32_t)qg);
+        const float4 r2 = raw24x4(key, kTagR2, t, gi, (uint32_t)qg);
+        move4<kB>(mp, x, v, pb, g, r1, r2, st + 4 * chunk, chunk, ql);
+        if ((d & 3) && qg == a.nvec_glob - 1) {
+          const int jj = 4 * qg;
+          if (jj + 1 >= d) x.y = v.y = 0.f;
+          if (jj + 2 >= d) x.z = v.z = 0.f;
+          if (jj + 3 >= d) x.w = v.w = 0.f;
+        }
+      }
+      xdst[ql] = x;
+      st[chunk + ql] = v;
+      if constexpr (!Obj::kNeighbor) map4<Obj>(acc, x, 0.f, 4 * qg, d);
+    }
+    if constexpr (Obj::kNeighbor) {
+      team_sync(nthr);  // every x' of the tile is in the stage
+      for (int ql = tid; ql < cnt; ql += nthr) {
+        const int qg = a.col_q0 + q0 + ql;
+        const float4 x = xdst[ql];
+        if (ql + 1 < cnt) {
+          map4<Obj>(acc, x, xdst[ql + 1].x, 4 * qg, d);
+        } else if (qg == a.nvec_glob - 1) {
+          map4<Obj>(acc, x, 0.f, 4 * qg, d);  // the row's last float4
+        } else {  // x_{j+1} of the tile's last dim is in the next tile: k_col_decide adds it
+          Obj::map(acc, x.x, x.y, 4 * qg, d);
+          Obj::map(acc, x.y, x.z, 4 * qg + 1, d);
+          Obj::map(acc, x.z, x.w, 4 * qg + 2, d);
+        }
+      }
+    }
+    warp_combine<Obj>(acc);
+    if (lane == 0) {
+#pragma unroll
+      for (int j = 0; j < Obj::kAcc; ++j) red[s][warp * Obj::kAcc + j] = acc[j];
+    }
+    fence_proxy_async_shared();  // x', v' visible to the finaliser's bulk stores
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&done[s]);
+    if (++s == stages) {
+      s = 0;
+      ph ^= 1u;
+    }
+  }
+}
+
+// One warp per row.
+template <class Obj>
+__global__ void __launch_bounds__(256) k_col_decide(const SwarmArgs a, int init) {
+  __shared__ unsigned long long s_best[8];
+  __shared__ unsigned s_nimp[8];
+  __shared__ int s_last;
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  const uint32_t t = init ? 0u : a.ctl->t + 1u;
+  const int par = (int)(t & 1u);
+  const int nbt = a.col_nbt;
+  if (a.world > 1 && tid == 0) {  // every rank's tiles of iteration t have landed
+    const unsigned long long want = ((unsigned long long)a.epoch << 32) | t;
+    const unsigned long long t0 = globaltimer_ns();
+    for (int q = 0; q < a.world; ++q) {
+      const void* tag = a.recv + ((size_t)par * a.world + q) * 8;
+      while (ld_acquire_sys_u64(tag) != want) {
+        __nanosleep(64);
+        if (globaltimer_ns() - t0 > 60ull * 1000000000ull) __trap();
+      }
+    }
+  }
+  __syncthreads();
+  const float4* P = col_parts<Obj>(const_cast<unsigned char*>(a.recv), a, par);
+  const uint32_t inc_ord = (uint32_t)(a.ctl->key_cur >> 32);
+  unsigned long long best = ~0ull;
+  unsigned nimp = 0;
+  const long long wpc = blockDim.x >> 5;
+  for (long long r = blockIdx.x * wpc + warp; r < a.n_local; r += (long long)gridDim.x * wpc) {
+    const float4* Pr = P + (size_t)r * nbt;
+    float c[Obj::kAcc];
+    Obj::init(c);
+    for (int bt = lane; bt < nbt; bt += 32) {
+      const float4 p = __ldcg(Pr + bt);
+      const float pa[2] = {p.x, p.y};
+      Obj::combine(c, pa);
+      if (Obj::kNeighbor && bt + 1 < nbt) {  // x_j, x_{j+1} across the tile border
+        float bterm[Obj::kAcc];
+        Obj::init(bterm);
+        Obj::map(bterm, p.w, __ldcg(Pr + bt + 1).z, 4 * (bt + 1) * a.col_chunk - 1, a.d);
+        Obj::combine(c, bterm);
+      }
+    }
+    warp_combine<Obj>(c);  // xor butterfly: every lane holds the same bits
+    if (lane == 0) {
+      const float f = Obj::finalize(c, a.d);
+      const uint32_t gi = (uint32_t)(a.row_begin + r);
+      float val = f;
+      if (init) {
+        val = (f != f) ? __int_as_float(0x7f800000) : f;  // reading 11: NaN -> +inf
+        a.pf[r] = val;
+        a.pbx[r] = 0;  // PB was stored (= x0)
+      } else {
+        const bool imp = f < a.pf[r];  // strict; NaN never improves
+        if (imp) {
+          a.pf[r] = f;
+          ++nimp;
+        }
+        a.pbx[r] = imp ? 1 : 0;
+      }
+      if (val == val && ord_f32(val) < inc_ord) {  // strictly below gf (Alg. 1 line 10)
+        const unsigned long long key = pack_key(val, gi);
+        best = key < best ? key : best;
+      }
+    }
+  }
+  if (lane == 0) {
+    s_best[warp] = best;
+    s_nimp[warp] = nimp;
+  }
+  __syncthreads();
+  if (tid == 0) {
+    for (int w = 1; w < (int)wpc; ++w) {
+      best = s_best[w] < best ? s_best[w] : best;
+      nimp += s_nimp[w];
+    }
+    if (best != ~0ull) atomicMin(&a.ctl->key_acc, best);
+    if (nimp) atomicAdd(&a.ctl->improvements, (unsigned long long)nimp);
+    __threadfence();
+    s_last = (atomicAdd(&a.ctl->done, 1u) == gridDim.x - 1) ? 1 : 0;
+  }
+  __syncthreads();
+  if (!s_last) return;
+  // last CTA: the winner's x' is its pbest (it improved); copy this rank's block
+  if (tid == 0) {
+    __threadfence();
+    s_best[0] = *(volatile unsigned long long*)&a.ctl->key_acc;
+    s_best[1] = a.ctl->key_cur;
+  }
+  __syncthreads();
+  const unsigned long long acc = s_best[0], cur = s_best[1];
+  if (acc < cur) {
+    const float4* x = reinterpret_cast<const float4*>(a.X) +
+                      ((long long)(uint32_t)acc - a.row_begin) * a.nvec;
+    float4* G4 = reinterpret_cast<float4*>(a.G);
+    for (int q = tid; q < a.nvec; q += blockDim.x) G4[q] = __ldcg(x + q);
+  }
+  __syncthreads();
+  if (tid == 0) {
+    if (acc < cur) a.ctl->key_cur = acc;
+    a.ctl->key_acc = ~0ull;
+    a.ctl->t = t;
+    a.ctl->done = 0;
+  }
+}

@@ -419,6 +419,62 @@ cudaError_t launch_init(int objective, const SwarmArgs& a, const LaunchCfg& c, c
                           dim3(c.init_threads), args, 0, s);
 }
 
+// ---------------------------------------------------------- column split
+cudaError_t plan_colsplit(int objective, int tile, int tiles_local, long long n, int sm_count,
+                          bool bounds, LaunchCfg* cfg) {
+  const KernelTable* t = kernel_table(objective);
+  if (!t) return cudaErrorInvalidDeviceFunction;
+  if (tile < 1 || tiles_local < 1 || n < 1) return cudaErrorInvalidConfiguration;
+  const int per = bounds ? 8 : 4;
+  const size_t stage = (size_t)per * tile * 16;
+  const int ctas = bounds ? 1 : 2;  // ~100 registers x 320 threads: 2 CTAs per SM
+  int stages = ring_stages(0, stage, ctas);
+  if (stages > 4) stages = 4;  // 4 tiles in flight per CTA cover the HBM latency
+  if (stages < 2) return cudaErrorInvalidConfiguration;
+  const void* fn = t->col_step[bounds ? 1 : 0];
+  const size_t smem = (size_t)stages * stage;
+  cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return e;
+  const long long items = n * tiles_local;
+  long long grid = (long long)sm_count * ctas;
+  if (grid > items) grid = items;
+  cfg->colsplit = 1;
+  cfg->chunk = tile;
+  cfg->col_grid = (int)grid;
+  cfg->col_stages = stages;
+  cfg->col_smem = smem;
+  cfg->threads = kColCompute + 64;
+  cfg->compute = kColCompute;
+  cfg->grid = (int)grid;
+  cfg->ctas_per_sm = ctas;
+  cfg->tma = 1;
+  cfg->stages = stages;
+  cfg->smem = smem;
+  cfg->bounds = bounds ? 1 : 0;
+  long long dg = (n + 7) / 8;
+  if (dg > (long long)sm_count * 8) dg = (long long)sm_count * 8;
+  cfg->col_decide_grid = (int)(dg < 1 ? 1 : dg);
+  return cudaSuccess;
+}
+
+cudaError_t launch_col_step(int objective, const SwarmArgs& a, const LaunchCfg& c, int init,
+                            cudaStream_t s) {
+  const KernelTable* t = kernel_table(objective);
+  if (!t) return cudaErrorInvalidDeviceFunction;
+  int stages = c.col_stages;
+  void* args[] = {const_cast<SwarmArgs*>(&a), &init, &stages};
+  return cudaLaunchKernel(t->col_step[c.bounds ? 1 : 0], dim3(c.col_grid), dim3(c.threads), args,
+                          c.col_smem, s);
+}
+
+cudaError_t launch_col_decide(int objective, const SwarmArgs& a, const LaunchCfg& c, int init,
+                              cudaStream_t s) {
+  const KernelTable* t = kernel_table(objective);
+  if (!t) return cudaErrorInvalidDeviceFunction;
+  void* args[] = {const_cast<SwarmArgs*>(&a), &init};
+  return cudaLaunchKernel(t->col_decide, dim3(c.col_decide_grid), dim3(256), args, 0, s);
+}
+
 cudaError_t launch_rebest(const SwarmArgs& a, unsigned t, cudaStream_t s) {
   long long blocks = (a.n_local + 255) / 256;
   if (blocks > 1024) blocks = 1024;

@@ -1537,10 +1537,13 @@ __global__ void __launch_bounds__(kMaxThreads, 1) k_gridres(const SwarmArgs a, i
 // handles float4 t, t + nthr, ... of a row (any d; the same accumulation
 // order as the register kernels); a neighbour functor's x_{j+1} across a
 // float4 boundary is recomputed from its Philox word.
-__device__ __forceinline__ void init_float4(const SwarmArgs& a, PhiloxKey key, uint32_t gi, int q,
-                                            float4& xo, float4& vo) {
-  const int nvec = a.nvec, d = a.d;
-  const float4* B4 = reinterpret_cast<const float4*>(a.bounds);  // null: scalar bounds
+// init_float4_at: dims 4 qg .. 4 qg + 3 of the row (qg: global float4 index,
+// the Philox counter and the padding test), bounds from float4 qb of a table
+// with `bstride` float4 per array (the column split keeps only its block).
+__device__ __forceinline__ void init_float4_at(const SwarmArgs& a, PhiloxKey key, uint32_t gi,
+                                               int qg, const float4* B4, int bstride, int qb,
+                                               float4& xo, float4& vo) {
+  const int q = qg, d = a.d;
   const float4 ux = uniforms4(key, kTagX0, 0u, gi, (uint32_t)q);
   const float4 uv = uniforms4(key, kTagV0, 0u, gi, (uint32_t)q);
   float xs[4] = {ux.x, ux.y, ux.z, ux.w};
@@ -1549,10 +1552,10 @@ __device__ __forceinline__ void init_float4(const SwarmArgs& a, PhiloxKey key, u
   float4 vhi4 = make_float4(a.vmax, a.vmax, a.vmax, a.vmax);
   float4 xlo4 = make_float4(a.lo, a.lo, a.lo, a.lo), xhi4 = make_float4(a.hi, a.hi, a.hi, a.hi);
   if (B4) {
-    vlo4 = B4[q];
-    vhi4 = B4[nvec + q];
-    xlo4 = B4[2 * nvec + q];
-    xhi4 = B4[3 * nvec + q];
+    vlo4 = B4[qb];
+    vhi4 = B4[bstride + qb];
+    xlo4 = B4[2 * bstride + qb];
+    xhi4 = B4[3 * bstride + qb];
   }
   const float vlo[4] = {vlo4.x, vlo4.y, vlo4.z, vlo4.w};
   const float vhi[4] = {vhi4.x, vhi4.y, vhi4.z, vhi4.w};
@@ -1568,6 +1571,10 @@ __device__ __forceinline__ void init_float4(const SwarmArgs& a, PhiloxKey key, u
   }
   xo = make_float4(xs[0], xs[1], xs[2], xs[3]);
   vo = make_float4(vs[0], vs[1], vs[2], vs[3]);
+}
+__device__ __forceinline__ void init_float4(const SwarmArgs& a, PhiloxKey key, uint32_t gi, int q,
+                                            float4& xo, float4& vo) {
+  init_float4_at(a, key, gi, q, reinterpret_cast<const float4*>(a.bounds), a.nvec, q, xo, vo);
 }
 
 template <class Obj, int VPT>
@@ -1639,6 +1646,8 @@ __global__ void __launch_bounds__(kMaxThreads) k_eval(const float* X, long long 
   }
 }
 
+#include "swarm_colsplit.cuh"
+
 template <class Obj>
 KernelTable make_kernel_table() {
   KernelTable t{};
@@ -1663,6 +1672,9 @@ KernelTable make_kernel_table() {
   t.eval[1] = (const void*)k_eval<Obj, 2>;
   t.eval[2] = (const void*)k_eval<Obj, 4>;
   t.eval[3] = (const void*)k_eval<Obj, 8>;
+  t.col_step[0] = (const void*)k_col_step<Obj, false>;
+  t.col_step[1] = (const void*)k_col_step<Obj, true>;
+  t.col_decide = (const void*)k_col_decide<Obj>;
   return t;
 }
 

@@ -58,7 +58,7 @@ def _create(n=10, d=10, w=0.9, c1=2.0, c2=2.0, lo=-1.0, hi=1.0, obj=1, seed=1, o
 
 
 @pytest.mark.parametrize("kw,status", [
-    (dict(n=0), 1), (dict(n=2**32), 1), (dict(d=0), 1), (dict(d=65537), 5),
+    (dict(n=0), 1), (dict(n=2**32), 1), (dict(d=0), 1), (dict(d=2**24 + 1), 5),
     (dict(lo=1.0, hi=1.0), 1), (dict(lo=2.0, hi=1.0), 1), (dict(hi=float("inf")), 1),
     (dict(w=float("nan")), 1), (dict(c1=float("inf")), 1), (dict(obj=0), 1), (dict(obj=63), 1),
 ])
@@ -67,6 +67,18 @@ def test_invalid_arguments_return_status(kw, status):
     assert st == status, fp.last_error()
     assert h.value is None  # *out is cleared on failure
     assert fp.last_error()
+
+
+def test_column_split_validation_before_any_device_call():
+    o = _lib.pso_opts()
+    o.device = -1
+    o.flags = fp.PSO_FLAG_COLUMN_SPLIT | _lib.PSO_FLAG_ASYNC_GBEST
+    assert _create(opts=o)[0] == 1 and "ASYNC" in fp.last_error()
+    # rows beyond the row kernels with a particle split: needs the column split
+    o = _lib.pso_opts()
+    o.device = -1
+    o.world, o.rank, o.flags = 2, 0, _lib.PSO_FLAG_DEFER_INIT
+    assert _create(d=65537, opts=o)[0] == 5 and "COLUMN_SPLIT" in fp.last_error()
 
 
 def test_invalid_flags_and_vmax():

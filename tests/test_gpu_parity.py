@@ -100,7 +100,7 @@ def test_init_bitexact(obj, n, d):
 
 
 # ------------------------------------------------------------------ single step
-def _step_and_compare(obj, n, d, seed, pf_mode, t0=0):
+def _step_and_compare(obj, n, d, seed, pf_mode, t0=0, **kw):
     lo, hi = DOMAINS[obj]
     X, V, PB, pf = random_state(n, d, lo, hi, 1.0, seed, pf_mode="inf")
     if pf_mode == "mixed":
@@ -110,7 +110,7 @@ def _step_and_compare(obj, n, d, seed, pf_mode, t0=0):
         rng = np.random.default_rng(seed + 1)
         pf = (probe.f * rng.choice([0.5, 1.5], size=n)).astype(np.float32)
         pf[probe.f < 0] = probe.f[probe.f < 0] * 0.5
-    g = gpu_swarm(n, d, obj, seed=seed).set_state(X, V, PB, pf, t=t0)
+    g = gpu_swarm(n, d, obj, seed=seed, **kw).set_state(X, V, PB, pf, t=t0)
     c = cpu_swarm(n, d, obj, seed=seed, create=False).set_state(X, V, PB, pf, t=t0)
     gf0, gi0, G0 = g.gbest()
     assert gi0 == c.gi and gf0 == c.gf
@@ -587,3 +587,93 @@ def test_async_gbest_single_rank_is_synchronous(monkeypatch):
         g.close()
     finally:
         fp.nccl_comm_destroy(comm)
+
+
+# ------------------------------------------------------------------ column split (NEXT-3)
+def _col_tiles(d):
+    nv = (d + 3) // 4
+    t = min(max((nv + 63) // 64, 32), 512, nv)
+    return -(-nv // t)
+
+
+@pytest.mark.parametrize("obj", OBJS)
+@pytest.mark.parametrize("n,d", [(20, 13), (33, 999), (9, 2049), (6, 5000), (4, 40001)])
+def test_column_split_single_gpu_matches_oracle(obj, n, d):
+    """PSO_FLAG_COLUMN_SPLIT on one GPU: rows cut into column tiles, tile
+    partials combined by k_col_decide.  Init bit-exact; one step from injected
+    state bit-exact in X / V, decisions as the oracle's; pf within tolerance."""
+    g = gpu_swarm(n, d, obj, seed=d + 3 * obj, column_split=True)
+    info = g.info()
+    assert info["column_split"] == 1 and info["col_begin"] == 0 and info["d_local"] == d
+    assert info["col_tiles"] == _col_tiles(d)
+    c = cpu_swarm(n, d, obj, seed=d + 3 * obj)
+    X, V, PB, pf, t = g.get_state()
+    assert t == 0
+    assert_bitwise(X, c.X, "X0")
+    assert_bitwise(V, c.V, "V0")
+    assert_bitwise(PB, c.PB, "PB0")
+    assert_fitness_close(obj, c.X, pf, c.pf, "pf0")
+    gf, gi, G = g.gbest()
+    assert_bitwise(G, PB[gi], "G == PB[gi]")
+    assert gf == pf.min() and gi == int(np.argmin(pf))
+    _step_and_compare(obj, n, d, seed=7000 + d, pf_mode="mixed", t0=3, column_split=True)
+    _step_and_compare(obj, n, d, seed=7100 + d, pf_mode="inf", t0=0, column_split=True)
+
+
+@pytest.mark.parametrize("obj,n,d", [(ROSENBROCK, 5, 9000), (GRIEWANK, 7, 3001),
+                                     (RASTRIGIN, 3, 70001), (ROSENBROCK, 2, 65537)])
+def test_column_split_lockstep_and_wide_rows(obj, n, d):
+    """Several iterations in lockstep with the oracle (the lazy pbest rows of
+    the split: deferred PB copies, materialised by get_state); d > PSO_D_MAX_ROW
+    selects the column split automatically."""
+    kw = {} if d > fp.PSO_D_MAX_ROW else {"column_split": True}
+    g = gpu_swarm(n, d, obj, seed=31, **kw)
+    assert g.info()["column_split"] == 1
+    c = cpu_swarm(n, d, obj, seed=31, create=False)
+    for _ in range(4):
+        X, V, PB, pf, t = g.get_state()
+        c.set_state(X, V, PB, pf, t=t)
+        g.step(1)
+        c.step(1)
+        X2, V2, PB2, pf2, _ = g.get_state()
+        assert_bitwise(X2, c.X, "X")
+        assert_bitwise(V2, c.V, "V")
+        assert_fitness_close(obj, c.PB, pf2, c.pf, "pf")
+        gf, gi, G = g.gbest()
+        assert gf == pf2.min() and gi == int(np.argmin(pf2))
+        assert_bitwise(G, PB2[gi], "G == PB[gi]")
+    info = g.info()
+    assert info["launches"] >= 2 + 2 * 4
+
+
+def test_column_split_with_bounds_lockstep():
+    n, d, obj = 6, 6001, ROSENBROCK
+    b = _dim_bounds(d, 5)
+    lo, hi = DOMAINS[obj]
+    g = fp.Swarm(n, d, 0.9, 2.0, 2.0, lo, hi, obj, 23, device=0, bounds=b, column_split=True)
+    c = orc.OracleSwarm(n, d, 0.9, 2.0, 2.0, lo, hi, obj, 23, bounds=b)
+    X, V, PB, pf, _ = g.get_state()
+    assert_bitwise(X, c.X, "X0")
+    assert_bitwise(V, c.V, "V0")
+    for _ in range(3):
+        X, V, PB, pf, t = g.get_state()
+        c.set_state(X, V, PB, pf, t=t)
+        g.step(1)
+        c.step(1)
+        X2, V2, _, pf2, _ = g.get_state()
+        assert_bitwise(X2, c.X, "X")
+        assert_bitwise(V2, c.V, "V")
+        assert_fitness_close(obj, c.PB, pf2, c.pf, "pf")
+
+
+def test_column_split_end_to_end_c1_gbest():
+    """C1 (Sphere 32 x 10, 100 iterations) through the column split: gbest
+    within relative 1e-4 of the oracle (north_star)."""
+    w = WORKLOADS["C1"]
+    g = fp.Swarm(w.n, w.d, w.w, w.c1, w.c2, w.lo, w.hi, w.objective, w.seed, vmax=w.vmax,
+                 device=0, column_split=True)
+    c = orc.OracleSwarm(w.n, w.d, w.w, w.c1, w.c2, w.lo, w.hi, w.objective, w.seed, vmax=w.vmax)
+    g.step(w.iters)
+    c.step(w.iters)
+    gf, _, _ = g.gbest()
+    assert abs(gf - c.gf) <= 1e-4 * abs(c.gf) + 1e-30
