@@ -258,7 +258,7 @@ def test_errors_do_not_abort():
         gpu_swarm(0, 10, SPHERE)
     assert e.value.status == 1
     with pytest.raises(fp.PsoError) as e:
-        gpu_swarm(10, 70000, SPHERE)
+        gpu_swarm(10, fp.PSO_D_MAX + 1, SPHERE)  # beyond the column split's limit
     assert e.value.status == 5
     g = gpu_swarm(10, 10, SPHERE)
     with pytest.raises(fp.PsoError):
