@@ -603,6 +603,7 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
   A.w = w; A.c1 = c1; A.c2 = c2; A.lo = lo; A.hi = hi; A.vmax = h->vmax;
   A.seed_lo = (unsigned)seed;
   A.seed_hi = (unsigned)(seed >> 32);
+  A.rk.set(seed);
 
   {
     cudaError_t e = cudaMemsetAsync(A.G, 0, gb + ctlb, h->stream);  // G and ctl

@@ -24,6 +24,24 @@ struct DevCtl {
 };
 static_assert(sizeof(DevCtl) == 128, "DevCtl is two 64-byte blocks");
 
+// Philox4x32-10 key schedule of the seed, precomputed on the host (round r:
+// seed_lo + r 0x9E3779B9, seed_hi + r 0xBB67AE85).  Read through a reference
+// to the kernel parameter, every round key is a constant-bank operand of the
+// LOP3 that consumes it instead of a per-call uniform add (philox.cuh).
+struct PhiloxRoundKeys {
+  unsigned int k0[10], k1[10];
+#ifdef __CUDACC__
+  __device__ __forceinline__ unsigned int rk0(int r) const { return k0[r]; }
+  __device__ __forceinline__ unsigned int rk1(int r) const { return k1[r]; }
+#endif
+  void set(unsigned long long seed) {
+    for (int r = 0; r < 10; ++r) {
+      k0[r] = (unsigned)seed + (unsigned)r * 0x9E3779B9u;
+      k1[r] = (unsigned)(seed >> 32) + (unsigned)r * 0xBB67AE85u;
+    }
+  }
+};
+
 // Exchange record for world > 1: the local candidate key and its PB row.
 // Layout: [u64 key][u64 pad][pitch floats].
 __host__ __device__ inline size_t record_bytes(int pitch) { return 16 + (size_t)pitch * 4; }
@@ -66,6 +84,7 @@ struct SwarmArgs {
   int col_nbt;      // tiles per row over all ranks
   float w, c1, c2, lo, hi, vmax;
   unsigned int seed_lo, seed_hi;
+  PhiloxRoundKeys rk;  // the same seed's Philox key schedule
 };
 
 // Column split geometry (host plan and decide kernel).  The tiling depends on

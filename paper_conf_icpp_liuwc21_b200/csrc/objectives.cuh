@@ -14,6 +14,9 @@
 //                                      // j: 0-based dim; xnext valid iff kNeighbor && j+1 < d
 //   __device__ static void  combine(float* a, const float* b);   // associative
 //   __device__ static float finalize(const float* a, int d);
+//   optional:
+//   __device__ static void  map4(float* a, float4 x, float xnext, int j, int d);
+//                                      // == map over dims j..j+3 (all < d), same bits
 //
 // The reduction order is fixed by the launch shape, which depends only on d,
 // so fitness bits do not depend on the grid or on the number of GPUs.
@@ -90,10 +93,27 @@ struct Griewank {
     a[0] = 0.f;
     a[1] = 1.f;
   }
-  __device__ static void map(float* a, float x, float, int j, int) {
+  // k = j + 1 >= 1 is never subnormal, so the flush-to-zero MUFU form is
+  // bitwise rsqrtf (whose non-FTZ form adds a subnormal-input rescale).
+  __device__ static float rsqrt_k(float k) {
+    float r;
+    asm("rsqrt.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(k));
+    return r;
+  }
+  __device__ static void term(float* a, float x, float k) {
     a[0] = fmaf(x, x, a[0]);
-    const float y = x * rsqrtf((float)(j + 1));  // x_k / sqrt(k)
+    const float y = x * rsqrt_k(k);  // x_k / sqrt(k)
     a[1] *= fmaf(-2.f, sinpi_sq(y * kInv2Pi), 1.f);  // cos(y)
+  }
+  __device__ static void map(float* a, float x, float, int j, int) { term(a, x, (float)(j + 1)); }
+  // Four consecutive dims j..j+3 (j + 4 <= d <= 2^24): (float)(j + 1 + m) ==
+  // (float)(j + 1) + m exactly, one conversion instead of four; same bits as map.
+  __device__ static void map4(float* a, float4 x, float, int j, int) {
+    const float k = (float)(j + 1);
+    term(a, x.x, k);
+    term(a, x.y, k + 1.f);
+    term(a, x.z, k + 2.f);
+    term(a, x.w, k + 3.f);
   }
   __device__ static void combine(float* a, const float* b) {
     a[0] += b[0];

@@ -17,25 +17,25 @@ namespace fastpso {
 
 enum : uint32_t { kTagR1 = 0, kTagR2 = 1, kTagX0 = 2, kTagV0 = 3 };
 
+constexpr uint32_t kPhiloxW0 = 0x9E3779B9u, kPhiloxW1 = 0xBB67AE85u;  // Weyl key bumps
+
 struct PhiloxKey {
   uint32_t k0, k1;
+  __device__ __forceinline__ uint32_t rk0(int r) const { return k0 + (uint32_t)r * kPhiloxW0; }
+  __device__ __forceinline__ uint32_t rk1(int r) const { return k1 + (uint32_t)r * kPhiloxW1; }
 };
 
 // Philox4x32-10 (Salmon et al., SC'11): 10 rounds of two 32x32->64 products;
 // the key is bumped by the Weyl constants between rounds.
-__device__ __forceinline__ uint4 philox4x32_10(uint4 c, PhiloxKey key) {
-  uint32_t k0 = key.k0, k1 = key.k1;
+template <class K>
+__device__ __forceinline__ uint4 philox4x32_10(uint4 c, const K& key) {
 #pragma unroll
   for (int r = 0; r < 10; ++r) {
-    if (r > 0) {
-      k0 += 0x9E3779B9u;
-      k1 += 0xBB67AE85u;
-    }
     const uint32_t lo0 = 0xD2511F53u * c.x;
     const uint32_t hi0 = __umulhi(0xD2511F53u, c.x);
     const uint32_t lo1 = 0xCD9E8D57u * c.z;
     const uint32_t hi1 = __umulhi(0xCD9E8D57u, c.z);
-    c = make_uint4(hi1 ^ c.y ^ k0, lo1, hi0 ^ c.w ^ k1, lo0);
+    c = make_uint4(hi1 ^ c.y ^ key.rk0(r), lo1, hi0 ^ c.w ^ key.rk1(r), lo0);
   }
   return c;
 }
@@ -56,13 +56,15 @@ __device__ __forceinline__ float4 raw24x4(uint4 w) {
 }
 
 // m of float4 q (dims 4q..4q+3) of particle i at iteration t.
-__device__ __forceinline__ float4 raw24x4(PhiloxKey key, uint32_t tag, uint32_t t, uint32_t i,
+template <class K>
+__device__ __forceinline__ float4 raw24x4(const K& key, uint32_t tag, uint32_t t, uint32_t i,
                                           uint32_t q) {
   return raw24x4(philox4x32_10(make_uint4(q, i, t, tag), key));
 }
 
 // The 4 uniforms of float4 q (dims 4q..4q+3) of particle i at iteration t.
-__device__ __forceinline__ float4 uniforms4(PhiloxKey key, uint32_t tag, uint32_t t,
+template <class K>
+__device__ __forceinline__ float4 uniforms4(const K& key, uint32_t tag, uint32_t t,
                                             uint32_t i, uint32_t q) {
   return u01x4(philox4x32_10(make_uint4(q, i, t, tag), key));
 }

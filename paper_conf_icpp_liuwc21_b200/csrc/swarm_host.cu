@@ -245,7 +245,8 @@ cudaError_t plan_launch(int objective, int d, long long n_local, int sm_count, c
   // ---- wide rows: thread-block cluster per row
   if (nvec > 2048 || h.cluster > 0) return plan_cluster(tab, nvec, n_local, h, cfg);
   shape_for(nvec, h.vpt, &cfg->vpt, &cfg->compute);
-  const int vi = vpt_index(cfg->vpt), bi = h.bounds ? 1 : 0;
+  int vi = vpt_index(cfg->vpt);
+  const int bi = h.bounds ? 1 : 0;
 
   // ---- resident single-CTA path for tiny swarms (single GPU only)
   if (h.allow_resident && nvec <= 32 && n_local * nvec * 4 <= kResidentElems) {
@@ -267,52 +268,80 @@ cudaError_t plan_launch(int objective, int d, long long n_local, int sm_count, c
     cudaGetLastError();
   }
 
-  // ---- streaming kernels: TMA pipeline for rows of >= 256 dims unless forced
+  // ---- streaming kernels: TMA pipeline for rows of >= 256 dims unless forced.
+  // Shape: (float4 per thread, CTAs per SM) from d only (never from n, so the
+  // per-row reduction order -- and every fitness bit -- is the same for every
+  // swarm size and world size).  Rule (measured, profiles/r01_tune_*): reach
+  // 16 compute warps per SM with >= 3 ring stages per CTA, and among shapes
+  // that do, prefer 2 float4 per thread (the per-row, per-warp bookkeeping --
+  // barrier waits, partial combine, arrivals -- is amortised over 8 elements
+  // per lane instead of 4; C3 Rosenbrock 10k x 1000: 45.8 -> 41.6 us).
   bool tma = h.kernel == 1 || (h.kernel == -1 && nvec >= 64);
   if (tma) {
-    const void* fn = tab->step_tma[vi][bi];
-    const int threads = cfg->compute + 64;  // + producer warp + finaliser warp
-    // CTAs per SM the registers allow, capped at 2; the ring fills the rest.
-    int by_regs = 0;
-    if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&by_regs, fn, threads, 0)) != cudaSuccess)
-      return e;
-    const int cap = (h.ctas >= 1 && h.ctas <= 8) ? h.ctas : 2;
-    int ctas = by_regs < 1 ? 1 : (by_regs > cap ? cap : by_regs);
-    // The most CTAs per SM (<= cap) that still keep >= 3 rows in flight per
-    // CTA; two rows only if nothing else fits (measured: 2-stage rings leave
-    // HBM idle between rows, 3-4 stages saturate it).
-    int c = ctas;
-    for (; c >= 1; --c)
-      if (ring_stages(row + btab, 3 * row, c) >= 3) break;
-    if (c >= 1) {
-      ctas = c;
-    } else {
-      for (c = ctas; c >= 1 && ring_stages(row + btab, 3 * row, c) < 2; --c) {
+    static const int kPref[] = {2, 1, 4, 8};
+    const int cap = (h.ctas >= 1 && h.ctas <= 8) ? h.ctas : 8;
+    int best_v = 0, best_c = 0, best_stages = 0, best_threads = 0, best_score = -1;
+    for (int v : kPref) {
+      if (h.vpt && v != h.vpt) continue;
+      const int t = (nvec + v - 1) / v;
+      if (t > kMaxThreads && v != 8) continue;
+      const int compute = ((t < kMaxThreads ? t : kMaxThreads) + 31) / 32 * 32;
+      const void* fn = tab->step_tma[vpt_index(v)][bi];
+      int by_regs = 0;
+      if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&by_regs, fn, compute + 64, 0)) !=
+          cudaSuccess)
+        return e;
+      int hi = by_regs < cap ? by_regs : cap;
+      // fewest CTAs that reach 16 compute warps, else as many as fit
+      const int want = (16 * 32 + compute - 1) / compute;
+      if (hi > want) hi = want;
+      int c = hi;
+      for (; c >= 1; --c)
+        if (ring_stages(row + btab, 3 * row, c) >= 3) break;
+      if (c < 1)  // two rows in flight only if nothing else fits
+        for (c = hi; c >= 1 && ring_stages(row + btab, 3 * row, c) < 2; --c) {
+        }
+      if (c < 1) continue;
+      const int warps = c * compute / 32;
+      const int score = warps < 16 ? warps : 16;
+      if (score > best_score) {
+        best_score = score;
+        best_v = v;
+        best_c = c;
+        best_threads = compute;
+        best_stages = ring_stages(row + btab, 3 * row, c);
       }
-      ctas = c < 1 ? 1 : c;
     }
-    int stages = ring_stages(row + btab, 3 * row, ctas);
-    if (h.stages >= 2 && h.stages <= kMaxStages) stages = stages < h.stages ? stages : h.stages;
-    if (stages > kMaxStages) stages = kMaxStages;
     tma = false;
-    if (stages >= 2) {
-      const size_t smem = row + btab + (size_t)stages * 3 * row;
-      if ((e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem)) !=
-          cudaSuccess)
-        return e;
-      int per_sm = 0;
-      if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, threads, smem)) !=
-          cudaSuccess)
-        return e;
-      if (per_sm >= 1) {
-        tma = true;
-        cfg->tma = 1;
-        cfg->stages = stages;
-        cfg->threads = threads;
-        cfg->smem = smem;
-        cfg->ctas_per_sm = per_sm;
+    if (best_score > 0) {
+      cfg->vpt = best_v;
+      cfg->compute = best_threads;
+      vi = vpt_index(best_v);
+      int stages = best_stages;
+      if (h.stages >= 2 && h.stages <= kMaxStages) stages = stages < h.stages ? stages : h.stages;
+      if (stages > kMaxStages) stages = kMaxStages;
+      const void* fn = tab->step_tma[vi][bi];
+      const int threads = cfg->compute + 64;  // + producer warp + finaliser warp
+      if (stages >= 2) {
+        const size_t smem = row + btab + (size_t)stages * 3 * row;
+        if ((e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem)) !=
+            cudaSuccess)
+          return e;
+        int per_sm = 0;
+        if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, threads, smem)) !=
+            cudaSuccess)
+          return e;
+        if (per_sm >= 1) {
+          tma = true;
+          cfg->tma = 1;
+          cfg->stages = stages;
+          cfg->threads = threads;
+          cfg->smem = smem;
+          cfg->ctas_per_sm = per_sm < best_c ? per_sm : best_c;
+        }
       }
     }
+    if (!tma) shape_for(nvec, h.vpt, &cfg->vpt, &cfg->compute), vi = vpt_index(cfg->vpt);
   }
   if (!tma) {
     const void* fn = tab->step_reg[vi][bi];
@@ -337,7 +366,7 @@ cudaError_t plan_launch(int objective, int d, long long n_local, int sm_count, c
   // ---- grid-resident path: the whole swarm in the grid's shared memory
   if (h.allow_resident && !cfg->resident && cfg->tma && nvec >= 64) {
     const void* fn = tab->gridres[vi][bi];
-    for (int per = 2; per >= 1 && !cfg->gridres; --per) {
+    for (int per = cfg->ctas_per_sm; per >= 1 && !cfg->gridres; --per) {
       long long g = (long long)per * sm_count;
       if (g > n_local) g = n_local;
       const long long rows = (n_local + g - 1) / g;
