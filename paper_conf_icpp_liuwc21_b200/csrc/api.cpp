@@ -539,6 +539,8 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
       return bail(fail(PSO_ERR_UNSUPPORTED, "no launch shape fits d=%d with the requested hints", d));
     }
     if (e != cudaSuccess) return bail(cuda_fail(nullptr, e, "plan_launch"));
+    const char* pdl = std::getenv("PSO_PDL");
+    h->cfg.pdl = (pdl && *pdl == '0') ? 0 : 1;
   }
 
   // ---- one arena: X, V, PB, pf, G, ctl, exchange records
@@ -673,10 +675,21 @@ pso_status pso_step(pso_handle h, int64_t iters) {
     h->t += (uint64_t)iters;
     return PSO_OK;
   }
+  // With programmatic dependent launch the step kernels of consecutive
+  // iterations overlap launch and drain, so an event between two of them would
+  // serialise the pair: time the whole back-to-back run of the call instead
+  // (per-launch average = its duration / iters).  A host-side exchange (NCCL)
+  // sits between the launches anyway, so there every launch is timed alone.
+  const bool per_call = timing && h->cfg.pdl && h->n_local > 0 && !(h->xchg && !h->args.p2p);
+  pso_swarm::Timed* call_ev = nullptr;
+  if (per_call) {
+    if ((st = next_event(h, &call_ev, (uint64_t)iters)) != PSO_OK) return st;
+    PSO_CUDA(h, cudaEventRecord(call_ev->start, h->stream));
+  }
   for (int64_t it = 0; it < iters; ++it) {
     if (h->n_local > 0) {
       pso_swarm::Timed* ev = nullptr;
-      if (timing && (st = next_event(h, &ev, 1)) != PSO_OK) return st;
+      if (timing && !per_call && (st = next_event(h, &ev, 1)) != PSO_OK) return st;
       if (ev) PSO_CUDA(h, cudaEventRecord(ev->start, h->stream));
       PSO_CUDA(h, launch_step(h->objective, h->args, h->cfg, h->stream));
       ++h->launches;
@@ -684,6 +697,7 @@ pso_status pso_step(pso_handle h, int64_t iters) {
     }
     if ((st = exchange(h, h->t + (uint64_t)it + 1, it + 1 == iters, false)) != PSO_OK) return st;
   }
+  if (call_ev) PSO_CUDA(h, cudaEventRecord(call_ev->stop, h->stream));
   h->t += (uint64_t)iters;
   return PSO_OK;
 }

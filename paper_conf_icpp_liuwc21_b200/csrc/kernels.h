@@ -135,6 +135,7 @@ struct LaunchCfg {
   size_t resident_smem = 0;
   size_t init_smem = 0;
   int bounds = 0;     // kernels instantiated with per-dimension bounds
+  int pdl = 1;        // step kernels: programmatic dependent launch (PSO_PDL=0 disables)
   int colsplit = 0;   // column split: k_col_step + k_col_decide per iteration
   int col_grid = 0, col_stages = 0, col_decide_grid = 0;
   size_t col_smem = 0, col_decide_smem = 0;

@@ -44,7 +44,7 @@ constexpr int kColCompute = 256;  // compute threads of k_col_step (+ producer +
 
 template <class Obj, bool kB>
 __global__ void __launch_bounds__(kColCompute + 64, 2)
-    k_col_step(const SwarmArgs a, int init, int stages) {
+    k_col_step(const __grid_constant__ SwarmArgs a, int init, int stages) {
   static_assert(Obj::kAcc <= 2, "the tile partial carries two accumulators");
   extern __shared__ __align__(128) unsigned char dsmem[];
   constexpr int nthr = kColCompute, nwarps = nthr / 32;
@@ -174,7 +174,7 @@ __global__ void __launch_bounds__(kColCompute + 64, 2)
   }
 
   // ---------------- compute warps
-  const PhiloxKey key{a.seed_lo, a.seed_hi};
+  const PhiloxRoundKeys& key = a.rk;
   const MoveParams mp = move_params(a);
   const float4* B4 = reinterpret_cast<const float4*>(a.bounds);
   int s = 0;
@@ -247,7 +247,7 @@ __global__ void __launch_bounds__(kColCompute + 64, 2)
 
 // One warp per row.
 template <class Obj>
-__global__ void __launch_bounds__(256) k_col_decide(const SwarmArgs a, int init) {
+__global__ void __launch_bounds__(256) k_col_decide(const __grid_constant__ SwarmArgs a, int init) {
   __shared__ unsigned long long s_best[8];
   __shared__ unsigned s_nimp[8];
   __shared__ int s_last;

@@ -398,26 +398,34 @@ cudaError_t launch_step(int objective, const SwarmArgs& a, const LaunchCfg& c, c
   if (!t) return cudaErrorInvalidDeviceFunction;
   const int vi = vpt_index(c.vpt), bi = c.bounds ? 1 : 0;
   int stages = c.stages;
-  if (c.cluster) {
-    int C = c.cluster, chunk = c.chunk;
-    void* args[] = {const_cast<SwarmArgs*>(&a), &stages, &C, &chunk};
-    cudaLaunchConfig_t lc{};
-    lc.gridDim = dim3(c.grid);
-    lc.blockDim = dim3(c.threads);
-    lc.dynamicSmemBytes = c.smem;
-    lc.stream = s;
-    cudaLaunchAttribute attr[1];
-    attr[0].id = cudaLaunchAttributeClusterDimension;
-    attr[0].val.clusterDim.x = C;
-    attr[0].val.clusterDim.y = 1;
-    attr[0].val.clusterDim.z = 1;
-    lc.attrs = attr;
-    lc.numAttrs = 1;
-    return cudaLaunchKernelExC(&lc, t->step_cluster[vi][bi], args);
+  int C = c.cluster, chunk = c.chunk;
+  void* args[] = {const_cast<SwarmArgs*>(&a), &stages, &C, &chunk};
+  cudaLaunchConfig_t lc{};
+  lc.gridDim = dim3(c.grid);
+  lc.blockDim = dim3(c.threads);
+  lc.dynamicSmemBytes = c.smem;
+  lc.stream = s;
+  cudaLaunchAttribute attr[2];
+  int na = 0;
+  if (c.pdl) {  // overlap this grid's launch with the previous step kernel's drain
+    attr[na].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[na].val.programmaticStreamSerializationAllowed = 1;
+    ++na;
   }
-  const void* fn = c.tma ? t->step_tma[vi][bi] : t->step_reg[vi][bi];
-  void* args[] = {const_cast<SwarmArgs*>(&a), &stages};
-  return cudaLaunchKernel(fn, dim3(c.grid), dim3(c.threads), args, c.smem, s);
+  const void* fn;
+  if (c.cluster) {
+    attr[na].id = cudaLaunchAttributeClusterDimension;
+    attr[na].val.clusterDim.x = C;
+    attr[na].val.clusterDim.y = 1;
+    attr[na].val.clusterDim.z = 1;
+    ++na;
+    fn = t->step_cluster[vi][bi];
+  } else {
+    fn = c.tma ? t->step_tma[vi][bi] : t->step_reg[vi][bi];
+  }
+  lc.attrs = attr;
+  lc.numAttrs = na;
+  return cudaLaunchKernelExC(&lc, fn, args);
 }
 
 cudaError_t launch_resident(int objective, const SwarmArgs& a, const LaunchCfg& c, int iters,

@@ -76,6 +76,17 @@ __device__ __forceinline__ void team_sync(int n) {
   asm volatile("bar.sync 1, %0;" ::"r"(n) : "memory");
 }
 
+// --- programmatic dependent launch (PDL): consecutive step kernels of one
+// stream are launched with programmatic stream serialization, so the next
+// iteration's grid is scheduled while this one drains; every global read of
+// the next kernel sits behind griddepcontrol.wait (the previous grid has
+// completed and its writes are visible).  Without the launch attribute both
+// are no-ops.
+__device__ __forceinline__ void pdl_wait_and_release() {
+  asm volatile("griddepcontrol.wait;" ::: "memory");
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+}
+
 // --- mbarrier + bulk async copy global -> shared (TMA engine) -------------
 __device__ __forceinline__ uint32_t smem_addr(const void* p) {
   return (uint32_t)__cvta_generic_to_shared(p);
@@ -628,13 +639,14 @@ __device__ __forceinline__ void row_bookkeeping(const SwarmArgs& a, long long r,
 // ------------------------------------------------- step kernel: registers
 template <class Obj, int VPT, bool kB>
 __global__ void __launch_bounds__(kMaxThreads, (VPT >= 8) ? 1 : 2)
-    k_step_reg(const SwarmArgs a, int /*stages: unused, same signature as k_step_tma*/) {
+    k_step_reg(const __grid_constant__ SwarmArgs a, int /*stages: unused, same signature as k_step_tma*/) {
   extern __shared__ __align__(128) unsigned char dsmem[];
   float4* sG = reinterpret_cast<float4*>(dsmem);
   float4* sB = sG + a.nvec;  // kB: [vlo | vhi | xlo | xhi]
   float* sFirst = reinterpret_cast<float*>(sB + (kB ? 4 * a.nvec : 0));
   __shared__ RowSmem<Obj> sm;
   const int tid = threadIdx.x, nthr = blockDim.x;
+  pdl_wait_and_release();
   const uint32_t t = a.ctl->t + 1u;
   if (tid == 0) {
     const unsigned row_bytes = (unsigned)a.nvec * 16u;
@@ -653,7 +665,7 @@ __global__ void __launch_bounds__(kMaxThreads, (VPT >= 8) ? 1 : 2)
   }
   __syncthreads();
   const uint32_t inc_ord = (uint32_t)(sm.inc >> 32);
-  const PhiloxKey key{a.seed_lo, a.seed_hi};
+  const PhiloxRoundKeys& key = a.rk;
   const MoveParams mp = move_params(a);
   const int nvec = a.nvec;
   mbar_wait(&sm.gbar, 0);
@@ -737,6 +749,7 @@ __global__ void __launch_bounds__(kMaxThreads + 64, 2)
     mbar_fence_init();
   }
   __syncthreads();
+  pdl_wait_and_release();
   const uint32_t t = a.ctl->t + 1u;
   const unsigned row_bytes = (unsigned)nvec * 16u;
 
@@ -930,7 +943,7 @@ __global__ void __launch_bounds__(kMaxThreads + 64, 2)
 // back to every CTA, which then bulk-stores its block of x', v' (and pb).
 template <class Obj, int VPT, bool kB>
 __global__ void __launch_bounds__(kMaxThreadsCluster + 64, 1)
-    k_step_cluster(const SwarmArgs a, int stages, int C, int chunk) {
+    k_step_cluster(const __grid_constant__ SwarmArgs a, int stages, int C, int chunk) {
   extern __shared__ __align__(128) unsigned char dsmem[];
   constexpr int kSlot = Obj::kAcc + 2;  // partial accumulators, first x', last x'
   const int nvec = a.nvec, d = a.d;
@@ -968,6 +981,7 @@ __global__ void __launch_bounds__(kMaxThreadsCluster + 64, 1)
   }
   __syncthreads();
   cluster_sync_all();  // every CTA's barriers exist before any remote arrival
+  pdl_wait_and_release();
   const uint32_t t = a.ctl->t + 1u;
   const unsigned blk_bytes = (unsigned)cnt * 16u;
 
@@ -1121,7 +1135,7 @@ __global__ void __launch_bounds__(kMaxThreadsCluster + 64, 1)
   }
 
   // ---------------- compute warps
-  const PhiloxKey key{a.seed_lo, a.seed_hi};
+  const PhiloxRoundKeys& key = a.rk;
   const MoveParams mp = move_params(a);
   mbar_wait(&gbar, 0);
   int s = 0;
@@ -1202,7 +1216,7 @@ __global__ void __launch_bounds__(kMaxThreadsCluster + 64, 1)
 // steps only add the identities of idle lanes), so fitness, decisions and
 // state are bitwise those of the streaming kernels.
 template <class Obj, bool kB>
-__global__ void __launch_bounds__(1024, 1) k_resident(const SwarmArgs a, int iters) {
+__global__ void __launch_bounds__(1024, 1) k_resident(const __grid_constant__ SwarmArgs a, int iters) {
   extern __shared__ __align__(16) unsigned char dsmem[];
   const int nvec = a.nvec, d = a.d;
   const int n = (int)a.n_local;
@@ -1241,7 +1255,7 @@ __global__ void __launch_bounds__(1024, 1) k_resident(const SwarmArgs a, int ite
     s_imp = 0;
   }
   __syncthreads();
-  const PhiloxKey key{a.seed_lo, a.seed_hi};
+  const PhiloxRoundKeys& key = a.rk;
   const MoveParams mp = move_params(a);
   unsigned long long cur = cur0;
   for (int it = 0; it < iters; ++it) {
@@ -1358,7 +1372,7 @@ __device__ __forceinline__ unsigned ld_acquire_u32(const unsigned* p) {
 }
 
 template <class Obj, int VPT, bool kB>
-__global__ void __launch_bounds__(kMaxThreads, 1) k_gridres(const SwarmArgs a, int iters) {
+__global__ void __launch_bounds__(kMaxThreads, 1) k_gridres(const __grid_constant__ SwarmArgs a, int iters) {
   extern __shared__ __align__(16) unsigned char dsmem[];
   const int nvec = a.nvec, d = a.d;
   const int nthr = blockDim.x, tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -1397,7 +1411,7 @@ __global__ void __launch_bounds__(kMaxThreads, 1) k_gridres(const SwarmArgs a, i
   const uint32_t t0 = a.ctl->t;
   __syncthreads();
 
-  const PhiloxKey key{a.seed_lo, a.seed_hi};
+  const PhiloxRoundKeys& key = a.rk;
   const MoveParams mp = move_params(a);
   unsigned long long cur = cur0;
   unsigned nimp = 0;
@@ -1555,7 +1569,8 @@ __global__ void __launch_bounds__(kMaxThreads, 1) k_gridres(const SwarmArgs a, i
 // init_float4_at: dims 4 qg .. 4 qg + 3 of the row (qg: global float4 index,
 // the Philox counter and the padding test), bounds from float4 qb of a table
 // with `bstride` float4 per array (the column split keeps only its block).
-__device__ __forceinline__ void init_float4_at(const SwarmArgs& a, PhiloxKey key, uint32_t gi,
+template <class K>
+__device__ __forceinline__ void init_float4_at(const SwarmArgs& a, const K& key, uint32_t gi,
                                                int qg, const float4* B4, int bstride, int qb,
                                                float4& xo, float4& vo) {
   const int q = qg, d = a.d;
@@ -1587,17 +1602,18 @@ __device__ __forceinline__ void init_float4_at(const SwarmArgs& a, PhiloxKey key
   xo = make_float4(xs[0], xs[1], xs[2], xs[3]);
   vo = make_float4(vs[0], vs[1], vs[2], vs[3]);
 }
-__device__ __forceinline__ void init_float4(const SwarmArgs& a, PhiloxKey key, uint32_t gi, int q,
+template <class K>
+__device__ __forceinline__ void init_float4(const SwarmArgs& a, const K& key, uint32_t gi, int q,
                                             float4& xo, float4& vo) {
   init_float4_at(a, key, gi, q, reinterpret_cast<const float4*>(a.bounds), a.nvec, q, xo, vo);
 }
 
 template <class Obj, int VPT>
 __global__ void __launch_bounds__(kMaxThreads, (VPT >= 8) ? 1 : 2)
-    k_init(const SwarmArgs a) {
+    k_init(const __grid_constant__ SwarmArgs a) {
   __shared__ RowSmem<Obj> sm;
   const int tid = threadIdx.x, nthr = blockDim.x;
-  const PhiloxKey key{a.seed_lo, a.seed_hi};
+  const PhiloxRoundKeys& key = a.rk;
   const int nvec = a.nvec, d = a.d;
   const uint32_t inc_ord = (uint32_t)(a.ctl->key_cur >> 32);
   unsigned long long best = ~0ull;
