@@ -120,6 +120,7 @@ struct LaunchCfg {
   int grid = 1;       // persistent grid
   int ctas_per_sm = 1;
   int tma = 0;        // 1: warp-specialised bulk-copy (TMA) pipeline; 0: register streaming
+  int wide = 0;       // TMA pipeline: the 512-compute-thread instantiation
   int stages = 0;     // TMA pipeline depth (rows in flight per CTA)
   size_t smem = 0;    // dynamic shared memory bytes of the step kernel
   int resident = 0;   // 1: tiny swarm, whole pso_step in one single-CTA launch
@@ -157,6 +158,7 @@ struct KernelTable {
   bool neighbor;
   const void* step_reg[4][2];
   const void* step_tma[4][2];
+  const void* step_tma_w[4][2];  // 512 compute threads, one CTA per SM (VPT 2 and 4 only)
   const void* gridres[4][2];
   const void* step_cluster[4][2];
   const void* resident[2];

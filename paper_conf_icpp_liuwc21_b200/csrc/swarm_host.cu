@@ -278,15 +278,20 @@ cudaError_t plan_launch(int objective, int d, long long n_local, int sm_count, c
   // per lane instead of 4; C3 Rosenbrock 10k x 1000: 45.8 -> 41.6 us).
   bool tma = h.kernel == 1 || (h.kernel == -1 && nvec >= 64);
   if (tma) {
-    static const int kPref[] = {2, 1, 4, 8};
+    // (float4 per thread, max compute threads) in order of preference; the
+    // 512-thread (wide) instantiations exist for VPT 2 and 4
+    static const int kPref[][2] = {{2, 256}, {1, 256}, {2, 512}, {4, 256}, {4, 512}, {8, 256}};
     const int cap = (h.ctas >= 1 && h.ctas <= 8) ? h.ctas : 8;
-    int best_v = 0, best_c = 0, best_stages = 0, best_threads = 0, best_score = -1;
-    for (int v : kPref) {
+    int best_v = 0, best_c = 0, best_stages = 0, best_threads = 0, best_score = -1, best_wide = 0;
+    for (const auto& pr : kPref) {
+      const int v = pr[0], maxt = pr[1];
       if (h.vpt && v != h.vpt) continue;
       const int t = (nvec + v - 1) / v;
-      if (t > kMaxThreads && v != 8) continue;
-      const int compute = ((t < kMaxThreads ? t : kMaxThreads) + 31) / 32 * 32;
-      const void* fn = tab->step_tma[vpt_index(v)][bi];
+      if (t > maxt && v != 8) continue;
+      if (maxt > kMaxThreads && t <= kMaxThreads) continue;  // the narrow variant covers it
+      const int compute = ((t < maxt ? t : maxt) + 31) / 32 * 32;
+      const void* fn = maxt > kMaxThreads ? tab->step_tma_w[vpt_index(v)][bi]
+                                          : tab->step_tma[vpt_index(v)][bi];
       int by_regs = 0;
       if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&by_regs, fn, compute + 64, 0)) !=
           cudaSuccess)
@@ -310,6 +315,7 @@ cudaError_t plan_launch(int objective, int d, long long n_local, int sm_count, c
         best_c = c;
         best_threads = compute;
         best_stages = ring_stages(row + btab, 3 * row, c);
+        best_wide = maxt > kMaxThreads ? 1 : 0;
       }
     }
     tma = false;
@@ -320,7 +326,7 @@ cudaError_t plan_launch(int objective, int d, long long n_local, int sm_count, c
       int stages = best_stages;
       if (h.stages >= 2 && h.stages <= kMaxStages) stages = stages < h.stages ? stages : h.stages;
       if (stages > kMaxStages) stages = kMaxStages;
-      const void* fn = tab->step_tma[vi][bi];
+      const void* fn = best_wide ? tab->step_tma_w[vi][bi] : tab->step_tma[vi][bi];
       const int threads = cfg->compute + 64;  // + producer warp + finaliser warp
       if (stages >= 2) {
         const size_t smem = row + btab + (size_t)stages * 3 * row;
@@ -334,6 +340,7 @@ cudaError_t plan_launch(int objective, int d, long long n_local, int sm_count, c
         if (per_sm >= 1) {
           tma = true;
           cfg->tma = 1;
+          cfg->wide = best_wide;
           cfg->stages = stages;
           cfg->threads = threads;
           cfg->smem = smem;
@@ -346,6 +353,7 @@ cudaError_t plan_launch(int objective, int d, long long n_local, int sm_count, c
   if (!tma) {
     const void* fn = tab->step_reg[vi][bi];
     cfg->tma = 0;
+    cfg->wide = 0;
     cfg->stages = 0;
     cfg->threads = cfg->compute;
     cfg->smem = row + btab + first;
@@ -421,7 +429,7 @@ cudaError_t launch_step(int objective, const SwarmArgs& a, const LaunchCfg& c, c
     ++na;
     fn = t->step_cluster[vi][bi];
   } else {
-    fn = c.tma ? t->step_tma[vi][bi] : t->step_reg[vi][bi];
+    fn = !c.tma ? t->step_reg[vi][bi] : c.wide ? t->step_tma_w[vi][bi] : t->step_tma[vi][bi];
   }
   lc.attrs = attr;
   lc.numAttrs = na;

@@ -44,6 +44,7 @@ namespace {
 
 constexpr int kMaxThreads = 256;         // compute threads per CTA
 constexpr int kMaxThreadsCluster = 512;  // compute threads per CTA of the cluster kernel
+constexpr int kMaxThreadsWide = 512;     // compute threads per CTA of the wide TMA variant
 constexpr int kMaxStages = 8;
 constexpr unsigned kFull = 0xFFFFFFFFu;
 
@@ -723,8 +724,11 @@ __global__ void __launch_bounds__(kMaxThreads, (VPT >= 8) ? 1 : 2)
 //                 bulk stores have read it (wait_group.read).
 // Barriers per stage: full (1 arrival + tx bytes), done (W arrivals), empty (1).
 // Shared memory: [G: nvec float4][stages x {x, v, pb}: nvec float4 each].
-template <class Obj, int VPT, bool kB>
-__global__ void __launch_bounds__(kMaxThreads + 64, 2)
+// kMaxT: compute threads the instantiation is built for -- 256 (two CTAs per
+// SM) or 512 (the wide variant: one CTA of 16 compute warps per SM, for rows
+// of 513-2048 float4 whose stages do not fit twice).
+template <class Obj, int VPT, bool kB, int kMaxT = kMaxThreads>
+__global__ void __launch_bounds__(kMaxT + 64, kMaxT > kMaxThreads ? 1 : 2)
     k_step_tma(const __grid_constant__ SwarmArgs a, int stages) {
   extern __shared__ __align__(128) unsigned char dsmem[];
   const int nvec = a.nvec, d = a.d;
@@ -733,7 +737,7 @@ __global__ void __launch_bounds__(kMaxThreads + 64, 2)
   float4* sG = reinterpret_cast<float4*>(dsmem);
   float4* sB = sG + nvec;  // kB: [vlo | vhi | xlo | xhi]
   float4* ring = sB + (kB ? 4 * nvec : 0);
-  __shared__ float red[kMaxStages][(kMaxThreads / 32) * 2];
+  __shared__ float red[kMaxStages][(kMaxT / 32) * 2];
   __shared__ unsigned long long full[kMaxStages], empty[kMaxStages], done[kMaxStages], gbar;
   __shared__ unsigned long long s_inc;  // incumbent of this iteration (after the exchange merge)
   __shared__ int s_src;
@@ -1372,7 +1376,7 @@ __device__ __forceinline__ unsigned ld_acquire_u32(const unsigned* p) {
 }
 
 template <class Obj, int VPT, bool kB>
-__global__ void __launch_bounds__(kMaxThreads, 1) k_gridres(const __grid_constant__ SwarmArgs a, int iters) {
+__global__ void __launch_bounds__(kMaxThreadsWide, 1) k_gridres(const __grid_constant__ SwarmArgs a, int iters) {
   extern __shared__ __align__(16) unsigned char dsmem[];
   const int nvec = a.nvec, d = a.d;
   const int nthr = blockDim.x, tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -1384,7 +1388,7 @@ __global__ void __launch_bounds__(kMaxThreads, 1) k_gridres(const __grid_constan
   float4* sB = sG + nvec;                          // kB: [vlo | vhi | xlo | xhi]
   float4* sRows = sB + (kB ? 4 * nvec : 0);        // [myrows][3][nvec]
   float* spf = reinterpret_cast<float*>(sRows + (size_t)myrows * 3 * nvec);
-  __shared__ float red[(kMaxThreads / 32) * 2];
+  __shared__ float red[(kMaxThreadsWide / 32) * 2];
   __shared__ float s_f;
   __shared__ int s_imp;
   __shared__ unsigned long long s_best;
@@ -1689,6 +1693,10 @@ KernelTable make_kernel_table() {
 #define PSO_ALLV(ARR, KER) PSO_T(ARR, KER, 1, 0) PSO_T(ARR, KER, 2, 1) PSO_T(ARR, KER, 4, 2) PSO_T(ARR, KER, 8, 3)
   PSO_ALLV(step_reg, k_step_reg)
   PSO_ALLV(step_tma, k_step_tma)
+  t.step_tma_w[1][0] = (const void*)k_step_tma<Obj, 2, false, kMaxThreadsWide>;
+  t.step_tma_w[1][1] = (const void*)k_step_tma<Obj, 2, true, kMaxThreadsWide>;
+  t.step_tma_w[2][0] = (const void*)k_step_tma<Obj, 4, false, kMaxThreadsWide>;
+  t.step_tma_w[2][1] = (const void*)k_step_tma<Obj, 4, true, kMaxThreadsWide>;
   PSO_ALLV(gridres, k_gridres)
   PSO_ALLV(step_cluster, k_step_cluster)
 #undef PSO_ALLV
