@@ -238,7 +238,6 @@ pso_status reset_ctl(pso_swarm* h, uint32_t t) {
   c.improvements = 0;
   c.done = 0;
   c.t = t;
-  c.key_par[0] = c.key_par[1] = ~0ull;
   c.bar_count = 0;
   h->args.t_base = t;  // async merges never reach back past the re-selection
   // improvements are preserved across set_state: read-modify-write
@@ -556,7 +555,9 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
                     (h->cfg.tma && !h->cfg.resident && !h->cfg.gridres && !(lz && *lz == '0'));
   const size_t pbxb = lazy ? align_up(rows, 256) : 0;
   const size_t rec = align_up(record_bytes(h->pitch), 256);
-  const size_t candb = h->cfg.gridres ? align_up(2 * (size_t)h->cfg.gridres_grid * h->pitch * 4, 256) : 0;
+  // grid-resident kernel: [2 parities][grid] candidate rows, then their keys
+  const size_t cand_rows = h->cfg.gridres ? align_up(2 * (size_t)h->cfg.gridres_grid * h->pitch * 4, 256) : 0;
+  const size_t candb = h->cfg.gridres ? cand_rows + align_up(2 * (size_t)h->cfg.gridres_grid * 8, 256) : 0;
   const size_t sendb = (h->xchg && !colsplit) ? rec : 0;
   const size_t recvb = colsplit ? col_tag_bytes(h->world) + 2 * rows * (size_t)col_nbt * 16
                        : h->xchg ? 4 * (size_t)h->world * record_bytes(h->pitch) : 0;
@@ -583,7 +584,9 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
   A.bounds = o.bounds ? (const float*)p : nullptr; p += boundb;
   A.pbx = lazy ? p : nullptr; p += pbxb;
   A.lazy_pb = lazy ? 1 : 0;
-  A.cand = h->cfg.gridres ? (float*)p : nullptr; p += candb;
+  A.cand = h->cfg.gridres ? (float*)p : nullptr;
+  A.cand_key = h->cfg.gridres ? (unsigned long long*)(p + cand_rows) : nullptr;
+  p += candb;
   A.G_view = async ? (float*)p : nullptr; p += viewb;
   A.async_gbest = async ? 1 : 0;
   A.send = sendb ? p : nullptr; p += sendb;

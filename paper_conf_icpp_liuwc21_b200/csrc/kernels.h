@@ -15,7 +15,7 @@ struct DevCtl {
   unsigned long long improvements;  // pbest improvements, summed
   unsigned int done;                // last-CTA ticket counter
   unsigned int t;                   // iterations done (low 32 bits; Philox ctr[2])
-  unsigned long long key_par[2];    // grid-resident kernel: per-iteration-parity accumulators
+  unsigned long long key_par[2];    // unused (the grid-resident kernel keeps per-CTA keys in cand_key)
   unsigned int bar_count, bar_gen;  // grid-resident kernel: grid barrier
   unsigned long long pb_loads;      // streaming kernels: pbest rows read from HBM
   unsigned long long pb_stores;     // streaming kernels: pbest rows written to HBM
@@ -53,6 +53,7 @@ struct SwarmArgs {
   float* pf;  // n_local
   float* G;   // pitch (gbest position)
   float* cand;                // grid-resident kernel: [2][grid][pitch] candidate rows
+  unsigned long long* cand_key;  // grid-resident kernel: [2][grid] candidate keys (~0: none)
   const float* bounds;        // per-dimension bounds [vlo | vhi | xlo | xhi] (4 x pitch), or null
   unsigned char* pbx;         // lazy pbest: 1 = the row's PB equals its X (PB not stored)
   int lazy_pb;

@@ -258,6 +258,47 @@ __device__ __forceinline__ void move4(const MoveParams& m, float4& x, float4& v,
   }
 }
 
+// Eq. 1 split at the gbest term, for work that overlaps the gbest exchange:
+// the pre part (ab = w v + (c1 r1)(pb - x)) needs no gbest, the post part
+// adds (c2 r2)(g - x), clamps and moves.  pre then post is move1 / move1b
+// operation for operation (same roundings, same order).
+__device__ __forceinline__ float move_pre1(const MoveParams& m, float x, float v, float pb, float m1) {
+  return __fadd_rn(__fmul_rn(m.w, v), __fmul_rn(__fmul_rn(m.c1s, m1), __fsub_rn(pb, x)));
+}
+template <bool kB>
+__device__ __forceinline__ void move_pre4(const MoveParams& m, const float4& x, const float4& v,
+                                          const float4& pb, const float4& r1, float4& ab) {
+  ab.x = move_pre1(m, x.x, v.x, pb.x, r1.x);
+  ab.y = move_pre1(m, x.y, v.y, pb.y, r1.y);
+  ab.z = move_pre1(m, x.z, v.z, pb.z, r1.z);
+  ab.w = move_pre1(m, x.w, v.w, pb.w, r1.w);
+}
+__device__ __forceinline__ void move_post1(const MoveParams& m, float& x, float& v, float g, float m2,
+                                           float ab, float vlo, float vhi, float xlo, float xhi) {
+  const float c = __fmul_rn(__fmul_rn(m.c2s, m2), __fsub_rn(g, x));
+  float vn = __fadd_rn(ab, c);
+  vn = fminf(fmaxf(vn, vlo), vhi);
+  x = fminf(fmaxf(__fadd_rn(x, vn), xlo), xhi);
+  v = vn;
+}
+template <bool kB>
+__device__ __forceinline__ void move_post4(const MoveParams& m, float4& x, float4& v, const float4& g,
+                                           const float4& r2, const float4& ab, const float4* sB,
+                                           int nvec, int q) {
+  if constexpr (kB) {
+    const float4 vlo = sB[q], vhi = sB[nvec + q], xlo = sB[2 * nvec + q], xhi = sB[3 * nvec + q];
+    move_post1(m, x.x, v.x, g.x, r2.x, ab.x, vlo.x, vhi.x, xlo.x, xhi.x);
+    move_post1(m, x.y, v.y, g.y, r2.y, ab.y, vlo.y, vhi.y, xlo.y, xhi.y);
+    move_post1(m, x.z, v.z, g.z, r2.z, ab.z, vlo.z, vhi.z, xlo.z, xhi.z);
+    move_post1(m, x.w, v.w, g.w, r2.w, ab.w, vlo.w, vhi.w, xlo.w, xhi.w);
+  } else {
+    move_post1(m, x.x, v.x, g.x, r2.x, ab.x, -m.vmax, m.vmax, m.lo, m.hi);
+    move_post1(m, x.y, v.y, g.y, r2.y, ab.y, -m.vmax, m.vmax, m.lo, m.hi);
+    move_post1(m, x.z, v.z, g.z, r2.z, ab.z, -m.vmax, m.vmax, m.lo, m.hi);
+    move_post1(m, x.w, v.w, g.w, r2.w, ab.w, -m.vmax, m.vmax, m.lo, m.hi);
+  }
+}
+
 // --- CTA reduction of the functor accumulators -----------------------------
 template <class Obj>
 __device__ __forceinline__ void warp_combine(float* a) {
@@ -1364,15 +1405,24 @@ __global__ void __launch_bounds__(1024, 1) k_resident(const __grid_constant__ Sw
 // no row data through L2/HBM at all.  Per row the arithmetic and the
 // reduction order are k_step_tma's (thread-sequential over its float4s, warp
 // butterfly, warps combined in index order by one thread), so results are
-// bitwise those of the streaming kernel.  Per iteration: each CTA publishes
-// its best candidate row to cand[parity][cta] and its key to key_par[parity];
-// a grid barrier (atomic ticket + generation flag; the last CTA resets the
-// other parity's accumulator); then every CTA pulls the winner's row into its
+// bitwise those of the streaming kernel (rows are processed in pairs, each
+// with its own accumulators).  Per iteration: each CTA publishes its best
+// candidate row to cand[parity][cta] and its key to cand_key[parity][cta]; a
+// grid barrier (acq_rel atomic ticket + release of a generation flag); then
+// every CTA folds all keys itself and pulls the winner's row into its
 // shared-memory G.
 __device__ __forceinline__ unsigned ld_acquire_u32(const unsigned* p) {
   unsigned v;
   asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
   return v;
+}
+__device__ __forceinline__ void st_release_u32(unsigned* p, unsigned v) {
+  asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ unsigned atom_add_acq_rel_u32(unsigned* p, unsigned v) {
+  unsigned o;
+  asm volatile("atom.acq_rel.gpu.global.add.u32 %0, [%1], %2;" : "=r"(o) : "l"(p), "r"(v) : "memory");
+  return o;
 }
 
 template <class Obj, int VPT, bool kB>
@@ -1388,11 +1438,12 @@ __global__ void __launch_bounds__(kMaxThreadsWide, 1) k_gridres(const __grid_con
   float4* sB = sG + nvec;                          // kB: [vlo | vhi | xlo | xhi]
   float4* sRows = sB + (kB ? 4 * nvec : 0);        // [myrows][3][nvec]
   float* spf = reinterpret_cast<float*>(sRows + (size_t)myrows * 3 * nvec);
-  __shared__ float red[(kMaxThreadsWide / 32) * 2];
-  __shared__ float s_f;
-  __shared__ int s_imp;
+  __shared__ float red[2 * (kMaxThreadsWide / 32) * 2];  // [row of the pair][warp][acc]
+  __shared__ float s_f2[2];
+  __shared__ int s_imp2[2];
   __shared__ unsigned long long s_best;
   __shared__ int s_best_row;
+  __shared__ unsigned long long s_kmin[kMaxThreadsWide / 32];
 
   // ---- load this CTA's rows and G
   for (int k = 0; k < myrows; ++k) {
@@ -1419,83 +1470,136 @@ __global__ void __launch_bounds__(kMaxThreadsWide, 1) k_gridres(const __grid_con
   const MoveParams mp = move_params(a);
   unsigned long long cur = cur0;
   unsigned nimp = 0;
+  unsigned long long* ckey = a.cand_key;  // [2 parities][grid] candidate keys
+  const unsigned gen0 = ld_acquire_u32(&a.ctl->bar_gen);  // barrier `it` completes at gen0 + it + 1
+  // Overlap (VPT <= 2): while the grid barrier of iteration t settles, every
+  // thread already computes the gbest-free part of iteration t + 1 for the
+  // CTA's first row pair -- both Philox draws and ab = w v + (c1 r1)(pb - x)
+  // -- and keeps it in registers; after the barrier only (c2 r2)(g - x), the
+  // clamps and the move remain.  Same operations in the same order.
+  constexpr bool kOverlap = VPT <= 2;
+  float4 pre_ab[2][kOverlap ? VPT : 1], pre_m2[2][kOverlap ? VPT : 1];
+  bool have_pre = false;
   for (int it = 0; it < iters; ++it) {
     const uint32_t t = t0 + 1u + (uint32_t)it;
     const int par = (int)(t & 1u);
     const uint32_t inc_ord = (uint32_t)(cur >> 32);
     unsigned long long best = ~0ull;
     int best_row = -1;
-    for (int k = 0; k < myrows; ++k) {
-      const long long r = b + (long long)k * grid;
-      const uint32_t gi = (uint32_t)(a.row_begin + r);
-      float4* st = sRows + (size_t)k * 3 * nvec;
-      float acc[Obj::kAcc];
-      Obj::init(acc);
+    // Rows in pairs: both rows' updates and maps in one pass (twice the
+    // independent work per thread), one reduction barrier for the pair.  Per
+    // row the operation order is unchanged (bitwise k_step_tma).
+    for (int k0 = 0; k0 < myrows; k0 += 2) {
+      const int nk = (myrows - k0) < 2 ? (myrows - k0) : 2;
+      const bool use_pre = kOverlap && have_pre && k0 == 0;
+      float acc[2][Obj::kAcc];
+#pragma unroll
+      for (int u = 0; u < 2; ++u) {
+        Obj::init(acc[u]);
+        if (u < nk) {
+          const int k = k0 + u;
+          const uint32_t gi = (uint32_t)(a.row_begin + b + (long long)k * grid);
+          float4* st = sRows + (size_t)k * 3 * nvec;
 #pragma unroll(VPT <= 2 ? VPT : 2)
-      for (int j = 0; j < VPT; ++j) {
-        const int q = tid + j * nthr;
-        if (q < nvec) {
-          float4 x = st[q], v = st[nvec + q];
-          const float4 pb = st[2 * nvec + q];
-          const float4 g = sG[q];
-          const float4 r1 = raw24x4(key, kTagR1, t, gi, (uint32_t)q);
-          const float4 r2 = raw24x4(key, kTagR2, t, gi, (uint32_t)q);
-          move4<kB>(mp, x, v, pb, g, r1, r2, sB, nvec, q);
-          if ((d & 3) && q == nvec - 1) {
-            const int jj = 4 * q;
-            if (jj + 1 >= d) x.y = v.y = 0.f;
-            if (jj + 2 >= d) x.z = v.z = 0.f;
-            if (jj + 3 >= d) x.w = v.w = 0.f;
+          for (int j = 0; j < VPT; ++j) {
+            const int q = tid + j * nthr;
+            if (q < nvec) {
+              float4 x = st[q], v = st[nvec + q];
+              const float4 g = sG[q];
+              if constexpr (kOverlap) {
+                if (use_pre) {
+                  move_post4<kB>(mp, x, v, g, pre_m2[u][j], pre_ab[u][j], sB, nvec, q);
+                } else {
+                  const float4 pb = st[2 * nvec + q];
+                  const float4 r1 = raw24x4(key, kTagR1, t, gi, (uint32_t)q);
+                  const float4 r2 = raw24x4(key, kTagR2, t, gi, (uint32_t)q);
+                  move4<kB>(mp, x, v, pb, g, r1, r2, sB, nvec, q);
+                }
+              } else {
+                const float4 pb = st[2 * nvec + q];
+                const float4 r1 = raw24x4(key, kTagR1, t, gi, (uint32_t)q);
+                const float4 r2 = raw24x4(key, kTagR2, t, gi, (uint32_t)q);
+                move4<kB>(mp, x, v, pb, g, r1, r2, sB, nvec, q);
+              }
+              if ((d & 3) && q == nvec - 1) {
+                const int jj = 4 * q;
+                if (jj + 1 >= d) x.y = v.y = 0.f;
+                if (jj + 2 >= d) x.z = v.z = 0.f;
+                if (jj + 3 >= d) x.w = v.w = 0.f;
+              }
+              st[q] = x;
+              st[nvec + q] = v;
+              if constexpr (!Obj::kNeighbor) map4<Obj>(acc[u], x, 0.f, 4 * q, d);
+            }
           }
-          st[q] = x;
-          st[nvec + q] = v;
-          if constexpr (!Obj::kNeighbor) map4<Obj>(acc, x, 0.f, 4 * q, d);
         }
       }
       if constexpr (Obj::kNeighbor) {
         __syncthreads();
+#pragma unroll
+        for (int u = 0; u < 2; ++u) {
+          if (u < nk) {
+            const float4* st = sRows + (size_t)(k0 + u) * 3 * nvec;
 #pragma unroll(VPT <= 2 ? VPT : 2)
-        for (int j = 0; j < VPT; ++j) {
-          const int q = tid + j * nthr;
-          if (q < nvec) map4<Obj>(acc, st[q], (q + 1 < nvec) ? st[q + 1].x : 0.f, 4 * q, d);
+            for (int j = 0; j < VPT; ++j) {
+              const int q = tid + j * nthr;
+              if (q < nvec) map4<Obj>(acc[u], st[q], (q + 1 < nvec) ? st[q + 1].x : 0.f, 4 * q, d);
+            }
+          }
         }
       }
-      warp_combine<Obj>(acc);
-      if (lane == 0) {
 #pragma unroll
-        for (int j = 0; j < Obj::kAcc; ++j) red[warp * Obj::kAcc + j] = acc[j];
+      for (int u = 0; u < 2; ++u) {
+        if (u < nk) {
+          warp_combine<Obj>(acc[u]);
+          if (lane == 0) {
+#pragma unroll
+            for (int j = 0; j < Obj::kAcc; ++j) red[(u * nwarps + warp) * Obj::kAcc + j] = acc[u][j];
+          }
+        }
       }
       __syncthreads();
-      if (tid == 0) {
+      if (tid < nk) {  // thread u finalises row k0 + u (warps combined in index order)
+        const int u = tid, k = k0 + u;
         float c[Obj::kAcc];
         Obj::init(c);
         for (int w = 0; w < nwarps; ++w) {
           float o[Obj::kAcc];
 #pragma unroll
-          for (int j = 0; j < Obj::kAcc; ++j) o[j] = red[w * Obj::kAcc + j];
+          for (int j = 0; j < Obj::kAcc; ++j) o[j] = red[(u * nwarps + w) * Obj::kAcc + j];
           Obj::combine(c, o);
         }
         const float f = Obj::finalize(c, d);
-        s_f = f;
-        s_imp = (f < spf[k]) ? 1 : 0;  // strict; NaN never improves
-        if (s_imp) {
-          spf[k] = f;
-          ++nimp;
-        }
-        if (f == f && ord_f32(f) < inc_ord) {
-          const unsigned long long kk = pack_key(f, gi);
-          if (kk < best) {
-            best = kk;
-            best_row = k;
+        const int imp = (f < spf[k]) ? 1 : 0;  // strict; NaN never improves
+        if (imp) spf[k] = f;
+        s_imp2[u] = imp;
+        s_f2[u] = f;
+      }
+      __syncthreads();
+      if (tid == 0) {  // gbest candidates in row order (equal keys: the lower global index)
+        for (int u = 0; u < nk; ++u) {
+          const float f = s_f2[u];
+          nimp += (unsigned)s_imp2[u];
+          const uint32_t gi = (uint32_t)(a.row_begin + b + (long long)(k0 + u) * grid);
+          if (f == f && ord_f32(f) < inc_ord) {  // strictly below gf (Alg. 1 line 10)
+            const unsigned long long kk = pack_key(f, gi);
+            if (kk < best) {
+              best = kk;
+              best_row = k0 + u;
+            }
           }
         }
       }
-      __syncthreads();
-      if (s_imp) {
-        for (int q = tid; q < nvec; q += nthr) st[2 * nvec + q] = st[q];
+#pragma unroll
+      for (int u = 0; u < 2; ++u) {
+        if (u < nk && s_imp2[u]) {  // pbest copy (Alg. 1 lines 7-9)
+          float4* st = sRows + (size_t)(k0 + u) * 3 * nvec;
+          for (int q = tid; q < nvec; q += nthr) st[2 * nvec + q] = st[q];
+        }
       }
+      __syncthreads();  // s_imp2 / s_f2 / red are reused by the next pair
     }
-    // ---- publish the CTA's candidate, grid barrier, pull the winner into G
+    // ---- publish the CTA's candidate (row + key), grid barrier, fold, pull the winner
     if (tid == 0) {
       s_best = best;
       s_best_row = best_row;
@@ -1506,28 +1610,72 @@ __global__ void __launch_bounds__(kMaxThreadsWide, 1) k_gridres(const __grid_con
       float4* dst = reinterpret_cast<float4*>(a.cand) + ((size_t)par * grid + b) * nvec;
       for (int q = tid; q < nvec; q += nthr) dst[q] = src[q];
     }
-    __syncthreads();
-    if (tid == 0) {
-      if (s_best != ~0ull) atomicMin(&a.ctl->key_par[par], s_best);
-      __threadfence();
-      const unsigned gen = ld_acquire_u32(&a.ctl->bar_gen);
-      if (atomicAdd(&a.ctl->bar_count, 1u) == (unsigned)grid - 1) {
+    if (tid == 0) ckey[(size_t)par * grid + b] = s_best;
+    __syncthreads();  // every candidate store of the CTA precedes thread 0's release
+    const unsigned gen_done = gen0 + (unsigned)it + 1u;
+    bool last = false;
+    if (tid == 0) {  // arrival: acq_rel ticket; the last CTA releases the generation
+      last = atom_add_acq_rel_u32(&a.ctl->bar_count, 1u) == (unsigned)grid - 1;
+      if (last) {
         a.ctl->bar_count = 0;
-        // the other parity serves the next iteration: reset it to the new incumbent
-        const unsigned long long winner = *(volatile unsigned long long*)&a.ctl->key_par[par];
-        a.ctl->key_par[par ^ 1] = winner < cur ? winner : cur;
-        __threadfence();
-        atomicAdd(&a.ctl->bar_gen, 1u);
-      } else {
-        while (ld_acquire_u32(&a.ctl->bar_gen) == gen) {
-        }
+        st_release_u32(&a.ctl->bar_gen, gen_done);
       }
-      __threadfence();
-      s_best = *(volatile unsigned long long*)&a.ctl->key_par[par];
+    }
+    // the gbest-free part of the next iteration while the barrier settles
+    have_pre = false;
+    if constexpr (kOverlap) {
+      if (it + 1 < iters) {
+        const uint32_t tn = t + 1u;
+#pragma unroll
+        for (int u = 0; u < 2; ++u) {
+          if (u < myrows) {
+            const uint32_t gi = (uint32_t)(a.row_begin + b + (long long)u * grid);
+            const float4* st = sRows + (size_t)u * 3 * nvec;
+#pragma unroll
+            for (int j = 0; j < VPT; ++j) {
+              const int q = tid + j * nthr;
+              if (q < nvec) {
+                const float4 r1 = raw24x4(key, kTagR1, tn, gi, (uint32_t)q);
+                pre_m2[u][j] = raw24x4(key, kTagR2, tn, gi, (uint32_t)q);
+                move_pre4<kB>(mp, st[q], st[nvec + q], st[2 * nvec + q], r1, pre_ab[u][j]);
+              }
+            }
+          }
+        }
+        have_pre = true;
+      }
+    }
+    if (tid == 0 && !last) {
+      while (ld_acquire_u32(&a.ctl->bar_gen) != gen_done) {
+      }
     }
     __syncthreads();
-    const unsigned long long win = s_best;
-    if (win < cur) {
+    // every CTA folds all candidate keys itself (one parallel L2 read instead
+    // of a serial fold by the last arriver); keys of this parity are
+    // rewritten only after the next barrier, which every CTA passes after
+    // this read
+    unsigned long long m = ~0ull;
+    const unsigned long long* keys = ckey + (size_t)par * grid;
+    for (int c0 = tid; c0 < grid; c0 += 8 * nthr) {  // 8 independent loads in flight per thread
+      unsigned long long kk[8];
+#pragma unroll
+      for (int i = 0; i < 8; ++i) {
+        const int c = c0 + i * nthr;
+        kk[i] = c < grid ? __ldcg(keys + c) : ~0ull;
+      }
+#pragma unroll
+      for (int i = 0; i < 8; ++i) m = kk[i] < m ? kk[i] : m;
+    }
+#pragma unroll
+    for (int off = 16; off > 0; off >>= 1) {
+      const unsigned long long o = __shfl_xor_sync(kFull, m, off);
+      m = o < m ? o : m;
+    }
+    if (lane == 0) s_kmin[warp] = m;
+    __syncthreads();
+    unsigned long long win = ~0ull;
+    for (int w = 0; w < nwarps; ++w) win = s_kmin[w] < win ? s_kmin[w] : win;
+    if (win < cur) {  // strictly better than the incumbent (candidates already are)
       const long long wr = (long long)(uint32_t)win - a.row_begin;
       const int owner = (int)(wr % grid);
       const float4* src = reinterpret_cast<const float4*>(a.cand) + ((size_t)par * grid + owner) * nvec;
