@@ -269,9 +269,11 @@ def test_errors_do_not_abort():
 
 
 # ------------------------------------------------------------------ full size, sampled
-@pytest.mark.parametrize("key", ["NS", "C4"])
+@pytest.mark.parametrize("key", ["NS", "C4", "C3", "C2"])
 def test_full_size_sampled_rows(key):
-    """Bench configuration (100k x 2000) in the bench's launch shape: the
+    """Bench configurations at full size in the bench's launch shape (NS / C4
+    streaming 100k x 2000, C3 streaming with a neighbour functor, C2 on the
+    grid-resident path): the
     oracle recomputes sampled rows of one iteration exactly (rows are
     independent given G), and the gbest invariants hold over the whole swarm."""
     w = WORKLOADS[key]
