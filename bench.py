@@ -32,6 +32,7 @@ METRIC = "particle-dim updates/sec and % of HBM roofline at 1/2/4/8 B200"
 UNIT = "particle-dim updates/s"
 L2_BYTES = 126 * 2**20
 FALLBACK_HBM_GBS = 6650.0  # B200_PROFILING.md fallback, used only without MEASURED_PEAKS.json
+SPEC_HBM_GBS = 8000.0      # B200 data-sheet HBM3e bandwidth (north_star's "~8 TB/s"), context only
 
 
 def parse():
@@ -368,6 +369,7 @@ def run_gpu(args, w):
             "gpu_launches": launches,
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "peak_source": peak_src,
+                         "frac_of_spec": achieved / SPEC_HBM_GBS,  # vs the 8 TB/s data-sheet figure
                          "traffic": ncu_traffic(w.name),
                          "kernel": "k_step (fused move+eval+pbest+gbest)",
                          "kernel_avg_us": kern_ms * 1e3,

@@ -253,6 +253,51 @@ def test_launch_counter_and_improvements(monkeypatch):
     assert 0 < info["improvements"] <= 20 * 1000
 
 
+@pytest.mark.parametrize("obj,n,d", [(RASTRIGIN, 600, 1000), (ROSENBROCK, 300, 2001),
+                                     (ACKLEY, 40, 4096), (SPHERE, 700, 256)])
+def test_pdl_and_timing_do_not_change_results(obj, n, d, monkeypatch):
+    """Programmatic dependent launch (default) vs plain stream order, with and
+    without the timing events: the same bits (PDL only moves the launch, every
+    global read of a step kernel sits behind griddepcontrol.wait)."""
+    monkeypatch.setenv("PSO_RESIDENT", "0")
+    runs = []
+    for pdl, timing in (("1", False), ("1", True), ("0", True)):
+        monkeypatch.setenv("PSO_PDL", pdl)
+        g = gpu_swarm(n, d, obj, seed=77, timing=timing)
+        g.step(9)
+        runs.append((g.get_state()[:4], g.gbest()))
+        info = g.info()
+        if timing:  # per-call events under PDL, one pair per launch without
+            assert info["step_kernel_count"] == 9 and info["step_kernel_ms"] > 0
+        g.close()
+    (s0, b0) = runs[0]
+    for s1, b1 in runs[1:]:
+        for x, y in zip(s0, s1):
+            assert_bitwise(x, y, "PDL / timing changed the state")
+        assert b0[:2] == b1[:2]
+        assert_bitwise(b0[2], b1[2], "G")
+
+
+@pytest.mark.parametrize("d,vpt,threads,ctas,stages", [
+    (1000, 2, 128 + 64, 4, 4),    # C3 shape: 4 CTAs x 4 compute warps
+    (2000, 2, 256 + 64, 2, 4),    # NS / C4: 2 CTAs x 8 warps
+    (4096, 2, 512 + 64, 1, 4),    # C5: the wide instantiation, 16 warps
+])
+def test_tma_launch_shape_rule(d, vpt, threads, ctas, stages, monkeypatch):
+    """The planner's shape rule: 16 compute warps per SM with
+    >= 3 stages, 2 float4 per thread preferred; it depends on d only."""
+    monkeypatch.setenv("PSO_RESIDENT", "0")
+    for n in (ctas * 148 + 5, 3):  # the shape must not depend on n
+        g = gpu_swarm(n, d, GRIEWANK, seed=5)
+        info = g.info()
+        assert info["tma_pipeline"] == 1
+        assert (info["vec_per_thread"], info["threads_per_cta"], info["pipeline_stages"]) == \
+            (vpt, threads, stages), info
+        if n > 3:
+            assert info["ctas_per_sm"] == ctas
+        g.close()
+
+
 def test_errors_do_not_abort():
     with pytest.raises(fp.PsoError) as e:
         gpu_swarm(0, 10, SPHERE)
