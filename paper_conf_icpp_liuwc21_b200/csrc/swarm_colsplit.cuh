@@ -198,11 +198,9 @@ __global__ void __launch_bounds__(kColCompute + 64, 2)
       } else {
         x = st[ql];
         v = st[chunk + ql];
-        const float4 pb = fl ? x : st[2 * chunk + ql];
         const float4 g = st[3 * chunk + ql];
-        const float4 r1 = raw24x4(key, kTagR1, t, gi, (uint32_t)qg);
-        const float4 r2 = raw24x4(key, kTagR2, t, gi, (uint32_t)qg);
-        move4<kB>(mp, x, v, pb, g, r1, r2, st + 4 * chunk, chunk, ql);
+        move4_draw<kB>(mp, key, t, gi, (uint32_t)qg, fl, x, v, st + 2 * chunk + ql, g,
+                       st + 4 * chunk, chunk, ql);
         if ((d & 3) && qg == a.nvec_glob - 1) {
           const int jj = 4 * qg;
           if (jj + 1 >= d) x.y = v.y = 0.f;

@@ -299,6 +299,36 @@ __device__ __forceinline__ void move_post4(const MoveParams& m, float4& x, float
   }
 }
 
+// One float4 of a staged row with its random draws (A1-A4).  fl: lazy pbest
+// row, PB == X bitwise (pbs is then not read).  x is finite there (every x the
+// kernels store is clamped to finite bounds), so pb - x = +0 and
+// (c1 r1)(pb - x) = copysign(0, c1) whatever r1 is: R1 is not drawn, and the
+// result is move4's bit for bit -- a + (+-0) is still rounded as the oracle
+// rounds it (-0 + +0 = +0).  Rows that improved the iteration before are lazy,
+// so a converging swarm (C4: every row, every iteration) skips a quarter of the
+// per-element instructions.
+template <bool kB, class K>
+__device__ __forceinline__ void move4_draw(const MoveParams& m, const K& key, uint32_t t, uint32_t gi,
+                                           uint32_t q, int fl, float4& x, float4& v,
+                                           const float4* pbs, const float4& g, const float4* sB,
+                                           int nb, int qb) {
+  if (fl) {
+    const float4 r2 = raw24x4(key, kTagR2, t, gi, q);
+    const float bz = copysignf(0.f, m.c1s);
+    float4 ab;
+    ab.x = __fadd_rn(__fmul_rn(m.w, v.x), bz);
+    ab.y = __fadd_rn(__fmul_rn(m.w, v.y), bz);
+    ab.z = __fadd_rn(__fmul_rn(m.w, v.z), bz);
+    ab.w = __fadd_rn(__fmul_rn(m.w, v.w), bz);
+    move_post4<kB>(m, x, v, g, r2, ab, sB, nb, qb);
+  } else {
+    const float4 pb = *pbs;
+    const float4 r1 = raw24x4(key, kTagR1, t, gi, q);
+    const float4 r2 = raw24x4(key, kTagR2, t, gi, q);
+    move4<kB>(m, x, v, pb, g, r1, r2, sB, nb, qb);
+  }
+}
+
 // --- CTA reduction of the functor accumulators -----------------------------
 template <class Obj>
 __device__ __forceinline__ void warp_combine(float* a) {
@@ -936,11 +966,8 @@ __global__ void __launch_bounds__(kMaxT + 64, kMaxT > kMaxThreads ? 1 : 2)
       const int q = tid + j * nthr;
       if (q < nvec) {
         float4 x = st[q], v = st[nvec + q];
-        const float4 pb = fl ? x : st[2 * nvec + q];
         const float4 g = sG[q];
-        const float4 r1 = raw24x4(key, kTagR1, t, gi, (uint32_t)q);
-        const float4 r2 = raw24x4(key, kTagR2, t, gi, (uint32_t)q);
-        move4<kB>(mp, x, v, pb, g, r1, r2, sB, nvec, q);
+        move4_draw<kB>(mp, key, t, gi, (uint32_t)q, fl, x, v, st + 2 * nvec + q, g, sB, nvec, q);
         if ((d & 3) && q == nvec - 1) {  // keep the row padding at zero
           const int jj = 4 * q;
           if (jj + 1 >= d) x.y = v.y = 0.f;
@@ -1199,11 +1226,8 @@ __global__ void __launch_bounds__(kMaxThreadsCluster + 64, 1)
       if (ql < cnt) {
         const int q = q0 + ql;
         float4 x = st[ql], v = st[chunk + ql];
-        const float4 pb = fl ? x : st[2 * chunk + ql];
         const float4 g = sG[ql];
-        const float4 r1 = raw24x4(key, kTagR1, t, gi, (uint32_t)q);
-        const float4 r2 = raw24x4(key, kTagR2, t, gi, (uint32_t)q);
-        move4<kB>(mp, x, v, pb, g, r1, r2, sB, chunk, ql);
+        move4_draw<kB>(mp, key, t, gi, (uint32_t)q, fl, x, v, st + 2 * chunk + ql, g, sB, chunk, ql);
         if ((d & 3) && q == nvec - 1) {
           const int jj = 4 * q;
           if (jj + 1 >= d) x.y = v.y = 0.f;

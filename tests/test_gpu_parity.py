@@ -614,6 +614,38 @@ def test_lazy_pbest_rows_lockstep(obj, n, d, monkeypatch):
     assert info["pb_loads"] < e.info()["pb_loads"]  # flagged rows skipped their pb load
 
 
+@pytest.mark.parametrize("w,c1,c2", [(0.0, 2.0, 0.0), (0.0, -1.5, 2.0), (0.5, 0.0, 2.0),
+                                     (0.9, -2.0, 2.0), (0.0, 0.0, 0.0)])
+@pytest.mark.parametrize("obj,n,d,kw", [(GRIEWANK, 300, 2000, {}), (SPHERE, 64, 1000, {}),
+                                        (ROSENBROCK, 5, 12000, {}),
+                                        (GRIEWANK, 9, 999, {"column_split": True})])
+def test_lazy_rows_skip_r1_signed_zeros(w, c1, c2, obj, n, d, kw, monkeypatch):
+    """A lazy row (PB == X) does not draw R1: (c1 r1)(pb - x) is copysign(0, c1)
+    for any r1.  The velocity must still be rounded as Eq. 1 rounds it: with
+    w = 0 a negative v gives a = -0, and -0 + (+0) = +0 must not become -0 when
+    c = 0 (c2 = 0, or g == x).  Negative and zero c1 give b = -0 / +0.  Lazy and
+    eager kernels and the oracle agree bit for bit (signs of zero included)."""
+    monkeypatch.setenv("PSO_RESIDENT", "0")
+    g = gpu_swarm(n, d, obj, seed=5, w=w, c1=c1, c2=c2, **kw)
+    c = cpu_swarm(n, d, obj, seed=5, w=w, c1=c1, c2=c2)
+    if not kw:
+        assert g.info()["lazy_pb"] == 1
+        monkeypatch.setenv("PSO_LAZY_PB", "0")
+        e = gpu_swarm(n, d, obj, seed=5, w=w, c1=c1, c2=c2)
+        assert e.info()["lazy_pb"] == 0
+    for k in (1, 1, 2, 1):
+        g.step(k)
+        c.step(k)
+        gs = g.get_state()
+        assert_bitwise(gs[0], c.X, "X vs oracle")
+        assert_bitwise(gs[1], c.V, "V vs oracle")
+        assert_bitwise(gs[2], c.PB, "PB vs oracle")
+        if not kw:
+            e.step(k)
+            for x, y, nm in zip(gs[:4], e.get_state()[:4], "X V PB pf".split()):
+                assert_bitwise(x, y, f"lazy vs eager {nm}")
+
+
 def test_async_gbest_single_rank_is_synchronous(monkeypatch):
     """With one rank the asynchronous split has nobody to lag behind: bitwise
     the synchronous single-GPU run."""
