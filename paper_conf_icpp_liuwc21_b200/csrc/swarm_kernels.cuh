@@ -142,6 +142,10 @@ template <int N>
 __device__ __forceinline__ void bulk_wait_read() {
   asm volatile("cp.async.bulk.wait_group.read %0;" ::"n"(N) : "memory");
 }
+// Hint: bring [src, src + bytes) into L2 (no shared memory, no completion).
+__device__ __forceinline__ void bulk_prefetch_l2(const void* src, unsigned bytes) {
+  asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(src), "r"(bytes) : "memory");
+}
 __device__ __forceinline__ void bulk_wait_all() {
   asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
 }
@@ -847,9 +851,26 @@ __global__ void __launch_bounds__(kMaxT + 64, kMaxT > kMaxThreads ? 1 : 2)
       int k = 0;
       // lazy pbest: rows whose PB equals X skip the pb load (flag prefetched one row ahead)
       int fl_next = (a.lazy_pb && blockIdx.x < a.n_local) ? a.pbx[blockIdx.x] : 0;
+      // L2 prefetch of the row l2pf rows beyond the load front: DRAM requests
+      // in flight beyond the ring.  Only lazy rows by default -- their stage
+      // loads 2 of its 3 slots, so the ring alone keeps a third fewer bytes in
+      // flight (C4: 547 -> 529 us); prefetching eager rows as well slows the
+      // ring-saturated case (NS 638 -> 671 us).  Flag read one row earlier.
+      const long long pd = (long long)a.l2pf * gridDim.x;
+      int pfl_next = (pd && blockIdx.x + pd < a.n_local) ? a.pbx[blockIdx.x + pd] : 0;
       for (long long r = blockIdx.x; r < a.n_local; r += gridDim.x, ++k) {
         const int fl = fl_next;
         if (a.lazy_pb && r + gridDim.x < a.n_local) fl_next = a.pbx[r + gridDim.x];
+        if (pd && r + pd < a.n_local) {
+          const int pfl = pfl_next;
+          if (r + pd + gridDim.x < a.n_local) pfl_next = a.pbx[r + pd + gridDim.x];
+          const size_t po = (size_t)(r + pd) * 4 * nvec;
+          if (pfl || a.l2pf_all) {
+            bulk_prefetch_l2(a.X + po, row_bytes);
+            bulk_prefetch_l2(a.V + po, row_bytes);
+            if (!pfl) bulk_prefetch_l2(a.PB + po, row_bytes);
+          }
+        }
         if (k >= stages) mbar_wait(&empty[s], ph ^ 1u);
         float4* st = ring + (size_t)s * 3 * nvec;
         sflag[s] = fl;
@@ -1079,9 +1100,21 @@ __global__ void __launch_bounds__(kMaxThreadsCluster + 64, 1)
       unsigned ph = 0;
       int k = 0;
       int fl_next = (a.lazy_pb && cid < a.n_local) ? a.pbx[cid] : 0;
+      const long long pd = (long long)a.l2pf * ncl;  // L2 prefetch, as in k_step_tma
+      int pfl_next = (pd && cid + pd < a.n_local) ? a.pbx[cid + pd] : 0;
       for (long long r = cid; r < a.n_local; r += ncl, ++k) {
         const int fl = fl_next;
         if (a.lazy_pb && r + ncl < a.n_local) fl_next = a.pbx[r + ncl];
+        if (pd && r + pd < a.n_local && cnt > 0) {
+          const int pfl = pfl_next;
+          if (r + pd + ncl < a.n_local) pfl_next = a.pbx[r + pd + ncl];
+          const size_t po = ((size_t)(r + pd) * nvec + q0) * 4;
+          if (pfl || a.l2pf_all) {
+            bulk_prefetch_l2(a.X + po, blk_bytes);
+            bulk_prefetch_l2(a.V + po, blk_bytes);
+            if (!pfl) bulk_prefetch_l2(a.PB + po, blk_bytes);
+          }
+        }
         if (k >= stages) mbar_wait(&empty[s], ph ^ 1u);
         float4* st = ring + (size_t)s * 3 * chunk;
         sflag[s] = fl;
