@@ -58,6 +58,7 @@ struct SwarmArgs {
   unsigned char* pbx;         // lazy pbest: 1 = the row's PB equals its X (PB not stored)
   int lazy_pb;
   int l2pf;                   // TMA producer: L2 prefetch distance in rows of this CTA (0: off)
+  int serp;                   // streaming kernels: odd iterations visit rows backwards (L2 reuse)
   int l2pf_all;               // prefetch every row (default: lazy rows only, whose stage loads 2 of 3 slots)
   unsigned char* send;        // world > 1: this rank's exchange record
   const unsigned char* recv;  // exchange: [2 iteration parities][world] records after the all-gather

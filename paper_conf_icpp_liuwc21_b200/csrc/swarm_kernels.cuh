@@ -303,6 +303,20 @@ __device__ __forceinline__ void move_post4(const MoveParams& m, float4& x, float
   }
 }
 
+// Row visiting order of the streaming kernels.  Rows are independent within an
+// iteration and every cross-row result (candidate key, counters) is an
+// order-free min / sum, so the order changes no bit.  Serpentine (a.serp):
+// odd iterations walk the rows backwards, so an iteration starts on the rows
+// the previous one wrote last -- still in L2 when the state is near its size.
+struct RowOrder {
+  long long n;
+  bool rev;
+  __device__ __forceinline__ long long operator()(long long i) const { return rev ? n - 1 - i : i; }
+};
+__device__ __forceinline__ RowOrder row_order(const SwarmArgs& a, uint32_t t) {
+  return RowOrder{a.n_local, a.serp != 0 && (t & 1u) != 0};
+}
+
 // One float4 of a staged row with its random draws (A1-A4).  fl: lazy pbest
 // row, PB == X bitwise (pbs is then not read).  x is finite there (every x the
 // kernels store is clamped to finite bounds), so pb - x = +0 and
@@ -850,21 +864,23 @@ __global__ void __launch_bounds__(kMaxT + 64, kMaxT > kMaxThreads ? 1 : 2)
       unsigned ph = 0;
       int k = 0;
       // lazy pbest: rows whose PB equals X skip the pb load (flag prefetched one row ahead)
-      int fl_next = (a.lazy_pb && blockIdx.x < a.n_local) ? a.pbx[blockIdx.x] : 0;
+      const RowOrder ro = row_order(a, t);
+      int fl_next = (a.lazy_pb && blockIdx.x < a.n_local) ? a.pbx[ro(blockIdx.x)] : 0;
       // L2 prefetch of the row l2pf rows beyond the load front: DRAM requests
       // in flight beyond the ring.  Only lazy rows by default -- their stage
       // loads 2 of its 3 slots, so the ring alone keeps a third fewer bytes in
       // flight (C4: 547 -> 529 us); prefetching eager rows as well slows the
       // ring-saturated case (NS 638 -> 671 us).  Flag read one row earlier.
       const long long pd = (long long)a.l2pf * gridDim.x;
-      int pfl_next = (pd && blockIdx.x + pd < a.n_local) ? a.pbx[blockIdx.x + pd] : 0;
-      for (long long r = blockIdx.x; r < a.n_local; r += gridDim.x, ++k) {
+      int pfl_next = (pd && blockIdx.x + pd < a.n_local) ? a.pbx[ro(blockIdx.x + pd)] : 0;
+      for (long long i = blockIdx.x; i < a.n_local; i += gridDim.x, ++k) {
+        const long long r = ro(i);
         const int fl = fl_next;
-        if (a.lazy_pb && r + gridDim.x < a.n_local) fl_next = a.pbx[r + gridDim.x];
-        if (pd && r + pd < a.n_local) {
+        if (a.lazy_pb && i + gridDim.x < a.n_local) fl_next = a.pbx[ro(i + gridDim.x)];
+        if (pd && i + pd < a.n_local) {
           const int pfl = pfl_next;
-          if (r + pd + gridDim.x < a.n_local) pfl_next = a.pbx[r + pd + gridDim.x];
-          const size_t po = (size_t)(r + pd) * 4 * nvec;
+          if (i + pd + gridDim.x < a.n_local) pfl_next = a.pbx[ro(i + pd + gridDim.x)];
+          const size_t po = (size_t)ro(i + pd) * 4 * nvec;
           if (pfl || a.l2pf_all) {
             bulk_prefetch_l2(a.X + po, row_bytes);
             bulk_prefetch_l2(a.V + po, row_bytes);
@@ -896,7 +912,9 @@ __global__ void __launch_bounds__(kMaxT + 64, kMaxT > kMaxThreads ? 1 : 2)
       unsigned nimp = 0, n_pbl = 0, n_pbs = 0;
       int s = 0, prev = -1;
       unsigned ph = 0;
-      for (long long r = blockIdx.x; r < a.n_local; r += gridDim.x) {
+      const RowOrder ro = row_order(a, t);
+      for (long long i = blockIdx.x; i < a.n_local; i += gridDim.x) {
+        const long long r = ro(i);
         const float pf_old = a.pf[r];
         const uint32_t gi = (uint32_t)(a.row_begin + r);
         mbar_wait(&done[s], ph);
@@ -971,8 +989,9 @@ __global__ void __launch_bounds__(kMaxT + 64, kMaxT > kMaxThreads ? 1 : 2)
   mbar_wait(&gbar, 0);
   int s = 0;
   unsigned ph = 0;
-  for (long long r = blockIdx.x; r < a.n_local; r += gridDim.x) {
-    const uint32_t gi = (uint32_t)(a.row_begin + r);
+  const RowOrder ro = row_order(a, t);
+  for (long long i = blockIdx.x; i < a.n_local; i += gridDim.x) {
+    const uint32_t gi = (uint32_t)(a.row_begin + ro(i));
     float4* st = ring + (size_t)s * 3 * nvec;
     mbar_wait(&full[s], ph);
     // lazy pbest row (PB == X): pb is the loaded x, and x' goes to the pb slot

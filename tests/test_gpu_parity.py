@@ -646,6 +646,29 @@ def test_lazy_rows_skip_r1_signed_zeros(w, c1, c2, obj, n, d, kw, monkeypatch):
                 assert_bitwise(x, y, f"lazy vs eager {nm}")
 
 
+@pytest.mark.parametrize("obj,n,d", [(ROSENBROCK, 301, 1000), (GRIEWANK, 300, 2000),
+                                     (RASTRIGIN, 7, 12000)])
+def test_row_order_is_invisible(obj, n, d, monkeypatch):
+    """Serpentine row order (odd iterations walk the rows backwards for L2
+    reuse) and the L2 prefetch change no bit: state, pf and gbest equal the
+    forward, prefetch-free run after every call."""
+    monkeypatch.setenv("PSO_RESIDENT", "0")
+    monkeypatch.setenv("PSO_SERP", "1")
+    monkeypatch.setenv("PSO_L2PF_ALL", "1")
+    g = gpu_swarm(n, d, obj, seed=12)
+    monkeypatch.setenv("PSO_SERP", "0")
+    monkeypatch.setenv("PSO_L2PF", "0")
+    monkeypatch.setenv("PSO_L2PF_ALL", "0")
+    e = gpu_swarm(n, d, obj, seed=12)
+    for k in (1, 2, 3, 1):
+        g.step(k)
+        e.step(k)
+        for x, y, nm in zip(g.get_state()[:4], e.get_state()[:4], "X V PB pf".split()):
+            assert_bitwise(x, y, f"serpentine vs forward {nm}")
+        assert g.gbest()[:2] == e.gbest()[:2]
+    assert g.info()["launches"] == e.info()["launches"]
+
+
 def test_async_gbest_single_rank_is_synchronous(monkeypatch):
     """With one rank the asynchronous split has nobody to lag behind: bitwise
     the synchronous single-GPU run."""
