@@ -79,6 +79,11 @@ WORKLOADS = {
     # NEXT-3: rows wider than one CTA (d > 8192), split over a thread-block cluster
     "W64K": Workload("wide-rastrigin-4096x65536", RASTRIGIN, 4096, 65536, 200),
     "W16K": Workload("wide-griewank-16384x16384", GRIEWANK, 16384, 16384, 200),
+    # one rank's shard of NS at 2 / 4 / 8 GPUs (rows floor(n r / k) ..), to time the
+    # per-rank step on one GPU (with PSO_FORCE_EXCHANGE=1: the exchange path too)
+    "NS_R2": Workload("northstar-shard-of-2-rastrigin-50000x2000", RASTRIGIN, 50_000, 2000, 500),
+    "NS_R4": Workload("northstar-shard-of-4-rastrigin-25000x2000", RASTRIGIN, 25_000, 2000, 500),
+    "NS_R8": Workload("northstar-shard-of-8-rastrigin-12500x2000", RASTRIGIN, 12_500, 2000, 500),
     # the paper's own default experiment, for the Table 2 plausibility band
     "PAPER": Workload("paper-default-5000x200", SPHERE, 5000, 200, 2000),
 }
