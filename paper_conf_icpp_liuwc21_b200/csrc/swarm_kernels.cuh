@@ -584,6 +584,47 @@ __device__ __forceinline__ unsigned long long exchange_merge(const SwarmArgs& a,
   *src = s;
   return best;
 }
+// The same merge by a whole warp (the producer warp of the TMA and cluster
+// kernels): lane r waits for and reads rank r's record, so the world's tags
+// and keys cost one round trip instead of one each; a shuffle takes the
+// minimum (keys are unique: global particle indices).  __syncwarp orders
+// every lane's acquire before lane 0's bulk copy of the winning row.
+__device__ __forceinline__ unsigned long long exchange_merge_warp(const SwarmArgs& a, uint32_t prev_t,
+                                                                  int lane, int* src) {
+  const size_t rec = record_bytes(a.nvec * 4);
+  const unsigned char* base = records(a, prev_t);
+  const unsigned long long want = ((unsigned long long)a.epoch << 32) | prev_t;
+  const unsigned long long cur = *(volatile unsigned long long*)&a.ctl->key_cur;
+  const unsigned long long t0 = globaltimer_ns();
+  unsigned long long best = cur;
+  int s = -1;
+  for (int r = lane; r < a.world; r += 32) {
+    if (a.p2p) {
+      while (ld_acquire_sys_u64(base + (size_t)r * rec + 8) != want) {
+        __nanosleep(64);
+        if (globaltimer_ns() - t0 > 60ull * 1000000000ull) __trap();
+      }
+    }
+    const unsigned long long k = *reinterpret_cast<const volatile unsigned long long*>(base + (size_t)r * rec);
+    if ((k >> 32) < (cur >> 32) && k < best) {  // strictly better fitness, then the lowest key
+      best = k;
+      s = r;
+    }
+  }
+#pragma unroll
+  for (int off = 16; off > 0; off >>= 1) {
+    const unsigned long long ob = __shfl_xor_sync(kFull, best, off);
+    const int os = __shfl_xor_sync(kFull, s, off);
+    if (ob < best) {
+      best = ob;
+      s = os;
+    }
+  }
+  __syncwarp();
+  if (a.p2p) fence_proxy_async_global();  // the records are then read by bulk copies too
+  *src = s;
+  return best;
+}
 __device__ __forceinline__ const float* merged_gbest_row(const SwarmArgs& a, uint32_t prev_t, int src) {
   return src < 0 ? a.G
                  : reinterpret_cast<const float*>(records(a, prev_t) +
@@ -654,21 +695,20 @@ __device__ __forceinline__ void epilogue_core(const SwarmArgs& a, uint32_t t, un
       hdr[1] = t;
     }
   } else {  // NVLink: store the record into recv[t & 1][rank] of every rank
+    // the row is read once and stored to every rank; thread r releases rank r's tag
     const size_t rec = record_bytes(a.nvec * 4);
     const size_t off = (size_t)(t & 3u) * a.world * rec + (size_t)a.rank * rec;
-    for (int r = 0; r < a.world; ++r) {
-      unsigned char* dst = a.peers[r] + off;
-      if (have) {
-        float4* row = reinterpret_cast<float4*>(dst + 16);
-        for (int q = tid; q < a.nvec; q += nthr) row[q] = __ldcg(pb + q);
+    if (have) {
+      for (int q = tid; q < a.nvec; q += nthr) {
+        const float4 v = __ldcg(pb + q);
+        for (int r = 0; r < a.world; ++r) reinterpret_cast<float4*>(a.peers[r] + off + 16)[q] = v;
       }
-      if (tid == 0) reinterpret_cast<unsigned long long*>(dst)[0] = key;
     }
+    for (int r = tid; r < a.world; r += nthr) reinterpret_cast<unsigned long long*>(a.peers[r] + off)[0] = key;
     __threadfence_system();
     sync();
-    if (tid == 0)
-      for (int r = 0; r < a.world; ++r)
-        st_release_sys_u64(a.peers[r] + off + 8, ((unsigned long long)a.epoch << 32) | t);
+    for (int r = tid; r < a.world; r += nthr)
+      st_release_sys_u64(a.peers[r] + off + 8, ((unsigned long long)a.epoch << 32) | t);
   }
   if (tid == 0) {
     if (local)
@@ -847,15 +887,17 @@ __global__ void __launch_bounds__(kMaxT + 64, kMaxT > kMaxThreads ? 1 : 2)
   const unsigned row_bytes = (unsigned)nvec * 16u;
 
   if (warp == nwarps) {  // ---------------- producer
+    int xsrc = -1;
+    unsigned long long xinc = 0;
+    if (a.exchange) xinc = exchange_merge_warp(a, merge_iter(a, t), lane, &xsrc);  // the all-gather's merge
     if (lane == 0) {
       const float* gsrc = a.G;
       s_src = -1;
       s_inc = a.ctl->key_cur;
-      if (a.exchange) {  // merge the previous iteration's records (the all-gather)
-        int src;
-        s_inc = exchange_merge(a, merge_iter(a, t), &src);
-        s_src = src;
-        gsrc = merged_gbest_row(a, merge_iter(a, t), src);
+      if (a.exchange) {
+        s_inc = xinc;
+        s_src = xsrc;
+        gsrc = merged_gbest_row(a, merge_iter(a, t), xsrc);
       }
       mbar_expect_tx(&gbar, row_bytes * (kB ? 5u : 1u));  // releases s_inc / s_src too
       bulk_g2s(sG, gsrc, row_bytes, &gbar);
@@ -1098,15 +1140,17 @@ __global__ void __launch_bounds__(kMaxThreadsCluster + 64, 1)
   const unsigned blk_bytes = (unsigned)cnt * 16u;
 
   if (warp == nwarps) {  // ---------------- producer
+    int xsrc = -1;
+    unsigned long long xinc = 0;
+    if (a.exchange) xinc = exchange_merge_warp(a, merge_iter(a, t), lane, &xsrc);  // the all-gather's merge
     if (lane == 0) {
       const float* gsrc = a.G;
       s_src = -1;
       s_inc = a.ctl->key_cur;
-      if (a.exchange) {  // merge the previous iteration's records (the all-gather)
-        int src;
-        s_inc = exchange_merge(a, merge_iter(a, t), &src);
-        s_src = src;
-        gsrc = merged_gbest_row(a, merge_iter(a, t), src);
+      if (a.exchange) {
+        s_inc = xinc;
+        s_src = xsrc;
+        gsrc = merged_gbest_row(a, merge_iter(a, t), xsrc);
       }
       mbar_expect_tx(&gbar, blk_bytes * (kB ? 5u : 1u));  // releases s_inc / s_src too
       if (cnt > 0) {
