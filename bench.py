@@ -60,6 +60,14 @@ def hbm_peak():
         return FALLBACK_HBM_GBS, "fallback (B200_PROFILING.md)"
 
 
+def _path_name(info) -> str:
+    if info["column_split"]:
+        return "column-split (%d tiles per row)" % info["col_tiles"]
+    if info["cluster"]:
+        return "cluster (%d CTAs per row)" % info["cluster"]
+    return ["streaming", "cta-resident", "grid-resident"][info["resident"]]
+
+
 def ncu_traffic(workload_name):
     """DRAM bytes per launch of the step kernel from the committed ncu --set full summary."""
     p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
@@ -371,7 +379,9 @@ def run_gpu(args, w):
                          "frac": achieved / peak, "peak_source": peak_src,
                          "frac_of_spec": achieved / SPEC_HBM_GBS,  # vs the 8 TB/s data-sheet figure
                          "traffic": ncu_traffic(w.name),
-                         "kernel": "k_step (fused move+eval+pbest+gbest)",
+                         "kernel": ("k_col_step (fused move+eval, tile partials; k_col_decide "
+                                    "takes the pbest/gbest decisions)" if info["column_split"]
+                                    else "k_step (fused move+eval+pbest+gbest)"),
                          "kernel_avg_us": kern_ms * 1e3,
                          "bytes_per_update": bytes_per_update, "rho": rho,
                          "pb_load_frac": pbl, "pb_store_frac": pbs,
@@ -383,7 +393,7 @@ def run_gpu(args, w):
                                  "tma_pipeline": info["tma_pipeline"],
                                  "stages": info["pipeline_stages"],
                                  "smem_bytes": info["smem_bytes"],
-                                 "path": ["streaming", "cta-resident", "grid-resident"][info["resident"]]}},
+                                 "path": _path_name(info)}},
             "clocks": clk.result, "e2e": e2e, "clocks_e2e": clk_e2e,
             "cpu_baseline": cpu, "gbest": {"fitness": gf, "index": gi},
         }

@@ -57,6 +57,9 @@ extern "C" {
                               above, a thread-block cluster of up to 16 CTAs per row */
 #define PSO_D_MAX (1 << 24) /* max dimension: above PSO_D_MAX_ROW the column split
                               (PSO_FLAG_COLUMN_SPLIT) is used on a single GPU */
+#define PSO_D_AUTO_COLSPLIT 16384 /* a single-GPU handle (no communicator, world <= 1)
+                              with d above this uses the column split: faster than
+                              clusters of 8-16 CTAs per row */
 
 typedef struct pso_swarm* pso_handle; /* opaque; owns all device memory */
 
@@ -108,7 +111,7 @@ enum {
                               rank's records at the end of the last pso_step call. */
   PSO_FLAG_COLUMN_SPLIT = 8 /* NEXT-3, "tile matrix": every rank holds ALL n
                               particles but only a block of the columns.  Rows are cut
-                              into column tiles of T = clamp(ceil(nv / 64), 32, 512)
+                              into column tiles of T = clamp(ceil(nv / 8), 32, 512)
                               float4 (nv = ceil(d / 4)); rank r owns tiles
                               [floor(nt r / world), floor(nt (r+1) / world)) of the nt
                               (dims [col_begin, col_begin + d_local), pso_get_info).
@@ -123,7 +126,8 @@ enum {
                               rank).  world > 1 needs the NVLink exchange (p2p connect +
                               enable before pso_init, so PSO_FLAG_DEFER_INIT) and
                               nt >= world.  Chosen automatically for a single
-                              GPU when d > PSO_D_MAX_ROW.  Not with ASYNC_GBEST. */
+                              GPU when d > PSO_D_AUTO_COLSPLIT (unless the PSO_CLUSTER
+                              tuning variable asks for a cluster).  Not with ASYNC_GBEST. */
 };
 
 /* Options; a zero-initialised struct means "defaults". */

@@ -11,7 +11,7 @@ import ctypes as C
 
 import numpy as np
 
-from ._lib import (EXPORTS, PSO_D_MAX, PSO_D_MAX_ROW, PSO_FLAG_ASYNC_GBEST, PSO_FLAG_COLUMN_SPLIT,
+from ._lib import (EXPORTS, PSO_D_AUTO_COLSPLIT, PSO_D_MAX, PSO_D_MAX_ROW, PSO_FLAG_ASYNC_GBEST, PSO_FLAG_COLUMN_SPLIT,
                    PSO_FLAG_DEFER_INIT, PSO_FLAG_TIMING, PSO_OBJ_ACKLEY, PSO_OBJ_CUSTOM_BASE,
                    PSO_OBJ_EASOM, PSO_OBJ_GRIEWANK, PSO_OBJ_RASTRIGIN, PSO_OBJ_ROSENBROCK,
                    PSO_OBJ_SPHERE, PSO_OK, PsoError, check, last_error, lib, pso_info, pso_opts,
@@ -22,7 +22,7 @@ __all__ = [
     "debug_philox", "debug_objective", "nccl_unique_id", "nccl_comm_init", "nccl_comm_destroy",
     "PSO_OBJ_SPHERE", "PSO_OBJ_RASTRIGIN", "PSO_OBJ_ROSENBROCK", "PSO_OBJ_GRIEWANK",
     "PSO_OBJ_ACKLEY", "PSO_OBJ_EASOM", "PSO_OBJ_CUSTOM_BASE", "PSO_FLAG_TIMING", "PSO_D_MAX",
-    "PSO_D_MAX_ROW",
+    "PSO_D_MAX_ROW", "PSO_D_AUTO_COLSPLIT",
     "EXPORTS",
 ]
 

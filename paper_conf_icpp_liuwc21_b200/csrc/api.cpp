@@ -392,6 +392,12 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
                   "PSO_FLAG_COLUMN_SPLIT", d, PSO_D_MAX_ROW);
     colsplit = true;  // one GPU: rows longer than a cluster are tiled
   }
+  // One GPU, rows that would need a cluster of 8 or 16 CTAs: the column split is
+  // faster (Rastrigin 4096 x 49152: 942 -> 739 us/iteration, 4096 x 65536:
+  // 1073 -> 998; Griewank 8192 x 32768: 991 -> 937; at d = 16384 the 4-CTA
+  // cluster stays faster, 831 vs 934).  PSO_CLUSTER (tuning) keeps the cluster.
+  if (!colsplit && !o.nccl_comm && o.world <= 1 && d > PSO_D_AUTO_COLSPLIT && !std::getenv("PSO_CLUSTER"))
+    colsplit = true;
   if (colsplit && (o.flags & PSO_FLAG_ASYNC_GBEST))
     return fail(PSO_ERR_INVALID, "PSO_FLAG_COLUMN_SPLIT excludes PSO_FLAG_ASYNC_GBEST");
   if (!finite(w) || !finite(c1) || !finite(c2))

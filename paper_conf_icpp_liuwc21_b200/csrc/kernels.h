@@ -93,14 +93,14 @@ struct SwarmArgs {
 
 // Column split geometry (host plan and decide kernel).  The tiling depends on
 // d only, never on the world size: rows of nvec = ceil(d / 4) float4 are cut
-// into tiles of T = clamp(ceil(nvec / 64), 32, 512) float4 (the last one
+// into tiles of T = clamp(ceil(nvec / 8), 32, 512) float4 (the last one
 // ragged), and rank r of `world` owns tiles [floor(nt r / world),
 // floor(nt (r+1) / world)).  The partial of a tile and the combine order over
 // tiles are therefore the same for every world size, so fitness, decisions
 // and state are bitwise independent of it.
 constexpr int kColTileMax = 512, kColTileMin = 32;
 __host__ __device__ inline int col_tile(int nvec) {
-  int t = (nvec + 63) / 64;
+  int t = (nvec + 7) / 8;  // >= 8 tiles (8 ranks) from 256 float4 up, 8 KB tiles for wide rows
   t = t < kColTileMin ? kColTileMin : (t > kColTileMax ? kColTileMax : t);
   return t < nvec ? t : nvec;
 }

@@ -79,6 +79,8 @@ WORKLOADS = {
     # NEXT-3: rows wider than one CTA (d > 8192), split over a thread-block cluster
     "W64K": Workload("wide-rastrigin-4096x65536", RASTRIGIN, 4096, 65536, 200),
     "W16K": Workload("wide-griewank-16384x16384", GRIEWANK, 16384, 16384, 200),
+    # NEXT-3 beyond one cluster's row (d > 65536): the column split on one GPU
+    "W256K": Workload("wide-rastrigin-1024x262144", RASTRIGIN, 1024, 262144, 200),
     # one rank's shard of NS at 2 / 4 / 8 GPUs (rows floor(n r / k) ..), to time the
     # per-rank step on one GPU (with PSO_FORCE_EXCHANGE=1: the exchange path too)
     "NS_R2": Workload("northstar-shard-of-2-rastrigin-50000x2000", RASTRIGIN, 50_000, 2000, 500),

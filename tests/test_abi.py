@@ -25,6 +25,14 @@ def test_header_and_binding_agree():
     assert sorted(_lib.EXPORTS) == syms
 
 
+def test_header_limits_match_binding():
+    src = open(os.path.join(ROOT, "include", "fastpso.h")).read()
+    for name in ("PSO_D_MAX_ROW", "PSO_D_AUTO_COLSPLIT"):
+        m = re.search(r"#define\s+%s\s+(\d+)" % name, src)
+        assert m and int(m.group(1)) == getattr(_lib, name), name
+    assert re.search(r"#define\s+PSO_D_MAX\s+\(1 << 24\)", src) and _lib.PSO_D_MAX == 1 << 24
+
+
 def test_library_exports_every_declared_symbol():
     L = fp.lib()
     for s in header_symbols():

@@ -500,9 +500,13 @@ WIDE = [(5, 8193), (3, 10000), (4, 16384), (2, 65536)]
 
 @pytest.mark.parametrize("obj", [SPHERE, RASTRIGIN, ROSENBROCK, GRIEWANK, ACKLEY])
 @pytest.mark.parametrize("n,d", WIDE)
-def test_wide_rows_cluster_path(obj, n, d):
+def test_wide_rows_cluster_path(obj, n, d, monkeypatch):
     """d > 8192: each row is split in column blocks over a thread-block cluster
-    (DSMEM partials, CTA 0 decides); init bit-exact, one step bit-exact in X/V."""
+    (DSMEM partials, CTA 0 decides); init bit-exact, one step bit-exact in X/V.
+    Above PSO_D_AUTO_COLSPLIT a single GPU picks the column split, so the
+    cluster is requested there (PSO_CLUSTER)."""
+    if d > fp.PSO_D_AUTO_COLSPLIT:
+        monkeypatch.setenv("PSO_CLUSTER", "16")
     g = gpu_swarm(n, d, obj, seed=d + obj)
     assert g.info()["cluster"] >= 2
     c = cpu_swarm(n, d, obj, seed=d + obj)
@@ -512,6 +516,21 @@ def test_wide_rows_cluster_path(obj, n, d):
     assert_fitness_close(obj, c.X, pf, c.pf, "pf0")
     _step_and_compare(obj, n, d, seed=5000 + d, pf_mode="mixed", t0=2)
     _step_and_compare(obj, n, d, seed=5100 + d, pf_mode="inf", t0=0)
+
+
+@pytest.mark.parametrize("d", [16385, 40000, 65536])
+def test_single_gpu_wide_rows_pick_the_column_split(d):
+    """One GPU, d > PSO_D_AUTO_COLSPLIT: the column split is chosen (it beats
+    8- and 16-CTA clusters); results as the oracle's (init bit-exact, one step
+    bit-exact in X / V)."""
+    g = gpu_swarm(3, d, RASTRIGIN, seed=d)
+    assert g.info()["column_split"] == 1 and g.info()["cluster"] == 0
+    c = cpu_swarm(3, d, RASTRIGIN, seed=d)
+    X, V, PB, pf, _ = g.get_state()
+    assert_bitwise(X, c.X, "X0")
+    assert_bitwise(V, c.V, "V0")
+    _step_and_compare(RASTRIGIN, 3, d, seed=5200 + d, pf_mode="mixed", t0=2)
+    assert gpu_swarm(3, fp.PSO_D_AUTO_COLSPLIT, RASTRIGIN).info()["column_split"] == 0
 
 
 @pytest.mark.parametrize("C", [2, 4, 8, 16])
@@ -694,7 +713,7 @@ def test_async_gbest_single_rank_is_synchronous(monkeypatch):
 # ------------------------------------------------------------------ column split (NEXT-3)
 def _col_tiles(d):
     nv = (d + 3) // 4
-    t = min(max((nv + 63) // 64, 32), 512, nv)
+    t = min(max((nv + 7) // 8, 32), 512, nv)
     return -(-nv // t)
 
 
