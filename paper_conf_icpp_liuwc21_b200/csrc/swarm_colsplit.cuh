@@ -41,6 +41,7 @@ __device__ __forceinline__ float4* col_parts(unsigned char* region, const SwarmA
 }
 
 constexpr int kColCompute = 256;  // compute threads of k_col_step (+ producer + finaliser warps)
+static_assert(kColTileMax <= 2 * kColCompute, "k_col_step: at most 2 float4 of a tile per thread");
 
 template <class Obj, bool kB>
 __global__ void __launch_bounds__(kColCompute + 64, 2)
@@ -190,27 +191,44 @@ __global__ void __launch_bounds__(kColCompute + 64, 2)
     float4* xdst = fl ? st + 2 * chunk : st;  // keep the old x for the deferred pbest copy
     float acc[Obj::kAcc];
     Obj::init(acc);
-    for (int ql = tid; ql < cnt; ql += nthr) {
-      const int qg = a.col_q0 + q0 + ql;  // global float4: Philox counter, functor index
-      float4 x, v;
-      if (init) {
-        init_float4_at(a, key, gi, qg, B4, nvl, q0 + ql, x, v);
-      } else {
-        x = st[ql];
-        v = st[chunk + ql];
-        const float4 g = st[3 * chunk + ql];
-        move4_draw<kB>(mp, key, t, gi, (uint32_t)qg, fl, x, v, st + 2 * chunk + ql, g,
-                       st + 4 * chunk, chunk, ql);
-        if ((d & 3) && qg == a.nvec_glob - 1) {
-          const int jj = 4 * qg;
-          if (jj + 1 >= d) x.y = v.y = 0.f;
-          if (jj + 2 >= d) x.z = v.z = 0.f;
-          if (jj + 3 >= d) x.w = v.w = 0.f;
+    // a tile is at most 2 float4 per compute thread: two unrolled, independent
+    // slots (thread-sequential order over ql = tid, tid + nthr, as before); the
+    // init and step bodies are separate loops so neither carries the other's
+    // registers
+    if (init) {
+#pragma unroll
+      for (int j = 0; j < 2; ++j) {
+        const int ql = tid + j * nthr;
+        if (ql < cnt) {
+          const int qg = a.col_q0 + q0 + ql;  // global float4: Philox counter, functor index
+          float4 x, v;
+          init_float4_at(a, key, gi, qg, B4, nvl, q0 + ql, x, v);
+          xdst[ql] = x;
+          st[chunk + ql] = v;
+          if constexpr (!Obj::kNeighbor) map4<Obj>(acc, x, 0.f, 4 * qg, d);
         }
       }
-      xdst[ql] = x;
-      st[chunk + ql] = v;
-      if constexpr (!Obj::kNeighbor) map4<Obj>(acc, x, 0.f, 4 * qg, d);
+    } else {
+#pragma unroll
+      for (int j = 0; j < 2; ++j) {
+        const int ql = tid + j * nthr;
+        if (ql < cnt) {
+          const int qg = a.col_q0 + q0 + ql;
+          float4 x = st[ql], v = st[chunk + ql];
+          const float4 g = st[3 * chunk + ql];
+          move4_draw<kB>(mp, key, t, gi, (uint32_t)qg, fl, x, v, st + 2 * chunk + ql, g,
+                         st + 4 * chunk, chunk, ql);
+          if ((d & 3) && qg == a.nvec_glob - 1) {
+            const int jj = 4 * qg;
+            if (jj + 1 >= d) x.y = v.y = 0.f;
+            if (jj + 2 >= d) x.z = v.z = 0.f;
+            if (jj + 3 >= d) x.w = v.w = 0.f;
+          }
+          xdst[ql] = x;
+          st[chunk + ql] = v;
+          if constexpr (!Obj::kNeighbor) map4<Obj>(acc, x, 0.f, 4 * qg, d);
+        }
+      }
     }
     if constexpr (Obj::kNeighbor) {
       team_sync(nthr);  // every x' of the tile is in the stage
