@@ -2,13 +2,14 @@
 """FastPSO hot-path benchmark (BASELINE.json metric: particle-dim updates/sec and
 % of HBM roofline at 1/2/4/8 B200).
 
-    python bench.py [--gpus N] [--steps K] [--warmup W] [--workload NS|C1|C2|C3|C4|C5]
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--workload NS|C1..C5|W16K|W64K|W256K|NS_R8|...]
     python -m torch.distributed.run --nproc-per-node N ... bench.py --gpus N ...
     python bench.py --impl reference ...   # the CPU oracle on a bounded sample
 
 A "step" is one PSO iteration over the whole swarm: the fused kernel (move,
-evaluate, pbest, gbest) plus, for N > 1, the NCCL all-gather + select of the
-gbest exchange.  Default workload: the north_star swarm, Rastrigin 100,000
+evaluate, pbest, gbest); for N > 1 the same kernel also stores the rank's gbest
+record into every peer over NVLink and merges the peers' records of the
+previous iteration (PSO_EXCHANGE=nccl: an NCCL all-gather instead).  Default workload: the north_star swarm, Rastrigin 100,000
 particles x 2,000 dims (2.4 GB of fp32 state, larger than the 126 MB L2, so no
 L2 flush is needed between steps).  N > 1 splits the same swarm by particles
 (strong scaling).  Prints ONE JSON line on rank 0.
