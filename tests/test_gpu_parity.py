@@ -767,11 +767,15 @@ def test_column_split_lockstep_and_wide_rows(obj, n, d):
     assert info["launches"] >= 2 + 2 * 4
 
 
-def test_column_split_with_bounds_lockstep():
-    n, d, obj = 6, 6001, ROSENBROCK
+@pytest.mark.parametrize("n,d,forced", [(6, 6001, True), (3, 20001, False)])
+def test_column_split_with_bounds_lockstep(n, d, forced):
+    """Per-dimension bounds through the column split, forced (d = 6001) or
+    chosen automatically on one GPU (d > PSO_D_AUTO_COLSPLIT)."""
+    obj = ROSENBROCK
     b = _dim_bounds(d, 5)
     lo, hi = DOMAINS[obj]
-    g = fp.Swarm(n, d, 0.9, 2.0, 2.0, lo, hi, obj, 23, device=0, bounds=b, column_split=True)
+    g = fp.Swarm(n, d, 0.9, 2.0, 2.0, lo, hi, obj, 23, device=0, bounds=b, column_split=forced)
+    assert g.info()["column_split"] == 1 and g.info()["bounds"] == 1
     c = orc.OracleSwarm(n, d, 0.9, 2.0, 2.0, lo, hi, obj, 23, bounds=b)
     X, V, PB, pf, _ = g.get_state()
     assert_bitwise(X, c.X, "X0")
