@@ -44,6 +44,21 @@ __device__ __forceinline__ float sinpi_sq(float x) {
   return u * p;
 }
 
+// 20 sin^2(pi x), the Rastrigin term, with the 20 folded into the coefficients
+// of sinpi_sq (each rounded once to fp32): one multiply less per element,
+// <= 4 ulp relative (checked on a 4e5-point grid over r in [-1/2, 1/2]).
+__device__ __forceinline__ float sinpi_sq20(float x) {
+  const float r = x - rintf(x);
+  const float u = r * r;
+  float p = -66.71456909179688f;
+  p = fmaf(p, u, 260.7359313964844f);
+  p = fmaf(p, u, -601.9696044921875f);
+  p = fmaf(p, u, 854.5384521484375f);
+  p = fmaf(p, u, -649.3932495117188f);
+  p = fmaf(p, u, 197.39208984375f);
+  return u * p;
+}
+
 constexpr float kInv2Pi = 0.15915494309189535f;
 
 // Sphere: sum x_k^2.
@@ -63,7 +78,7 @@ struct Rastrigin {
   static constexpr bool kNeighbor = false;
   __device__ static void init(float* a) { a[0] = 0.f; }
   __device__ static void map(float* a, float x, float, int, int) {
-    a[0] += fmaf(x, x, 20.f * sinpi_sq(x));
+    a[0] += fmaf(x, x, sinpi_sq20(x));
   }
   __device__ static void combine(float* a, const float* b) { a[0] += b[0]; }
   __device__ static float finalize(const float* a, int) { return a[0]; }
