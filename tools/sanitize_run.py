@@ -1,18 +1,60 @@
-"""Small runs of every kernel variant, for compute-sanitizer (memcheck/racecheck/synccheck)."""
+"""Small runs of every kernel path, for compute-sanitizer (memcheck / racecheck / synccheck).
+
+Paths: register streaming and TMA pipeline (eager and lazy pbest rows, L2 prefetch, serpentine
+order), the CTA-resident and grid-resident latency kernels, the thread-block cluster, the column
+split (forced and automatic), per-dimension bounds, and the gbest exchange on a 1-rank NCCL
+communicator (records, merge in the next prologue, select kernel).
+"""
 import os
 import sys
 
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np  # noqa: E402
+
 import paper_conf_icpp_liuwc21_b200 as fp  # noqa: E402
 from synth import DOMAINS  # noqa: E402
 
-for kernel in ("reg", "tma"):
-    os.environ["PSO_KERNEL"] = kernel
-    for obj, n, d in ((2, 40, 1000), (3, 33, 999), (4, 20, 2000), (5, 7, 4096), (1, 5, 13)):
+
+def run(tag, obj, n, d, steps=3, env=None, **kw):
+    saved = {k: os.environ.get(k) for k in (env or {})}
+    os.environ.update(env or {})
+    try:
         lo, hi = DOMAINS[obj]
-        s = fp.Swarm(n, d, 0.9, 2.0, 2.0, lo, hi, obj, 7, device=0)
-        s.step(3)
+        s = fp.Swarm(n, d, 0.9, 2.0, 2.0, lo, hi, obj, 7, device=0, **kw)
+        s.step(steps)
         f, i, _ = s.gbest()
+        X, V, PB, pf, t = s.get_state()
         info = s.info()
-        print(kernel, obj, n, d, "tma" if info["tma_pipeline"] else "reg", f, i, flush=True)
+        path = ("colsplit" if info["column_split"] else "cluster" if info["cluster"] else
+                ["reg", "cta-resident", "grid-resident"][info["resident"]] if not info["tma_pipeline"]
+                else "tma")
+        print(f"{tag:14s} obj={obj} n={n} d={d} path={path} lazy={info['lazy_pb']} f={f:.6g} i={i} "
+              f"t={t}", flush=True)
         s.close()
+    finally:
+        for k, v in saved.items():
+            if v is None:
+                os.environ.pop(k, None)
+            else:
+                os.environ[k] = v
+
+
+for kernel in ("reg", "tma"):
+    for obj, n, d in ((2, 40, 1000), (3, 33, 999), (4, 20, 2000), (5, 7, 4096), (1, 5, 13)):
+        run(kernel, obj, n, d, env={"PSO_KERNEL": kernel, "PSO_RESIDENT": "0"})
+run("lazy+prefetch", 4, 300, 2000, steps=4, env={"PSO_RESIDENT": "0", "PSO_L2PF_ALL": "1"})
+run("cta-resident", 1, 32, 10, steps=10)
+run("grid-resident", 2, 256, 1000, steps=5)
+run("cluster", 3, 5, 12000, steps=3)
+run("cluster-C16", 4, 3, 40000, steps=2, env={"PSO_CLUSTER": "16"})
+run("colsplit-auto", 2, 3, 20001, steps=3)
+run("colsplit", 3, 9, 999, steps=3, column_split=True)
+b = np.stack([np.full(1000, -0.5, np.float32), np.full(1000, 0.5, np.float32),
+              np.full(1000, -3.0, np.float32), np.full(1000, 4.0, np.float32)])
+run("bounds", 2, 40, 1000, steps=3, bounds=b)
+comm = fp.nccl_comm_init(1, fp.nccl_unique_id(), 0, 0)
+try:
+    run("exchange-nccl", 2, 300, 1000, steps=3, env={"PSO_FORCE_EXCHANGE": "1"}, nccl_comm=comm)
+finally:
+    fp.nccl_comm_destroy(comm)
+print("sanitize_run done", flush=True)
