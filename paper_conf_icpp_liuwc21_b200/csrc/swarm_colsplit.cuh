@@ -55,6 +55,9 @@ __global__ void __launch_bounds__(kColCompute + 64, 2)
   __shared__ float red[kMaxStages][nwarps * 2];
   __shared__ unsigned long long full[kMaxStages], empty[kMaxStages], done[kMaxStages];
   __shared__ int sflag[kMaxStages];
+  // the tile's first and last x' for the neighbour terms across tiles, handed to
+  // the finaliser by the arriving lanes themselves (ordered by their own release)
+  __shared__ float s_edge[kMaxStages][2];
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   if (tid == 0) {
     for (int s = 0; s < stages; ++s) {
@@ -129,8 +132,7 @@ __global__ void __launch_bounds__(kColCompute + 64, 2)
         const float4* st = ring + (size_t)s * per * chunk;
         const int fl = sflag[s];
         const float4* xnew = fl ? st + 2 * chunk : st;  // where the compute warps put x'
-        const float4 msg =
-            make_float4(c[0], Obj::kAcc > 1 ? c[Obj::kAcc - 1] : 0.f, xnew[0].x, xnew[cnt - 1].w);
+        const float4 msg = make_float4(c[0], Obj::kAcc > 1 ? c[Obj::kAcc - 1] : 0.f, s_edge[s][0], s_edge[s][1]);
         const size_t pidx = (size_t)r * a.col_nbt + (size_t)(a.col_bbase + b);
         if (a.world > 1) {
           for (int q = 0; q < a.world; ++q) col_parts<Obj>(a.peers[q], a, par)[pidx] = msg;
@@ -191,6 +193,7 @@ __global__ void __launch_bounds__(kColCompute + 64, 2)
     float4* xdst = fl ? st + 2 * chunk : st;  // keep the old x for the deferred pbest copy
     float acc[Obj::kAcc];
     Obj::init(acc);
+    float e_first = 0.f, e_last = 0.f;  // x' of the tile's first / last float4 (owners only)
     // a tile is at most 2 float4 per compute thread: two unrolled, independent
     // slots (thread-sequential order over ql = tid, tid + nthr, as before); the
     // init and step bodies are separate loops so neither carries the other's
@@ -203,6 +206,8 @@ __global__ void __launch_bounds__(kColCompute + 64, 2)
           const int qg = a.col_q0 + q0 + ql;  // global float4: Philox counter, functor index
           float4 x, v;
           init_float4_at(a, key, gi, qg, B4, nvl, q0 + ql, x, v);
+          if (ql == 0) e_first = x.x;
+          if (ql == cnt - 1) e_last = x.w;
           xdst[ql] = x;
           st[chunk + ql] = v;
           if constexpr (!Obj::kNeighbor) map4<Obj>(acc, x, 0.f, 4 * qg, d);
@@ -224,6 +229,8 @@ __global__ void __launch_bounds__(kColCompute + 64, 2)
             if (jj + 2 >= d) x.z = v.z = 0.f;
             if (jj + 3 >= d) x.w = v.w = 0.f;
           }
+          if (ql == 0) e_first = x.x;
+          if (ql == cnt - 1) e_last = x.w;
           xdst[ql] = x;
           st[chunk + ql] = v;
           if constexpr (!Obj::kNeighbor) map4<Obj>(acc, x, 0.f, 4 * qg, d);
@@ -247,6 +254,12 @@ __global__ void __launch_bounds__(kColCompute + 64, 2)
       }
     }
     warp_combine<Obj>(acc);
+    {  // ql = 0 is thread 0 (lane 0 of warp 0); ql = cnt - 1 is thread (cnt - 1) % nthr
+      const int lt = (cnt - 1) % nthr;
+      const float el = __shfl_sync(kFull, e_last, lt & 31);
+      if (lane == 0 && warp == (lt >> 5)) s_edge[s][1] = el;
+      if (tid == 0) s_edge[s][0] = e_first;
+    }
     if (lane == 0) {
 #pragma unroll
       for (int j = 0; j < Obj::kAcc; ++j) red[s][warp * Obj::kAcc + j] = acc[j];
