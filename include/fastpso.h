@@ -54,7 +54,9 @@ extern "C" {
 #define FASTPSO_VERSION_MAJOR 0
 #define FASTPSO_VERSION_MINOR 1
 #define PSO_D_MAX_ROW 65536 /* max dimension of the row kernels: <= 8192 one CTA per row;
-                              above, a thread-block cluster of up to 16 CTAs per row */
+                              above, a thread-block cluster of up to 16 CTAs per row (a
+                              single GPU switches to the column split above
+                              PSO_D_AUTO_COLSPLIT) */
 #define PSO_D_MAX (1 << 24) /* max dimension: above PSO_D_MAX_ROW the column split
                               (PSO_FLAG_COLUMN_SPLIT) is used on a single GPU */
 #define PSO_D_AUTO_COLSPLIT 16384 /* a single-GPU handle (no communicator, world <= 1)
