@@ -314,14 +314,17 @@ def test_errors_do_not_abort():
 
 
 # ------------------------------------------------------------------ full size, sampled
-@pytest.mark.parametrize("key", ["NS", "C4", "C3", "C2"])
+@pytest.mark.parametrize("key", ["NS", "C4", "C3", "C2", "W16K", "W64K", "C5@40000"])
 def test_full_size_sampled_rows(key):
     """Bench configurations at full size in the bench's launch shape (NS / C4
     streaming 100k x 2000, C3 streaming with a neighbour functor, C2 on the
-    grid-resident path): the
+    grid-resident path, W16K on 4-CTA clusters, W64K on the automatic column
+    split; C5's wide 16-warp instantiation at d = 4096 with n cut to 40,000 --
+    the launch shape depends on d only -- so the host copies stay ~2 GB): the
     oracle recomputes sampled rows of one iteration exactly (rows are
     independent given G), and the gbest invariants hold over the whole swarm."""
-    w = WORKLOADS[key]
+    name, _, n_cut = key.partition("@")
+    w = WORKLOADS[name].with_(n=int(n_cut)) if n_cut else WORKLOADS[name]
     g = gpu_swarm(w.n, w.d, w.objective, seed=w.seed)
     idx = sample_rows(w.n, 48, seed=7)
     X0, V0, _, _, _ = g.get_state()
