@@ -336,24 +336,37 @@ def run_gpu(args, w):
         pf = torch.empty((n_local,), dtype=torch.float32).pin_memory()
         _, _, _, _, t_ck = sw.get_state(out=(X, V, PB, pf))  # a host checkpoint of the swarm
         sw.close()
-        sw2, _ = make_swarm()
         gpos = torch.empty((w.d,), dtype=torch.float32).pin_memory()
-        with ClockSampler(local) as clk2:
-            barrier()
-            t0 = time.perf_counter()
-            sw2.set_state(X, V, PB, pf, t=t_ck)  # H2D of the whole swarm state
-            sw2.step(K)
-            res = sw2.gbest(out=gpos)            # D2H of the result (synchronises)
-            barrier()
-            e2e_s = max_over_ranks(time.perf_counter() - t0)
-        clk_e2e = clk2.result
-        sw2.close()
+
+        def e2e_run(per_step: bool):
+            s2, _ = make_swarm()
+            with ClockSampler(local) as ck:
+                barrier()
+                t0 = time.perf_counter()
+                s2.set_state(X, V, PB, pf, t=t_ck)  # H2D of the whole swarm state
+                if per_step:  # every step: pso_step(1) + D2H of its result (gbest fitness, index)
+                    for _ in range(K):
+                        s2.step(1)
+                        s2.gbest(pos=False)
+                else:
+                    s2.step(K)
+                r = s2.gbest(out=gpos)  # D2H of the final gbest position (synchronises)
+                barrier()
+                sec = max_over_ranks(time.perf_counter() - t0)
+            s2.close()
+            return sec, r, ck.result
+
+        e2e_s, res, clk_e2e = e2e_run(per_step=True)
+        batched_s, _, _ = e2e_run(per_step=False)
         h2d = 3 * n_local * w.d * 4 + n_local * 4
-        d2h = 4 + 8 + 4 * w.d
+        d2h = K * (4 + 8) + 4 * w.d
         e2e = {"value": total_updates / e2e_s, "unit": UNIT,
                "h2d_bytes_per_step": h2d / K, "d2h_bytes_per_step": d2h / K,
                "seconds": e2e_s,
-               "path": "pso_set_state(pinned host X,V,PB,pf) + pso_step(K) + pso_get_gbest(pinned host)",
+               "path": ("pso_set_state(pinned host X,V,PB,pf) once, then per step pso_step(1) + "
+                        "pso_get_gbest (fitness, index to host), then pso_get_gbest(position)"),
+               "batched": {"value": total_updates / batched_s, "seconds": batched_s,
+                           "path": "pso_set_state + pso_step(K) + pso_get_gbest(position)"},
                "gbest": res[0]}
     else:
         sw.close()
