@@ -17,6 +17,11 @@
 //   optional:
 //   __device__ static void  map4(float* a, float4 x, float xnext, int j, int d);
 //                                      // == map over dims j..j+3 (all < d), same bits
+//   static constexpr bool kRowTable;   // with table4 / map4r: per-dimension factors
+//   __device__ static float4 table4(int j);          // computed once per kernel (the
+//   __device__ static void  map4r(float* a, float4 x, int d, const float4& t);
+//                                      // TMA kernel's threads own fixed dims); map4r
+//                                      // with t = table4(j) == map4 at j, same bits
 //
 // The reduction order is fixed by the launch shape, which depends only on d,
 // so fitness bits do not depend on the grid or on the number of GPUs.
@@ -115,10 +120,26 @@ struct Griewank {
     asm("rsqrt.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(k));
     return r;
   }
-  __device__ static void term(float* a, float x, float k) {
+  __device__ static void term_r(float* a, float x, float r) {  // r = rsqrt_k(k)
     a[0] = fmaf(x, x, a[0]);
-    const float y = x * rsqrt_k(k);  // x_k / sqrt(k)
+    const float y = x * r;  // x_k / sqrt(k)
     a[1] *= fmaf(-2.f, sinpi_sq(y * kInv2Pi), 1.f);  // cos(y)
+  }
+  __device__ static void term(float* a, float x, float k) { term_r(a, x, rsqrt_k(k)); }
+  // Row-invariant per-dimension factors: a streaming kernel whose threads own
+  // the same dims in every row computes rsqrt(k) once per kernel (table4) and
+  // maps with them (map4r) -- the same bits as map4, one MUFU + one add fewer
+  // per element.
+  static constexpr bool kRowTable = true;
+  __device__ static float4 table4(int j) {
+    const float k = (float)(j + 1);
+    return make_float4(rsqrt_k(k), rsqrt_k(k + 1.f), rsqrt_k(k + 2.f), rsqrt_k(k + 3.f));
+  }
+  __device__ static void map4r(float* a, float4 x, int, const float4& r) {
+    term_r(a, x.x, r.x);
+    term_r(a, x.y, r.y);
+    term_r(a, x.z, r.z);
+    term_r(a, x.w, r.w);
   }
   __device__ static void map(float* a, float x, float, int j, int) { term(a, x, (float)(j + 1)); }
   // Four consecutive dims j..j+3 (j + 4 <= d <= 2^24): (float)(j + 1 + m) ==

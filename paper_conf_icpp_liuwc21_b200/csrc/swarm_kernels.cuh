@@ -34,6 +34,7 @@
 #include <cuda_runtime.h>
 
 #include <cstdint>
+#include <type_traits>
 
 #include "kernels.h"
 #include "objectives.cuh"
@@ -405,6 +406,11 @@ __device__ __forceinline__ float cta_fitness(float* a, RowSmem<Obj>& sm, int d, 
 }
 
 // Map one float4 of new positions (dims j..j+3; nx = x_{j+4} for neighbours).
+template <class Obj, class = void>
+struct HasRowTable : std::false_type {};
+template <class Obj>
+struct HasRowTable<Obj, std::enable_if_t<Obj::kRowTable>> : std::true_type {};
+
 template <class Obj, class = void>
 struct HasMap4 {
   static constexpr bool value = false;
@@ -1031,6 +1037,16 @@ __global__ void __launch_bounds__(kMaxT + 64, kMaxT > kMaxThreads ? 1 : 2)
   // ---------------- compute warps
   const PhiloxRoundKeys& key = a.rk;
   const MoveParams mp = move_params(a);
+  // row-invariant functor factors of this thread's float4 slots (VPT <= 2: registers)
+  constexpr bool kTab = HasRowTable<Obj>::value && !Obj::kNeighbor && VPT <= 2;
+  float4 rtab[VPT];
+  if constexpr (kTab) {
+#pragma unroll
+    for (int j = 0; j < VPT; ++j) {
+      const int q = tid + j * nthr;
+      rtab[j] = q < nvec ? Obj::table4(4 * q) : make_float4(0.f, 0.f, 0.f, 0.f);
+    }
+  }
   mbar_wait(&gbar, 0);
   int s = 0;
   unsigned ph = 0;
@@ -1061,7 +1077,10 @@ __global__ void __launch_bounds__(kMaxT + 64, kMaxT > kMaxThreads ? 1 : 2)
         }
         xdst[q] = x;
         st[nvec + q] = v;
-        if constexpr (!Obj::kNeighbor) map4<Obj>(acc, x, 0.f, 4 * q, d);
+        if constexpr (kTab)
+          Obj::map4r(acc, x, d, rtab[j]);
+        else if constexpr (!Obj::kNeighbor)
+          map4<Obj>(acc, x, 0.f, 4 * q, d);
       }
     }
     if constexpr (Obj::kNeighbor) {
