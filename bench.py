@@ -154,16 +154,39 @@ def oracle_sample(w, budget_s: float, steps_hint: int | None = None):
     return s, rows, k
 
 
+class _PinnedCore:
+    """Pin this process to one host core while the oracle is timed (the
+    oracle runs single-threaded on one core of the GPU box's host); restored after."""
+
+    def __enter__(self):
+        self.core, self.saved = None, None
+        try:
+            self.saved = os.sched_getaffinity(0)
+            self.core = max(self.saved)
+            os.sched_setaffinity(0, {self.core})
+        except (AttributeError, OSError):
+            self.core = None
+        return self
+
+    def __exit__(self, *exc):
+        if self.saved:
+            try:
+                os.sched_setaffinity(0, self.saved)
+            except OSError:
+                pass
+
+
 def cpu_baseline(w, budget_s: float):
-    s, rows, k = oracle_sample(w, budget_s)
-    t0 = time.perf_counter()
-    s.step(k)
-    dt = time.perf_counter() - t0
+    with _PinnedCore() as pin:
+        s, rows, k = oracle_sample(w, budget_s)
+        t0 = time.perf_counter()
+        s.step(k)
+        dt = time.perf_counter() - t0
     rate = rows * w.d * k / dt
     return {"value": rate, "unit": UNIT, "cores": 1, "kind": "oracle",
             "sample": f"oracle (single-threaded C++ -O3 -ffp-contract=off) on the first {rows} of "
                       f"{w.n} particles x {w.d} dims, {k} iterations ({dt:.1f} s), create excluded",
-            "host_cpu": _cpu_model()}
+            "host_cpu": _cpu_model(), "pinned_core": pin.core}
 
 
 def _cpu_model():
@@ -183,11 +206,12 @@ def run_reference(args, w):
         return 0
     K, W = args.steps, args.warmup
     budget = args.ref_seconds  # whole --steps K --warmup W run
-    s, rows, _ = oracle_sample(w, budget / max(K + W, 1), steps_hint=1)
-    s.step(W)
-    t0 = time.perf_counter()
-    s.step(K)
-    dt = time.perf_counter() - t0
+    with _PinnedCore() as pin:
+        s, rows, _ = oracle_sample(w, budget / max(K + W, 1), steps_hint=1)
+        s.step(W)
+        t0 = time.perf_counter()
+        s.step(K)
+        dt = time.perf_counter() - t0
     rate = rows * w.d * K / dt
     sample = (f"oracle (single-threaded C++ -O3 -ffp-contract=off) on the first {rows} of {w.n} "
               f"particles x {w.d} dims; {W} warm-up + {K} timed iterations ({dt:.1f} s)")
@@ -197,7 +221,7 @@ def run_reference(args, w):
         "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f32",
         "data": "synthetic", "config": _config(w, args.gpus, K, extra={"sample_rows": rows}),
         "cpu_baseline": {"value": rate, "unit": UNIT, "cores": 1, "kind": "oracle",
-                         "sample": sample, "host_cpu": _cpu_model()},
+                         "sample": sample, "host_cpu": _cpu_model(), "pinned_core": pin.core},
         "e2e": {"value": rate, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)
