@@ -40,6 +40,10 @@
 #include "objectives.cuh"
 #include "philox.cuh"
 
+#ifndef PSO_SLOT_PHILOX
+#define PSO_SLOT_PHILOX 1
+#endif
+
 namespace fastpso {
 namespace {
 
@@ -344,6 +348,32 @@ __device__ __forceinline__ void move4_draw(const MoveParams& m, const K& key, ui
     const float4 pb = *pbs;
     const float4 r1 = raw24x4(key, kTagR1, t, gi, q);
     const float4 r2 = raw24x4(key, kTagR2, t, gi, q);
+    move4<kB>(m, x, v, pb, g, r1, r2, sB, nb, qb);
+  }
+}
+
+// move4_draw with the row-independent Philox rounds precomputed per thread
+// slot (philox.cuh PhiloxSlot): the same draws bit for bit.
+template <bool kB, class K>
+__device__ __forceinline__ void move4_draw_slot(const MoveParams& m, const K& key, const PhiloxIter& it,
+                                                const PhiloxSlot& s1, const PhiloxSlot& s2,
+                                                uint32_t gi, int fl, float4& x, float4& v,
+                                                const float4* pbs, const float4& g, const float4* sB,
+                                                int nb, int qb) {
+  uint32_t lo0r1, hi1r2, lo1r2;
+  philox_row_shared(it, s2, gi, lo0r1, hi1r2, lo1r2);
+  const float4 r2 = raw24x4(philox_slot_row(key, s2, lo0r1, hi1r2, lo1r2));
+  if (fl) {
+    const float bz = copysignf(0.f, m.c1s);
+    float4 ab;
+    ab.x = __fadd_rn(__fmul_rn(m.w, v.x), bz);
+    ab.y = __fadd_rn(__fmul_rn(m.w, v.y), bz);
+    ab.z = __fadd_rn(__fmul_rn(m.w, v.z), bz);
+    ab.w = __fadd_rn(__fmul_rn(m.w, v.w), bz);
+    move_post4<kB>(m, x, v, g, r2, ab, sB, nb, qb);
+  } else {
+    const float4 pb = *pbs;
+    const float4 r1 = raw24x4(philox_slot_row(key, s1, lo0r1, hi1r2, lo1r2));
     move4<kB>(m, x, v, pb, g, r1, r2, sB, nb, qb);
   }
 }
@@ -1047,6 +1077,20 @@ __global__ void __launch_bounds__(kMaxT + 64, kMaxT > kMaxThreads ? 1 : 2)
       rtab[j] = q < nvec ? Obj::table4(4 * q) : make_float4(0.f, 0.f, 0.f, 0.f);
     }
   }
+  // row-invariant Philox rounds of this thread's slots (VPT <= 2: registers)
+  // Only in the wide (512-thread, 1 CTA/SM) instantiation: C5 12.62 -> 12.36 ms; in the
+  // 256-thread one it cost NS 618 -> 623 us and Rosenbrock 11 registers (A/B of two builds)
+  constexpr bool kSlotRng = PSO_SLOT_PHILOX && VPT <= 2 && !Obj::kNeighbor && (kMaxT > kMaxThreads);
+  const PhiloxIter pit = philox_iter(key, t);
+  PhiloxSlot ps1[VPT], ps2[VPT];
+  if constexpr (kSlotRng) {
+#pragma unroll
+    for (int j = 0; j < VPT; ++j) {
+      const uint32_t q = (uint32_t)(tid + j * nthr);
+      ps1[j] = philox_slot(key, pit, q, kTagR1);
+      ps2[j] = philox_slot(key, pit, q, kTagR2);
+    }
+  }
   mbar_wait(&gbar, 0);
   int s = 0;
   unsigned ph = 0;
@@ -1068,7 +1112,10 @@ __global__ void __launch_bounds__(kMaxT + 64, kMaxT > kMaxThreads ? 1 : 2)
       if (q < nvec) {
         float4 x = st[q], v = st[nvec + q];
         const float4 g = sG[q];
-        move4_draw<kB>(mp, key, t, gi, (uint32_t)q, fl, x, v, st + 2 * nvec + q, g, sB, nvec, q);
+        if constexpr (kSlotRng)
+          move4_draw_slot<kB>(mp, key, pit, ps1[j], ps2[j], gi, fl, x, v, st + 2 * nvec + q, g, sB, nvec, q);
+        else
+          move4_draw<kB>(mp, key, t, gi, (uint32_t)q, fl, x, v, st + 2 * nvec + q, g, sB, nvec, q);
         if ((d & 3) && q == nvec - 1) {  // keep the row padding at zero
           const int jj = 4 * q;
           if (jj + 1 >= d) x.y = v.y = 0.f;
