@@ -70,13 +70,19 @@ def _path_name(info) -> str:
 
 
 def ncu_traffic(workload_name):
-    """DRAM bytes per launch of the step kernel from the committed ncu --set full summary."""
+    """(DRAM bytes per launch of the step kernel, where that number comes from):
+    the committed ncu --set full summary, NOT a measurement of this run (a run
+    under ncu is never a bench run)."""
     p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     try:
         with open(p) as fh:
-            return json.load(fh).get(workload_name)
+            j = json.load(fh)
     except Exception:
-        return None
+        return None, None
+    v = j.get(workload_name)
+    if v is None:
+        return None, None
+    return v, "committed ncu capture, not this run: profiles/ncu_traffic.json (" + j.get("_source", "") + ")"
 
 
 # ------------------------------------------------------------------ clocks
@@ -271,6 +277,9 @@ def run_gpu(args, w):
     if share:
         dist.init_process_group("gloo")
     elif use_comm:
+        if world > 1:  # the communicator setup of every rank stays visible on stderr
+            os.environ.setdefault("NCCL_DEBUG", "INFO")
+            os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
         dist.init_process_group("nccl", device_id=dev)
         comm = init_comm(local)
 
@@ -314,6 +323,13 @@ def run_gpu(args, w):
     # iteration late); default synchronous (bitwise independent of N)
     async_gbest = use_comm and os.environ.get("PSO_GBEST", "sync") == "async"
     sw, p2p = make_swarm(timing=True)
+    # NCCL exchange (fallback): the timed run replays the library's captured
+    # [step, all-gather] graphs, which carry no timing events; the step kernel's
+    # own duration is then measured on a second handle with per-launch events.
+    graphs = use_comm and not p2p and not share
+    if graphs:
+        sw.close()
+        sw, _ = make_swarm(timing=False)
     sw.step(W)
     sw.synchronize()
     sw.reset_counters()
@@ -328,6 +344,12 @@ def run_gpu(args, w):
         barrier()
     ms = max_over_ranks(ev0.elapsed_time(ev1))
     info = sw.info()
+    if graphs:
+        tk, _ = make_swarm(timing=True)
+        tk.step(min(K, 100))
+        ti = tk.info()
+        info["step_kernel_ms"], info["step_kernel_count"] = ti["step_kernel_ms"], ti["step_kernel_count"]
+        tk.close()
     kern_ms = max_over_ranks(info["step_kernel_ms"] / max(info["step_kernel_count"], 1))
     launches = int(info["launches"])
     improvements = info["improvements"]
@@ -348,6 +370,9 @@ def run_gpu(args, w):
     bytes_per_update = 16.0 + 4.0 * pbl + 4.0 * pbs
     alg_bytes = n_local * w.d * bytes_per_update + n_local * (4.0 + 4.0 * rho)
     achieved = alg_bytes / (kern_ms / 1e3) / 1e9
+    # (20 + 4 rho + 8/d) B per update, pbest read for every row
+    survey_gbs = n_local * w.d * (20.0 + 4.0 * rho + 8.0 / w.d) / (kern_ms / 1e3) / 1e9
+    traffic, traffic_src = ncu_traffic(w.name)
     peak, peak_src = hbm_peak()
 
     # ---------------- end to end through the public API, host buffers
@@ -409,14 +434,17 @@ def run_gpu(args, w):
             "scaling": "strong", "vs_baseline": None, "dtype": "f32",
             "data": "synthetic (swarm initialised from Philox streams, seed %d)" % w.seed,
             "config": _config(w, world, K, extra={"gbest_exchange": (
-                "nvlink-peer-stores" if p2p else "nccl-allgather") if use_comm else None,
+                "nvlink-peer-stores" if p2p else "nccl-allgather (CUDA graph)") if use_comm else None,
                 "gbest_mode": ("async" if async_gbest else "sync") if use_comm else None,
                 **({"shared_gpu_harness_test": True} if share else {})}),
             "gpu_launches": launches,
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "peak_source": peak_src,
                          "frac_of_spec": achieved / SPEC_HBM_GBS,  # vs the 8 TB/s data-sheet figure
-                         "traffic": ncu_traffic(w.name),
+                         "traffic": traffic, "traffic_source": traffic_src,
+                         # SURVEY 8(d)'s accounting: every pbest row read, 4 rho written
+                         "frac_survey_formula": survey_gbs / peak,
+                         "achieved_survey_formula": survey_gbs,
                          "kernel": ("k_col_step (fused move+eval, tile partials; k_col_decide "
                                     "takes the pbest/gbest decisions)" if info["column_split"]
                                     else "k_step (fused move+eval+pbest+gbest)"),
@@ -442,8 +470,33 @@ def run_gpu(args, w):
     return 0
 
 
+def _free_port() -> int:
+    import socket
+    with socket.socket() as sk:
+        sk.bind(("127.0.0.1", 0))
+        return sk.getsockname()[1]
+
+
+def self_launch(args) -> int:
+    """`python bench.py --gpus N` (N > 1) outside torchrun: re-run this script
+    as N ranks (one process per GPU) through torch.distributed.run on
+    127.0.0.1; rank 0 prints the one JSON line.  NCCL's init lines stay on
+    stderr (NCCL_DEBUG=INFO, INIT subsystem) so every rank's communicator
+    setup is visible."""
+    env = dict(os.environ)
+    env.setdefault("NCCL_DEBUG", "INFO")
+    env.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1",
+           f"--nproc-per-node={args.gpus}", "--master-addr", "127.0.0.1",
+           f"--master-port={_free_port()}", os.path.abspath(__file__)] + sys.argv[1:]
+    print("[bench] launching %d ranks: %s" % (args.gpus, " ".join(cmd)), file=sys.stderr, flush=True)
+    return subprocess.run(cmd, env=env).returncode
+
+
 def main():
     args = parse()
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        return self_launch(args)
     w = WORKLOADS[args.workload]
     if args.impl == "reference":
         return run_reference(args, w)

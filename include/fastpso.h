@@ -111,6 +111,9 @@ enum {
                               world = 1 identical to the synchronous mode.
                               pso_get_gbest returns the global view folded from every
                               rank's records at the end of the last pso_step call. */
+  PSO_FLAG_DEVICE = 16,     /* use pso_opts.device as the CUDA ordinal; without it the
+                              handle runs on the caller's current device (so a
+                              zero-initialised pso_opts means "defaults") */
   PSO_FLAG_COLUMN_SPLIT = 8 /* NEXT-3, "tile matrix": every rank holds ALL n
                               particles but only a block of the columns.  Rows are cut
                               into column tiles of T = clamp(ceil(nv / 8), 32, 512)
@@ -135,8 +138,8 @@ enum {
 /* Options; a zero-initialised struct means "defaults". */
 typedef struct {
   float vmax;      /* Eq. 5 bound |v| <= vmax; <= 0 -> 1.0 (reading 3) */
-  int32_t device;  /* CUDA ordinal; < 0 -> the caller's current device.  NOTE:
-                      zero-initialised means device 0 unless set to -1 */
+  int32_t device;  /* CUDA ordinal, read only with PSO_FLAG_DEVICE (else the
+                      caller's current device is used) */
   void* stream;    /* cudaStream_t to enqueue on; NULL -> a library-owned stream */
   void* nccl_comm; /* ncclComm_t (see pso_nccl_comm_init); NULL -> single GPU */
   uint32_t flags;  /* PSO_FLAG_* */
@@ -180,8 +183,19 @@ pso_status pso_init(pso_handle h);
 
 /* Enqueue iters >= 0 iterations; each is one fused kernel: move (Eq. 1, 5,
  * 2), evaluate (Sec 3.2), pbest (Sec 3.3, strict <) and gbest (strict <,
- * lowest index among equal new minima).  With world > 1 each iteration adds
- * one NCCL all-gather of (key, candidate row) and a select kernel. */
+ * lowest index among equal new minima).  Tiny and shared-memory-sized swarms
+ * on one GPU run the whole call as one launch (pso_info.resident).
+ * world > 1 (particle split): with the NVLink exchange (pso_p2p_*)
+ * the same kernel stores the rank's (key, candidate row) record into every
+ * rank over NVLink and the next iteration's kernel merges them, so an
+ * iteration is still one kernel; one select kernel per call folds the last
+ * records for the host.  With the NCCL fallback each iteration adds an
+ * ncclAllGather of the records (runs of 4 iterations are replayed as a
+ * captured CUDA graph).  A rank without particles runs a one-warp record
+ * kernel per iteration instead of the step kernel.  The column split
+ * (PSO_FLAG_COLUMN_SPLIT) runs two kernels per iteration.
+ * PSO_ERR_UNSUPPORTED if the iteration counter would reach 2^32 (it is the
+ * 32-bit Philox counter word t). */
 pso_status pso_step(pso_handle h, int64_t iters);
 
 /* Wait for all enqueued work and report asynchronous errors. */
@@ -278,6 +292,13 @@ pso_status pso_nccl_comm_destroy(void* comm);
 pso_status pso_p2p_handle(pso_handle h, void* ipc_handle /* 64 bytes */, uint64_t* offset);
 pso_status pso_p2p_connect(pso_handle h, const void* ipc_handles /* world x 64 bytes */,
                            const uint64_t* offsets /* world */);
+/* Probe the mapped data path before enabling it (collective, two phases with a
+ * host barrier between them): phase 0 stores this rank's token into its slot of
+ * every rank's probe area with a system-scope release; phase 1 acquires our own
+ * slots and sets *ok = 1 if every rank's token arrived (then clears them).  A
+ * connected but non-working mapping is caught here rather than by the 60 s
+ * trap of the first step kernel. */
+pso_status pso_p2p_probe(pso_handle h, int32_t phase, int32_t* ok);
 pso_status pso_p2p_enable(pso_handle h, int32_t on); /* 1: NVLink records, 0: NCCL all-gather */
 
 /* --- Device-side primitives exposed for parity tests ---------------------- */

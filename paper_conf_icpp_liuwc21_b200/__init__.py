@@ -11,8 +11,8 @@ import ctypes as C
 
 import numpy as np
 
-from ._lib import (EXPORTS, PSO_D_AUTO_COLSPLIT, PSO_D_MAX, PSO_D_MAX_ROW, PSO_FLAG_ASYNC_GBEST, PSO_FLAG_COLUMN_SPLIT,
-                   PSO_FLAG_DEFER_INIT, PSO_FLAG_TIMING, PSO_OBJ_ACKLEY, PSO_OBJ_CUSTOM_BASE,
+from ._lib import (EXPORTS, PSO_D_AUTO_COLSPLIT, PSO_D_MAX, PSO_D_MAX_ROW, PSO_FLAG_ASYNC_GBEST,
+                   PSO_FLAG_COLUMN_SPLIT, PSO_FLAG_DEFER_INIT, PSO_FLAG_DEVICE, PSO_FLAG_TIMING, PSO_OBJ_ACKLEY, PSO_OBJ_CUSTOM_BASE,
                    PSO_OBJ_EASOM, PSO_OBJ_GRIEWANK, PSO_OBJ_RASTRIGIN, PSO_OBJ_ROSENBROCK,
                    PSO_OBJ_SPHERE, PSO_OK, PsoError, check, last_error, lib, pso_info, pso_opts,
                    status_string)
@@ -27,19 +27,34 @@ __all__ = [
 ]
 
 
-def _ptr(a, dtype=np.float32, writable=False):
-    """Raw host pointer of a C-contiguous numpy array or CPU torch tensor (or None)."""
+def _ptr(a, count=None, writable=False, dtype=np.float32):
+    """Raw host pointer of a C-contiguous numpy array or CPU torch tensor (or None).
+
+    The library reads or writes exactly ``count`` elements of ``dtype`` behind
+    the pointer, so both the element type and the element count are checked
+    here (a float16 or undersized output would be a host heap overflow, a
+    float64 input would be silently reinterpreted)."""
     if a is None:
         return None
     if hasattr(a, "data_ptr"):  # torch.Tensor
+        import torch
+        want = {np.dtype(np.float32): torch.float32}[np.dtype(dtype)]
         if a.device.type != "cpu" or not a.is_contiguous():
             raise ValueError("host tensors must be contiguous CPU tensors")
-        return C.c_void_p(a.data_ptr())
-    if not isinstance(a, np.ndarray) or a.dtype != dtype or not a.flags.c_contiguous:
-        raise ValueError(f"expected a C-contiguous numpy {np.dtype(dtype).name} array")
-    if writable and not a.flags.writeable:
-        raise ValueError("output array is read-only")
-    return C.c_void_p(a.ctypes.data)
+        if a.dtype != want:
+            raise ValueError(f"expected a {want} tensor, got {a.dtype}")
+        size = a.numel()
+        ptr = a.data_ptr()
+    else:
+        if not isinstance(a, np.ndarray) or a.dtype != dtype or not a.flags.c_contiguous:
+            raise ValueError(f"expected a C-contiguous numpy {np.dtype(dtype).name} array")
+        if writable and not a.flags.writeable:
+            raise ValueError("output array is read-only")
+        size = a.size
+        ptr = a.ctypes.data
+    if count is not None and size != count:
+        raise ValueError(f"buffer holds {size} elements, the call needs exactly {count}")
+    return C.c_void_p(ptr)
 
 
 def objective_registered(obj: int) -> bool:
@@ -57,13 +72,14 @@ class Swarm:
         L = lib()
         opts = pso_opts()
         opts.vmax = float(vmax)
-        opts.device = int(device)
+        opts.device = int(device) if device >= 0 else 0  # < 0: the current device
         if stream is not None:
             opts.stream = int(getattr(stream, "cuda_stream", stream))
         opts.nccl_comm = nccl_comm
         opts.flags = ((PSO_FLAG_TIMING if timing else 0) | (PSO_FLAG_DEFER_INIT if defer_init else 0)
                       | (PSO_FLAG_ASYNC_GBEST if async_gbest else 0)
-                      | (PSO_FLAG_COLUMN_SPLIT if column_split else 0))
+                      | (PSO_FLAG_COLUMN_SPLIT if column_split else 0)
+                      | (PSO_FLAG_DEVICE if device >= 0 else 0))
         opts.world, opts.rank = int(world), int(rank)
         if bounds is not None:  # per-dimension [vlo | vhi | xlo | xhi], 4 x d
             bounds = np.ascontiguousarray(bounds, dtype=np.float32).reshape(4 * int(d))
@@ -122,7 +138,8 @@ class Swarm:
         buf = None
         if pos:
             buf = out if out is not None else np.empty(self.d_local, np.float32)
-        check(lib().pso_get_gbest(self._h, C.byref(f), C.byref(i), _ptr(buf, writable=True)),
+        check(lib().pso_get_gbest(self._h, C.byref(f), C.byref(i),
+                                  _ptr(buf, self.d_local, writable=True)),
               "pso_get_gbest")
         return float(np.float32(f.value)), int(i.value), buf
 
@@ -134,8 +151,10 @@ class Swarm:
                    np.empty((m, d), np.float32), np.empty(m, np.float32))
         X, V, PB, pf = out
         t = C.c_uint64()
-        check(lib().pso_get_state(self._h, _ptr(X, writable=True), _ptr(V, writable=True),
-                                  _ptr(PB, writable=True), _ptr(pf, writable=True), C.byref(t)),
+        m = self.n_local * self.d_local
+        check(lib().pso_get_state(self._h, _ptr(X, m, writable=True), _ptr(V, m, writable=True),
+                                  _ptr(PB, m, writable=True), _ptr(pf, self.n_local, writable=True),
+                                  C.byref(t)),
               "pso_get_state")
         return X, V, PB, pf, int(t.value)
 
@@ -150,7 +169,9 @@ class Swarm:
                          (PB, (self.n_local, dl)), (pf, (self.n_local,))):
             if tuple(a.shape) != shape:
                 raise ValueError(f"state shape {tuple(a.shape)} != {shape}")
-        check(lib().pso_set_state(self._h, _ptr(X), _ptr(V), _ptr(PB), _ptr(pf), int(t)),
+        m = self.n_local * dl
+        check(lib().pso_set_state(self._h, _ptr(X, m), _ptr(V, m), _ptr(PB, m),
+                                  _ptr(pf, self.n_local), int(t)),
               "pso_set_state")
         return self
 
@@ -172,6 +193,14 @@ class Swarm:
         offs = (C.c_uint64 * len(offsets))(*[int(o) for o in offsets])
         check(lib().pso_p2p_connect(self._h, blob, offs), "pso_p2p_connect")
         return self
+
+    def p2p_probe(self, phase: int) -> bool:
+        """Collective two-phase check of the mapped NVLink path (phase 0: store
+        this rank's token into every peer; barrier; phase 1: True if every
+        peer's token arrived)."""
+        ok = C.c_int32(0)
+        check(lib().pso_p2p_probe(self._h, int(phase), C.byref(ok)), "pso_p2p_probe")
+        return bool(ok.value)
 
     def p2p_enable(self, on: bool = True) -> "Swarm":
         check(lib().pso_p2p_enable(self._h, int(bool(on))), "pso_p2p_enable")

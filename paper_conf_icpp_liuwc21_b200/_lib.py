@@ -17,6 +17,7 @@ PSO_ERR_NCCL, PSO_ERR_UNSUPPORTED, PSO_ERR_POISONED = 4, 5, 6
 PSO_OBJ_SPHERE, PSO_OBJ_RASTRIGIN, PSO_OBJ_ROSENBROCK = 1, 2, 3
 PSO_OBJ_GRIEWANK, PSO_OBJ_ACKLEY, PSO_OBJ_EASOM, PSO_OBJ_CUSTOM_BASE = 4, 5, 6, 64
 PSO_FLAG_TIMING, PSO_FLAG_DEFER_INIT, PSO_FLAG_ASYNC_GBEST, PSO_FLAG_COLUMN_SPLIT = 1, 2, 4, 8
+PSO_FLAG_DEVICE = 16
 PSO_D_MAX_ROW = 65536
 PSO_D_AUTO_COLSPLIT = 16384
 PSO_D_MAX = 1 << 24
@@ -27,7 +28,7 @@ EXPORTS = (
     "pso_get_state", "pso_set_state", "pso_set_bounds", "pso_get_info", "pso_reset_counters", "pso_destroy",
     "pso_status_string", "pso_last_error", "pso_objective_registered",
     "pso_nccl_get_unique_id", "pso_nccl_comm_init", "pso_nccl_comm_destroy",
-    "pso_p2p_handle", "pso_p2p_connect", "pso_p2p_enable",
+    "pso_p2p_handle", "pso_p2p_connect", "pso_p2p_probe", "pso_p2p_enable",
     "pso_debug_philox", "pso_debug_objective",
 )
 
@@ -104,6 +105,7 @@ def lib() -> C.CDLL:
     L.pso_nccl_comm_destroy.argtypes = [C.c_void_p]
     L.pso_p2p_handle.argtypes = [H, C.c_void_p, u64p]
     L.pso_p2p_connect.argtypes = [H, C.c_void_p, u64p]
+    L.pso_p2p_probe.argtypes = [H, C.c_int32, C.POINTER(C.c_int32)]
     L.pso_p2p_enable.argtypes = [H, C.c_int32]
     L.pso_debug_philox.argtypes = [C.c_uint64, C.c_uint32, C.c_uint32, C.c_uint32, C.c_uint32,
                                    C.c_int64, u32p, C.c_int32, C.c_int32]

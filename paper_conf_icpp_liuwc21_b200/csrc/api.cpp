@@ -19,11 +19,33 @@
 #include <utility>
 #include <vector>
 
+#include <nvtx3/nvToolsExt.h>
+
 #include "kernels.h"
 
 using namespace fastpso;
 
 namespace {
+
+// NVTX ranges around every entry point that enqueues or waits for GPU work
+// (header-only NVTX v3: free unless a profiler such as nsys / ncu attaches).
+nvtxDomainHandle_t nvtx_domain() {
+  static nvtxDomainHandle_t d = nvtxDomainCreateA("fastpso");
+  return d;
+}
+struct NvtxRange {
+  explicit NvtxRange(const char* name) {
+    nvtxEventAttributes_t ev{};
+    ev.version = NVTX_VERSION;
+    ev.size = NVTX_EVENT_ATTRIB_STRUCT_SIZE;
+    ev.messageType = NVTX_MESSAGE_TYPE_ASCII;
+    ev.message.ascii = name;
+    nvtxDomainRangePushEx(nvtx_domain(), &ev);
+  }
+  ~NvtxRange() { nvtxDomainRangePop(nvtx_domain()); }
+  NvtxRange(const NvtxRange&) = delete;
+  NvtxRange& operator=(const NvtxRange&) = delete;
+};
 
 thread_local std::string g_last_error;
 
@@ -144,9 +166,14 @@ struct pso_swarm {
   // NVLink peer exchange (pso_p2p_connect)
   std::vector<void*> ipc_opened;
   void* peers_dev = nullptr;
+  // NCCL exchange: captured [step, all-gather] x kGraphIters, one per slot phase
+  cudaGraphExec_t nccl_graph[4] = {nullptr, nullptr, nullptr, nullptr};
+  bool graph_off = false;
 };
 
 namespace {
+
+constexpr int kGraphIters = 4;  // iterations per captured NCCL-exchange graph
 
 pso_status cuda_fail(pso_swarm* h, cudaError_t e, const char* what) {
   if (h) h->poisoned = true;
@@ -185,6 +212,7 @@ pso_status use_device(pso_swarm* h) {
 // prologue; `fold` additionally runs the select kernel so key_cur / G are
 // final for the host (end of create, set_state and every pso_step call).
 pso_status exchange(pso_swarm* h, uint64_t t, bool fold, bool into_local) {
+  NvtxRange nvtx_range("gbest exchange");
   if (!h->xchg || h->colsplit) return PSO_OK;  // the column split exchanges inside its kernels
   const size_t rec = record_bytes(h->pitch);
   if (h->args.p2p) {  // records travel by NVLink peer stores inside the kernels
@@ -213,6 +241,42 @@ pso_status exchange(pso_swarm* h, uint64_t t, bool fold, bool into_local) {
     PSO_CUDA(h, launch_select(h->args, (unsigned)t, into_local, h->stream));
     ++h->launches;
   }
+  return PSO_OK;
+}
+
+// Capture kGraphIters iterations of the NCCL exchange path starting at slot
+// phase `phase` ([step kernel, all-gather into recv slot (t & 3)] each) into an
+// executable graph.  The step kernel reads its iteration from the control block,
+// so the graph is valid for every start iteration with the same t & 3.  If the
+// capture fails (e.g. NCCL without graph support) the handle stays eager.
+pso_status capture_nccl_graph(pso_swarm* h, int phase) {
+  NvtxRange nvtx_range("capture NCCL graph");
+  NcclApi* a = nccl();
+  if (!a || !h->comm) return PSO_OK;
+  cudaGraph_t g = nullptr;
+  cudaError_t e = cudaStreamBeginCapture(h->stream, cudaStreamCaptureModeThreadLocal);
+  bool ok = e == cudaSuccess;
+  const size_t rec = record_bytes(h->pitch);
+  for (int k = 0; ok && k < kGraphIters; ++k) {
+    ok = launch_step(h->objective, h->args, h->cfg, h->stream) == cudaSuccess;
+    unsigned char* dst = const_cast<unsigned char*>(h->args.recv) +
+                         (size_t)((phase + k) & 3) * (size_t)h->world * rec;
+    ok = ok && a->AllGather(h->args.send, dst, rec, kNcclUint8, h->comm, h->stream) == 0;
+  }
+  if (e == cudaSuccess) {
+    cudaError_t e2 = cudaStreamEndCapture(h->stream, &g);
+    ok = ok && e2 == cudaSuccess && g;
+  }
+  cudaGraphExec_t ex = nullptr;
+  if (ok) ok = cudaGraphInstantiate(&ex, g, 0) == cudaSuccess;
+  if (g) cudaGraphDestroy(g);
+  cudaGetLastError();
+  if (!ok) {
+    if (ex) cudaGraphExecDestroy(ex);
+    h->graph_off = true;
+    return PSO_OK;
+  }
+  h->nccl_graph[phase] = ex;
   return PSO_OK;
 }
 
@@ -325,6 +389,9 @@ pso_status run_init(pso_swarm* h) {
   if (h->n_local > 0) {
     PSO_CUDA(h, launch_init(h->objective, h->args, h->cfg, h->stream));
     ++h->launches;
+  } else if (h->xchg) {  // no particles: publish a "no candidate" record of t = 0
+    PSO_CUDA(h, launch_empty_step(h->args, 0, false, h->stream));
+    ++h->launches;
   }
   pso_status st = exchange(h, 0, true, true);
   if (st != PSO_OK) return st;
@@ -368,18 +435,17 @@ int pso_objective_registered(int32_t objective) { return objective_registered(ob
 
 pso_status pso_create(pso_handle* out, int64_t n, int32_t d, float w, float c1, float c2, float lo,
                       float hi, int32_t objective, uint64_t seed) {
-  pso_opts o{};
-  o.device = -1;
+  pso_opts o{};  // zero-initialised: defaults (current device, own stream, 1 GPU)
   return pso_create_ex(out, n, d, w, c1, c2, lo, hi, objective, seed, &o);
 }
 
 pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c1, float c2,
                          float lo, float hi, int32_t objective, uint64_t seed,
                          const pso_opts* opts) {
+  NvtxRange nvtx_range("pso_create");
   if (!out) return fail(PSO_ERR_INVALID, "out is NULL");
   *out = nullptr;
   pso_opts o{};
-  o.device = -1;
   if (opts) o = *opts;
   // ---- validation (nothing touches the GPU before this passes)
   if (n < 1 || n >= (int64_t)1 << 32) return fail(PSO_ERR_INVALID, "n=%lld outside [1, 2^32)", (long long)n);
@@ -410,7 +476,7 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
   if (!objective_registered(objective))
     return fail(PSO_ERR_INVALID, "objective %d is not registered", objective);
   if (o.flags & ~(uint32_t)(PSO_FLAG_TIMING | PSO_FLAG_DEFER_INIT | PSO_FLAG_ASYNC_GBEST |
-                            PSO_FLAG_COLUMN_SPLIT))
+                            PSO_FLAG_COLUMN_SPLIT | PSO_FLAG_DEVICE))
     return fail(PSO_ERR_INVALID, "unknown flags 0x%x", o.flags);
   if (o.bounds) {
     pso_status bs = check_bounds(o.bounds, d);
@@ -438,7 +504,9 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
   };
 
   // ---- device and stream
-  if (o.device >= 0) {
+  if ((o.flags & PSO_FLAG_DEVICE) && o.device < 0)
+    return bail(fail(PSO_ERR_INVALID, "PSO_FLAG_DEVICE with device=%d < 0", o.device));
+  if (o.flags & PSO_FLAG_DEVICE) {
     cudaError_t e = cudaSetDevice(o.device);
     if (e != cudaSuccess) return bail(cuda_fail(nullptr, e, "cudaSetDevice"));
     h->device = o.device;
@@ -518,6 +586,7 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
   if (const char* v = std::getenv("PSO_STAGES")) hints.stages = std::atoi(v);
   if (const char* v = std::getenv("PSO_CTAS")) hints.ctas = std::atoi(v);
   if (const char* v = std::getenv("PSO_CLUSTER")) hints.cluster = std::atoi(v);
+  if (const char* v = std::getenv("PSO_GRAPH")) h->graph_off = *v == '0';
   if (const char* v = std::getenv("PSO_KERNEL")) {
     if (!std::strcmp(v, "reg")) hints.kernel = 0;
     if (!std::strcmp(v, "tma")) hints.kernel = 1;
@@ -569,8 +638,10 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
                        : h->xchg ? 4 * (size_t)h->world * record_bytes(h->pitch) : 0;
   const bool async = (o.flags & PSO_FLAG_ASYNC_GBEST) != 0 && h->xchg;  // needs an exchange
   const size_t viewb = async ? gb : 0;  // the host's global gbest view
-  h->arena_bytes =
-      3 * mat + pfb + gb + ctlb + boundb + pbxb + candb + viewb + sendb + align_up(recvb, 256);
+  // NVLink connect probe slots (pso_p2p_probe) after the receive area
+  const size_t probeb = (recvb && h->xchg) ? align_up((size_t)h->world * 8, 256) : 0;
+  h->arena_bytes = 3 * mat + pfb + gb + ctlb + boundb + pbxb + candb + viewb + sendb +
+                   align_up(recvb, 256) + probeb;
   {
     cudaError_t e = cudaMalloc(&h->arena, h->arena_bytes);
     if (e == cudaErrorMemoryAllocation) {
@@ -604,6 +675,7 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
   A.async_gbest = async ? 1 : 0;
   A.send = sendb ? p : nullptr; p += sendb;
   A.recv = recvb ? p : nullptr;
+  A.probe_off = align_up(recvb, 256);
   A.n_local = h->n_local;
   A.row_begin = h->row_begin;
   A.d = d;
@@ -630,23 +702,21 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
     if (e == cudaSuccess && recvb)  // record tags that no iteration matches until written
       e = cudaMemsetAsync(const_cast<unsigned char*>(A.recv), 0xFF,
                           colsplit ? col_tag_bytes(h->world) : recvb, h->stream);
+    if (e == cudaSuccess && probeb)
+      e = cudaMemsetAsync(const_cast<unsigned char*>(A.recv) + A.probe_off, 0, probeb, h->stream);
     if (e != cudaSuccess) return bail(cuda_fail(nullptr, e, "cudaMemsetAsync"));
   }
   pso_status st = reset_ctl(h, 0);
   if (st != PSO_OK) return bail(st);
   if (o.bounds && (st = upload_bounds(h, o.bounds)) != PSO_OK) return bail(st);
 
-  if (h->n_local == 0 && h->xchg && !colsplit) {  // empty shard: contribute "no candidate"
-    unsigned long long none[2] = {~0ull, 0ull};
-    cudaError_t e = cudaMemcpyAsync(A.send, none, 16, cudaMemcpyHostToDevice, h->stream);
-    if (e != cudaSuccess) return bail(cuda_fail(nullptr, e, "cudaMemcpyAsync"));
-  }
   if (!(o.flags & PSO_FLAG_DEFER_INIT) && (st = run_init(h)) != PSO_OK) return bail(st);
   *out = h;
   return PSO_OK;
 }
 
 pso_status pso_init(pso_handle h) {
+  NvtxRange nvtx_range("pso_init");
   pso_status st = check_handle(h);
   if (st != PSO_OK) return st;
   if (h->inited) return fail(PSO_ERR_INVALID, "already initialised");
@@ -655,10 +725,15 @@ pso_status pso_init(pso_handle h) {
 }
 
 pso_status pso_step(pso_handle h, int64_t iters) {
+  NvtxRange nvtx_range("pso_step");
   pso_status st = check_ready(h);
   if (st != PSO_OK) return st;
   if (iters < 0) return fail(PSO_ERR_INVALID, "iters=%lld < 0", (long long)iters);
   if (iters == 0) return PSO_OK;
+  // the iteration counter is 32-bit on the device (Philox ctr[2], record tags)
+  if (h->t + (uint64_t)iters >= ((uint64_t)1 << 32))
+    return fail(PSO_ERR_UNSUPPORTED, "t=%llu + iters=%lld reaches 2^32 (32-bit iteration counter)",
+                (unsigned long long)h->t, (long long)iters);
   if ((st = use_device(h)) != PSO_OK) return st;
   const bool timing = (h->flags & PSO_FLAG_TIMING) != 0;
   if (h->colsplit) {  // two kernels per iteration; the partials travel inside them
@@ -702,16 +777,42 @@ pso_status pso_step(pso_handle h, int64_t iters) {
     if ((st = next_event(h, &call_ev, (uint64_t)iters)) != PSO_OK) return st;
     PSO_CUDA(h, cudaEventRecord(call_ev->start, h->stream));
   }
-  for (int64_t it = 0; it < iters; ++it) {
-    if (h->n_local > 0) {
+  const bool empty = h->n_local == 0;
+  int64_t it = 0;
+  // NCCL exchange: whole runs of kGraphIters iterations [step kernel, all-gather]
+  // replay a captured CUDA graph (one per slot phase), so the host issues one
+  // launch per kGraphIters iterations instead of 2 kGraphIters.
+  if (!empty && !timing && h->xchg && !h->args.p2p && !h->graph_off) {
+    while (iters - it > kGraphIters) {  // the last iteration stays eager (it folds)
+      const int phase = (int)((h->t + (uint64_t)it + 1) & 3u);
+      if (!h->nccl_graph[phase] && (st = capture_nccl_graph(h, phase)) != PSO_OK) return st;
+      if (!h->nccl_graph[phase]) break;  // capture unavailable: eager from here on
+      PSO_CUDA(h, cudaGraphLaunch(h->nccl_graph[phase], h->stream));
+      h->launches += kGraphIters;
+      it += kGraphIters;
+    }
+  }
+  for (; it < iters; ++it) {
+    const uint64_t ti = h->t + (uint64_t)it + 1;
+    if (!empty) {
       pso_swarm::Timed* ev = nullptr;
       if (timing && !per_call && (st = next_event(h, &ev, 1)) != PSO_OK) return st;
       if (ev) PSO_CUDA(h, cudaEventRecord(ev->start, h->stream));
       PSO_CUDA(h, launch_step(h->objective, h->args, h->cfg, h->stream));
       ++h->launches;
       if (ev) PSO_CUDA(h, cudaEventRecord(ev->stop, h->stream));
+    } else if (h->xchg) {
+      // A rank without particles runs no step kernel: k_empty_step publishes its
+      // "no candidate" record (NVLink: after merging t - 1 as a prologue would).
+      // Over NCCL nothing merges on this rank, so every iteration's records are
+      // folded (a record only carries candidates strictly better than its
+      // sender's incumbent: a gbest of an earlier iteration would otherwise
+      // never reach this rank).
+      PSO_CUDA(h, launch_empty_step(h->args, (unsigned)ti, true, h->stream));
+      ++h->launches;
     }
-    if ((st = exchange(h, h->t + (uint64_t)it + 1, it + 1 == iters, false)) != PSO_OK) return st;
+    const bool fold = it + 1 == iters || (empty && !h->args.p2p);
+    if ((st = exchange(h, ti, fold, empty)) != PSO_OK) return st;
   }
   if (call_ev) PSO_CUDA(h, cudaEventRecord(call_ev->stop, h->stream));
   h->t += (uint64_t)iters;
@@ -719,6 +820,7 @@ pso_status pso_step(pso_handle h, int64_t iters) {
 }
 
 pso_status pso_synchronize(pso_handle h) {
+  NvtxRange nvtx_range("pso_synchronize");
   pso_status st = check_handle(h);
   if (st != PSO_OK) return st;
   if ((st = use_device(h)) != PSO_OK) return st;
@@ -726,6 +828,7 @@ pso_status pso_synchronize(pso_handle h) {
 }
 
 pso_status pso_get_gbest(pso_handle h, float* fitness, int64_t* index, float* pos) {
+  NvtxRange nvtx_range("pso_get_gbest");
   pso_status st = check_ready(h);
   if (st != PSO_OK) return st;
   if ((st = use_device(h)) != PSO_OK) return st;
@@ -743,6 +846,7 @@ pso_status pso_get_gbest(pso_handle h, float* fitness, int64_t* index, float* po
 }
 
 pso_status pso_get_state(pso_handle h, float* x, float* v, float* pb, float* pf, uint64_t* t) {
+  NvtxRange nvtx_range("pso_get_state");
   pso_status st = check_ready(h);
   if (st != PSO_OK) return st;
   if ((st = use_device(h)) != PSO_OK) return st;
@@ -766,6 +870,7 @@ pso_status pso_get_state(pso_handle h, float* x, float* v, float* pb, float* pf,
 
 pso_status pso_set_state(pso_handle h, const float* x, const float* v, const float* pb,
                          const float* pf, uint64_t t) {
+  NvtxRange nvtx_range("pso_set_state");
   pso_status st = check_handle(h);
   if (st != PSO_OK) return st;
   if (h->n_local > 0 && (!x || !v || !pb || !pf))
@@ -788,12 +893,15 @@ pso_status pso_set_state(pso_handle h, const float* x, const float* v, const flo
   }
   if ((st = reset_ctl(h, (uint32_t)t)) != PSO_OK) return st;
   ++h->args.epoch;  // p2p: records written before this call can never match again
+  // captured graphs hold the kernel parameters by value (epoch, t_base)
+  for (cudaGraphExec_t& g : h->nccl_graph)
+    if (g) cudaGraphExecDestroy(g), g = nullptr;
   if (rows > 0) {
     PSO_CUDA(h, launch_rebest(h->args, (unsigned)t, h->stream));
     ++h->launches;
-  } else if (h->xchg) {
-    unsigned long long none[2] = {~0ull, 0ull};
-    PSO_CUDA(h, cudaMemcpyAsync(h->args.send, none, 16, cudaMemcpyHostToDevice, h->stream));
+  } else if (h->xchg) {  // no particles: a "no candidate" record of t (new epoch)
+    PSO_CUDA(h, launch_empty_step(h->args, (unsigned)t, false, h->stream));
+    ++h->launches;
   }
   if ((st = exchange(h, t, true, true)) != PSO_OK) return st;
   if ((st = sync_and_check(h)) != PSO_OK) return st;
@@ -828,6 +936,7 @@ pso_status pso_p2p_handle(pso_handle h, void* ipc_handle, uint64_t* offset) {
 }
 
 pso_status pso_p2p_connect(pso_handle h, const void* ipc_handles, const uint64_t* offsets) {
+  NvtxRange nvtx_range("pso_p2p_connect");
   pso_status st = check_handle(h);
   if (st != PSO_OK) return st;
   if (!ipc_handles || !offsets) return fail(PSO_ERR_INVALID, "ipc_handles/offsets is NULL");
@@ -836,8 +945,6 @@ pso_status pso_p2p_connect(pso_handle h, const void* ipc_handles, const uint64_t
   if ((st = use_device(h)) != PSO_OK) return st;
   if ((st = sync_and_check(h)) != PSO_OK) return st;
   if (h->peers_dev) return fail(PSO_ERR_INVALID, "already connected");
-  if (h->n_local == 0)  // records are written by step kernels; an empty shard runs none
-    return fail(PSO_ERR_UNSUPPORTED, "rank owns no particles: use the NCCL exchange");
   // Failures here leave the handle usable (NCCL exchange): nothing is poisoned.
   auto undo = [&](cudaError_t e, const char* what) {
     for (void* p : h->ipc_opened) cudaIpcCloseMemHandle(p);
@@ -866,6 +973,27 @@ pso_status pso_p2p_connect(pso_handle h, const void* ipc_handles, const uint64_t
                  cudaMemcpyHostToDevice);
   if (e != cudaSuccess) return undo(e, "cudaMemcpy");
   h->args.peers = (unsigned char* const*)h->peers_dev;
+  return PSO_OK;
+}
+
+pso_status pso_p2p_probe(pso_handle h, int32_t phase, int32_t* ok) {
+  NvtxRange nvtx_range("pso_p2p_probe");
+  pso_status st = check_handle(h);
+  if (st != PSO_OK) return st;
+  if (phase != 0 && phase != 1) return fail(PSO_ERR_INVALID, "phase must be 0 or 1");
+  if (phase == 1 && !ok) return fail(PSO_ERR_INVALID, "ok is NULL");
+  if (!h->peers_dev) return fail(PSO_ERR_INVALID, "pso_p2p_connect first");
+  if ((st = use_device(h)) != PSO_OK) return st;
+  int* dev_ok = nullptr;
+  if (phase == 1) PSO_CUDA(h, cudaMalloc(&dev_ok, sizeof(int)));
+  cudaError_t e = launch_p2p_probe(h->args, phase, dev_ok, h->stream);
+  int host_ok = 0;
+  if (e == cudaSuccess && phase == 1)
+    e = cudaMemcpyAsync(&host_ok, dev_ok, sizeof(int), cudaMemcpyDeviceToHost, h->stream);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(h->stream);
+  if (dev_ok) cudaFree(dev_ok);
+  if (e != cudaSuccess) return cuda_fail(h, e, "p2p probe");
+  if (phase == 1) *ok = host_ok;
   return PSO_OK;
 }
 
@@ -958,6 +1086,8 @@ void pso_destroy(pso_handle h) {
     cudaEventDestroy(e.start);
     cudaEventDestroy(e.stop);
   }
+  for (cudaGraphExec_t g : h->nccl_graph)
+    if (g) cudaGraphExecDestroy(g);
   for (void* p : h->ipc_opened) cudaIpcCloseMemHandle(p);
   if (h->peers_dev) cudaFree(h->peers_dev);
   if (h->arena) cudaFree(h->arena);

@@ -15,7 +15,7 @@ struct DevCtl {
   unsigned long long improvements;  // pbest improvements, summed
   unsigned int done;                // last-CTA ticket counter
   unsigned int t;                   // iterations done (low 32 bits; Philox ctr[2])
-  unsigned long long key_par[2];    // unused (the grid-resident kernel keeps per-CTA keys in cand_key)
+  unsigned long long spare[2];
   unsigned int bar_count, bar_gen;  // grid-resident kernel: grid barrier
   unsigned long long pb_loads;      // streaming kernels: pbest rows read from HBM
   unsigned long long pb_stores;     // streaming kernels: pbest rows written to HBM
@@ -75,6 +75,7 @@ struct SwarmArgs {
   unsigned epoch;             // p2p: record tags are (epoch << 32 | t); set_state starts an epoch
   unsigned t_base;            // async: iteration of the last create/set_state (records start there)
   unsigned char* const* peers;  // p2p: device array, world pointers to every rank's recv
+  unsigned long long probe_off; // p2p: offset from a recv base to the connect probe slots (world u64)
   // Column split (NEXT-3, "tile matrix"): this rank holds float4 columns
   // [col_q0, col_q0 + nvec) of every row (n_local = n); X, V, PB, G, bounds are
   // that block (pitch 4 nvec).  recv = [2][world] u64 tags, then the partials
@@ -196,6 +197,13 @@ cudaError_t launch_rebest(const SwarmArgs& a, unsigned t, cudaStream_t s);
 // Fold the records of iteration t (and, asynchronous, of t - 1) for the host;
 // into_local: also into the kernels' incumbent (create / set_state).
 cudaError_t launch_select(const SwarmArgs& a, unsigned t, bool into_local, cudaStream_t s);
+// A rank without particles: its share of iteration t of the exchange (merge the
+// records of t - 1 if `merge`, publish a "no candidate" record of t).
+cudaError_t launch_empty_step(const SwarmArgs& a, unsigned t, bool merge, cudaStream_t s);
+// NVLink connect probe: phase 0 stores this rank's token into every peer's probe
+// slot; phase 1 (after a host barrier) checks that every peer's token arrived in
+// ours (*ok_dev = 1) and clears the slots.
+cudaError_t launch_p2p_probe(const SwarmArgs& a, int phase, int* ok_dev, cudaStream_t s);
 // lazy pbest: copy X -> PB for flagged rows and clear the flags (host reads)
 cudaError_t launch_materialize_pb(const SwarmArgs& a, cudaStream_t s);
 

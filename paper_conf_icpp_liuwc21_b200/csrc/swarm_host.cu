@@ -1,5 +1,11 @@
 // swarm_host.cu — launch planning and dispatch of the fused kernels, and the
 // objective-independent kernels (gbest rebest after set_state, multi-GPU select).
+#include <algorithm>
+#include <cstdlib>
+#include <map>
+#include <mutex>
+#include <utility>
+
 #include "swarm_kernels.cuh"
 
 namespace fastpso {
@@ -90,6 +96,74 @@ __global__ void __launch_bounds__(128) k_select(const SwarmArgs a, unsigned t, i
   }
 }
 
+// ---------------------------------------------------------- empty shard
+// A rank that owns no particles (n < world) runs no step kernel, yet its peers
+// wait for its record of every iteration.  This one-warp kernel plays the
+// rank's part of iteration t.  NVLink exchange: merge the records of t - 1
+// into the incumbent (`merge`: what a step kernel's prologue does) and publish
+// a "no candidate" record of t to every rank (its epilogue).  NCCL exchange:
+// write the "no candidate" record of t into `send` for the all-gather (the host
+// folds every iteration's records with k_select).  Records carry the same
+// (epoch, iteration) tag as a step kernel's, so switching exchanges is safe.
+__global__ void __launch_bounds__(32) k_empty_step(const SwarmArgs a, unsigned t, int merge) {
+  const int lane = threadIdx.x;
+  const unsigned long long tag = ((unsigned long long)a.epoch << 32) | t;
+  if (!a.p2p) {
+    if (lane == 0) {
+      unsigned long long* hdr = reinterpret_cast<unsigned long long*>(a.send);
+      hdr[0] = ~0ull;
+      hdr[1] = tag;
+    }
+    return;
+  }
+  if (merge) {
+    int src = -1;
+    const unsigned long long best = exchange_merge_warp(a, t - 1u, lane, &src);
+    if (src >= 0) {
+      const float4* w = reinterpret_cast<const float4*>(merged_gbest_row(a, t - 1u, src));
+      for (int q = lane; q < a.nvec; q += 32) {
+        const float4 v = w[q];
+        reinterpret_cast<float4*>(a.G)[q] = v;
+        if (a.G_view) reinterpret_cast<float4*>(a.G_view)[q] = v;
+      }
+    }
+    if (lane == 0) {
+      a.ctl->key_cur = best;
+      a.ctl->key_view = best;
+      a.ctl->t = t;
+    }
+  }
+  const size_t rec = record_bytes(a.nvec * 4);
+  const size_t off = (size_t)(t & 3u) * a.world * rec + (size_t)a.rank * rec;
+  for (int r = lane; r < a.world; r += 32) reinterpret_cast<unsigned long long*>(a.peers[r] + off)[0] = ~0ull;
+  __syncwarp();
+  for (int r = lane; r < a.world; r += 32) st_release_sys_u64(a.peers[r] + off + 8, tag);
+}
+
+// ---------------------------------------------------------- NVLink probe
+// Proves the peer mappings carry data before the exchange relies on them: a
+// system-scope release store of token(rank) into slot `rank` of every rank's
+// probe area, then (after the host barrier) acquire loads of our own slots.
+__device__ __forceinline__ unsigned long long probe_token(int r) {
+  return 0x50534F5000000000ull | (unsigned)(r + 1);
+}
+__global__ void __launch_bounds__(32) k_p2p_probe(const SwarmArgs a, int phase, int* ok) {
+  const int lane = threadIdx.x;
+  if (phase == 0) {
+    for (int r = lane; r < a.world; r += 32)
+      st_release_sys_u64(a.peers[r] + a.probe_off + 8ull * a.rank, probe_token(a.rank));
+    return;
+  }
+  unsigned char* mine = const_cast<unsigned char*>(a.recv) + a.probe_off;
+  int good = 1;
+  for (int r = lane; r < a.world; r += 32) {
+    good &= ld_acquire_sys_u64(mine + 8ull * r) == probe_token(r);
+    reinterpret_cast<unsigned long long*>(mine)[r] = 0ull;
+  }
+  good = __all_sync(kFull, good);
+  if (lane == 0) *ok = good;
+}
+
 // ---------------------------------------------------------- materialize PB
 // Lazy pbest rows (PB == X, not stored): one warp per flagged row copies X -> PB.
 __global__ void __launch_bounds__(256) k_materialize_pb(const SwarmArgs a) {
@@ -151,6 +225,24 @@ constexpr long long kResidentElems = 8192;      // resident path: n d <= this
 
 }  // namespace
 
+// cudaFuncAttributeMaxDynamicSharedMemorySize is one setting per kernel function
+// (per device), shared by every handle of the process: it is only ever RAISED,
+// to the largest ring any handle planned, so creating a handle never lowers the
+// limit an older handle of the same instantiation launches with.
+cudaError_t allow_dynamic_smem(const void* fn, size_t bytes) {
+  static std::mutex mu;
+  static std::map<std::pair<int, const void*>, size_t> granted;
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return e;
+  std::lock_guard<std::mutex> lock(mu);
+  size_t& g = granted[{dev, fn}];
+  if (bytes <= g) return cudaSuccess;
+  e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes);
+  if (e == cudaSuccess) g = bytes;
+  return e;
+}
+
 bool objective_registered(int objective) {
   bool nb;
   return kernel_for(objective, Which::Init, 1, false, &nb) != nullptr;
@@ -165,31 +257,29 @@ int ring_stages(size_t fixed, size_t stage_bytes, int ctas) {
   return budget > fixed ? (int)((budget - fixed) / stage_bytes) : 0;
 }
 
-// Cluster path (NEXT-3): rows of more than 2048 float4 (d > 8192), or forced.
-cudaError_t plan_cluster(const KernelTable* t, int nvec, long long n_local, const PlanHints& h,
-                         LaunchCfg* cfg) {
-  int C = h.cluster > 0 ? h.cluster : 2;
-  if (h.cluster <= 0)
-    while (C < 16 && (nvec + C - 1) / C > 1024) C *= 2;
+// One cluster shape: C CTAs per row, the ring sized for one CTA per SM.  Fills
+// *cfg and reports how many SMs its clusters cover (0 if it does not fit).
+cudaError_t cluster_shape(const KernelTable* t, int nvec, int C, const PlanHints& h, LaunchCfg* cfg,
+                          int* sms_covered) {
+  *sms_covered = 0;
   const int chunk = (nvec + C - 1) / C;
-  if (C < 2 || C > 16 || (C & (C - 1)) || chunk > 2048) return cudaErrorInvalidConfiguration;
+  if (C < 2 || C > 16 || chunk > 2048) return cudaSuccess;
   int vpt, compute;
   shape_for(chunk, h.vpt, &vpt, &compute, kMaxThreadsCluster);
+  if ((chunk + vpt - 1) / vpt > kMaxThreadsCluster) return cudaSuccess;
   const void* fn = t->step_cluster[vpt_index(vpt)][h.bounds ? 1 : 0];
   const size_t crow = (size_t)chunk * 16, btab = h.bounds ? 4 * crow : 0;
   const int per_sm = (h.ctas >= 1 && h.ctas <= 4) ? h.ctas : 1;  // CTAs per SM to size the ring for
   int stages = ring_stages(crow + btab, 3 * crow, per_sm);
   if (h.stages >= 2 && h.stages < stages) stages = h.stages;
   if (stages > kMaxStages) stages = kMaxStages;
-  if (stages < 2) return cudaErrorInvalidConfiguration;
+  if (stages < 2) return cudaSuccess;
   const size_t smem = crow + btab + (size_t)stages * 3 * crow;
   cudaError_t e;
   if (C > 8 &&
       (e = cudaFuncSetAttribute(fn, cudaFuncAttributeNonPortableClusterSizeAllowed, 1)) != cudaSuccess)
     return e;
-  if ((e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem)) !=
-      cudaSuccess)
-    return e;
+  if ((e = allow_dynamic_smem(fn, smem)) != cudaSuccess) return e;
   cudaLaunchConfig_t lc{};
   lc.gridDim = dim3(C);
   lc.blockDim = dim3(compute + 64);
@@ -202,9 +292,11 @@ cudaError_t plan_cluster(const KernelTable* t, int nvec, long long n_local, cons
   lc.attrs = attr;
   lc.numAttrs = 1;
   int ncl = 0;
-  if ((e = cudaOccupancyMaxActiveClusters(&ncl, fn, &lc)) != cudaSuccess) return e;
-  if (ncl < 1) return cudaErrorInvalidConfiguration;
-  long long clusters = ncl < n_local ? ncl : n_local;
+  if ((e = cudaOccupancyMaxActiveClusters(&ncl, fn, &lc)) != cudaSuccess) {
+    cudaGetLastError();  // e.g. a cluster size the device cannot co-schedule
+    return cudaSuccess;
+  }
+  if (ncl < 1) return cudaSuccess;
   cfg->cluster = C;
   cfg->chunk = chunk;
   cfg->vpt = vpt;
@@ -213,8 +305,52 @@ cudaError_t plan_cluster(const KernelTable* t, int nvec, long long n_local, cons
   cfg->tma = 1;
   cfg->stages = stages;
   cfg->smem = smem;
-  cfg->grid = (int)(clusters * C);
+  cfg->grid = ncl * C;  // clipped to the rows by the caller
   cfg->ctas_per_sm = 1;
+  *sms_covered = ncl * C / per_sm;
+  return cudaSuccess;
+}
+
+// Cluster path (NEXT-3): rows of more than 2048 float4 (d > 8192), or forced.
+// The cluster size is chosen for SM coverage: clusters are placed within one
+// GPC, so C CTAs of one SM each leave (GPC size mod C) SMs of every GPC idle --
+// on a 148-SM B200 four-CTA clusters fit 33 per GPU (132 SMs) while three-
+// or six-CTA ones cover more.  Among the sizes with >= 3 ring stages the one
+// covering the most SMs wins (ties: the smaller C, fewer DSMEM messages per
+// row).  The choice depends on d and the device only (never on n or the world
+// size), so the block combine order -- and every fitness bit -- is the same on
+// every rank.
+cudaError_t plan_cluster(const KernelTable* t, int nvec, long long n_local, const PlanHints& h,
+                         LaunchCfg* cfg) {
+  LaunchCfg best = *cfg;
+  int best_sms = 0, best_stages = 0;
+  const int c_lo = h.cluster > 0 ? h.cluster : 2, c_hi = h.cluster > 0 ? h.cluster : 16;
+  for (int C = c_lo; C <= c_hi; ++C) {
+    LaunchCfg c = *cfg;
+    int sms = 0;
+    cudaError_t e = cluster_shape(t, nvec, C, h, &c, &sms);
+    if (e != cudaSuccess) return e;
+    if (sms == 0) continue;
+    const bool deep = c.stages >= 3, best_deep = best_stages >= 3;
+    if (best_sms == 0 || (deep && !best_deep) || (deep == best_deep && sms > best_sms)) {
+      best = c;
+      best_sms = sms;
+      best_stages = c.stages;
+    }
+  }
+  if (best_sms == 0) return cudaErrorInvalidConfiguration;
+  if (std::getenv("PSO_CLUSTER_POW2") && h.cluster <= 0) {  // round-1 rule, for A/B runs
+    int C = 2;
+    while (C < 16 && (nvec + C - 1) / C > 1024) C *= 2;
+    int sms = 0;
+    LaunchCfg c = *cfg;
+    cudaError_t e = cluster_shape(t, nvec, C, h, &c, &sms);
+    if (e != cudaSuccess) return e;
+    if (sms) best = c;
+  }
+  *cfg = best;
+  const long long clusters = std::min<long long>(cfg->grid / cfg->cluster, n_local);
+  cfg->grid = (int)(clusters * cfg->cluster);
   return cudaSuccess;
 }
 
@@ -254,7 +390,7 @@ cudaError_t plan_launch(int objective, int d, long long n_local, int sm_count, c
         (size_t)n_local * nvec * 16 * 3 + (size_t)nvec * 16 + btab + (size_t)n_local * 4;
     const void* fn = tab->resident[bi];
     if (smem <= kSmemPerCtaMax - kStaticReserve &&
-        cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) ==
+        allow_dynamic_smem(fn, smem) ==
             cudaSuccess) {
       int gs = 1;
       while (gs < nvec) gs <<= 1;
@@ -330,7 +466,7 @@ cudaError_t plan_launch(int objective, int d, long long n_local, int sm_count, c
       const int threads = cfg->compute + 64;  // + producer warp + finaliser warp
       if (stages >= 2) {
         const size_t smem = row + btab + (size_t)stages * 3 * row;
-        if ((e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem)) !=
+        if ((e = allow_dynamic_smem(fn, smem)) !=
             cudaSuccess)
           return e;
         int per_sm = 0;
@@ -357,8 +493,7 @@ cudaError_t plan_launch(int objective, int d, long long n_local, int sm_count, c
     cfg->stages = 0;
     cfg->threads = cfg->compute;
     cfg->smem = row + btab + first;
-    if ((e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                  (int)cfg->smem)) != cudaSuccess)
+    if ((e = allow_dynamic_smem(fn, cfg->smem)) != cudaSuccess)
       return e;
     int per_sm = 0;
     if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, cfg->threads, cfg->smem)) !=
@@ -381,7 +516,7 @@ cudaError_t plan_launch(int objective, int d, long long n_local, int sm_count, c
       const size_t smem = row + btab + (size_t)rows * 3 * row + (size_t)rows * 4;
       if (smem > kSmemPerCtaMax - kStaticReserve || smem * per > kSmemPerSm - per * kStaticReserve)
         continue;
-      if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) !=
+      if (allow_dynamic_smem(fn, smem) !=
           cudaSuccess) {
         cudaGetLastError();
         continue;
@@ -478,7 +613,7 @@ cudaError_t plan_colsplit(int objective, int tile, int tiles_local, long long n,
   if (stages < 2) return cudaErrorInvalidConfiguration;
   const void* fn = t->col_step[bounds ? 1 : 0];
   const size_t smem = (size_t)stages * stage;
-  cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  cudaError_t e = allow_dynamic_smem(fn, smem);
   if (e != cudaSuccess) return e;
   const long long items = n * tiles_local;
   long long grid = (long long)sm_count * ctas;
@@ -533,6 +668,16 @@ cudaError_t launch_materialize_pb(const SwarmArgs& a, cudaStream_t s) {
   long long blocks = (a.n_local + 7) / 8;
   if (blocks > 2048) blocks = 2048;
   k_materialize_pb<<<(unsigned)blocks, 256, 0, s>>>(a);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_p2p_probe(const SwarmArgs& a, int phase, int* ok_dev, cudaStream_t s) {
+  k_p2p_probe<<<1, 32, 0, s>>>(a, phase, ok_dev);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_empty_step(const SwarmArgs& a, unsigned t, bool merge, cudaStream_t s) {
+  k_empty_step<<<1, 32, 0, s>>>(a, t, merge ? 1 : 0);
   return cudaGetLastError();
 }
 

@@ -728,7 +728,9 @@ __device__ __forceinline__ void epilogue_core(const SwarmArgs& a, uint32_t t, un
     if (tid == 0) {
       unsigned long long* hdr = reinterpret_cast<unsigned long long*>(a.send);
       hdr[0] = key;
-      hdr[1] = t;
+      // the same (epoch, iteration) tag as the NVLink records, so a handle that
+      // switches to p2p after set_state finds its last all-gathered records
+      hdr[1] = ((unsigned long long)a.epoch << 32) | t;
     }
   } else {  // NVLink: store the record into recv[t & 1][rank] of every rank
     // the row is read once and stored to every rank; thread r releases rank r's tag

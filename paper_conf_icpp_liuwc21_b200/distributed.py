@@ -1,13 +1,17 @@
 """Process-group plumbing for the particle-split multi-GPU path.
 
-One process per GPU.  torch.distributed (any backend) only carries the
-128-byte NCCL unique id from rank 0 to the others; the per-iteration exchange
-(one ncclAllGather of the (key, candidate row) records + a select kernel)
-runs inside the C library on the handle's stream.
+One process per GPU.  torch.distributed (any backend) only carries
+out-of-band setup data: the 128-byte NCCL unique id, and the CUDA IPC handles
+of the NVLink peer exchange.  Per iteration the gbest exchange runs inside the
+step kernels (NVLink peer stores of each rank's record, merged by the next
+kernel's prologue); the NCCL all-gather of the same records (+ a select
+kernel at the end of each pso_step call) is the fallback when a rank cannot
+map or probe its peers.
 """
 from __future__ import annotations
 
 import os
+import sys
 
 from . import nccl_comm_destroy, nccl_comm_init, nccl_unique_id
 
@@ -45,25 +49,53 @@ def destroy_comm(comm: int) -> None:
         nccl_comm_destroy(comm)
 
 
+def _log(msg: str) -> None:
+    if os.environ.get("PSO_QUIET", "0") in ("", "0"):
+        print(f"[fastpso] {msg}", file=sys.stderr, flush=True)
+
+
 def connect_p2p(swarm, group=None) -> bool:
-    """Switch `swarm` (created with a communicator) to the NVLink peer exchange:
-    all-gather every rank's CUDA IPC handle + receive-buffer offset over
-    torch.distributed, map the peers' buffers, and enable the mode only if every
-    rank succeeded (else all ranks stay on the NCCL all-gather).  Returns
+    """Switch `swarm` to the NVLink peer exchange: all-gather every rank's CUDA
+    IPC handle + receive-buffer offset over torch.distributed, map the peers'
+    buffers, then PROBE the mapped path (every rank stores a token into every
+    peer with a system-scope release; after a barrier every rank checks it
+    received all of them).  The mode is enabled only if every rank mapped and
+    probed successfully; otherwise every rank stays on the NCCL all-gather (a
+    handle with a communicator) and the reason is logged to stderr.  Returns
     whether the peer exchange is on.  Collective."""
     import torch.distributed as dist
     from . import PsoError
+    world = dist.get_world_size(group)
+    rank = dist.get_rank(group)
     mine = swarm.p2p_handle()
-    everyone = [None] * dist.get_world_size(group)
+    everyone = [None] * world
     dist.all_gather_object(everyone, mine, group=group)
-    ok = True
+    why = ""
     try:
         swarm.p2p_connect([h for h, _ in everyone], [o for _, o in everyone])
-    except PsoError:
-        ok = False
-    votes = [None] * dist.get_world_size(group)
-    dist.all_gather_object(votes, ok, group=group)
-    if all(votes):
+    except PsoError as e:
+        why = f"rank {rank}: peer mapping failed: {e}"
+    votes = [None] * world
+    dist.all_gather_object(votes, why, group=group)
+    reasons = [v for v in votes if v]
+    if not reasons:
+        probe_ok = False
+        try:
+            swarm.p2p_probe(0)
+            dist.barrier(group=group)
+            probe_ok = swarm.p2p_probe(1)
+        except PsoError as e:
+            why = f"rank {rank}: probe failed: {e}"
+        if not probe_ok and not why:
+            why = f"rank {rank}: probe tokens missing"
+        votes = [None] * world
+        dist.all_gather_object(votes, why, group=group)
+        reasons = [v for v in votes if v]
+    if not reasons:
         swarm.p2p_enable(True)
+        if rank == 0:
+            _log(f"gbest exchange: NVLink peer stores, {world} ranks mapped and probed")
         return True
+    if rank == 0:
+        _log("gbest exchange: falling back to the NCCL all-gather (" + "; ".join(reasons) + ")")
     return False

@@ -86,6 +86,11 @@ WORKLOADS = {
     "NS_R2": Workload("northstar-shard-of-2-rastrigin-50000x2000", RASTRIGIN, 50_000, 2000, 500),
     "NS_R4": Workload("northstar-shard-of-4-rastrigin-25000x2000", RASTRIGIN, 25_000, 2000, 500),
     "NS_R8": Workload("northstar-shard-of-8-rastrigin-12500x2000", RASTRIGIN, 12_500, 2000, 500),
+    # reading 3 (vmax = 1) made visible: the survey's C4 velocity bound (vmax = 600, the
+    # domain half-width) and the north-star swarm at vmax = 5.12 (its domain half-width)
+    "C4_V600": Workload("C4-griewank-100000x2000-vmax600", GRIEWANK, 100_000, 2000, 500, vmax=600.0),
+    "NS_V512": Workload("northstar-rastrigin-100000x2000-vmax5.12", RASTRIGIN, 100_000, 2000, 500,
+                        vmax=5.12),
     # the paper's own default experiment, for the Table 2 plausibility band
     "PAPER": Workload("paper-default-5000x200", SPHERE, 5000, 200, 2000),
 }

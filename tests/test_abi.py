@@ -154,3 +154,33 @@ def test_bounds_validation_without_gpu():
     b[25] = -1.0
     b[3] = np.nan
     assert _create(opts=o)[0] == 1
+
+
+def test_device_flag_validation_without_gpu():
+    """pso_opts.device is read only with PSO_FLAG_DEVICE (zero-initialised opts
+    are the defaults: the caller's current device); a negative ordinal with
+    the flag is rejected before any device call."""
+    o = _lib.pso_opts()
+    o.flags = _lib.PSO_FLAG_DEVICE
+    o.device = -2
+    assert _create(opts=o)[0] == 1 and "PSO_FLAG_DEVICE" in fp.last_error()
+
+
+def test_host_buffer_validation():
+    """The binding checks element type and count of every host buffer the
+    library reads or writes (no silent reinterpretation, no overflow)."""
+    import numpy as np
+    import torch
+    from paper_conf_icpp_liuwc21_b200 import _ptr
+    assert _ptr(None) is None
+    assert _ptr(np.zeros(6, np.float32), 6).value
+    assert _ptr(torch.zeros(2, 3), 6).value
+    for bad, count in ((np.zeros(6, np.float64), 6), (np.zeros(5, np.float32), 6),
+                       (torch.zeros(6, dtype=torch.float16), 6), (torch.zeros(7), 6),
+                       (torch.zeros(6, dtype=torch.float64), None), (np.zeros((6, 2), np.float32)[:, 0], 6)):
+        with pytest.raises(ValueError):
+            _ptr(bad, count)
+    ro = np.zeros(3, np.float32)
+    ro.flags.writeable = False
+    with pytest.raises(ValueError):
+        _ptr(ro, 3, writable=True)

@@ -90,6 +90,27 @@ def test_gpu_arm_two_ranks_share_one_gpu(mode):
     assert j["value"] > 0 and j["e2e"]["value"] > 0
 
 
+@pytest.mark.gpu
+def test_gpu_arm_self_launches_ranks():
+    """`python bench.py --gpus N` without torchrun launches the N ranks itself
+    (the driver's SCALE run may call it either way) and still prints one line;
+    here 3 ranks share GPU 0 (PSO_SHARE_GPU harness), NS_R8-sized swarm split 3 ways."""
+    lines = _run("--gpus", "3", "--steps", "20", "--warmup", "3", "--workload", "NS_R8",
+                 env={"PSO_SHARE_GPU": "1"})
+    lines = [ln for ln in lines if ln.startswith("{")]
+    assert len(lines) == 1
+    j = json.loads(lines[0])
+    assert j["n_gpus"] == 3 and j["value"] > 0 and j["gpu_launches"] >= 20
+    assert j["config"]["gbest_exchange"] == "nvlink-peer-stores"
+
+
+def test_self_launch_reference_arm_prints_once():
+    lines = _run("--impl", "reference", "--gpus", "2", "--steps", "2", "--warmup", "1",
+                 "--workload", "C1", "--ref-seconds", "3")
+    lines = [ln for ln in lines if ln.startswith("{")]
+    assert len(lines) == 1 and json.loads(lines[0])["impl"] == "reference"
+
+
 def test_reference_arm_under_torchrun_prints_once():
     lines = _torchrun(2, "--impl", "reference", "--gpus", "2", "--steps", "2", "--warmup", "1",
                       "--workload", "C1", "--ref-seconds", "3")

@@ -1,9 +1,10 @@
-"""Ranks of the particle split as 2-4 processes on ONE GPU, with
+"""Ranks of the particle split as 2-8 processes on ONE GPU, with
 the NVLink peer exchange (CUDA IPC mappings between the processes): every
-iteration each rank's step kernel stores its gbest record into both ranks'
-receive buffers and the next step kernel acquires both tags — the real
-multi-rank protocol (parity double-buffering, epoch tags, merge order), not a
-1-rank stand-in.  Results must equal a single-process run bit for bit."""
+iteration each rank's step kernel stores its gbest record into every rank's
+receive buffer and the next step kernel acquires the tags -- the real
+multi-rank protocol (slot rotation, epoch tags, merge order), not a 1-rank
+stand-in.  Every call's result is checked against the oracle run as `world`
+virtual shards, and the whole run against a single-process run bit for bit."""
 import os
 import socket
 
@@ -12,8 +13,10 @@ import pytest
 import torch.distributed as dist
 import torch.multiprocessing as mp
 
+import oracle as orc
 import paper_conf_icpp_liuwc21_b200 as fp
-from synth import DOMAINS, GRIEWANK, RASTRIGIN, ROSENBROCK, row_range
+from pso_testutil import assert_bitwise, oracle_lockstep
+from synth import DOMAINS, GRIEWANK, RASTRIGIN, ROSENBROCK, SPHERE, random_state, row_range
 
 pytestmark = pytest.mark.gpu
 
@@ -24,60 +27,182 @@ def _free_port():
         return s.getsockname()[1]
 
 
-def _worker(rank, world, port, n, d, obj, steps, out_dir):
+def _snap(s):
+    X, V, PB, pf, t = s.get_state()
+    f, i, G = s.gbest()
+    return dict(X=X, V=V, PB=PB, pf=pf, t=t, f=f, i=i, G=G)
+
+
+def _run_ops(s, ops, rows=None, cols=None):
+    """Apply ops to a handle; a snapshot after create / init and after each op.
+    ("step", k); ("restore", None): set_state with the handle's own state (a new
+    epoch: records of the previous state must never match); ("set_state",
+    (X, V, PB, pf, t)) with the whole swarm, of which this rank takes its rows
+    (particle split) or its column block (column split)."""
+    snaps = [_snap(s)]
+    for op, arg in ops:
+        if op == "step":
+            s.step(arg)
+        elif op == "restore":
+            X, V, PB, pf, t = s.get_state()
+            s.set_state(X, V, PB, pf, t=t)
+        else:
+            X, V, PB, pf, t = arg
+            if rows is not None:
+                b, e = rows
+                X, V, PB, pf = X[b:e], V[b:e], PB[b:e], pf[b:e]
+            if cols is not None:
+                b, e = cols
+                X, V, PB = X[:, b:e], V[:, b:e], PB[:, b:e]
+            s.set_state(np.ascontiguousarray(X), np.ascontiguousarray(V), np.ascontiguousarray(PB),
+                        pf, t=t)
+        snaps.append(_snap(s))
+    return snaps
+
+
+def _save(out_dir, tag, rank, snaps, **extra):
+    flat = {f"{k}{j}": np.asarray(v) for j, sn in enumerate(snaps) for k, v in sn.items()}
+    np.savez(os.path.join(out_dir, f"{tag}{rank}.npz"), nsnap=len(snaps), **flat, **extra)
+
+
+def _load(path):
+    z = np.load(path)
+    out = []
+    for j in range(int(z["nsnap"])):
+        sn = {k: z[f"{k}{j}"] for k in ("X", "V", "PB", "pf", "G")}
+        sn.update(t=int(z[f"t{j}"]), f=float(z[f"f{j}"]), i=int(z[f"i{j}"]))
+        out.append(sn)
+    return out, z
+
+
+def _worker(rank, world, port, n, d, obj, seed, ops, out_dir, params=(0.9, 2.0, 2.0, None)):
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)
     dist.init_process_group("gloo", rank=rank, world_size=world)
     from paper_conf_icpp_liuwc21_b200.distributed import connect_p2p
-    lo, hi = DOMAINS[obj]
-    s = fp.Swarm(n, d, 0.9, 2.0, 2.0, lo, hi, obj, 4242, device=0, world=world, rank=rank,
+    w, c1, c2, dom = params
+    lo, hi = dom or DOMAINS[obj]
+    s = fp.Swarm(n, d, w, c1, c2, lo, hi, obj, seed, device=0, world=world, rank=rank,
                  defer_init=True)
     assert connect_p2p(s)
     s.init()
-    for k in steps:
-        s.step(k)
-    X, V, PB, pf, t = s.get_state()
-    f, i, G = s.gbest()
-    # set_state starts a new epoch: records of the previous state must never match
-    s.set_state(X, V, PB, pf, t=t)
-    s.step(2)
-    X2, V2, PB2, pf2, t2 = s.get_state()
-    f2, i2, G2 = s.gbest()
-    np.savez(os.path.join(out_dir, f"r{rank}.npz"), X=X, V=V, PB=PB, pf=pf, G=G, f=f, i=i, t=t,
-             X2=X2, PB2=PB2, pf2=pf2, G2=G2, f2=f2, i2=i2, launches=s.info()["launches"])
+    snaps = _run_ops(s, ops, rows=row_range(n, rank, world))
+    _save(out_dir, "r", rank, snaps, launches=s.info()["launches"])
     s.close()
     dist.barrier()
     dist.destroy_process_group()
 
 
-@pytest.mark.parametrize("world,obj,n,d", [(2, RASTRIGIN, 300, 1000), (2, GRIEWANK, 41, 13),
-                                           (2, ROSENBROCK, 6, 10000), (3, RASTRIGIN, 7, 2000),
-                                           (4, GRIEWANK, 9, 999)])
-def test_processes_nvlink_exchange_matches_single_gpu(tmp_path, world, obj, n, d):
-    steps = (1, 4, 3)
-    mp.spawn(_worker, args=(world, _free_port(), n, d, obj, steps, str(tmp_path)), nprocs=world,
-             join=True)
+def _gathered(tmp_path, tag, world, axis=0):
+    per_rank = [_load(tmp_path / f"{tag}{r}.npz")[0] for r in range(world)]
+    out = []
+    for j in range(len(per_rank[0])):
+        sn = dict(per_rank[0][j])
+        for k in ("X", "V", "PB"):
+            sn[k] = np.concatenate([pr[j][k] for pr in per_rank], axis=axis)
+        if axis == 0:
+            sn["pf"] = np.concatenate([pr[j]["pf"] for pr in per_rank])
+        else:
+            sn["G"] = np.concatenate([pr[j]["G"] for pr in per_rank])
+            for pr in per_rank[1:]:  # every rank holds all n pf and the same gbest
+                assert_bitwise(pr[j]["pf"], sn["pf"], f"pf rank-identical, snapshot {j}")
+        for pr in per_rank[1:]:  # the gbest is bitwise identical on every rank
+            assert (pr[j]["f"], pr[j]["i"], pr[j]["t"]) == (sn["f"], sn["i"], sn["t"])
+            if axis == 0:
+                assert_bitwise(pr[j]["G"], sn["G"], f"G rank-identical, snapshot {j}")
+        out.append(sn)
+    return out
+
+
+def _oracle_ops(ops, snaps):
+    """The ops as the oracle replays them (restore = set_state of the previous snapshot)."""
+    out = []
+    for k, (op, arg) in enumerate(ops):
+        if op == "restore":
+            p = snaps[k]
+            arg = (p["X"], p["V"], p["PB"], p["pf"], p["t"])
+            op = "set_state"
+        out.append((op, arg))
+    return out
+
+
+def _injected_state(n, d, t):
+    """A random injected state: every pbest above every fitness (all rows
+    improve) and a NaN pbest at row 0 (read as +inf)."""
+    lo, hi = DOMAINS[RASTRIGIN]
+    X, V, PB, pf = random_state(n, d, lo, hi, 1.0, 99 + n, pf_mode="rand")
+    pf = (pf + np.float32(5e4)).astype(np.float32)
+    pf[0] = np.nan
+    return X, V, PB, pf, t
+
+
+WORLDS = [(2, RASTRIGIN, 300, 1000), (2, GRIEWANK, 41, 13), (2, ROSENBROCK, 6, 10000),
+          (3, RASTRIGIN, 7, 2000), (4, GRIEWANK, 9, 999), (8, RASTRIGIN, 203, 1000),
+          (8, GRIEWANK, 37, 2001), (3, SPHERE, 2, 300)]
+
+
+@pytest.mark.parametrize("world,obj,n,d", WORLDS)
+def test_processes_nvlink_exchange_match_the_oracle(tmp_path, world, obj, n, d):
+    """Each rank's shard after every call equals the oracle run as `world`
+    virtual particle shards (X, V, PB bitwise, pf within the
+    fitness tolerance, (gi, G) the oracle's), replayed call by call from the
+    gathered GPU state; the gbest is bitwise identical on every rank; and the
+    whole run equals a single-process run bit for bit (world invariance).
+    (3, SPHERE, 2, 300): rank 0 owns no particle (n < world)."""
+    seed = 4242
+    ops = [("step", 1), ("step", 4), ("step", 3), ("restore", None), ("step", 2)]
+    if obj == RASTRIGIN:
+        ops += [("set_state", _injected_state(n, d, t=17)), ("step", 1), ("step", 2)]
+    mp.spawn(_worker, args=(world, _free_port(), n, d, obj, seed, ops, str(tmp_path)),
+             nprocs=world, join=True)
+    snaps = _gathered(tmp_path, "r", world)
     lo, hi = DOMAINS[obj]
-    ref = fp.Swarm(n, d, 0.9, 2.0, 2.0, lo, hi, obj, 4242, device=0)
-    for k in steps:
-        ref.step(k)
-    RX, RV, RPB, Rpf, Rt = ref.get_state()
-    rf, ri, RG = ref.gbest()
-    ref.set_state(RX, RV, RPB, Rpf, t=Rt)
-    ref.step(2)
-    RX2, _, RPB2, Rpf2, _ = ref.get_state()
-    rf2, ri2, RG2 = ref.gbest()
-    for r in range(world):
-        z = np.load(tmp_path / f"r{r}.npz")
-        b, e = row_range(n, r, world)
-        for name, full in (("X", RX), ("V", RV), ("PB", RPB), ("pf", Rpf), ("X2", RX2),
-                           ("PB2", RPB2), ("pf2", Rpf2)):
-            assert np.array_equal(z[name].view(np.uint32), full[b:e].view(np.uint32)), (r, name)
-        assert int(z["t"]) == Rt
-        assert (float(z["f"]), int(z["i"])) == (rf, ri)
-        assert (float(z["f2"]), int(z["i2"])) == (rf2, ri2)
-        assert np.array_equal(z["G"].view(np.uint32), RG.view(np.uint32))
-        assert np.array_equal(z["G2"].view(np.uint32), RG2.view(np.uint32))
+
+    def make_oracle(create):
+        return orc.OracleSwarm(n, d, 0.9, 2.0, 2.0, lo, hi, obj, seed, nshards=world,
+                               create=create)
+
+    skip_state, skip_g = oracle_lockstep(make_oracle, obj, snaps, _oracle_ops(ops, snaps),
+                                         f"world={world}")
+    assert skip_state <= 1 and skip_g <= 2, (skip_state, skip_g)
+    # world invariance: the single-process run of the same ops
+    ref = fp.Swarm(n, d, 0.9, 2.0, 2.0, lo, hi, obj, seed, device=0)
+    rsnaps = _run_ops(ref, ops)
+    for j, (a, b) in enumerate(zip(snaps, rsnaps)):
+        for k in ("X", "V", "PB", "pf", "G"):
+            assert_bitwise(a[k], b[k], f"snapshot {j} {k} vs 1 process")
+        assert (a["f"], a["i"], a["t"]) == (b["f"], b["i"], b["t"])
+
+
+@pytest.mark.parametrize("case", ["ties", "zero", "minf"])
+@pytest.mark.parametrize("world", [3, 8])
+def test_processes_decisions_across_ranks(tmp_path, world, case):
+    """The decision pins (readings 9-11) with the rows of the case in different
+    ranks (row 1 on rank 0, row n - 2 on the last rank): equal fitness in two
+    ranks goes to the lower global index through the NVLink merge, -0 ties +0
+    across ranks, a -inf pbest on the last rank wins everywhere.  Frozen swarm,
+    so every value is exact: compared with the oracle bit for bit."""
+    from pso_testutil import crafted_expect, crafted_state
+    n, d = 48, 1000
+    obj, lo, hi, X, V, PB, pf, a, b = crafted_state(case, n, d)
+    assert row_range(n, 0, world)[1] > a and row_range(n, world - 1, world)[0] <= b
+    ops = [("set_state", (X, V, PB, pf, 5)), ("step", 1), ("step", 1),
+           ("set_state", (X, V, PB, pf, 8)), ("step", 2)]
+    mp.spawn(_worker, args=(world, _free_port(), n, d, obj, 7, ops, str(tmp_path),
+                            (0.0, 0.0, 0.0, (lo, hi))), nprocs=world, join=True)
+    snaps = _gathered(tmp_path, "r", world)
+    c = orc.OracleSwarm(n, d, 0.0, 0.0, 0.0, lo, hi, obj, 7, nshards=world, create=False)
+    expect_steps = [None, 0, 1, 2, 0, 2]
+    for j, (op, arg) in enumerate(ops, start=1):
+        if op == "set_state":
+            c.set_state(*arg[:4], t=arg[4])
+        else:
+            c.step(arg)
+        sn = snaps[j]
+        for k, ref in (("X", c.X), ("V", c.V), ("PB", c.PB), ("pf", c.pf), ("G", c.G)):
+            assert_bitwise(sn[k], ref, f"{case} world={world} snapshot {j}: {k}")
+        assert (sn["i"], sn["t"]) == (c.gi, c.t) and sn["f"] == c.gf
+        assert (sn["i"], sn["f"]) == crafted_expect(case, n, d, expect_steps[j])
 
 
 def _async_worker(rank, world, port, n, d, obj, steps, out_dir):
@@ -138,68 +263,56 @@ def test_async_split_matches_the_async_oracle(tmp_path, world, obj, n, d):
             assert abs(gf - mf) <= 1e-5 * abs(mf) + 1e-6
 
 
-def _col_worker(rank, world, port, n, d, obj, steps, out_dir):
+def _col_worker(rank, world, port, n, d, obj, seed, ops, out_dir):
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)
     dist.init_process_group("gloo", rank=rank, world_size=world)
     from paper_conf_icpp_liuwc21_b200.distributed import connect_p2p
     lo, hi = DOMAINS[obj]
-    s = fp.Swarm(n, d, 0.9, 2.0, 2.0, lo, hi, obj, 99, device=0, world=world, rank=rank,
+    s = fp.Swarm(n, d, 0.9, 2.0, 2.0, lo, hi, obj, seed, device=0, world=world, rank=rank,
                  defer_init=True, column_split=True)
     assert connect_p2p(s)
     s.init()
-    for k in steps:
-        s.step(k)
-    X, V, PB, pf, t = s.get_state()
-    f, i, G = s.gbest()
-    s.set_state(X, V, PB, pf, t=t)  # new epoch: stale tags never match
-    s.step(2)
-    X2, _, PB2, pf2, _ = s.get_state()
-    f2, i2, G2 = s.gbest()
     info = s.info()
-    np.savez(os.path.join(out_dir, f"c{rank}.npz"), X=X, V=V, PB=PB, pf=pf, G=G, f=f, i=i, t=t,
-             X2=X2, PB2=PB2, pf2=pf2, G2=G2, f2=f2, i2=i2, col_begin=info["col_begin"],
-             d_local=info["d_local"])
+    snaps = _run_ops(s, ops, cols=(info["col_begin"], info["col_begin"] + info["d_local"]))
+    _save(out_dir, "c", rank, snaps, col_begin=info["col_begin"], d_local=info["d_local"])
     s.close()
     dist.barrier()
     dist.destroy_process_group()
 
 
 @pytest.mark.parametrize("world,obj,n,d", [(2, ROSENBROCK, 50, 6000), (3, GRIEWANK, 17, 9001),
-                                           (4, RASTRIGIN, 64, 4096), (2, ROSENBROCK, 3, 70001)])
-def test_column_split_processes_match_single_gpu(tmp_path, world, obj, n, d):
+                                           (4, RASTRIGIN, 64, 4096), (2, ROSENBROCK, 3, 70001),
+                                           (8, RASTRIGIN, 40, 8192)])
+def test_column_split_processes_match_the_oracle(tmp_path, world, obj, n, d):
     """NEXT-3 across ranks ("tile matrix"): each rank process owns a
     block of column tiles of every row; tile partials travel by NVLink peer
     stores, every rank decides pbest / gbest from the same partial table.  The
-    tiling depends on d only, so the ranks' blocks, pf and gbest equal the
-    single-GPU column split bit for bit."""
-    steps = (1, 3, 2)
-    mp.spawn(_col_worker, args=(world, _free_port(), n, d, obj, steps, str(tmp_path)),
+    blocks tile the row in rank order; the gathered state after every call
+    equals the oracle (replayed call by call), pf and the gbest are identical
+    on every rank, and the run equals the single-GPU column split bit for bit."""
+    seed = 99
+    ops = [("step", 1), ("step", 3), ("step", 1), ("restore", None), ("step", 2), ("step", 1)]
+    mp.spawn(_col_worker, args=(world, _free_port(), n, d, obj, seed, ops, str(tmp_path)),
              nprocs=world, join=True)
-    lo, hi = DOMAINS[obj]
-    ref = fp.Swarm(n, d, 0.9, 2.0, 2.0, lo, hi, obj, 99, device=0, column_split=True)
-    for k in steps:
-        ref.step(k)
-    RX, RV, RPB, Rpf, Rt = ref.get_state()
-    rf, ri, RG = ref.gbest()
-    ref.set_state(RX, RV, RPB, Rpf, t=Rt)
-    ref.step(2)
-    RX2, _, RPB2, Rpf2, _ = ref.get_state()
-    rf2, ri2, RG2 = ref.gbest()
     covered = 0
     for r in range(world):
         z = np.load(tmp_path / f"c{r}.npz")
-        b = int(z["col_begin"])
-        e = b + int(z["d_local"])
-        assert b == covered  # blocks tile the row in rank order
-        covered = e
-        for name, full in (("X", RX), ("V", RV), ("PB", RPB), ("X2", RX2), ("PB2", RPB2)):
-            assert np.array_equal(z[name].view(np.uint32), full[:, b:e].view(np.uint32)), (r, name)
-        for name, full in (("pf", Rpf), ("pf2", Rpf2)):
-            assert np.array_equal(z[name].view(np.uint32), full.view(np.uint32)), (r, name)
-        assert np.array_equal(z["G"].view(np.uint32), RG[b:e].view(np.uint32))
-        assert np.array_equal(z["G2"].view(np.uint32), RG2[b:e].view(np.uint32))
-        assert (float(z["f"]), int(z["i"])) == (rf, ri)
-        assert (float(z["f2"]), int(z["i2"])) == (rf2, ri2)
-        assert int(z["t"]) == Rt
+        assert int(z["col_begin"]) == covered  # blocks tile the row in rank order
+        covered += int(z["d_local"])
     assert covered == d
+    snaps = _gathered(tmp_path, "c", world, axis=1)
+    lo, hi = DOMAINS[obj]
+
+    def make_oracle(create):
+        return orc.OracleSwarm(n, d, 0.9, 2.0, 2.0, lo, hi, obj, seed, create=create)
+
+    skip_state, skip_g = oracle_lockstep(make_oracle, obj, snaps, _oracle_ops(ops, snaps),
+                                         f"colsplit world={world}")
+    assert skip_state <= 1 and skip_g <= 2, (skip_state, skip_g)
+    ref = fp.Swarm(n, d, 0.9, 2.0, 2.0, lo, hi, obj, seed, device=0, column_split=True)
+    rsnaps = _run_ops(ref, ops)
+    for j, (a, b) in enumerate(zip(snaps, rsnaps)):
+        for k in ("X", "V", "PB", "pf", "G"):
+            assert_bitwise(a[k], b[k], f"snapshot {j} {k} vs 1 process")
+        assert (a["f"], a["i"], a["t"]) == (b["f"], b["i"], b["t"])

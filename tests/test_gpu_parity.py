@@ -313,6 +313,37 @@ def test_errors_do_not_abort():
     fp.lib().pso_destroy(None)
 
 
+def test_iteration_counter_limit():
+    """The device iteration counter (Philox ctr[2], record tags) is 32-bit:
+    pso_step refuses to cross 2^32 instead of repeating random streams."""
+    g = gpu_swarm(40, 300, RASTRIGIN)
+    X, V, PB, pf, _ = g.get_state()
+    g.set_state(X, V, PB, pf, t=2**32 - 3)
+    g.step(2)  # reaches 2^32 - 1
+    with pytest.raises(fp.PsoError) as e:
+        g.step(1)
+    assert e.value.status == 5
+    assert g.get_state()[4] == 2**32 - 1  # not poisoned, nothing ran
+
+
+@pytest.mark.parametrize("first,second", [(2000, 1600), (1000, 700), (16384, 12288)])
+def test_handles_sharing_a_kernel_keep_their_shared_memory(first, second, monkeypatch):
+    """The dynamic shared memory limit is one attribute per kernel function:
+    planning a second handle of the same instantiation with a smaller ring must
+    not lower the limit the first one launches with (both keep stepping, each
+    equal to a fresh single handle)."""
+    monkeypatch.setenv("PSO_RESIDENT", "0")
+    a = gpu_swarm(300, first, RASTRIGIN, seed=1)
+    b = gpu_swarm(300, second, RASTRIGIN, seed=2)
+    ia, ib = a.info(), b.info()
+    assert ia["smem_bytes"] > ib["smem_bytes"] and ia["vec_per_thread"] == ib["vec_per_thread"]
+    a.step(3)
+    b.step(3)
+    a2 = gpu_swarm(300, first, RASTRIGIN, seed=1).step(3)
+    for x, y in zip(a.get_state()[:4], a2.get_state()[:4]):
+        assert_bitwise(x, y, "first handle after a smaller plan")
+
+
 # ------------------------------------------------------------------ full size, sampled
 @pytest.mark.parametrize("key", ["NS", "C4", "C3", "C2", "W16K", "W64K", "C5@40000"])
 def test_full_size_sampled_rows(key):
@@ -602,6 +633,36 @@ def test_nvlink_peer_exchange_single_rank(obj, n, d, monkeypatch):
         rf, ri, RG = ref.gbest()
         assert (gf, gi) == (rf, ri)
         assert_bitwise(G, RG, "G")
+        g.close()
+    finally:
+        fp.nccl_comm_destroy(comm)
+
+
+def test_switch_to_nvlink_after_set_state(monkeypatch):
+    """Records all-gathered over NCCL carry the same (epoch, iteration) tag as
+    NVLink records: a handle that runs set_state (a new epoch) on the NCCL
+    exchange and only then switches to NVLink finds its last records instead
+    of waiting for a tag that never comes."""
+    import torch  # noqa: F401
+    monkeypatch.setenv("PSO_FORCE_EXCHANGE", "1")
+    comm = fp.nccl_comm_init(1, fp.nccl_unique_id(), 0, 0)
+    try:
+        g = gpu_swarm(200, 1000, RASTRIGIN, seed=12, nccl_comm=comm)
+        ref = gpu_swarm(200, 1000, RASTRIGIN, seed=12)
+        g.step(3)
+        ref.step(3)
+        X, V, PB, pf, t = g.get_state()
+        g.set_state(X, V, PB, pf, t=t)
+        ref.set_state(X, V, PB, pf, t=t)
+        g.step(2)
+        ref.step(2)
+        h, off = g.p2p_handle()
+        g.p2p_connect([h], [off]).p2p_enable(True)
+        g.step(3)
+        ref.step(3)
+        for x, y in zip(g.get_state()[:4], ref.get_state()[:4]):
+            assert_bitwise(x, y, "state after the switch")
+        assert g.gbest()[:2] == ref.gbest()[:2]
         g.close()
     finally:
         fp.nccl_comm_destroy(comm)

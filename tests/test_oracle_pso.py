@@ -219,6 +219,67 @@ def test_gbest_ties_and_nan():
     assert s.gi == 3
 
 
+def test_signed_zero_fitness_ties_and_minus_inf_winner():
+    """Readings 10-11: -0 and +0 are the same fitness (strict <, lowest index
+    among equal minima); -inf is a legal winner and nothing beats it."""
+    s = make(n=6, d=4, w=0.0, c1=0.0, c2=0.0)
+    X = np.full((6, 4), 2.0, np.float32)  # f = 16
+    pf = np.array([9, 9, 0.0, 9, 9, -0.0], np.float32)  # +0 at row 2, -0 at row 5
+    s.set_state(X, np.zeros_like(X), X.copy(), pf, t=0)
+    assert s.gi == 2 and s.gf == 0.0  # -0 is not below +0: the lower index wins
+    pf = np.array([9, 9, -0.0, 9, 9, 0.0], np.float32)
+    s.set_state(X, np.zeros_like(X), X.copy(), pf, t=0)
+    assert s.gi == 2 and np.signbit(np.float32(s.gf))  # the incumbent's own bits are kept
+    s.step(1)  # f = 16 everywhere: no improvement, no new gbest
+    assert s.gi == 2
+    pf = np.array([9, 9, 0.0, 9, -np.inf, 9], np.float32)
+    s.set_state(X, np.zeros_like(X), X.copy(), pf, t=0)
+    assert s.gi == 4 and s.gf == -np.inf
+    X[0] = 0.0  # f = +0 on the next step: below every finite pbest, not below -inf
+    s.set_state(X, np.zeros_like(X), X.copy(), pf, t=0)
+    s.step(1)
+    assert s.pf[0] == 0.0 and s.gi == 4 and s.gf == -np.inf
+
+
+def test_easom_far_from_pi_is_minus_zero_and_not_an_improvement():
+    """Easom with even d and exp(-sum (x - pi)^2) underflowing: f = -0 exactly
+    (-(-1)^d prod cos^2 * 0).  Against a +0 incumbent it is a tie (reading 10):
+    pbest +inf rows improve to -0, the +0 gbest stays."""
+    s = orc.OracleSwarm(5, 8, 0.0, 0.0, 0.0, -100.0, 100.0, orc.EASOM, 1)
+    X = np.full((5, 8), -50.0, np.float32)
+    f = orc.objective(orc.EASOM, X[0])
+    assert f == 0.0 and np.signbit(np.float32(f))
+    pf = np.array([np.inf, np.inf, 0.0, np.inf, np.inf], np.float32)
+    s.set_state(X, np.zeros_like(X), X.copy(), pf, t=3)
+    assert s.gi == 2
+    s.step(1)
+    assert s.gi == 2 and not np.signbit(np.float32(s.gf))
+    assert all(np.signbit(s.pf[[0, 1, 3, 4]])) and not np.signbit(s.pf[2])
+
+
+@pytest.mark.parametrize("obj,lo,hi,n,d", [(orc.RASTRIGIN, -5.12, 5.12, 23, 37),
+                                           (orc.ROSENBROCK, -2.048, 2.048, 9, 1001),
+                                           (orc.GRIEWANK, -600.0, 600.0, 17, 13)])
+def test_rows_step_is_one_step_of_the_sampled_rows(obj, lo, hi, n, d):
+    """orc_rows_step (the full-size GPU tests' per-row checker) is one
+    iteration of Alg. 1's body for the given rows: over all rows at t + 1 it
+    equals orc_step's move, evaluation and pbest update from the same state,
+    and any subset (shuffled, with repeats) equals the same rows of it."""
+    s = make(n=n, d=d, obj=obj, lo=lo, hi=hi, seed=77)
+    s.step(3)
+    X, V, PB, pf, G, t = s.X.copy(), s.V.copy(), s.PB.copy(), s.pf.copy(), s.G.copy(), s.t
+    s.step(1)
+    idx = np.arange(n)
+    rX, rV, rPB, rpf, rf = s.rows_step(t + 1, G, idx, X, V, PB, pf)
+    assert_same((rX, rV, rPB, rpf, rf), (s.X, s.V, s.PB, s.pf, s.f))
+    sub = np.array([n - 1, 0, n // 2, 0, 3])
+    sX, sV, sPB, spf, sf = s.rows_step(t + 1, G, sub, X[sub], V[sub], PB[sub], pf[sub])
+    assert_same((sX, sV, sPB, spf, sf), (s.X[sub], s.V[sub], s.PB[sub], s.pf[sub], s.f[sub]))
+    # the iteration number selects the random streams: t + 2 moves differently
+    oX = s.rows_step(t + 2, G, idx, X, V, PB, pf)[0]
+    assert not np.array_equal(oX, s.X)
+
+
 def test_all_infinite_pbest_gives_index_zero():
     s = make(n=4, d=2)
     s.set_state(s.X, s.V, s.PB, np.full(4, np.inf, np.float32), t=0)
