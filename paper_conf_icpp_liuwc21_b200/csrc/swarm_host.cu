@@ -311,44 +311,27 @@ cudaError_t cluster_shape(const KernelTable* t, int nvec, int C, const PlanHints
   return cudaSuccess;
 }
 
-// Cluster path (NEXT-3): rows of more than 2048 float4 (d > 8192), or forced.
-// The cluster size is chosen for SM coverage: clusters are placed within one
-// GPC, so C CTAs of one SM each leave (GPC size mod C) SMs of every GPC idle --
-// on a 148-SM B200 four-CTA clusters fit 33 per GPU (132 SMs) while three-
-// or six-CTA ones cover more.  Among the sizes with >= 3 ring stages the one
-// covering the most SMs wins (ties: the smaller C, fewer DSMEM messages per
-// row).  The choice depends on d and the device only (never on n or the world
-// size), so the block combine order -- and every fitness bit -- is the same on
-// every rank.
+// Cluster path (NEXT-3): rows of more than 2048 float4 (d > 8192), or forced
+// (PSO_CLUSTER = any size 2-16).  Automatic size: the smallest power of two
+// whose column block is <= 1024 float4 (d only, never n or the world size, so
+// the block combine order -- and every fitness bit -- is the same on every
+// rank).  Measured at W16K (Griewank 16384 x 16384, round 2): C = 4 (132 SMs,
+// 4 stages) 821 us; C = 3 (135 SMs, 3 stages) 1122; C = 5 (130 SMs) 978; C = 8
+// 1478; C = 16 (2 CTAs per SM) 1626 -- covering more SMs does not pay: the
+// cluster's per-row handshake, not SM coverage, set the pace.
 cudaError_t plan_cluster(const KernelTable* t, int nvec, long long n_local, const PlanHints& h,
                          LaunchCfg* cfg) {
-  LaunchCfg best = *cfg;
-  int best_sms = 0, best_stages = 0;
-  const int c_lo = h.cluster > 0 ? h.cluster : 2, c_hi = h.cluster > 0 ? h.cluster : 16;
-  for (int C = c_lo; C <= c_hi; ++C) {
-    LaunchCfg c = *cfg;
-    int sms = 0;
-    cudaError_t e = cluster_shape(t, nvec, C, h, &c, &sms);
-    if (e != cudaSuccess) return e;
-    if (sms == 0) continue;
-    const bool deep = c.stages >= 3, best_deep = best_stages >= 3;
-    if (best_sms == 0 || (deep && !best_deep) || (deep == best_deep && sms > best_sms)) {
-      best = c;
-      best_sms = sms;
-      best_stages = c.stages;
-    }
-  }
-  if (best_sms == 0) return cudaErrorInvalidConfiguration;
-  if (std::getenv("PSO_CLUSTER_POW2") && h.cluster <= 0) {  // round-1 rule, for A/B runs
-    int C = 2;
+  int C = h.cluster;
+  if (C <= 0) {
+    C = 2;
     while (C < 16 && (nvec + C - 1) / C > 1024) C *= 2;
-    int sms = 0;
-    LaunchCfg c = *cfg;
-    cudaError_t e = cluster_shape(t, nvec, C, h, &c, &sms);
-    if (e != cudaSuccess) return e;
-    if (sms) best = c;
   }
-  *cfg = best;
+  int sms = 0;
+  LaunchCfg c = *cfg;
+  cudaError_t e = cluster_shape(t, nvec, C, h, &c, &sms);
+  if (e != cudaSuccess) return e;
+  if (sms == 0) return cudaErrorInvalidConfiguration;
+  *cfg = c;
   const long long clusters = std::min<long long>(cfg->grid / cfg->cluster, n_local);
   cfg->grid = (int)(clusters * cfg->cluster);
   return cudaSuccess;

@@ -55,6 +55,21 @@ run("bounds", 2, 40, 1000, steps=3, bounds=b)
 comm = fp.nccl_comm_init(1, fp.nccl_unique_id(), 0, 0)
 try:
     run("exchange-nccl", 2, 300, 1000, steps=3, env={"PSO_FORCE_EXCHANGE": "1"}, nccl_comm=comm)
+    # runs of 4 iterations replay the captured [step, all-gather] CUDA graph
+    run("nccl-graph", 2, 300, 1000, steps=11, env={"PSO_FORCE_EXCHANGE": "1"}, nccl_comm=comm)
+    # NVLink records on a 1-rank group: IPC mapping, connect probe, peer stores
+    os.environ["PSO_FORCE_EXCHANGE"] = "1"
+    lo, hi = DOMAINS[2]
+    s = fp.Swarm(300, 1000, 0.9, 2.0, 2.0, lo, hi, 2, 7, device=0, nccl_comm=comm)
+    h, off = s.p2p_handle()
+    s.p2p_connect([h], [off])
+    s.p2p_probe(0)
+    assert s.p2p_probe(1)
+    s.p2p_enable(True)
+    s.step(3)
+    print("p2p-probe      f=%.6g i=%d" % s.gbest()[:2], flush=True)
+    s.close()
+    os.environ.pop("PSO_FORCE_EXCHANGE")
 finally:
     fp.nccl_comm_destroy(comm)
 print("sanitize_run done", flush=True)
