@@ -445,8 +445,9 @@ def run_gpu(args, w):
                          # SURVEY 8(d)'s accounting: every pbest row read, 4 rho written
                          "frac_survey_formula": survey_gbs / peak,
                          "achieved_survey_formula": survey_gbs,
-                         "kernel": ("k_col_step (fused move+eval, tile partials; k_col_decide "
-                                    "takes the pbest/gbest decisions)" if info["column_split"]
+                         "kernel": ("k_col_step + k_col_decide per iteration (fused move+eval "
+                                    "with tile partials, then the pbest/gbest decisions; PDL "
+                                    "launches, timed together)" if info["column_split"]
                                     else "k_step (fused move+eval+pbest+gbest)"),
                          "kernel_avg_us": kern_ms * 1e3,
                          "bytes_per_update": bytes_per_update, "rho": rho,

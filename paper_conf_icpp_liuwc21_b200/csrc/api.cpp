@@ -599,6 +599,8 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
       return bail(fail(PSO_ERR_UNSUPPORTED, "no column-split plan for d=%d", d));
     }
     if (e != cudaSuccess) return bail(cuda_fail(nullptr, e, "plan_colsplit"));
+    const char* pdl = std::getenv("PSO_PDL");
+    h->cfg.pdl = (pdl && *pdl == '0') ? 0 : 1;
   }
   if (!colsplit) {
     const char* v = std::getenv("PSO_RESIDENT");
@@ -737,15 +739,24 @@ pso_status pso_step(pso_handle h, int64_t iters) {
   if ((st = use_device(h)) != PSO_OK) return st;
   const bool timing = (h->flags & PSO_FLAG_TIMING) != 0;
   if (h->colsplit) {  // two kernels per iteration; the partials travel inside them
+    // With PDL (default) the kernels overlap launch and drain, so one event pair
+    // brackets the whole call: the timed "step kernel" is then k_col_step +
+    // k_col_decide per iteration.  PSO_PDL=0: an event pair around each k_col_step.
+    pso_swarm::Timed* call_ev = nullptr;
+    if (timing && h->cfg.pdl) {
+      if ((st = next_event(h, &call_ev, (uint64_t)iters)) != PSO_OK) return st;
+      PSO_CUDA(h, cudaEventRecord(call_ev->start, h->stream));
+    }
     for (int64_t it = 0; it < iters; ++it) {
       pso_swarm::Timed* ev = nullptr;
-      if (timing && (st = next_event(h, &ev, 1)) != PSO_OK) return st;
+      if (timing && !call_ev && (st = next_event(h, &ev, 1)) != PSO_OK) return st;
       if (ev) PSO_CUDA(h, cudaEventRecord(ev->start, h->stream));
       PSO_CUDA(h, launch_col_step(h->objective, h->args, h->cfg, 0, h->stream));
       if (ev) PSO_CUDA(h, cudaEventRecord(ev->stop, h->stream));
       PSO_CUDA(h, launch_col_decide(h->objective, h->args, h->cfg, 0, h->stream));
       h->launches += 2;
     }
+    if (call_ev) PSO_CUDA(h, cudaEventRecord(call_ev->stop, h->stream));
     h->t += (uint64_t)iters;
     return PSO_OK;
   }

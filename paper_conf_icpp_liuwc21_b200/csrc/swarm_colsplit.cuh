@@ -40,6 +40,28 @@ __device__ __forceinline__ float4* col_parts(unsigned char* region, const SwarmA
          (size_t)par * (size_t)a.n_local * (size_t)a.col_nbt;
 }
 
+// The items k = k0, k0 + step, ... of the (row, tile) sequence, k = r nb + b,
+// advanced without a 64-bit division per item (every thread of the CTA walks
+// the sequence; a division per item cost ~100 instructions each).
+struct ItemWalk {
+  long long r, dr;
+  int b, db, nb;
+  __device__ __forceinline__ ItemWalk(long long k0, long long step, int nb_) : nb(nb_) {
+    r = k0 / nb_;
+    b = (int)(k0 - r * nb_);
+    dr = step / nb_;
+    db = (int)(step - dr * nb_);
+  }
+  __device__ __forceinline__ void next() {
+    r += dr;
+    b += db;
+    if (b >= nb) {
+      b -= nb;
+      ++r;
+    }
+  }
+};
+
 constexpr int kColCompute = 256;  // compute threads of k_col_step (+ producer + finaliser warps)
 static_assert(kColTileMax <= 2 * kColCompute, "k_col_step: at most 2 float4 of a tile per thread");
 
@@ -68,6 +90,7 @@ __global__ void __launch_bounds__(kColCompute + 64, 2)
     mbar_fence_init();
   }
   __syncthreads();
+  pdl_wait_and_release();  // the previous iteration's decisions, G and t are visible
   const uint32_t t = init ? 0u : a.ctl->t + 1u;
   const long long items = a.n_local * (long long)nb;
 
@@ -76,18 +99,27 @@ __global__ void __launch_bounds__(kColCompute + 64, 2)
       int s = 0;
       unsigned ph = 0;
       long long i = 0;
-      for (long long k = blockIdx.x; k < items; k += gridDim.x, ++i) {
-        const long long r = k / nb;
-        const int q0 = (int)(k - r * nb) * chunk;
+      ItemWalk it(blockIdx.x, gridDim.x, nb);
+      // the lazy-pbest flag of the next item is loaded one item ahead, so its L2
+      // latency overlaps the wait for a free stage instead of delaying the copies
+      int fl_next = (!init && blockIdx.x < items) ? a.pbx[it.r] : 0;
+      for (long long k = blockIdx.x; k < items; k += gridDim.x, ++i, it.next()) {
+        const long long r = it.r;
+        const int q0 = it.b * chunk;
         const int cnt = min(chunk, nvl - q0);
         const unsigned bytes = (unsigned)cnt * 16u;
+        const int fl = fl_next;
+        if (!init && k + gridDim.x < items) {
+          ItemWalk nx = it;
+          nx.next();
+          fl_next = a.pbx[nx.r];
+        }
         if (i >= stages) mbar_wait(&empty[s], ph ^ 1u);
         float4* st = ring + (size_t)s * per * chunk;
         if (init) {
           sflag[s] = 0;
           mbar_arrive(&full[s]);
         } else {
-          const int fl = a.pbx[r];
           sflag[s] = fl;
           mbar_expect_tx(&full[s], bytes * ((fl ? 3u : 4u) + (kB ? 4u : 0u)));
           const size_t off = ((size_t)r * nvl + q0) * 4;
@@ -114,9 +146,10 @@ __global__ void __launch_bounds__(kColCompute + 64, 2)
       unsigned n_pbl = 0, n_pbs = 0;
       int s = 0, prev = -1;
       unsigned ph = 0;
-      for (long long k = blockIdx.x; k < items; k += gridDim.x) {
-        const long long r = k / nb;
-        const int b = (int)(k - r * nb);
+      ItemWalk it(blockIdx.x, gridDim.x, nb);
+      for (long long k = blockIdx.x; k < items; k += gridDim.x, it.next()) {
+        const long long r = it.r;
+        const int b = it.b;
         const int q0 = b * chunk;
         const int cnt = min(chunk, nvl - q0);
         const unsigned bytes = (unsigned)cnt * 16u;
@@ -182,9 +215,10 @@ __global__ void __launch_bounds__(kColCompute + 64, 2)
   const float4* B4 = reinterpret_cast<const float4*>(a.bounds);
   int s = 0;
   unsigned ph = 0;
-  for (long long k = blockIdx.x; k < items; k += gridDim.x) {
-    const long long r = k / nb;
-    const int q0 = (int)(k - r * nb) * chunk;
+  ItemWalk it(blockIdx.x, gridDim.x, nb);
+  for (long long k = blockIdx.x; k < items; k += gridDim.x, it.next()) {
+    const long long r = it.r;
+    const int q0 = it.b * chunk;
     const int cnt = min(chunk, nvl - q0);
     const uint32_t gi = (uint32_t)(a.row_begin + r);
     float4* st = ring + (size_t)s * per * chunk;
@@ -281,6 +315,7 @@ __global__ void __launch_bounds__(256) k_col_decide(const __grid_constant__ Swar
   __shared__ unsigned s_nimp[8];
   __shared__ int s_last;
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  pdl_wait_and_release();  // k_col_step's partials and flags are visible
   const uint32_t t = init ? 0u : a.ctl->t + 1u;
   const int par = (int)(t & 1u);
   const int nbt = a.col_nbt;

@@ -583,6 +583,24 @@ cudaError_t launch_init(int objective, const SwarmArgs& a, const LaunchCfg& c, c
 }
 
 // ---------------------------------------------------------- column split
+// A launch with programmatic stream serialization (PDL) when `pdl`: the kernel
+// is scheduled while the previous one drains and waits for it with
+// griddepcontrol.wait before its first global read.
+cudaError_t launch_pdl(const void* fn, dim3 grid, dim3 block, void** args, size_t smem, cudaStream_t s,
+                       int pdl) {
+  cudaLaunchConfig_t lc{};
+  lc.gridDim = grid;
+  lc.blockDim = block;
+  lc.dynamicSmemBytes = smem;
+  lc.stream = s;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  lc.attrs = attr;
+  lc.numAttrs = pdl ? 1 : 0;
+  return cudaLaunchKernelExC(&lc, fn, args);
+}
+
 cudaError_t plan_colsplit(int objective, int tile, int tiles_local, long long n, int sm_count,
                           bool bounds, LaunchCfg* cfg) {
   const KernelTable* t = kernel_table(objective);
@@ -590,9 +608,12 @@ cudaError_t plan_colsplit(int objective, int tile, int tiles_local, long long n,
   if (tile < 1 || tiles_local < 1 || n < 1) return cudaErrorInvalidConfiguration;
   const int per = bounds ? 8 : 4;
   const size_t stage = (size_t)per * tile * 16;
-  const int ctas = bounds ? 1 : 2;  // ~100 registers x 320 threads: 2 CTAs per SM
+  int ctas = bounds ? 1 : 2;  // ~100 registers x 320 threads: 2 CTAs per SM
+  if (const char* v = std::getenv("PSO_COL_CTAS")) ctas = std::max(1, std::min(2, std::atoi(v)));
   int stages = ring_stages(0, stage, ctas);
-  if (stages > 4) stages = 4;  // 4 tiles in flight per CTA cover the HBM latency
+  int max_st = 4;  // 4 tiles in flight per CTA cover the HBM latency
+  if (const char* v = std::getenv("PSO_COL_STAGES")) max_st = std::max(2, std::min(kMaxStages, std::atoi(v)));
+  if (stages > max_st) stages = max_st;
   if (stages < 2) return cudaErrorInvalidConfiguration;
   const void* fn = t->col_step[bounds ? 1 : 0];
   const size_t smem = (size_t)stages * stage;
@@ -626,8 +647,8 @@ cudaError_t launch_col_step(int objective, const SwarmArgs& a, const LaunchCfg& 
   if (!t) return cudaErrorInvalidDeviceFunction;
   int stages = c.col_stages;
   void* args[] = {const_cast<SwarmArgs*>(&a), &init, &stages};
-  return cudaLaunchKernel(t->col_step[c.bounds ? 1 : 0], dim3(c.col_grid), dim3(c.threads), args,
-                          c.col_smem, s);
+  return launch_pdl(t->col_step[c.bounds ? 1 : 0], dim3(c.col_grid), dim3(c.threads), args,
+                    c.col_smem, s, c.pdl);
 }
 
 cudaError_t launch_col_decide(int objective, const SwarmArgs& a, const LaunchCfg& c, int init,
@@ -635,7 +656,7 @@ cudaError_t launch_col_decide(int objective, const SwarmArgs& a, const LaunchCfg
   const KernelTable* t = kernel_table(objective);
   if (!t) return cudaErrorInvalidDeviceFunction;
   void* args[] = {const_cast<SwarmArgs*>(&a), &init};
-  return cudaLaunchKernel(t->col_decide, dim3(c.col_decide_grid), dim3(256), args, 0, s);
+  return launch_pdl(t->col_decide, dim3(c.col_decide_grid), dim3(256), args, 0, s, c.pdl);
 }
 
 cudaError_t launch_rebest(const SwarmArgs& a, unsigned t, cudaStream_t s) {

@@ -86,6 +86,10 @@ WORKLOADS = {
     "NS_R2": Workload("northstar-shard-of-2-rastrigin-50000x2000", RASTRIGIN, 50_000, 2000, 500),
     "NS_R4": Workload("northstar-shard-of-4-rastrigin-25000x2000", RASTRIGIN, 25_000, 2000, 500),
     "NS_R8": Workload("northstar-shard-of-8-rastrigin-12500x2000", RASTRIGIN, 12_500, 2000, 500),
+    # C5's optional HBM-capacity sweep: n doubled until the state nears ~80 % of
+    # the 180 GB of one B200 (12 B per element: X, V, PB; 2.9M x 4096 = 142.5 GB)
+    "C5_2M": Workload("C5-ackley-2000000x4096", ACKLEY, 2_000_000, 4096, 200),
+    "C5_2900K": Workload("C5-ackley-2900000x4096", ACKLEY, 2_900_000, 4096, 200),
     # reading 3 (vmax = 1) made visible: the survey's C4 velocity bound (vmax = 600, the
     # domain half-width) and the north-star swarm at vmax = 5.12 (its domain half-width)
     "C4_V600": Workload("C4-griewank-100000x2000-vmax600", GRIEWANK, 100_000, 2000, 500, vmax=600.0),
