@@ -306,16 +306,22 @@ def run_gpu(args, w):
             s.init()
             return s, True
         s = fp.Swarm(w.n, w.d, w.w, w.c1, w.c2, w.lo, w.hi, w.objective, w.seed, vmax=w.vmax,
-                     device=local, stream=stream, nccl_comm=comm, async_gbest=async_gbest, **kw)
+                     device=local, stream=stream, nccl_comm=comm, async_gbest=async_gbest,
+                     allreduce_exchange=xmode == "allreduce", **kw)
         # gbest exchange between ranks: NVLink peer stores from the step kernels
         # (default), or the NCCL all-gather (PSO_EXCHANGE=nccl, or if any rank
         # cannot map its peers)
         on = False
-        if use_comm and os.environ.get("PSO_EXCHANGE", "p2p") == "p2p":
+        if use_comm and xmode == "p2p":
             from paper_conf_icpp_liuwc21_b200.distributed import connect_p2p
             on = connect_p2p(s)
         return s, on
 
+    # gbest exchange for N > 1: "p2p" NVLink peer stores from the step kernels
+    # (default; falls back to the all-gather if any rank cannot map / probe its
+    # peers), "nccl" the all-gather, "allreduce" north_star's allreduce-min of the
+    # key + bit-exact sum-broadcast of the winner's row
+    xmode = os.environ.get("PSO_EXCHANGE", "p2p")
     stream = torch.cuda.Stream(device=dev)  # the library enqueues on this stream
     torch.cuda.set_stream(stream)
     K, W = args.steps, args.warmup
@@ -434,7 +440,9 @@ def run_gpu(args, w):
             "scaling": "strong", "vs_baseline": None, "dtype": "f32",
             "data": "synthetic (swarm initialised from Philox streams, seed %d)" % w.seed,
             "config": _config(w, world, K, extra={"gbest_exchange": (
-                "nvlink-peer-stores" if p2p else "nccl-allgather (CUDA graph)") if use_comm else None,
+                "nvlink-peer-stores" if p2p else
+                "nccl-allreduce-min + sum-broadcast (CUDA graph)" if xmode == "allreduce" else
+                "nccl-allgather (CUDA graph)") if use_comm else None,
                 "gbest_mode": ("async" if async_gbest else "sync") if use_comm else None,
                 **({"shared_gpu_harness_test": True} if share else {})}),
             "gpu_launches": launches,

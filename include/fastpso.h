@@ -111,6 +111,15 @@ enum {
                               world = 1 identical to the synchronous mode.
                               pso_get_gbest returns the global view folded from every
                               rank's records at the end of the last pso_step call. */
+  PSO_FLAG_ALLREDUCE = 32,  /* NCCL exchange as north_star states it:
+                              per iteration an ncclAllReduce(min) of the u64 packed
+                              (fitness, index) keys, then the owning rank's candidate
+                              row is broadcast bit-exactly by an ncclAllReduce(sum) of
+                              the row as u32 words to which every other rank adds
+                              zeros (root decided on the device, no host sync).
+                              Default: one ncclAllGather of the (key, row) records.
+                              Either is replaced by the NVLink peer exchange once
+                              pso_p2p_enable(h, 1) succeeds. */
   PSO_FLAG_DEVICE = 16,     /* use pso_opts.device as the CUDA ordinal; without it the
                               handle runs on the caller's current device (so a
                               zero-initialised pso_opts means "defaults") */

@@ -12,7 +12,7 @@ import ctypes as C
 import numpy as np
 
 from ._lib import (EXPORTS, PSO_D_AUTO_COLSPLIT, PSO_D_MAX, PSO_D_MAX_ROW, PSO_FLAG_ASYNC_GBEST,
-                   PSO_FLAG_COLUMN_SPLIT, PSO_FLAG_DEFER_INIT, PSO_FLAG_DEVICE, PSO_FLAG_TIMING, PSO_OBJ_ACKLEY, PSO_OBJ_CUSTOM_BASE,
+                   PSO_FLAG_ALLREDUCE, PSO_FLAG_COLUMN_SPLIT, PSO_FLAG_DEFER_INIT, PSO_FLAG_DEVICE, PSO_FLAG_TIMING, PSO_OBJ_ACKLEY, PSO_OBJ_CUSTOM_BASE,
                    PSO_OBJ_EASOM, PSO_OBJ_GRIEWANK, PSO_OBJ_RASTRIGIN, PSO_OBJ_ROSENBROCK,
                    PSO_OBJ_SPHERE, PSO_OK, PsoError, check, last_error, lib, pso_info, pso_opts,
                    status_string)
@@ -68,7 +68,8 @@ class Swarm:
                  objective: int, seed: int, *, vmax: float = 0.0, device: int = -1,
                  stream=None, nccl_comm=None, timing: bool = False, bounds=None,
                  world: int = 1, rank: int = 0, defer_init: bool = False,
-                 async_gbest: bool = False, column_split: bool = False):
+                 async_gbest: bool = False, column_split: bool = False,
+                 allreduce_exchange: bool = False):
         L = lib()
         opts = pso_opts()
         opts.vmax = float(vmax)
@@ -79,7 +80,8 @@ class Swarm:
         opts.flags = ((PSO_FLAG_TIMING if timing else 0) | (PSO_FLAG_DEFER_INIT if defer_init else 0)
                       | (PSO_FLAG_ASYNC_GBEST if async_gbest else 0)
                       | (PSO_FLAG_COLUMN_SPLIT if column_split else 0)
-                      | (PSO_FLAG_DEVICE if device >= 0 else 0))
+                      | (PSO_FLAG_DEVICE if device >= 0 else 0)
+                      | (PSO_FLAG_ALLREDUCE if allreduce_exchange else 0))
         opts.world, opts.rank = int(world), int(rank)
         if bounds is not None:  # per-dimension [vlo | vhi | xlo | xhi], 4 x d
             bounds = np.ascontiguousarray(bounds, dtype=np.float32).reshape(4 * int(d))

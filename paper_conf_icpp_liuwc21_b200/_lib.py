@@ -18,6 +18,7 @@ PSO_OBJ_SPHERE, PSO_OBJ_RASTRIGIN, PSO_OBJ_ROSENBROCK = 1, 2, 3
 PSO_OBJ_GRIEWANK, PSO_OBJ_ACKLEY, PSO_OBJ_EASOM, PSO_OBJ_CUSTOM_BASE = 4, 5, 6, 64
 PSO_FLAG_TIMING, PSO_FLAG_DEFER_INIT, PSO_FLAG_ASYNC_GBEST, PSO_FLAG_COLUMN_SPLIT = 1, 2, 4, 8
 PSO_FLAG_DEVICE = 16
+PSO_FLAG_ALLREDUCE = 32
 PSO_D_MAX_ROW = 65536
 PSO_D_AUTO_COLSPLIT = 16384
 PSO_D_MAX = 1 << 24

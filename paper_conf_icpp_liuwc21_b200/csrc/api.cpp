@@ -66,7 +66,8 @@ typedef struct {
   char internal[128];
 } ncclUniqueId;
 typedef int ncclResult_t;  // ncclSuccess == 0
-enum { kNcclUint8 = 1 };
+enum { kNcclUint8 = 1, kNcclUint32 = 3, kNcclUint64 = 5 };  // ncclDataType_t
+enum { kNcclSum = 0, kNcclMin = 3 };                          // ncclRedOp_t
 
 struct NcclApi {
   void* handle = nullptr;
@@ -77,6 +78,7 @@ struct NcclApi {
   ncclResult_t (*CommUserRank)(ncclComm_t, int*) = nullptr;
   ncclResult_t (*CommGetAsyncError)(ncclComm_t, ncclResult_t*) = nullptr;
   ncclResult_t (*AllGather)(const void*, void*, size_t, int, ncclComm_t, cudaStream_t) = nullptr;
+  ncclResult_t (*AllReduce)(const void*, void*, size_t, int, int, ncclComm_t, cudaStream_t) = nullptr;
   const char* (*GetErrorString)(ncclResult_t) = nullptr;
   std::string error;
 };
@@ -114,6 +116,7 @@ NcclApi* nccl() {
   PSO_SYM(CommUserRank, "ncclCommUserRank")
   PSO_SYM(CommGetAsyncError, "ncclCommGetAsyncError")
   PSO_SYM(AllGather, "ncclAllGather")
+  PSO_SYM(AllReduce, "ncclAllReduce")
   PSO_SYM(GetErrorString, "ncclGetErrorString")
 #undef PSO_SYM
   return &api;
@@ -169,6 +172,7 @@ struct pso_swarm {
   // NCCL exchange: captured [step, all-gather] x kGraphIters, one per slot phase
   cudaGraphExec_t nccl_graph[4] = {nullptr, nullptr, nullptr, nullptr};
   bool graph_off = false;
+  bool allreduce = false;  // PSO_FLAG_ALLREDUCE: NCCL exchange as allreduce-min + sum-broadcast
 };
 
 namespace {
@@ -207,14 +211,31 @@ pso_status use_device(pso_swarm* h) {
   return PSO_OK;
 }
 
-// All-gather the records of iteration t (one per rank: its best candidate key
-// and row) into recv[t & 1].  The next step kernel merges them in its
+// The NCCL exchange of one iteration (records of iteration t into slot t & 3):
+// the all-gather of every rank's record, or -- PSO_FLAG_ALLREDUCE, the north
+// star's collective -- an allreduce-min of the u64 keys into record 0, the
+// owner kernel (the winner's row or zeros), and an allreduce-sum of the row as
+// u32 words (a bit-exact broadcast from the device-decided owner).
+ncclResult_t nccl_exchange(pso_swarm* h, NcclApi* a, uint64_t t, bool* launched_kernel) {
+  const size_t rec = record_bytes(h->pitch);
+  unsigned char* dst = const_cast<unsigned char*>(h->args.recv) + (t & 3) * (size_t)h->world * rec;
+  *launched_kernel = false;
+  if (!h->allreduce) return a->AllGather(h->args.send, dst, rec, kNcclUint8, h->comm, h->stream);
+  ncclResult_t r = a->AllReduce(h->args.send, dst, 1, kNcclUint64, kNcclMin, h->comm, h->stream);
+  if (r != 0) return r;
+  if (launch_owner_row(h->args, h->stream) != cudaSuccess) return 1;  // reported as an NCCL failure
+  *launched_kernel = true;
+  return a->AllReduce(dst + 16, dst + 16, (size_t)h->pitch, kNcclUint32, kNcclSum, h->comm, h->stream);
+}
+
+// Exchange the records of iteration t (one per rank: its best candidate key
+// and row) into recv slot t & 3 (NCCL: nccl_exchange; NVLink: already stored
+// by the step kernels).  The next step kernel merges them in its
 // prologue; `fold` additionally runs the select kernel so key_cur / G are
 // final for the host (end of create, set_state and every pso_step call).
 pso_status exchange(pso_swarm* h, uint64_t t, bool fold, bool into_local) {
   NvtxRange nvtx_range("gbest exchange");
   if (!h->xchg || h->colsplit) return PSO_OK;  // the column split exchanges inside its kernels
-  const size_t rec = record_bytes(h->pitch);
   if (h->args.p2p) {  // records travel by NVLink peer stores inside the kernels
     if (fold) {
       PSO_CUDA(h, launch_select(h->args, (unsigned)t, into_local, h->stream));
@@ -231,11 +252,13 @@ pso_status exchange(pso_swarm* h, uint64_t t, bool fold, bool into_local) {
     h->poisoned = true;
     return fail(PSO_ERR_NCCL, "NCCL unavailable");
   }
-  unsigned char* dst = const_cast<unsigned char*>(h->args.recv) + (t & 3) * (size_t)h->world * rec;
-  ncclResult_t r = a->AllGather(h->args.send, dst, rec, kNcclUint8, h->comm, h->stream);
+  bool kern = false;
+  ncclResult_t r = nccl_exchange(h, a, t, &kern);
+  if (kern) ++h->launches;
   if (r != 0) {
     h->poisoned = true;
-    return fail(PSO_ERR_NCCL, "ncclAllGather: %s", nccl_str(r));
+    return fail(PSO_ERR_NCCL, "%s: %s", h->allreduce ? "ncclAllReduce exchange" : "ncclAllGather",
+                nccl_str(r));
   }
   if (fold) {
     PSO_CUDA(h, launch_select(h->args, (unsigned)t, into_local, h->stream));
@@ -245,8 +268,8 @@ pso_status exchange(pso_swarm* h, uint64_t t, bool fold, bool into_local) {
 }
 
 // Capture kGraphIters iterations of the NCCL exchange path starting at slot
-// phase `phase` ([step kernel, all-gather into recv slot (t & 3)] each) into an
-// executable graph.  The step kernel reads its iteration from the control block,
+// phase `phase` ([step kernel, nccl_exchange into recv slot (t & 3)] each) into
+// an executable graph.  The step kernel reads its iteration from the control block,
 // so the graph is valid for every start iteration with the same t & 3.  If the
 // capture fails (e.g. NCCL without graph support) the handle stays eager.
 pso_status capture_nccl_graph(pso_swarm* h, int phase) {
@@ -256,12 +279,10 @@ pso_status capture_nccl_graph(pso_swarm* h, int phase) {
   cudaGraph_t g = nullptr;
   cudaError_t e = cudaStreamBeginCapture(h->stream, cudaStreamCaptureModeThreadLocal);
   bool ok = e == cudaSuccess;
-  const size_t rec = record_bytes(h->pitch);
   for (int k = 0; ok && k < kGraphIters; ++k) {
     ok = launch_step(h->objective, h->args, h->cfg, h->stream) == cudaSuccess;
-    unsigned char* dst = const_cast<unsigned char*>(h->args.recv) +
-                         (size_t)((phase + k) & 3) * (size_t)h->world * rec;
-    ok = ok && a->AllGather(h->args.send, dst, rec, kNcclUint8, h->comm, h->stream) == 0;
+    bool kern = false;
+    ok = ok && nccl_exchange(h, a, (uint64_t)((phase + k) & 3), &kern) == 0;
   }
   if (e == cudaSuccess) {
     cudaError_t e2 = cudaStreamEndCapture(h->stream, &g);
@@ -476,7 +497,7 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
   if (!objective_registered(objective))
     return fail(PSO_ERR_INVALID, "objective %d is not registered", objective);
   if (o.flags & ~(uint32_t)(PSO_FLAG_TIMING | PSO_FLAG_DEFER_INIT | PSO_FLAG_ASYNC_GBEST |
-                            PSO_FLAG_COLUMN_SPLIT | PSO_FLAG_DEVICE))
+                            PSO_FLAG_COLUMN_SPLIT | PSO_FLAG_DEVICE | PSO_FLAG_ALLREDUCE))
     return fail(PSO_ERR_INVALID, "unknown flags 0x%x", o.flags);
   if (o.bounds) {
     pso_status bs = check_bounds(o.bounds, d);
@@ -685,6 +706,8 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
   A.world = h->world;
   A.rank = h->rank;
   A.exchange = (h->xchg && !colsplit) ? 1 : 0;
+  h->allreduce = (o.flags & PSO_FLAG_ALLREDUCE) != 0;
+  A.xrecs = h->allreduce ? 1 : h->world;
   A.colsplit = colsplit ? 1 : 0;
   A.col_q0 = col_q0;
   A.nvec_glob = (d + 3) / 4;
@@ -799,7 +822,7 @@ pso_status pso_step(pso_handle h, int64_t iters) {
       if (!h->nccl_graph[phase] && (st = capture_nccl_graph(h, phase)) != PSO_OK) return st;
       if (!h->nccl_graph[phase]) break;  // capture unavailable: eager from here on
       PSO_CUDA(h, cudaGraphLaunch(h->nccl_graph[phase], h->stream));
-      h->launches += kGraphIters;
+      h->launches += kGraphIters * (h->allreduce ? 2 : 1);  // step (+ owner-row) kernels
       it += kGraphIters;
     }
   }
@@ -1017,6 +1040,9 @@ pso_status pso_p2p_enable(pso_handle h, int32_t on) {
   if ((st = use_device(h)) != PSO_OK) return st;
   if ((st = sync_and_check(h)) != PSO_OK) return st;
   h->args.p2p = on ? 1 : 0;
+  h->args.xrecs = (on || !h->allreduce) ? h->world : 1;
+  for (cudaGraphExec_t& g : h->nccl_graph)  // captured with the previous exchange's arguments
+    if (g) cudaGraphExecDestroy(g), g = nullptr;
   return PSO_OK;
 }
 

@@ -69,6 +69,8 @@ struct SwarmArgs {
   int world;
   int rank;
   int exchange;               // 1: publish (key, row) records for the all-gather + select
+  int xrecs;                  // records per iteration slot the merges read: world (all-gather,
+                              // NVLink), or 1 (allreduce exchange: the reduced record)
   int p2p;                    // exchange over NVLink peer stores instead of NCCL
   int async_gbest;            // NEXT-4: merge peers' records with a one-iteration lag
   float* G_view;              // async: the host's global gbest view (pitch floats)
@@ -200,6 +202,10 @@ cudaError_t launch_select(const SwarmArgs& a, unsigned t, bool into_local, cudaS
 // A rank without particles: its share of iteration t of the exchange (merge the
 // records of t - 1 if `merge`, publish a "no candidate" record of t).
 cudaError_t launch_empty_step(const SwarmArgs& a, unsigned t, bool merge, cudaStream_t s);
+// Allreduce exchange: after the allreduce-min of the keys into record 0 of the
+// current slot, the owner of the winning key writes its candidate row there and
+// every other rank zeros it (the allreduce-sum that follows broadcasts the bits).
+cudaError_t launch_owner_row(const SwarmArgs& a, cudaStream_t s);
 // NVLink connect probe: phase 0 stores this rank's token into every peer's probe
 // slot; phase 1 (after a host barrier) checks that every peer's token arrived in
 // ours (*ok_dev = 1) and clears the slots.

@@ -68,7 +68,7 @@ __global__ void __launch_bounds__(128) k_select(const SwarmArgs a, unsigned t, i
       const unsigned it = t - (unsigned)k;
       if (a.p2p) wait_records(a, it);
       const unsigned char* base = records(a, it);
-      for (int r = 0; r < a.world; ++r) {
+      for (int r = 0; r < a.xrecs; ++r) {
         const unsigned long long key =
             *reinterpret_cast<const unsigned long long*>(base + (size_t)r * rec);
         if ((key >> 32) < (cur >> 32) && key < best) {
@@ -113,6 +113,7 @@ __global__ void __launch_bounds__(32) k_empty_step(const SwarmArgs a, unsigned t
       unsigned long long* hdr = reinterpret_cast<unsigned long long*>(a.send);
       hdr[0] = ~0ull;
       hdr[1] = tag;
+      a.ctl->t = t;  // the allreduce exchange's owner kernel reads the slot from it
     }
     return;
   }
@@ -130,14 +131,38 @@ __global__ void __launch_bounds__(32) k_empty_step(const SwarmArgs a, unsigned t
     if (lane == 0) {
       a.ctl->key_cur = best;
       a.ctl->key_view = best;
-      a.ctl->t = t;
     }
   }
+  if (lane == 0) a.ctl->t = t;
   const size_t rec = record_bytes(a.nvec * 4);
   const size_t off = (size_t)(t & 3u) * a.world * rec + (size_t)a.rank * rec;
   for (int r = lane; r < a.world; r += 32) reinterpret_cast<unsigned long long*>(a.peers[r] + off)[0] = ~0ull;
   __syncwarp();
   for (int r = lane; r < a.world; r += 32) st_release_sys_u64(a.peers[r] + off + 8, tag);
+}
+
+// ---------------------------------------------------------- allreduce exchange
+// The north star's collective: the records of iteration t are
+// reduced into record 0 of slot t & 3 -- ncclAllReduce(min) of the u64 keys,
+// then this kernel, then ncclAllReduce(sum) of the row as u32 words.  Here the
+// rank whose candidate is the global minimum writes its row, every other rank
+// zeros, so the sum is the owner's row bit for bit (a broadcast whose root is
+// decided on the device, no host round trip).  Keys hold the global particle
+// index, so exactly one rank owns a winning key; with no candidate anywhere
+// (key ~0) every rank writes zeros and the merge ignores the record.  The
+// iteration comes from the control block (graph-capturable).
+__global__ void __launch_bounds__(256) k_owner_row(const SwarmArgs a) {
+  const uint32_t t = a.ctl->t;
+  unsigned char* rec = const_cast<unsigned char*>(records(a, t));
+  const unsigned long long g = *reinterpret_cast<const volatile unsigned long long*>(rec);
+  const unsigned long long mine = *reinterpret_cast<const unsigned long long*>(a.send);
+  const bool own = g != ~0ull && g == mine;
+  const float4* src = reinterpret_cast<const float4*>(a.send + 16);
+  float4* dst = reinterpret_cast<float4*>(rec + 16);
+  for (int q = threadIdx.x; q < a.nvec; q += blockDim.x)
+    dst[q] = own ? src[q] : make_float4(0.f, 0.f, 0.f, 0.f);
+  if (threadIdx.x == 0)
+    reinterpret_cast<unsigned long long*>(rec)[1] = ((unsigned long long)a.epoch << 32) | t;
 }
 
 // ---------------------------------------------------------- NVLink probe
@@ -672,6 +697,11 @@ cudaError_t launch_materialize_pb(const SwarmArgs& a, cudaStream_t s) {
   long long blocks = (a.n_local + 7) / 8;
   if (blocks > 2048) blocks = 2048;
   k_materialize_pb<<<(unsigned)blocks, 256, 0, s>>>(a);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_owner_row(const SwarmArgs& a, cudaStream_t s) {
+  k_owner_row<<<1, 256, 0, s>>>(a);
   return cudaGetLastError();
 }
 

@@ -608,7 +608,7 @@ __device__ __forceinline__ unsigned long long exchange_merge(const SwarmArgs& a,
   const unsigned long long cur = *(volatile unsigned long long*)&a.ctl->key_cur;
   unsigned long long best = cur;
   int s = -1;
-  for (int r = 0; r < a.world; ++r) {
+  for (int r = 0; r < a.xrecs; ++r) {
     const unsigned long long k = *reinterpret_cast<const unsigned long long*>(base + (size_t)r * rec);
     // strictly better fitness than the incumbent (Alg. 1 line 10), then the
     // lowest key: in the synchronous mode every record already satisfies it
@@ -634,7 +634,7 @@ __device__ __forceinline__ unsigned long long exchange_merge_warp(const SwarmArg
   const unsigned long long t0 = globaltimer_ns();
   unsigned long long best = cur;
   int s = -1;
-  for (int r = lane; r < a.world; r += 32) {
+  for (int r = lane; r < a.xrecs; r += 32) {
     if (a.p2p) {
       while (ld_acquire_sys_u64(base + (size_t)r * rec + 8) != want) {
         __nanosleep(64);

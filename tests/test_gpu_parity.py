@@ -387,24 +387,32 @@ def test_full_size_sampled_rows(key):
 
 
 # ------------------------------------------------------------------ exchange path
+@pytest.mark.parametrize("mode", ["allgather", "allreduce", "allgather-eager", "allreduce-eager"])
 @pytest.mark.parametrize("obj,n,d", [(RASTRIGIN, 300, 1000), (GRIEWANK, 50, 13),
                                      (ROSENBROCK, 6, 10000)])
-def test_exchange_path_with_single_rank_comm(obj, n, d, monkeypatch):
-    """The multi-GPU exchange (records -> ncclAllGather -> k_select) forced on a
-    1-rank NCCL communicator must give the single-GPU results bitwise."""
+def test_exchange_path_with_single_rank_comm(obj, n, d, mode, monkeypatch):
+    """The NCCL exchanges forced on a 1-rank communicator must give the
+    single-GPU results bitwise: the all-gather of the (key, row) records, and
+    north_star's allreduce-min of the key + sum-broadcast of the owner's row
+    (PSO_FLAG_ALLREDUCE); both replayed as captured CUDA graphs of 4
+    iterations, or launched eagerly (PSO_GRAPH=0)."""
     import torch  # noqa: F401  (loads the NCCL the library resolves)
     monkeypatch.setenv("PSO_FORCE_EXCHANGE", "1")
+    if mode.endswith("-eager"):
+        monkeypatch.setenv("PSO_GRAPH", "0")
     comm = fp.nccl_comm_init(1, fp.nccl_unique_id(), 0, 0)
     try:
-        g = gpu_swarm(n, d, obj, seed=5, nccl_comm=comm)
+        g = gpu_swarm(n, d, obj, seed=5, nccl_comm=comm,
+                      allreduce_exchange=mode.startswith("allreduce"))
         ref = gpu_swarm(n, d, obj, seed=5)
         assert g.gbest()[:2] == ref.gbest()[:2]
         g.reset_counters()
         g.step(20)
         ref.step(20)
         # one step kernel per iteration (the exchange merge runs in the next
-        # step's prologue) + one select kernel at the end of the call
-        assert g.info()["launches"] == 21
+        # step's prologue) + one select kernel at the end of the call; the
+        # allreduce exchange adds its owner-row kernel per iteration
+        assert g.info()["launches"] == (41 if mode.startswith("allreduce") else 21)
         g.step(1).step(2)
         ref.step(3)
         for x, y in zip(g.get_state()[:4], ref.get_state()[:4]):

@@ -18,7 +18,7 @@ timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -c 40 --cs
 R=${NCU_REP_DIR:-/tmp/ncu_reps}
 mkdir -p $R
 for w in ${NCU_WORKLOADS:-NS C4 C3 C5 W16K W64K}; do
-  timeout 900 ncu --set full --clock-control none --import-source on -k regex:"k_step|k_col_step" -s 8 -c 1 \
+  timeout 900 ncu --set full --metrics lts__t_bytes.sum,lts__t_sector_hit_rate.pct --clock-control none --import-source on -k regex:"k_step|k_col_step" -s 8 -c 1 \
     -o $R/prof_$w -f python bench.py --workload $w --steps 10 --warmup 5 --no-e2e --no-cpu-baseline > $O/ncu_$w.log 2>&1
   python tools/ncu_summary.py $R/prof_$w.ncu-rep > $O/ncu_summary_$w.txt 2>&1
 done
