@@ -12,6 +12,7 @@ NCCL_INC ?= $(shell python -c "import os, nvidia.nccl as m; print(os.path.join(l
 ARCH     := -gencode arch=compute_100a,code=sm_100a
 NVFLAGS  := $(ARCH) -O3 -lineinfo -std=c++17 -Xcompiler -fPIC,-O3,-Wall \
             -Xptxas -v -I include -I $(CSRC) $(if $(NCCL_INC),-I $(NCCL_INC) -DPSO_HAVE_NCCL_H=1,)
+NVFLAGS  += $(EXTRA)
 CU_SRCS  := $(wildcard $(CSRC)/*.cu)
 CPP_SRCS := $(wildcard $(CSRC)/*.cpp)
 HDRS     := $(wildcard $(CSRC)/*.cuh) $(wildcard $(CSRC)/*.h) include/fastpso.h
