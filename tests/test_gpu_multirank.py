@@ -231,7 +231,8 @@ def _async_worker(rank, world, port, n, d, obj, steps, out_dir):
 
 
 @pytest.mark.parametrize("world,obj,n,d", [(2, RASTRIGIN, 40, 300), (3, GRIEWANK, 30, 13),
-                                           (2, ROSENBROCK, 4, 9000)])
+                                           (2, ROSENBROCK, 4, 9000), (3, SPHERE, 2, 300),
+                                           (8, RASTRIGIN, 50, 1000)])
 def test_async_split_matches_the_async_oracle(tmp_path, world, obj, n, d):
     """NEXT-4: each rank adopts its own candidates at once and its peers' one
     iteration late (merging records of t - 2 over NVLink); set_state mid-run
