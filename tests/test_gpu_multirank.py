@@ -75,7 +75,8 @@ def _load(path):
     return out, z
 
 
-def _worker(rank, world, port, n, d, obj, seed, ops, out_dir, params=(0.9, 2.0, 2.0, None)):
+def _worker(rank, world, port, n, d, obj, seed, ops, out_dir, params=(0.9, 2.0, 2.0, None),
+            bounds=None, column_split=False):
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)
     dist.init_process_group("gloo", rank=rank, world_size=world)
@@ -83,11 +84,15 @@ def _worker(rank, world, port, n, d, obj, seed, ops, out_dir, params=(0.9, 2.0, 
     w, c1, c2, dom = params
     lo, hi = dom or DOMAINS[obj]
     s = fp.Swarm(n, d, w, c1, c2, lo, hi, obj, seed, device=0, world=world, rank=rank,
-                 defer_init=True)
+                 defer_init=True, bounds=bounds, column_split=column_split)
     assert connect_p2p(s)
     s.init()
-    snaps = _run_ops(s, ops, rows=row_range(n, rank, world))
-    _save(out_dir, "r", rank, snaps, launches=s.info()["launches"])
+    info = s.info()
+    if column_split:
+        snaps = _run_ops(s, ops, cols=(info["col_begin"], info["col_begin"] + info["d_local"]))
+    else:
+        snaps = _run_ops(s, ops, rows=row_range(n, rank, world))
+    _save(out_dir, "r", rank, snaps, launches=info["launches"])
     s.close()
     dist.barrier()
     dist.destroy_process_group()
@@ -317,3 +322,35 @@ def test_column_split_processes_match_the_oracle(tmp_path, world, obj, n, d):
         for k in ("X", "V", "PB", "pf", "G"):
             assert_bitwise(a[k], b[k], f"snapshot {j} {k} vs 1 process")
         assert (a["f"], a["i"], a["t"]) == (b["f"], b["i"], b["t"])
+
+
+@pytest.mark.parametrize("split,world,obj,n,d", [("particle", 3, RASTRIGIN, 40, 1000),
+                                                 ("particle", 2, ROSENBROCK, 9, 2001),
+                                                 ("column", 3, RASTRIGIN, 12, 6001),
+                                                 ("column", 2, GRIEWANK, 7, 9000)])
+def test_processes_with_per_dimension_bounds_match_the_oracle(tmp_path, split, world, obj, n, d):
+    """NEXT-2's per-dimension velocity bounds and domains (Eq. 5's
+    lower/upper_bound_j) across rank processes: the particle split
+    (every rank holds the whole bounds table) and the column split (each rank
+    its block of it) equal the oracle call by call."""
+    rng = np.random.default_rng(d)
+    xlo = rng.uniform(-5, -0.5, d).astype(np.float32)
+    xhi = (xlo + rng.uniform(0.5, 6, d)).astype(np.float32)
+    vhi = rng.uniform(0.05, 2, d).astype(np.float32)
+    vlo = (-rng.uniform(0.05, 2, d)).astype(np.float32)
+    bounds = np.stack([vlo, vhi, xlo, xhi])
+    seed = 31
+    ops = [("step", 1), ("step", 3), ("restore", None), ("step", 2)]
+    lo, hi = DOMAINS[obj]
+    mp.spawn(_worker, args=(world, _free_port(), n, d, obj, seed, ops, str(tmp_path),
+                            (0.9, 2.0, 2.0, None), bounds, split == "column"),
+             nprocs=world, join=True)
+    snaps = _gathered(tmp_path, "r", world, axis=1 if split == "column" else 0)
+
+    def make_oracle(create):
+        return orc.OracleSwarm(n, d, 0.9, 2.0, 2.0, lo, hi, obj, seed, create=create, bounds=bounds,
+                               nshards=world if split == "particle" else 1)
+
+    skip_state, skip_g = oracle_lockstep(make_oracle, obj, snaps, _oracle_ops(ops, snaps),
+                                         f"{split} bounds world={world}")
+    assert skip_state <= 1 and skip_g <= 2, (skip_state, skip_g)
