@@ -40,6 +40,13 @@
 #include "objectives.cuh"
 #include "philox.cuh"
 
+// The row-invariant Philox rounds in the 256-thread instantiation as well (scalar
+// bounds only; the per-dimension-bounds variants would pass 88 registers).
+// Round 2, A/B of two builds on one box: C4 526.6 -> 523.9 us, NS 642.9 -> 641.0 us
+// (round 1 had measured NS +0.8 % with an earlier version of the kernel).
+#ifndef PSO_SLOT_PHILOX_NARROW
+#define PSO_SLOT_PHILOX_NARROW 1
+#endif
 #ifndef PSO_SLOT_PHILOX
 #define PSO_SLOT_PHILOX 1
 #endif
@@ -1083,9 +1090,11 @@ __global__ void __launch_bounds__(kMaxT + 64, kMaxT > kMaxThreads ? 1 : 2)
     }
   }
   // row-invariant Philox rounds of this thread's slots (VPT <= 2: registers)
-  // Only in the wide (512-thread, 1 CTA/SM) instantiation: C5 12.62 -> 12.36 ms; in the
-  // 256-thread one it cost NS 618 -> 623 us and Rosenbrock 11 registers (A/B of two builds)
-  constexpr bool kSlotRng = PSO_SLOT_PHILOX && VPT <= 2 && !Obj::kNeighbor && (kMaxT > kMaxThreads);
+  // Wide (512-thread, 1 CTA/SM) instantiation: C5 12.62 -> 12.36 ms; 256-thread one:
+  // see PSO_SLOT_PHILOX_NARROW (scalar bounds; not for neighbour functors: Rosenbrock
+  // +11 registers)
+  constexpr bool kSlotRng = PSO_SLOT_PHILOX && VPT <= 2 && !Obj::kNeighbor &&
+                            (kMaxT > kMaxThreads || (PSO_SLOT_PHILOX_NARROW && !kB));
   const PhiloxIter pit = philox_iter(key, t);
   PhiloxSlot ps1[VPT], ps2[VPT];
   if constexpr (kSlotRng) {
