@@ -184,3 +184,14 @@ def test_host_buffer_validation():
     ro.flags.writeable = False
     with pytest.raises(ValueError):
         _ptr(ro, 3, writable=True)
+
+
+def test_header_flags_and_objectives_match_binding():
+    src = open(os.path.join(ROOT, "include", "fastpso.h")).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    consts = dict((k, int(v)) for k, v in re.findall(r"\b(PSO_(?:FLAG|OBJ)_[A-Z_]+)\s*=\s*(\d+)", src))
+    assert len(consts) >= 13
+    for k, v in consts.items():
+        assert getattr(_lib, k) == v, k
+    flags = [v for k, v in consts.items() if k.startswith("PSO_FLAG_")]
+    assert all(f & (f - 1) == 0 for f in flags) and len(set(flags)) == len(flags)
