@@ -297,7 +297,9 @@ pso_status pso_nccl_comm_destroy(void* comm);
  * ranks agree that all connected, and then every rank calls
  * pso_p2p_enable(h, 1).  Record tags carry an epoch that pso_set_state
  * advances, so records of an earlier state never match.  A peer that stops
- * delivering makes the waiting kernels trap after 60 s. */
+ * delivering makes the waiting kernels trap after 60 s (PSO_PEER_TIMEOUT_S sets
+ * another limit, read at create): the handle is then poisoned (PSO_ERR_CUDA at the
+ * next synchronising call) instead of the GPU hanging. */
 pso_status pso_p2p_handle(pso_handle h, void* ipc_handle /* 64 bytes */, uint64_t* offset);
 pso_status pso_p2p_connect(pso_handle h, const void* ipc_handles /* world x 64 bytes */,
                            const uint64_t* offsets /* world */);

@@ -699,6 +699,11 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
   A.send = sendb ? p : nullptr; p += sendb;
   A.recv = recvb ? p : nullptr;
   A.probe_off = align_up(recvb, 256);
+  A.peer_timeout_ns = 60ull * 1000000000ull;  // PSO_PEER_TIMEOUT_S overrides (seconds)
+  if (const char* v = std::getenv("PSO_PEER_TIMEOUT_S")) {
+    const double sec = std::atof(v);
+    if (sec > 0) A.peer_timeout_ns = (unsigned long long)(sec * 1e9);
+  }
   A.n_local = h->n_local;
   A.row_begin = h->row_begin;
   A.d = d;

@@ -77,6 +77,8 @@ struct SwarmArgs {
   unsigned epoch;             // p2p: record tags are (epoch << 32 | t); set_state starts an epoch
   unsigned t_base;            // async: iteration of the last create/set_state (records start there)
   unsigned char* const* peers;  // p2p: device array, world pointers to every rank's recv
+  unsigned long long peer_timeout_ns;  // p2p: a peer record not arriving within this traps the
+                                       // kernel (a dead rank poisons the handle instead of hanging)
   unsigned long long probe_off; // p2p: offset from a recv base to the connect probe slots (world u64)
   // Column split (NEXT-3, "tile matrix"): this rank holds float4 columns
   // [col_q0, col_q0 + nvec) of every row (n_local = n); X, V, PB, G, bounds are

@@ -326,7 +326,7 @@ __global__ void __launch_bounds__(256) k_col_decide(const __grid_constant__ Swar
       const void* tag = a.recv + ((size_t)par * a.world + q) * 8;
       while (ld_acquire_sys_u64(tag) != want) {
         __nanosleep(64);
-        if (globaltimer_ns() - t0 > 60ull * 1000000000ull) __trap();
+        if (globaltimer_ns() - t0 > a.peer_timeout_ns) __trap();
       }
     }
   }

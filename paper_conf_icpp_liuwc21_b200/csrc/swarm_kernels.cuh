@@ -599,7 +599,7 @@ __device__ __forceinline__ void wait_records(const SwarmArgs& a, uint32_t t) {
     const unsigned long long want = ((unsigned long long)a.epoch << 32) | t;
     while (ld_acquire_sys_u64(tag) != want) {
       __nanosleep(64);
-      if (globaltimer_ns() - t0 > 60ull * 1000000000ull) __trap();
+      if (globaltimer_ns() - t0 > a.peer_timeout_ns) __trap();
     }
   }
   fence_proxy_async_global();  // the records are then read by bulk copies too
@@ -645,7 +645,7 @@ __device__ __forceinline__ unsigned long long exchange_merge_warp(const SwarmArg
     if (a.p2p) {
       while (ld_acquire_sys_u64(base + (size_t)r * rec + 8) != want) {
         __nanosleep(64);
-        if (globaltimer_ns() - t0 > 60ull * 1000000000ull) __trap();
+        if (globaltimer_ns() - t0 > a.peer_timeout_ns) __trap();
       }
     }
     const unsigned long long k = *reinterpret_cast<const volatile unsigned long long*>(base + (size_t)r * rec);

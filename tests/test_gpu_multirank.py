@@ -354,3 +354,43 @@ def test_processes_with_per_dimension_bounds_match_the_oracle(tmp_path, split, w
     skip_state, skip_g = oracle_lockstep(make_oracle, obj, snaps, _oracle_ops(ops, snaps),
                                          f"{split} bounds world={world}")
     assert skip_state <= 1 and skip_g <= 2, (skip_state, skip_g)
+
+
+def _dead_peer_worker(rank, world, port, out_dir):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    os.environ["PSO_PEER_TIMEOUT_S"] = "2"
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    import time
+    from paper_conf_icpp_liuwc21_b200.distributed import connect_p2p
+    s = fp.Swarm(64, 300, 0.9, 2.0, 2.0, -5.12, 5.12, RASTRIGIN, 5, device=0, world=world,
+                 rank=rank, defer_init=True)
+    assert connect_p2p(s)
+    s.init()
+    if rank == 0:  # rank 1 never steps: the second iteration's prologue waits for its record
+        t0 = time.time()
+        status, msg = -1, ""
+        try:
+            s.step(3)
+            s.gbest()
+        except fp.PsoError as e:
+            status, msg = e.status, str(e)
+        try:
+            s.gbest()
+        except fp.PsoError as e:
+            msg += " | then: " + str(e)
+        with open(os.path.join(out_dir, "dead_peer.txt"), "w") as fh:
+            fh.write(f"{status}\n{time.time() - t0:.2f}\n{msg}\n")
+    dist.barrier()  # rank 1 stays alive (its memory mapped) until rank 0 has seen the failure
+    os._exit(0)
+
+
+def test_dead_peer_traps_and_poisons_instead_of_hanging(tmp_path):
+    """A rank that stops delivering its records (here: it never steps) makes
+    the waiting step kernel trap after the peer timeout (PSO_PEER_TIMEOUT_S=2)
+    -- the handle reports PSO_ERR_CUDA and is poisoned, nothing hangs."""
+    mp.spawn(_dead_peer_worker, args=(2, _free_port(), str(tmp_path)), nprocs=2, join=True)
+    status, secs, msg = open(tmp_path / "dead_peer.txt").read().split("\n")[:3]
+    assert int(status) == 3, msg  # PSO_ERR_CUDA
+    assert 1.5 < float(secs) < 30, secs
+    assert "POISONED" in msg, msg
