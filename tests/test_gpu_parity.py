@@ -874,3 +874,26 @@ def test_column_split_end_to_end_c1_gbest():
     c.step(w.iters)
     gf, _, _ = g.gbest()
     assert abs(gf - c.gf) <= 1e-4 * abs(c.gf) + 1e-30
+
+
+@pytest.mark.parametrize("obj", [RASTRIGIN, GRIEWANK])
+def test_maximum_dimension(obj):
+    """d = PSO_D_MAX (2^24, the column split on one GPU, 4096 tiles per row):
+    init and two steps equal the oracle -- X, V, PB bitwise, fitness within the
+    tolerance (Griewank: the product of 16.7M factors), gbest as the oracle's."""
+    n, d = 2, fp.PSO_D_MAX
+    g = gpu_swarm(n, d, obj, seed=77)
+    assert g.info()["column_split"] == 1
+    c = cpu_swarm(n, d, obj, seed=77)
+    for k in (0, 1, 1):
+        g.step(k)
+        c.step(k)
+        X, V, PB, pf, t = g.get_state()
+        assert t == c.t
+        assert_bitwise(X, c.X, f"X t={t}")
+        assert_bitwise(V, c.V, f"V t={t}")
+        assert_bitwise(PB, c.PB, f"PB t={t}")
+        assert_fitness_close(obj, c.PB, pf, c.pf, f"pf t={t}")
+        gf, gi, G = g.gbest()
+        assert gi == c.gi
+        assert_bitwise(G, PB[gi], "G == PB[gi]")
