@@ -143,6 +143,9 @@ __global__ void __launch_bounds__(kColCompute + 64, 2)
   if (warp == nwarps + 1) {  // ---------------- finaliser
     if (lane == 0) {
       const int par = (int)(t & 1u);
+      // byte offset of this iteration's partial table within every rank's region
+      const size_t parts_off =  // = col_parts(region, a, par) - region
+          col_tag_bytes(a.world) + (size_t)par * (size_t)a.n_local * (size_t)a.col_nbt * sizeof(float4);
       unsigned n_pbl = 0, n_pbs = 0;
       int s = 0, prev = -1;
       unsigned ph = 0;
@@ -165,12 +168,14 @@ __global__ void __launch_bounds__(kColCompute + 64, 2)
         const float4* st = ring + (size_t)s * per * chunk;
         const int fl = sflag[s];
         const float4* xnew = fl ? st + 2 * chunk : st;  // where the compute warps put x'
-        const float4 msg = make_float4(c[0], Obj::kAcc > 1 ? c[Obj::kAcc - 1] : 0.f, s_edge[s][0], s_edge[s][1]);
+        const float4 msg = make_float4(c[0], Obj::kAcc > 1 ? c[Obj::kAcc - 1] : 0.f,
+                                       Obj::kNeighbor ? s_edge[s][0] : 0.f,
+                                       Obj::kNeighbor ? s_edge[s][1] : 0.f);
         const size_t pidx = (size_t)r * a.col_nbt + (size_t)(a.col_bbase + b);
         if (a.world > 1) {
-          for (int q = 0; q < a.world; ++q) col_parts<Obj>(a.peers[q], a, par)[pidx] = msg;
+          for (int q = 0; q < a.world; ++q) reinterpret_cast<float4*>(a.peers[q] + parts_off)[pidx] = msg;
         } else {
-          col_parts<Obj>(const_cast<unsigned char*>(a.recv), a, par)[pidx] = msg;
+          reinterpret_cast<float4*>(const_cast<unsigned char*>(a.recv) + parts_off)[pidx] = msg;
         }
         const size_t off = ((size_t)r * nvl + q0) * 4;
         bulk_s2g(a.X + off, xnew, bytes);
@@ -240,8 +245,10 @@ __global__ void __launch_bounds__(kColCompute + 64, 2)
           const int qg = a.col_q0 + q0 + ql;  // global float4: Philox counter, functor index
           float4 x, v;
           init_float4_at(a, key, gi, qg, B4, nvl, q0 + ql, x, v);
-          if (ql == 0) e_first = x.x;
-          if (ql == cnt - 1) e_last = x.w;
+          if constexpr (Obj::kNeighbor) {
+            if (ql == 0) e_first = x.x;
+            if (ql == cnt - 1) e_last = x.w;
+          }
           xdst[ql] = x;
           st[chunk + ql] = v;
           if constexpr (!Obj::kNeighbor) map4<Obj>(acc, x, 0.f, 4 * qg, d);
@@ -263,8 +270,10 @@ __global__ void __launch_bounds__(kColCompute + 64, 2)
             if (jj + 2 >= d) x.z = v.z = 0.f;
             if (jj + 3 >= d) x.w = v.w = 0.f;
           }
-          if (ql == 0) e_first = x.x;
-          if (ql == cnt - 1) e_last = x.w;
+          if constexpr (Obj::kNeighbor) {
+            if (ql == 0) e_first = x.x;
+            if (ql == cnt - 1) e_last = x.w;
+          }
           xdst[ql] = x;
           st[chunk + ql] = v;
           if constexpr (!Obj::kNeighbor) map4<Obj>(acc, x, 0.f, 4 * qg, d);
@@ -288,8 +297,10 @@ __global__ void __launch_bounds__(kColCompute + 64, 2)
       }
     }
     warp_combine<Obj>(acc);
-    {  // ql = 0 is thread 0 (lane 0 of warp 0); ql = cnt - 1 is thread (cnt - 1) % nthr
-      const int lt = (cnt - 1) % nthr;
+    if constexpr (Obj::kNeighbor) {  // only neighbour functors need the tile's edge x'
+      // ql = 0 is thread 0 (lane 0 of warp 0); ql = cnt - 1 (< 2 nthr) is thread
+      // (cnt - 1) mod nthr
+      const int lt = cnt - 1 >= nthr ? cnt - 1 - nthr : cnt - 1;
       const float el = __shfl_sync(kFull, e_last, lt & 31);
       if (lane == 0 && warp == (lt >> 5)) s_edge[s][1] = el;
       if (tid == 0) s_edge[s][0] = e_first;
@@ -309,10 +320,11 @@ __global__ void __launch_bounds__(kColCompute + 64, 2)
 }
 
 // One warp per row.
+constexpr int kColDecideThreads = 512;
 template <class Obj>
-__global__ void __launch_bounds__(256) k_col_decide(const __grid_constant__ SwarmArgs a, int init) {
-  __shared__ unsigned long long s_best[8];
-  __shared__ unsigned s_nimp[8];
+__global__ void __launch_bounds__(kColDecideThreads) k_col_decide(const __grid_constant__ SwarmArgs a, int init) {
+  __shared__ unsigned long long s_best[kColDecideThreads / 32];
+  __shared__ unsigned s_nimp[kColDecideThreads / 32];
   __shared__ int s_last;
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   pdl_wait_and_release();  // k_col_step's partials and flags are visible
@@ -338,6 +350,7 @@ __global__ void __launch_bounds__(256) k_col_decide(const __grid_constant__ Swar
   const long long wpc = blockDim.x >> 5;
   for (long long r = blockIdx.x * wpc + warp; r < a.n_local; r += (long long)gridDim.x * wpc) {
     const float4* Pr = P + (size_t)r * nbt;
+    const float pf_old = (lane == 0 && !init) ? a.pf[r] : 0.f;  // in flight with the partials
     float c[Obj::kAcc];
     Obj::init(c);
     for (int bt = lane; bt < nbt; bt += 32) {
@@ -361,7 +374,7 @@ __global__ void __launch_bounds__(256) k_col_decide(const __grid_constant__ Swar
         a.pf[r] = val;
         a.pbx[r] = 0;  // PB was stored (= x0)
       } else {
-        const bool imp = f < a.pf[r];  // strict; NaN never improves
+        const bool imp = f < pf_old;  // strict; NaN never improves
         if (imp) {
           a.pf[r] = f;
           ++nimp;
@@ -399,11 +412,24 @@ __global__ void __launch_bounds__(256) k_col_decide(const __grid_constant__ Swar
   }
   __syncthreads();
   const unsigned long long acc = s_best[0], cur = s_best[1];
-  if (acc < cur) {
+  if (acc < cur) {  // the block is up to 1 MB: 8 independent loads in flight per thread
     const float4* x = reinterpret_cast<const float4*>(a.X) +
                       ((long long)(uint32_t)acc - a.row_begin) * a.nvec;
     float4* G4 = reinterpret_cast<float4*>(a.G);
-    for (int q = tid; q < a.nvec; q += blockDim.x) G4[q] = __ldcg(x + q);
+    const int nt = blockDim.x;
+    for (int q0 = tid; q0 < a.nvec; q0 += 8 * nt) {
+      float4 v[8];
+#pragma unroll
+      for (int u = 0; u < 8; ++u) {
+        const int q = q0 + u * nt;
+        if (q < a.nvec) v[u] = __ldcg(x + q);
+      }
+#pragma unroll
+      for (int u = 0; u < 8; ++u) {
+        const int q = q0 + u * nt;
+        if (q < a.nvec) G4[q] = v[u];
+      }
+    }
   }
   __syncthreads();
   if (tid == 0) {

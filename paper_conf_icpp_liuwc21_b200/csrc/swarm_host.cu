@@ -660,8 +660,9 @@ cudaError_t plan_colsplit(int objective, int tile, int tiles_local, long long n,
   cfg->stages = stages;
   cfg->smem = smem;
   cfg->bounds = bounds ? 1 : 0;
-  long long dg = (n + 7) / 8;
-  if (dg > (long long)sm_count * 8) dg = (long long)sm_count * 8;
+  const int rows_per_cta = kColDecideThreads / 32;  // one warp per row
+  long long dg = (n + rows_per_cta - 1) / rows_per_cta;
+  if (dg > (long long)sm_count * 4) dg = (long long)sm_count * 4;
   cfg->col_decide_grid = (int)(dg < 1 ? 1 : dg);
   return cudaSuccess;
 }
@@ -681,7 +682,7 @@ cudaError_t launch_col_decide(int objective, const SwarmArgs& a, const LaunchCfg
   const KernelTable* t = kernel_table(objective);
   if (!t) return cudaErrorInvalidDeviceFunction;
   void* args[] = {const_cast<SwarmArgs*>(&a), &init};
-  return launch_pdl(t->col_decide, dim3(c.col_decide_grid), dim3(256), args, 0, s, c.pdl);
+  return launch_pdl(t->col_decide, dim3(c.col_decide_grid), dim3(kColDecideThreads), args, 0, s, c.pdl);
 }
 
 cudaError_t launch_rebest(const SwarmArgs& a, unsigned t, cudaStream_t s) {
