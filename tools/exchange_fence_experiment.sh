@@ -1,4 +1,8 @@
 # Exchange-latency experiment on the 1-rank proxy (NS_R8 with the NVLink exchange forced).
+# Round 2 measured the record tag's system-scope release by building once with a relaxed store
+# in its place (-DPSO_EXP_RELAXED_TAG around st_release_sys_u64 in epilogue_core); that
+# experiment-only switch is not kept in the kernels (it has no ordering guarantee), so the
+# second pair of runs below now repeats the baseline unless it is re-added.
 exec > gpurun_out/exp1.log 2>&1
 run() { PSO_FORCE_EXCHANGE=1 timeout 600 python -m torch.distributed.run --nnodes=1 --nproc-per-node 1 --master-addr 127.0.0.1 --master-port 29517 bench.py --workload NS_R8 --steps 1000 --warmup 20 --no-e2e --no-cpu-baseline 2>/dev/null | tail -1 | python -c "
 import json,sys
