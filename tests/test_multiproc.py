@@ -97,3 +97,62 @@ def test_row_partition_covers_every_row_once(n, world):
         assert e0 == b1 and b0 <= e0
     sizes = [e - b for b, e in spans]
     assert max(sizes) - min(sizes) <= 1
+
+
+class _FakeSwarm:
+    """The four p2p calls of a handle, scripted per rank (no GPU): connect_p2p's
+    collective decision logic is what is under test."""
+
+    def __init__(self, rank, fail_connect=False, fail_probe=False):
+        self.rank, self.fail_connect, self.fail_probe = rank, fail_connect, fail_probe
+        self.enabled = False
+        self.calls = []
+
+    def p2p_handle(self):
+        return bytes([self.rank]) * 64, 4096 + self.rank
+
+    def p2p_connect(self, handles, offsets):
+        from paper_conf_icpp_liuwc21_b200 import PsoError
+        self.calls.append(("connect", [h[0] for h in handles], list(offsets)))
+        if self.fail_connect:
+            raise PsoError(3, "pso_p2p_connect", "cudaIpcOpenMemHandle failed (scripted)")
+
+    def p2p_probe(self, phase):
+        self.calls.append(("probe", phase))
+        return not self.fail_probe
+
+    def p2p_enable(self, on=True):
+        self.enabled = bool(on)
+
+
+def _connect_worker(rank, world, port, fail_connect_rank, fail_probe_rank, out_dir):
+    _init(rank, world, port)
+    os.environ["PSO_QUIET"] = "1"
+    from paper_conf_icpp_liuwc21_b200.distributed import connect_p2p
+    s = _FakeSwarm(rank, fail_connect=rank == fail_connect_rank, fail_probe=rank == fail_probe_rank)
+    on = connect_p2p(s)
+    import json
+    with open(os.path.join(out_dir, f"c{rank}.json"), "w") as fh:
+        json.dump({"on": on, "enabled": s.enabled, "calls": s.calls}, fh)
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world,fail_connect,fail_probe", [(2, -1, -1), (3, 1, -1), (2, -1, 0),
+                                                           (3, -1, 2)])
+def test_connect_p2p_is_all_or_nothing(tmp_path, world, fail_connect, fail_probe):
+    """The NVLink exchange is switched on only if every rank mapped its peers
+    AND every rank's probe saw every token; otherwise no rank enables it (all
+    stay on the NCCL exchange).  Handles and offsets reach every rank in rank
+    order; a failed mapping skips the probe on every rank."""
+    import json
+    mp.spawn(_connect_worker, args=(world, _free_port(), fail_connect, fail_probe, str(tmp_path)),
+             nprocs=world, join=True)
+    res = [json.load(open(tmp_path / f"c{r}.json")) for r in range(world)]
+    expect = fail_connect < 0 and fail_probe < 0
+    for r in res:
+        assert r["on"] == expect and r["enabled"] == expect
+        connect = [c for c in r["calls"] if c[0] == "connect"][0]
+        assert connect[1] == list(range(world)) and connect[2] == [4096 + k for k in range(world)]
+        probes = [c[1] for c in r["calls"] if c[0] == "probe"]
+        assert probes == ([] if fail_connect >= 0 else [0, 1])
