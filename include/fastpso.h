@@ -219,6 +219,15 @@ pso_status pso_get_gbest(pso_handle h, float* fitness, int64_t* index, float* po
  * x, v, pb: n_local x d floats; pf: n_local floats; t: iterations done. */
 pso_status pso_get_state(pso_handle h, float* x, float* v, float* pb, float* pf, uint64_t* t);
 
+/* Synchronise and copy m rank-local rows (local indices rows[k] in [0, n_local);
+ * row k is particle row_begin + rows[k]) to host buffers (any may be NULL):
+ * x, v, pb: m x d floats; pf: m floats.  The state is not changed (a pbest
+ * deferred by the lazy rows is read from x).  For sampling swarms too large
+ * to copy whole (e.g. 2.9M x 4096: 142 GB).  PSO_ERR_INVALID for an index
+ * outside [0, n_local) or m < 0. */
+pso_status pso_get_rows(pso_handle h, const int64_t* rows, int64_t m, float* x, float* v, float* pb,
+                        float* pf);
+
 /* Replace the rank-local state from host buffers (all required: x, v, pb are
  * n_local x d, pf is n_local; NaN pf is read as +inf) and set the iteration
  * counter to t.  The gbest is recomputed from pf/pb exactly as after create.

@@ -160,6 +160,19 @@ class Swarm:
               "pso_get_state")
         return X, V, PB, pf, int(t.value)
 
+    def get_rows(self, rows):
+        """(X, V, PB, pf) of the given rank-local rows (dense numpy arrays) without
+        copying the rest of the swarm -- synchronises."""
+        idx = np.ascontiguousarray(rows, dtype=np.int64).reshape(-1)
+        m, d = idx.size, self.d_local
+        X, V, PB = (np.empty((m, d), np.float32) for _ in range(3))
+        pf = np.empty(m, np.float32)
+        check(lib().pso_get_rows(self._h, idx.ctypes.data_as(C.POINTER(C.c_int64)), m,
+                                 _ptr(X, m * d, writable=True), _ptr(V, m * d, writable=True),
+                                 _ptr(PB, m * d, writable=True), _ptr(pf, m, writable=True)),
+              "pso_get_rows")
+        return X, V, PB, pf
+
     def set_state(self, X, V, PB, pf, t: int = 0) -> "Swarm":
         def prep(a):
             if hasattr(a, "data_ptr"):

@@ -26,7 +26,7 @@ PSO_D_MAX = 1 << 24
 # every symbol include/fastpso.h declares
 EXPORTS = (
     "pso_create", "pso_create_ex", "pso_init", "pso_step", "pso_synchronize", "pso_get_gbest",
-    "pso_get_state", "pso_set_state", "pso_set_bounds", "pso_get_info", "pso_reset_counters", "pso_destroy",
+    "pso_get_state", "pso_get_rows", "pso_set_state", "pso_set_bounds", "pso_get_info", "pso_reset_counters", "pso_destroy",
     "pso_status_string", "pso_last_error", "pso_objective_registered",
     "pso_nccl_get_unique_id", "pso_nccl_comm_init", "pso_nccl_comm_destroy",
     "pso_p2p_handle", "pso_p2p_connect", "pso_p2p_probe", "pso_p2p_enable",
@@ -89,6 +89,7 @@ def lib() -> C.CDLL:
     L.pso_synchronize.argtypes = [H]
     L.pso_get_gbest.argtypes = [H, fp, i64p, C.c_void_p]
     L.pso_get_state.argtypes = [H, C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p, u64p]
+    L.pso_get_rows.argtypes = [H, i64p, C.c_int64, C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p]
     L.pso_set_state.argtypes = [H, C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p, C.c_uint64]
     L.pso_get_info.argtypes = [H, C.POINTER(pso_info)]
     L.pso_set_bounds.argtypes = [H, C.c_void_p]

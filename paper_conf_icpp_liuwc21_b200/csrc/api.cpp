@@ -907,6 +907,42 @@ pso_status pso_get_state(pso_handle h, float* x, float* v, float* pb, float* pf,
   return PSO_OK;
 }
 
+pso_status pso_get_rows(pso_handle h, const int64_t* rows, int64_t m, float* x, float* v, float* pb,
+                        float* pf) {
+  NvtxRange nvtx_range("pso_get_rows");
+  pso_status st = check_ready(h);
+  if (st != PSO_OK) return st;
+  if (m < 0 || (m > 0 && !rows)) return fail(PSO_ERR_INVALID, "bad rows / m");
+  for (int64_t k = 0; k < m; ++k)
+    if (rows[k] < 0 || rows[k] >= h->n_local)
+      return fail(PSO_ERR_INVALID, "row %lld outside [0, %lld)", (long long)rows[k], (long long)h->n_local);
+  if ((st = use_device(h)) != PSO_OK) return st;
+  if ((st = sync_and_check(h)) != PSO_OK) return st;
+  // lazy pbest rows (PB == X, not stored): their pbest is read from X
+  std::vector<unsigned char> lazy;
+  if (pb && h->args.lazy_pb && m > 0) {
+    lazy.resize((size_t)h->n_local);
+    PSO_CUDA(h, cudaMemcpy(lazy.data(), h->args.pbx, lazy.size(), cudaMemcpyDeviceToHost));
+  }
+  const size_t w = (size_t)h->d_local * 4, sp = (size_t)h->pitch * 4;
+  for (int64_t k = 0; k < m; ++k) {
+    const size_t r = (size_t)rows[k], o = (size_t)k * h->d_local;
+    const unsigned char* xr = reinterpret_cast<const unsigned char*>(h->args.X) + r * sp;
+    if (x) PSO_CUDA(h, cudaMemcpyAsync(x + o, xr, w, cudaMemcpyDeviceToHost, h->stream));
+    if (v)
+      PSO_CUDA(h, cudaMemcpyAsync(v + o, reinterpret_cast<const unsigned char*>(h->args.V) + r * sp, w,
+                                  cudaMemcpyDeviceToHost, h->stream));
+    if (pb) {
+      const unsigned char* src = (!lazy.empty() && lazy[r])
+                                     ? xr
+                                     : reinterpret_cast<const unsigned char*>(h->args.PB) + r * sp;
+      PSO_CUDA(h, cudaMemcpyAsync(pb + o, src, w, cudaMemcpyDeviceToHost, h->stream));
+    }
+    if (pf) PSO_CUDA(h, cudaMemcpyAsync(pf + k, h->args.pf + r, 4, cudaMemcpyDeviceToHost, h->stream));
+  }
+  return sync_and_check(h);
+}
+
 pso_status pso_set_state(pso_handle h, const float* x, const float* v, const float* pb,
                          const float* pf, uint64_t t) {
   NvtxRange nvtx_range("pso_set_state");

@@ -345,45 +345,74 @@ def test_handles_sharing_a_kernel_keep_their_shared_memory(first, second, monkey
 
 
 # ------------------------------------------------------------------ full size, sampled
-@pytest.mark.parametrize("key", ["NS", "C4", "C3", "C2", "W16K", "W64K", "C5@40000"])
+@pytest.mark.parametrize("key", ["NS", "C4", "C3", "C2", "W16K", "W64K", "C5", "C5_2900K"])
 def test_full_size_sampled_rows(key):
     """Bench configurations at full size in the bench's launch shape (NS / C4
     streaming 100k x 2000, C3 streaming with a neighbour functor, C2 on the
     grid-resident path, W16K on 4-CTA clusters, W64K on the automatic column
-    split; C5's wide 16-warp instantiation at d = 4096 with n cut to 40,000 --
-    the launch shape depends on d only -- so the host copies stay ~2 GB): the
-    oracle recomputes sampled rows of one iteration exactly (rows are
-    independent given G), and the gbest invariants hold over the whole swarm."""
-    name, _, n_cut = key.partition("@")
-    w = WORKLOADS[name].with_(n=int(n_cut)) if n_cut else WORKLOADS[name]
+    split, C5 1M x 4096 on the wide 16-warp instantiation, and the capacity
+    sweep's 2.9M x 4096 -- 142.5 GB of state): sampled rows read back with
+    pso_get_rows are recomputed by the oracle exactly (rows are independent
+    given G): init bit-exact, one iteration's X / V bit-exact, decisions as the
+    oracle's; the gbest is min pf with the lowest index and G = PB[gi]."""
+    w = WORKLOADS[key]
     g = gpu_swarm(w.n, w.d, w.objective, seed=w.seed)
     idx = sample_rows(w.n, 48, seed=7)
-    X0, V0, _, _, _ = g.get_state()
-    # init rows are bit-exact
-    for i in idx[:8]:
+    X0, V0, _, _ = g.get_rows(idx[:8])
+    for k, i in enumerate(idx[:8]):  # init rows are bit-exact
         c = orc.OracleSwarm(w.n, w.d, w.w, w.c1, w.c2, w.lo, w.hi, w.objective, w.seed,
                             row_begin=int(i), nrows=1, create=False)
         c.init_local()
-        assert_bitwise(X0[i], c.X[0], f"X0 row {i}")
-        assert_bitwise(V0[i], c.V[0], f"V0 row {i}")
-    del X0, V0
+        assert_bitwise(X0[k], c.X[0], f"X0 row {i}")
+        assert_bitwise(V0[k], c.V[0], f"V0 row {i}")
     g.step(2)
-    X, V, PB, pf, t = g.get_state()
+    X, V, PB, pf = g.get_rows(idx)
+    t = g.info()["t"]
     _, _, G = g.gbest()
     g.step(1)
-    X2, V2, PB2, pf2, t2 = g.get_state()
+    X2, V2, PB2, pf2s = g.get_rows(idx)
+    pf2 = np.empty(w.n, np.float32)
+    g.get_state(out=(None, None, None, pf2))
     gf, gi, G2 = g.gbest()
     c = cpu_swarm(w.n, w.d, w.objective, seed=w.seed, create=False)
-    cX, cV, cPB, cpf, cf = c.rows_step(t + 1, G, idx, X[idx], V[idx], PB[idx], pf[idx])
-    assert_bitwise(X2[idx], cX, "X rows")
-    assert_bitwise(V2[idx], cV, "V rows")
+    cX, cV, cPB, cpf, cf = c.rows_step(t + 1, G, idx, X, V, PB, pf)
+    assert_bitwise(X2, cX, "X rows")
+    assert_bitwise(V2, cV, "V rows")
+    assert_bitwise(pf2s, pf2[idx], "pf rows (get_rows vs get_state)")
     tol = fit_tol(w.objective, cX, cf)
-    amb = np.abs(cf.astype(np.float64) - pf[idx].astype(np.float64)) <= tol
+    amb = np.abs(cf.astype(np.float64) - pf.astype(np.float64)) <= tol
     ok = ~amb
-    assert_bitwise(PB2[idx][ok], cPB[ok], "PB rows")
-    assert_fitness_close(w.objective, cPB[ok], pf2[idx][ok], cpf[ok], "pf rows")
+    assert_bitwise(PB2[ok], cPB[ok], "PB rows")
+    assert_fitness_close(w.objective, cPB[ok], pf2s[ok], cpf[ok], "pf rows")
     assert gf == pf2.min() and gi == int(np.argmin(pf2))
-    assert_bitwise(G2, PB2[gi], "G == PB[gi]")
+    Xg, _, PBg, _ = g.get_rows([gi])
+    assert_bitwise(G2, PBg[0], "G == PB[gi]")
+    g.close()
+
+
+def test_get_rows_reads_without_changing_the_state(monkeypatch):
+    """pso_get_rows returns exactly the rows pso_get_state returns (a deferred
+    pbest read from x), and reading does not change the following iterations."""
+    monkeypatch.setenv("PSO_RESIDENT", "0")
+    a = gpu_swarm(500, 2000, GRIEWANK, seed=3)
+    b = gpu_swarm(500, 2000, GRIEWANK, seed=3)
+    assert a.info()["lazy_pb"] == 1
+    a.step(4)
+    b.step(4)
+    idx = np.array([499, 0, 17, 17, 250])
+    Xr, Vr, PBr, pfr = a.get_rows(idx)
+    a.step(3)
+    b.step(3)
+    X, V, PB, pf, _ = b.get_state()
+    Xa, Va, PBa, pfa, _ = a.get_state()
+    for x, y in zip((Xa, Va, PBa, pfa), (X, V, PB, pf)):
+        assert_bitwise(x, y, "a run read with get_rows equals one that was not")
+    c = gpu_swarm(500, 2000, GRIEWANK, seed=3).step(4)
+    Xc, Vc, PBc, pfc, _ = c.get_state()
+    for got, ref in zip((Xr, Vr, PBr, pfr), (Xc[idx], Vc[idx], PBc[idx], pfc[idx])):
+        assert_bitwise(got, ref, "get_rows vs get_state")
+    with pytest.raises(fp.PsoError):
+        a.get_rows([500])
 
 
 # ------------------------------------------------------------------ exchange path
