@@ -15,7 +15,9 @@ struct DevCtl {
   unsigned long long improvements;  // pbest improvements, summed
   unsigned int done;                // last-CTA ticket counter
   unsigned int t;                   // iterations done (low 32 bits; Philox ctr[2])
-  unsigned long long spare[2];
+  unsigned long long row_claim;     // TMA streaming kernel, dynamic rows: rows claimed beyond the
+                                    // grid's first (reset by the iteration's last CTA)
+  unsigned long long spare;
   unsigned int bar_count, bar_gen;  // grid-resident kernel: grid barrier
   unsigned long long pb_loads;      // streaming kernels: pbest rows read from HBM
   unsigned long long pb_stores;     // streaming kernels: pbest rows written to HBM
@@ -60,6 +62,7 @@ struct SwarmArgs {
   int l2pf;                   // TMA producer: L2 prefetch distance in rows of this CTA (0: off)
   int serp;                   // streaming kernels: odd iterations visit rows backwards (L2 reuse)
   int l2pf_all;               // prefetch every row (default: lazy rows only, whose stage loads 2 of 3 slots)
+  int dyn_rows;               // TMA streaming kernel: CTAs claim rows from a counter (else round robin)
   unsigned char* send;        // world > 1: this rank's exchange record
   const unsigned char* recv;  // exchange: [2 iteration parities][world] records after the all-gather
   DevCtl* ctl;

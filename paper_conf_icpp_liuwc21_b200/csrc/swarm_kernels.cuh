@@ -945,6 +945,7 @@ __global__ void __launch_bounds__(kMaxT + 64, kMaxT > kMaxThreads ? 1 : 2)
   __shared__ unsigned long long s_inc;  // incumbent of this iteration (after the exchange merge)
   __shared__ int s_src;
   __shared__ int sflag[kMaxStages];     // lazy pbest: the stage's row had PB == X (pb not loaded)
+  __shared__ long long srow[kMaxStages];  // the stage's row (local index), -1: no more rows
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   if (tid == 0) {
     mbar_init(&gbar, 1);
@@ -981,21 +982,42 @@ __global__ void __launch_bounds__(kMaxT + 64, kMaxT > kMaxThreads ? 1 : 2)
       int k = 0;
       // lazy pbest: rows whose PB equals X skip the pb load (flag prefetched one row ahead)
       const RowOrder ro = row_order(a, t);
-      int fl_next = (a.lazy_pb && blockIdx.x < a.n_local) ? a.pbx[ro(blockIdx.x)] : 0;
-      // L2 prefetch of the row l2pf rows beyond the load front: DRAM requests
-      // in flight beyond the ring.  Only lazy rows by default -- their stage
-      // loads 2 of its 3 slots, so the ring alone keeps a third fewer bytes in
-      // flight (C4: 547 -> 529 us); prefetching eager rows as well slows the
-      // ring-saturated case (NS 638 -> 671 us).  Flag read one row earlier.
+      const long long n = a.n_local;
+      // Row schedule.  Round robin (row i to CTA i mod grid), or dynamic: a
+      // CTA's first row is its blockIdx, every further one is claimed from
+      // ctl->row_claim, so CTAs that run faster (SM placement, the co-resident
+      // CTA's lazy-row share) take more rows and the grid ends together.  A
+      // claim is issued two rows ahead (its value is needed one row ahead, for
+      // the lazy flag) and only while the previous claim was a row, so every
+      // claim's value is consumed before the sentinel below: the last CTA's
+      // reset of the counter then follows every claim of the iteration.  Which
+      // CTA computes a row changes no bit (rows are independent; the candidate
+      // key and the counters are order-free min / sums).
+      unsigned long long* claim_ctr = &a.ctl->row_claim;
+      const bool dyn = a.dyn_rows != 0;
+      long long i = blockIdx.x;
+      long long i_next =
+          i >= n ? n : (dyn ? (long long)atomicAdd(claim_ctr, 1ull) + gridDim.x : i + gridDim.x);
+      int fl_next = (a.lazy_pb && i < n) ? a.pbx[ro(i)] : 0;
+      // L2 prefetch of the row l2pf rounds of the grid beyond the load front:
+      // DRAM requests in flight beyond the ring.  Only lazy rows by default --
+      // their stage loads 2 of its 3 slots, so the ring alone keeps a third
+      // fewer bytes in flight (C4: 547 -> 529 us); prefetching eager rows as
+      // well slows the ring-saturated case (NS 638 -> 671 us).  Flag read one
+      // row earlier.  (Dynamic rows: the prefetched row is claimed by whichever
+      // CTA reaches it; L2 is shared.)
       const long long pd = (long long)a.l2pf * gridDim.x;
-      int pfl_next = (pd && blockIdx.x + pd < a.n_local) ? a.pbx[ro(blockIdx.x + pd)] : 0;
-      for (long long i = blockIdx.x; i < a.n_local; i += gridDim.x, ++k) {
+      int pfl_next = (pd && i + pd < n) ? a.pbx[ro(i + pd)] : 0;
+      for (; i < n; ++k) {
         const long long r = ro(i);
         const int fl = fl_next;
-        if (a.lazy_pb && i + gridDim.x < a.n_local) fl_next = a.pbx[ro(i + gridDim.x)];
-        if (pd && i + pd < a.n_local) {
+        const long long i_nn = i_next >= n ? n
+                               : (dyn ? (long long)atomicAdd(claim_ctr, 1ull) + gridDim.x
+                                      : i_next + gridDim.x);
+        if (a.lazy_pb && i_next < n) fl_next = a.pbx[ro(i_next)];
+        if (pd && i + pd < n) {
           const int pfl = pfl_next;
-          if (i + pd + gridDim.x < a.n_local) pfl_next = a.pbx[ro(i + pd + gridDim.x)];
+          if (i_next + pd < n) pfl_next = a.pbx[ro(i_next + pd)];
           const size_t po = (size_t)ro(i + pd) * 4 * nvec;
           if (pfl || a.l2pf_all) {
             bulk_prefetch_l2(a.X + po, row_bytes);
@@ -1003,10 +1025,13 @@ __global__ void __launch_bounds__(kMaxT + 64, kMaxT > kMaxThreads ? 1 : 2)
             if (!pfl) bulk_prefetch_l2(a.PB + po, row_bytes);
           }
         }
+        i = i_next;
+        i_next = i_nn;
         if (k >= stages) mbar_wait(&empty[s], ph ^ 1u);
         float4* st = ring + (size_t)s * 3 * nvec;
         sflag[s] = fl;
-        mbar_expect_tx(&full[s], (fl ? 2u : 3u) * row_bytes);  // releases sflag[s] too
+        srow[s] = r;
+        mbar_expect_tx(&full[s], (fl ? 2u : 3u) * row_bytes);  // releases sflag[s], srow[s] too
         bulk_g2s(st, a.X + (size_t)r * 4 * nvec, row_bytes, &full[s]);
         bulk_g2s(st + nvec, a.V + (size_t)r * 4 * nvec, row_bytes, &full[s]);
         if (!fl) bulk_g2s(st + 2 * nvec, a.PB + (size_t)r * 4 * nvec, row_bytes, &full[s]);
@@ -1015,6 +1040,10 @@ __global__ void __launch_bounds__(kMaxT + 64, kMaxT > kMaxThreads ? 1 : 2)
           ph ^= 1u;
         }
       }
+      // sentinel: the compute warps and the finaliser stop at a stage without a row
+      if (k >= stages) mbar_wait(&empty[s], ph ^ 1u);
+      srow[s] = -1;
+      mbar_arrive(&full[s]);
     }
     return;
   }
@@ -1028,9 +1057,10 @@ __global__ void __launch_bounds__(kMaxT + 64, kMaxT > kMaxThreads ? 1 : 2)
       unsigned nimp = 0, n_pbl = 0, n_pbs = 0;
       int s = 0, prev = -1;
       unsigned ph = 0;
-      const RowOrder ro = row_order(a, t);
-      for (long long i = blockIdx.x; i < a.n_local; i += gridDim.x) {
-        const long long r = ro(i);
+      for (;;) {
+        mbar_wait(&full[s], ph);
+        const long long r = srow[s];
+        if (r < 0) break;
         const float pf_old = a.pf[r];
         const uint32_t gi = (uint32_t)(a.row_begin + r);
         mbar_wait(&done[s], ph);
@@ -1093,6 +1123,7 @@ __global__ void __launch_bounds__(kMaxT + 64, kMaxT > kMaxThreads ? 1 : 2)
       if (n_pbs) atomicAdd(&a.ctl->pb_stores, (unsigned long long)n_pbs);
       __threadfence();
       s_last = (atomicAdd(&a.ctl->done, 1u) == gridDim.x - 1) ? 1 : 0;
+      if (s_last) a.ctl->row_claim = 0;  // every CTA's claims are done (see the producer)
     }
     __syncwarp();
     if (s_last) warp_gbest_epilogue(a, t, lane, s_inc, s_src);
@@ -1131,11 +1162,12 @@ __global__ void __launch_bounds__(kMaxT + 64, kMaxT > kMaxThreads ? 1 : 2)
   mbar_wait(&gbar, 0);
   int s = 0;
   unsigned ph = 0;
-  const RowOrder ro = row_order(a, t);
-  for (long long i = blockIdx.x; i < a.n_local; i += gridDim.x) {
-    const uint32_t gi = (uint32_t)(a.row_begin + ro(i));
+  for (;;) {
     float4* st = ring + (size_t)s * 3 * nvec;
     mbar_wait(&full[s], ph);
+    const long long r = srow[s];
+    if (r < 0) break;
+    const uint32_t gi = (uint32_t)(a.row_begin + r);
     // lazy pbest row (PB == X): pb is the loaded x, and x' goes to the pb slot
     // so the old x stays available for a deferred PB store
     const int fl = sflag[s];

@@ -767,18 +767,24 @@ def test_lazy_rows_skip_r1_signed_zeros(w, c1, c2, obj, n, d, kw, monkeypatch):
 
 
 @pytest.mark.parametrize("obj,n,d", [(ROSENBROCK, 301, 1000), (GRIEWANK, 300, 2000),
-                                     (RASTRIGIN, 7, 12000)])
+                                     (RASTRIGIN, 7, 12000), (SPHERE, 5000, 600),
+                                     (GRIEWANK, 1200, 4096), (RASTRIGIN, 100, 2000)])
 def test_row_order_is_invisible(obj, n, d, monkeypatch):
     """Serpentine row order (odd iterations walk the rows backwards for L2
-    reuse) and the L2 prefetch change no bit: state, pf and gbest equal the
-    forward, prefetch-free run after every call."""
+    reuse), the L2 prefetch and the dynamic row claims (a CTA takes its next
+    row from a counter the iteration's last CTA resets) change no bit: state,
+    pf and gbest equal the forward, prefetch-free, round-robin run after every
+    call (many rows per CTA, the wide 512-thread kernel at d = 4096, fewer rows
+    than CTAs)."""
     monkeypatch.setenv("PSO_RESIDENT", "0")
     monkeypatch.setenv("PSO_SERP", "1")
     monkeypatch.setenv("PSO_L2PF_ALL", "1")
+    monkeypatch.setenv("PSO_DYN_ROWS", "1")
     g = gpu_swarm(n, d, obj, seed=12)
     monkeypatch.setenv("PSO_SERP", "0")
     monkeypatch.setenv("PSO_L2PF", "0")
     monkeypatch.setenv("PSO_L2PF_ALL", "0")
+    monkeypatch.setenv("PSO_DYN_ROWS", "0")
     e = gpu_swarm(n, d, obj, seed=12)
     for k in (1, 2, 3, 1):
         g.step(k)
