@@ -40,28 +40,6 @@ __device__ __forceinline__ float4* col_parts(unsigned char* region, const SwarmA
          (size_t)par * (size_t)a.n_local * (size_t)a.col_nbt;
 }
 
-// The items k = k0, k0 + step, ... of the (row, tile) sequence, k = r nb + b,
-// advanced without a 64-bit division per item (every thread of the CTA walks
-// the sequence; a division per item cost ~100 instructions each).
-struct ItemWalk {
-  long long r, dr;
-  int b, db, nb;
-  __device__ __forceinline__ ItemWalk(long long k0, long long step, int nb_) : nb(nb_) {
-    r = k0 / nb_;
-    b = (int)(k0 - r * nb_);
-    dr = step / nb_;
-    db = (int)(step - dr * nb_);
-  }
-  __device__ __forceinline__ void next() {
-    r += dr;
-    b += db;
-    if (b >= nb) {
-      b -= nb;
-      ++r;
-    }
-  }
-};
-
 constexpr int kColCompute = 256;  // compute threads of k_col_step (+ producer + finaliser warps)
 static_assert(kColTileMax <= 2 * kColCompute, "k_col_step: at most 2 float4 of a tile per thread");
 
@@ -77,6 +55,8 @@ __global__ void __launch_bounds__(kColCompute + 64, 2)
   __shared__ float red[kMaxStages][nwarps * 2];
   __shared__ unsigned long long full[kMaxStages], empty[kMaxStages], done[kMaxStages];
   __shared__ int sflag[kMaxStages];
+  __shared__ long long s_r[kMaxStages];  // the stage's item: row (-1: no more items) ...
+  __shared__ int s_b[kMaxStages];        // ... and tile
   // the tile's first and last x' for the neighbour terms across tiles, handed to
   // the finaliser by the arriving lanes themselves (ordered by their own release)
   __shared__ float s_edge[kMaxStages][2];
@@ -99,23 +79,36 @@ __global__ void __launch_bounds__(kColCompute + 64, 2)
       int s = 0;
       unsigned ph = 0;
       long long i = 0;
-      ItemWalk it(blockIdx.x, gridDim.x, nb);
+      // Item schedule as k_step_tma's rows: round robin, or (a.dyn_rows) the
+      // first item is blockIdx.x and every further one is claimed from
+      // ctl->row_claim two items ahead, each claim's value consumed before the
+      // sentinel (the last CTA resets the counter).  The producer passes the
+      // item's (row, tile) to the other warps with the stage.
+      unsigned long long* claim_ctr = &a.ctl->row_claim;
+      const bool dyn = a.dyn_rows != 0;
+      long long k = blockIdx.x;
+      long long k_next =
+          k >= items ? items : (dyn ? (long long)atomicAdd(claim_ctr, 1ull) + gridDim.x : k + gridDim.x);
       // the lazy-pbest flag of the next item is loaded one item ahead, so its L2
       // latency overlaps the wait for a free stage instead of delaying the copies
-      int fl_next = (!init && blockIdx.x < items) ? a.pbx[it.r] : 0;
-      for (long long k = blockIdx.x; k < items; k += gridDim.x, ++i, it.next()) {
-        const long long r = it.r;
-        const int q0 = it.b * chunk;
+      int fl_next = (!init && k < items) ? a.pbx[k / nb] : 0;
+      for (; k < items; ++i) {
+        const long long r = k / nb;
+        const int b = (int)(k - r * nb);
+        const int q0 = b * chunk;
         const int cnt = min(chunk, nvl - q0);
         const unsigned bytes = (unsigned)cnt * 16u;
         const int fl = fl_next;
-        if (!init && k + gridDim.x < items) {
-          ItemWalk nx = it;
-          nx.next();
-          fl_next = a.pbx[nx.r];
-        }
+        const long long k_nn = k_next >= items ? items
+                               : (dyn ? (long long)atomicAdd(claim_ctr, 1ull) + gridDim.x
+                                      : k_next + gridDim.x);
+        if (!init && k_next < items) fl_next = a.pbx[k_next / nb];
+        k = k_next;
+        k_next = k_nn;
         if (i >= stages) mbar_wait(&empty[s], ph ^ 1u);
         float4* st = ring + (size_t)s * per * chunk;
+        s_r[s] = r;
+        s_b[s] = b;
         if (init) {
           sflag[s] = 0;
           mbar_arrive(&full[s]);
@@ -136,6 +129,10 @@ __global__ void __launch_bounds__(kColCompute + 64, 2)
           ph ^= 1u;
         }
       }
+      // sentinel: the compute warps and the finaliser stop at a stage without an item
+      if (i >= stages) mbar_wait(&empty[s], ph ^ 1u);
+      s_r[s] = -1;
+      mbar_arrive(&full[s]);
     }
     return;
   }
@@ -149,10 +146,11 @@ __global__ void __launch_bounds__(kColCompute + 64, 2)
       unsigned n_pbl = 0, n_pbs = 0;
       int s = 0, prev = -1;
       unsigned ph = 0;
-      ItemWalk it(blockIdx.x, gridDim.x, nb);
-      for (long long k = blockIdx.x; k < items; k += gridDim.x, it.next()) {
-        const long long r = it.r;
-        const int b = it.b;
+      for (;;) {
+        mbar_wait(&full[s], ph);
+        const long long r = s_r[s];
+        if (r < 0) break;
+        const int b = s_b[s];
         const int q0 = b * chunk;
         const int cnt = min(chunk, nvl - q0);
         const unsigned bytes = (unsigned)cnt * 16u;
@@ -204,6 +202,7 @@ __global__ void __launch_bounds__(kColCompute + 64, 2)
       if (atomicAdd(&a.ctl->done, 1u) == gridDim.x - 1) {
         __threadfence_system();
         a.ctl->done = 0;
+        a.ctl->row_claim = 0;  // every CTA's claims are done (see the producer)
         if (a.world > 1) {
           const unsigned long long tag = ((unsigned long long)a.epoch << 32) | t;
           for (int q = 0; q < a.world; ++q)
@@ -220,14 +219,14 @@ __global__ void __launch_bounds__(kColCompute + 64, 2)
   const float4* B4 = reinterpret_cast<const float4*>(a.bounds);
   int s = 0;
   unsigned ph = 0;
-  ItemWalk it(blockIdx.x, gridDim.x, nb);
-  for (long long k = blockIdx.x; k < items; k += gridDim.x, it.next()) {
-    const long long r = it.r;
-    const int q0 = it.b * chunk;
-    const int cnt = min(chunk, nvl - q0);
-    const uint32_t gi = (uint32_t)(a.row_begin + r);
+  for (;;) {
     float4* st = ring + (size_t)s * per * chunk;
     mbar_wait(&full[s], ph);
+    const long long r = s_r[s];
+    if (r < 0) break;
+    const int q0 = s_b[s] * chunk;
+    const int cnt = min(chunk, nvl - q0);
+    const uint32_t gi = (uint32_t)(a.row_begin + r);
     const int fl = sflag[s];
     float4* xdst = fl ? st + 2 * chunk : st;  // keep the old x for the deferred pbest copy
     float acc[Obj::kAcc];
