@@ -85,6 +85,37 @@ def ncu_traffic(workload_name):
     return v, "committed ncu capture, not this run: profiles/ncu_traffic.json (" + j.get("_source", "") + ")"
 
 
+def mix_peak(read_fraction):
+    """HBM bandwidth at the kernel's read:write mix, from the committed probe
+    (profiles/r02_hbm_mix_probe.json: torch kernels of 1R:1W, 2R:1W, 3R:1W,
+    read-only and write-only mixes over 4 GiB operands on a B200), linearly
+    interpolated between the two nearest measured mixes.  Context beside the
+    contract's peak (the 1:1 copy of MEASURED_PEAKS.json), not a replacement:
+    a read-heavy kernel can run above the copy figure."""
+    p = os.path.join(ROOT, "profiles", "r02_hbm_mix_probe.json")
+    try:
+        with open(p) as fh:
+            cases = json.load(fh)["cases"]
+    except Exception:
+        return None
+    pts = sorted((c["read_fraction"], c["GBps"]) for k, c in cases.items()
+                 if 0.0 < c["read_fraction"] < 1.0)  # the mixed cases (the one-sided ones differ in kind)
+    if not pts:
+        return None
+    if read_fraction <= pts[0][0]:
+        g = pts[0][1]
+    elif read_fraction >= pts[-1][0]:
+        g = pts[-1][1]
+    else:
+        for (f0, g0), (f1, g1) in zip(pts, pts[1:]):
+            if f0 <= read_fraction <= f1:
+                g = g0 + (g1 - g0) * (read_fraction - f0) / (f1 - f0)
+                break
+    return {"GBps": g, "read_fraction": read_fraction,
+            "source": "profiles/r02_hbm_mix_probe.json (tools/hbm_mix_probe.py; torch kernels, "
+                      "interpolated between the nearest mixes; context, not the contract's peak)"}
+
+
 # ------------------------------------------------------------------ clocks
 class ClockSampler:
     """nvidia-smi clocks / throttle reasons sampled during the timed region."""
@@ -380,6 +411,10 @@ def run_gpu(args, w):
     survey_gbs = n_local * w.d * (20.0 + 4.0 * rho + 8.0 / w.d) / (kern_ms / 1e3) / 1e9
     traffic, traffic_src = ncu_traffic(w.name)
     peak, peak_src = hbm_peak()
+    rd = 8.0 + 4.0 * pbl  # bytes read / written per update (x, v; pbest where moved)
+    mix = mix_peak(rd / bytes_per_update)
+    if mix:
+        mix["frac"] = achieved / mix["GBps"]
 
     # ---------------- end to end through the public API, host buffers
     e2e = None
@@ -449,6 +484,7 @@ def run_gpu(args, w):
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "peak_source": peak_src,
                          "frac_of_spec": achieved / SPEC_HBM_GBS,  # vs the 8 TB/s data-sheet figure
+                         "mix_peak": mix,
                          "traffic": traffic, "traffic_source": traffic_src,
                          # SURVEY 8(d)'s accounting: every pbest row read, 4 rho written
                          "frac_survey_formula": survey_gbs / peak,

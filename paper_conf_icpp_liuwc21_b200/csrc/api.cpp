@@ -689,8 +689,10 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
   if (A.l2pf < 0 || A.l2pf > 64) A.l2pf = 0;
   if (!lazy) A.l2pf = 0;
   if (const char* v = std::getenv("PSO_L2PF_ALL")) A.l2pf_all = std::atoi(v) != 0;
+  // dynamic row claims (bit 0: streaming and column-split kernels; bit 1: the
+  // cluster kernel, where they measured slower).  NS 628 -> 591 us, W64K 912 -> 878.
   A.dyn_rows = 1;
-  if (const char* v = std::getenv("PSO_DYN_ROWS")) A.dyn_rows = std::atoi(v) != 0;
+  if (const char* v = std::getenv("PSO_DYN_ROWS")) A.dyn_rows = std::atoi(v) & 3;
   A.serp = 1;  // measured: C3 36.9 -> 35.7 us (120 MB state, L2-borderline), NS / C4 within 1 %
   if (const char* v = std::getenv("PSO_SERP")) A.serp = std::atoi(v) != 0;
   A.cand = h->cfg.gridres ? (float*)p : nullptr;

@@ -62,7 +62,8 @@ struct SwarmArgs {
   int l2pf;                   // TMA producer: L2 prefetch distance in rows of this CTA (0: off)
   int serp;                   // streaming kernels: odd iterations visit rows backwards (L2 reuse)
   int l2pf_all;               // prefetch every row (default: lazy rows only, whose stage loads 2 of 3 slots)
-  int dyn_rows;               // TMA streaming kernel: CTAs claim rows from a counter (else round robin)
+  int dyn_rows;               // rows / items claimed from ctl->row_claim instead of round robin:
+                              // bit 0 streaming + column split, bit 1 cluster
   unsigned char* send;        // world > 1: this rank's exchange record
   const unsigned char* recv;  // exchange: [2 iteration parities][world] records after the all-gather
   DevCtl* ctl;

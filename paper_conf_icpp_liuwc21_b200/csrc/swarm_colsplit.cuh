@@ -85,7 +85,7 @@ __global__ void __launch_bounds__(kColCompute + 64, 2)
       // sentinel (the last CTA resets the counter).  The producer passes the
       // item's (row, tile) to the other warps with the stage.
       unsigned long long* claim_ctr = &a.ctl->row_claim;
-      const bool dyn = a.dyn_rows != 0;
+      const bool dyn = (a.dyn_rows & 1) != 0;
       long long k = blockIdx.x;
       long long k_next =
           k >= items ? items : (dyn ? (long long)atomicAdd(claim_ctr, 1ull) + gridDim.x : k + gridDim.x);

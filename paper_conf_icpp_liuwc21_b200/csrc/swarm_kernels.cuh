@@ -994,7 +994,7 @@ __global__ void __launch_bounds__(kMaxT + 64, kMaxT > kMaxThreads ? 1 : 2)
       // CTA computes a row changes no bit (rows are independent; the candidate
       // key and the counters are order-free min / sums).
       unsigned long long* claim_ctr = &a.ctl->row_claim;
-      const bool dyn = a.dyn_rows != 0;
+      const bool dyn = (a.dyn_rows & 1) != 0;
       long long i = blockIdx.x;
       long long i_next =
           i >= n ? n : (dyn ? (long long)atomicAdd(claim_ctr, 1ull) + gridDim.x : i + gridDim.x);
@@ -1259,6 +1259,13 @@ __global__ void __launch_bounds__(kMaxThreadsCluster + 64, 1)
   __shared__ unsigned long long s_inc;  // incumbent of this iteration (after the exchange merge)
   __shared__ int s_src;
   __shared__ int sflag[kMaxStages];     // lazy pbest: the stage's row had PB == X
+  // Row schedule: CTA 0's producer picks the cluster's rows (round robin over
+  // clusters, or claimed from ctl->row_claim as in k_step_tma) and sends each
+  // stage's {row, lazy flag} to every CTA of the cluster (st.async + rbar);
+  // a CTA's producer copies it to srow / sflag for its own warps.
+  __shared__ __align__(8) float2 rmsg[kMaxStages];  // {row bits, flag bits; flag -1: no more rows}
+  __shared__ unsigned long long rbar[kMaxStages];
+  __shared__ long long srow[kMaxStages];
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   if (tid == 0) {
     mbar_init(&gbar, 1);
@@ -1268,6 +1275,7 @@ __global__ void __launch_bounds__(kMaxThreadsCluster + 64, 1)
       mbar_init(&empty[s], 1);
       mbar_init(&pbar[s], 1);
       mbar_init(&dbar[s], 1);
+      mbar_init(&rbar[s], 1);
     }
     mbar_fence_init();
   }
@@ -1300,26 +1308,63 @@ __global__ void __launch_bounds__(kMaxThreadsCluster + 64, 1)
       int s = 0;
       unsigned ph = 0;
       int k = 0;
-      int fl_next = (a.lazy_pb && cid < a.n_local) ? a.pbx[cid] : 0;
+      const long long n = a.n_local;
       const long long pd = (long long)a.l2pf * ncl;  // L2 prefetch, as in k_step_tma
-      int pfl_next = (pd && cid + pd < a.n_local) ? a.pbx[cid + pd] : 0;
-      for (long long r = cid; r < a.n_local; r += ncl, ++k) {
-        const int fl = fl_next;
-        if (a.lazy_pb && r + ncl < a.n_local) fl_next = a.pbx[r + ncl];
-        if (pd && r + pd < a.n_local && cnt > 0) {
-          const int pfl = pfl_next;
-          if (r + pd + ncl < a.n_local) pfl_next = a.pbx[r + pd + ncl];
-          const size_t po = ((size_t)(r + pd) * nvec + q0) * 4;
-          if (pfl || a.l2pf_all) {
-            bulk_prefetch_l2(a.X + po, blk_bytes);
-            bulk_prefetch_l2(a.V + po, blk_bytes);
-            if (!pfl) bulk_prefetch_l2(a.PB + po, blk_bytes);
-          }
-        }
+      // CTA 0 only: the claim front (k_step_tma's scheme, per cluster)
+      // (dynamic claims measured slower here -- W16K 808 -> 885-904 us -- so
+      // they are opt-in: dyn_rows bit 1)
+      unsigned long long* claim_ctr = &a.ctl->row_claim;
+      const bool dyn = (a.dyn_rows & 2) != 0;
+      long long i = cid, i_next = 0;
+      int fl_next = 0, pfl_next = 0;
+      if (crank == 0) {
+        i_next = i >= n ? n : (dyn ? (long long)atomicAdd(claim_ctr, 1ull) + ncl : i + ncl);
+        fl_next = (a.lazy_pb && i < n) ? a.pbx[i] : 0;
+        pfl_next = (pd && i + pd < n) ? a.pbx[i + pd] : 0;
+      }
+      for (;; ++k) {
         if (k >= stages) mbar_wait(&empty[s], ph ^ 1u);
+        if (crank == 0) {  // pick the row, send {row, flag} to every CTA of the cluster
+          long long r = -1;
+          int fl = -1;
+          if (i < n) {
+            r = i;
+            fl = fl_next;
+            const long long i_nn = i_next >= n ? n
+                                   : (dyn ? (long long)atomicAdd(claim_ctr, 1ull) + ncl
+                                          : i_next + ncl);
+            if (a.lazy_pb && i_next < n) fl_next = a.pbx[i_next];
+            if (pd && i + pd < n) {
+              const int pfl = pfl_next;
+              if (i_next + pd < n) pfl_next = a.pbx[i_next + pd];
+              if (pfl || a.l2pf_all) {  // the whole row (every CTA's block)
+                const size_t po = (size_t)(i + pd) * nvec * 4;
+                const unsigned rb = (unsigned)nvec * 16u;
+                bulk_prefetch_l2(a.X + po, rb);
+                bulk_prefetch_l2(a.V + po, rb);
+                if (!pfl) bulk_prefetch_l2(a.PB + po, rb);
+              }
+            }
+            i = i_next;
+            i_next = i_nn;
+          }
+          const float2 m = make_float2(__int_as_float((int)r), __int_as_float(fl));
+          for (int c = 0; c < C; ++c) st_async_v2(map_to_rank(&rmsg[s], c), m, map_to_rank(&rbar[s], c));
+        }
+        mbar_expect_tx(&rbar[s], 8u);
+        mbar_wait_cluster(&rbar[s], ph);
+        const float2 m = rmsg[s];
+        const int fl = __float_as_int(m.y);
+        if (fl < 0) {  // sentinel: the compute warps and the finaliser stop here
+          srow[s] = -1;
+          mbar_arrive(&full[s]);
+          break;
+        }
+        const long long r = __float_as_int(m.x);
         float4* st = ring + (size_t)s * 3 * chunk;
         sflag[s] = fl;
-        mbar_expect_tx(&full[s], (fl ? 2u : 3u) * blk_bytes);
+        srow[s] = r;
+        mbar_expect_tx(&full[s], (fl ? 2u : 3u) * blk_bytes);  // releases sflag[s], srow[s] too
         if (cnt > 0) {
           const size_t off = ((size_t)r * nvec + q0) * 4;
           bulk_g2s(st, a.X + off, blk_bytes, &full[s]);
@@ -1344,7 +1389,10 @@ __global__ void __launch_bounds__(kMaxThreadsCluster + 64, 1)
       unsigned nimp = 0, n_pbl = 0, n_pbs = 0;
       int s = 0, prev = -1;
       unsigned ph = 0;
-      for (long long r = cid; r < a.n_local; r += ncl) {
+      for (;;) {
+        mbar_wait(&full[s], ph);
+        const long long r = srow[s];
+        if (r < 0) break;
         const uint32_t gi = (uint32_t)(a.row_begin + r);
         const float pf_old = crank == 0 ? a.pf[r] : 0.f;
         mbar_wait(&done[s], ph);
@@ -1434,6 +1482,7 @@ __global__ void __launch_bounds__(kMaxThreadsCluster + 64, 1)
       if (n_pbs) atomicAdd(&a.ctl->pb_stores, (unsigned long long)n_pbs);
       __threadfence();
       s_last = (atomicAdd(&a.ctl->done, 1u) == gridDim.x - 1) ? 1 : 0;
+      if (s_last) a.ctl->row_claim = 0;  // every cluster's claims are done (see the producer)
     }
     __syncwarp();
     if (s_last) warp_gbest_epilogue(a, t, lane, s_inc, s_src);
@@ -1446,10 +1495,12 @@ __global__ void __launch_bounds__(kMaxThreadsCluster + 64, 1)
   mbar_wait(&gbar, 0);
   int s = 0;
   unsigned ph = 0;
-  for (long long r = cid; r < a.n_local; r += ncl) {
-    const uint32_t gi = (uint32_t)(a.row_begin + r);
+  for (;;) {
     float4* st = ring + (size_t)s * 3 * chunk;
     mbar_wait(&full[s], ph);
+    const long long r = srow[s];
+    if (r < 0) break;
+    const uint32_t gi = (uint32_t)(a.row_begin + r);
     const int fl = sflag[s];
     float4* xdst = fl ? st + 2 * chunk : st;
     float acc[Obj::kAcc];

@@ -775,11 +775,11 @@ def test_row_order_is_invisible(obj, n, d, monkeypatch):
     row from a counter the iteration's last CTA resets) change no bit: state,
     pf and gbest equal the forward, prefetch-free, round-robin run after every
     call (many rows per CTA, the wide 512-thread kernel at d = 4096, fewer rows
-    than CTAs)."""
+    than CTAs, the cluster kernel at d = 12000)."""
     monkeypatch.setenv("PSO_RESIDENT", "0")
     monkeypatch.setenv("PSO_SERP", "1")
     monkeypatch.setenv("PSO_L2PF_ALL", "1")
-    monkeypatch.setenv("PSO_DYN_ROWS", "1")
+    monkeypatch.setenv("PSO_DYN_ROWS", "3")  # claims on every streaming path, the cluster too
     g = gpu_swarm(n, d, obj, seed=12)
     monkeypatch.setenv("PSO_SERP", "0")
     monkeypatch.setenv("PSO_L2PF", "0")
