@@ -9,6 +9,6 @@ python -c "import __graft_entry__ as g; g.smoke()" 2>&1 | tail -2
 timeout 2400 python -m pytest tests -m gpu -q 2>&1 | tail -15
 timeout 900 python bench.py --gpus 1 --steps 20 --warmup 5 2>&1 | tail -1 > gpurun_out/final/bench_driver_cmd.json
 PSO_SHARE_GPU=1 PSO_QUIET=1 timeout 900 python bench.py --gpus 8 --steps 50 --warmup 5 --workload NS 2>/dev/null | grep '^{' > gpurun_out/final/bench_8ranks_shared_gpu.json
-WORKLOADS="C1 C2 C3 C4 NS C5 W16K W64K W256K NS_R8 C4_V600 NS_V512" NCU_WORKLOADS="NS C4 C3 W16K W64K" bash tools/profile_round.sh
+WORKLOADS="C1 C2 C3 C4 NS C5 W16K W64K W256K NS_R8 C4_V600 NS_V512" NCU_WORKLOADS="NS C4 C3 C5 W16K W64K" bash tools/profile_round.sh
 bash tools/gpu_sanitize.sh
 bash tools/capacity_sweep.sh

@@ -6,6 +6,7 @@ set -x
 O=gpurun_out/prof
 mkdir -p $O
 nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm,power.draw --format=csv > $O/gpu.txt
+python tools/hbm_mix_probe.py > $O/hbm_mix_probe.json 2>&1
 timeout 900 python bench.py 2>&1 | tail -1 > $O/bench_default.json
 timeout 900 python bench.py --impl reference --steps 3 --warmup 3 2>&1 | tail -1 > $O/bench_reference.json
 for w in ${WORKLOADS:-C1 C2 C3 C4 NS C5 W16K W64K}; do
