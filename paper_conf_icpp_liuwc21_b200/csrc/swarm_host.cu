@@ -295,12 +295,18 @@ cudaError_t cluster_shape(const KernelTable* t, int nvec, int C, const PlanHints
   const void* fn = t->step_cluster[vpt_index(vpt)][h.bounds ? 1 : 0];
   const size_t crow = (size_t)chunk * 16, btab = h.bounds ? 4 * crow : 0;
   const int per_sm = (h.ctas >= 1 && h.ctas <= 4) ? h.ctas : 1;  // CTAs per SM to size the ring for
+  cudaError_t e;
   int stages = ring_stages(crow + btab, 3 * crow, per_sm);
+  if (per_sm == 1) {  // one CTA per SM: the exact budget next to the kernel's static shared memory
+    cudaFuncAttributes fa{};
+    if ((e = cudaFuncGetAttributes(&fa, fn)) != cudaSuccess) return e;
+    const size_t budget = kSmemPerCtaMax - fa.sharedSizeBytes, fixed = crow + btab;
+    stages = budget > fixed ? (int)((budget - fixed) / (3 * crow)) : 0;
+  }
   if (h.stages >= 2 && h.stages < stages) stages = h.stages;
-  if (stages > kMaxStages) stages = kMaxStages;
+  if (stages > kClusterStages) stages = kClusterStages;
   if (stages < 2) return cudaSuccess;
   const size_t smem = crow + btab + (size_t)stages * 3 * crow;
-  cudaError_t e;
   if (C > 8 &&
       (e = cudaFuncSetAttribute(fn, cudaFuncAttributeNonPortableClusterSizeAllowed, 1)) != cudaSuccess)
     return e;

@@ -58,6 +58,9 @@ constexpr int kMaxThreads = 256;         // compute threads per CTA
 constexpr int kMaxThreadsCluster = 512;  // compute threads per CTA of the cluster kernel
 constexpr int kMaxThreadsWide = 512;     // compute threads per CTA of the wide TMA variant
 constexpr int kMaxStages = 8;
+// ring stages of the cluster kernel (its static shared arrays are sized by it; a
+// 2-CTA cluster's two 96 KB stages fit only with the static part this small)
+constexpr int kClusterStages = 4;
 constexpr unsigned kFull = 0xFFFFFFFFu;
 
 // ---------------------------------------------------------------- helpers
@@ -1249,23 +1252,23 @@ __global__ void __launch_bounds__(kMaxThreadsCluster + 64, 1)
   float4* sG = reinterpret_cast<float4*>(dsmem);
   float4* sB = sG + chunk;
   float4* ring = sB + (kB ? 4 * chunk : 0);
-  __shared__ float red[kMaxStages][(kMaxThreadsCluster / 32) * 2];
+  __shared__ float red[kClusterStages][(kMaxThreadsCluster / 32) * 2];
   // CTA 0: per rank {acc0, acc1, first x', last x'}; every CTA: {improved, f}.
   // Both arrive by st.async, which signals the receiver's mbarrier (complete_tx).
-  __shared__ __align__(16) float4 parts[kMaxStages][16];
-  __shared__ __align__(8) float2 dec[kMaxStages];
-  __shared__ unsigned long long full[kMaxStages], empty[kMaxStages], done[kMaxStages];
-  __shared__ unsigned long long pbar[kMaxStages], dbar[kMaxStages], gbar;
+  __shared__ __align__(16) float4 parts[kClusterStages][16];
+  __shared__ __align__(8) float2 dec[kClusterStages];
+  __shared__ unsigned long long full[kClusterStages], empty[kClusterStages], done[kClusterStages];
+  __shared__ unsigned long long pbar[kClusterStages], dbar[kClusterStages], gbar;
   __shared__ unsigned long long s_inc;  // incumbent of this iteration (after the exchange merge)
   __shared__ int s_src;
-  __shared__ int sflag[kMaxStages];     // lazy pbest: the stage's row had PB == X
+  __shared__ int sflag[kClusterStages];     // lazy pbest: the stage's row had PB == X
   // Row schedule: CTA 0's producer picks the cluster's rows (round robin over
   // clusters, or claimed from ctl->row_claim as in k_step_tma) and sends each
   // stage's {row, lazy flag} to every CTA of the cluster (st.async + rbar);
   // a CTA's producer copies it to srow / sflag for its own warps.
-  __shared__ __align__(8) float2 rmsg[kMaxStages];  // {row bits, flag bits; flag -1: no more rows}
-  __shared__ unsigned long long rbar[kMaxStages];
-  __shared__ long long srow[kMaxStages];
+  __shared__ __align__(8) float2 rmsg[kClusterStages];  // {row bits, flag bits; flag -1: no more rows}
+  __shared__ unsigned long long rbar[kClusterStages];
+  __shared__ long long srow[kClusterStages];
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   if (tid == 0) {
     mbar_init(&gbar, 1);
