@@ -59,9 +59,10 @@ extern "C" {
                               PSO_D_AUTO_COLSPLIT) */
 #define PSO_D_MAX (1 << 24) /* max dimension: above PSO_D_MAX_ROW the column split
                               (PSO_FLAG_COLUMN_SPLIT) is used on a single GPU */
-#define PSO_D_AUTO_COLSPLIT 16384 /* a single-GPU handle (no communicator, world <= 1)
+#define PSO_D_AUTO_COLSPLIT 9216 /* a single-GPU handle (no communicator, world <= 1)
                               with d above this uses the column split: faster than
-                              clusters of 8-16 CTAs per row */
+                              the 4-16-CTA clusters per row from d = 9728 up (W16K
+                              16384^2: 708 vs 806 us) */
 
 typedef struct pso_swarm* pso_handle; /* opaque; owns all device memory */
 

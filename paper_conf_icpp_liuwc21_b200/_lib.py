@@ -20,7 +20,7 @@ PSO_FLAG_TIMING, PSO_FLAG_DEFER_INIT, PSO_FLAG_ASYNC_GBEST, PSO_FLAG_COLUMN_SPLI
 PSO_FLAG_DEVICE = 16
 PSO_FLAG_ALLREDUCE = 32
 PSO_D_MAX_ROW = 65536
-PSO_D_AUTO_COLSPLIT = 16384
+PSO_D_AUTO_COLSPLIT = 9216
 PSO_D_MAX = 1 << 24
 
 # every symbol include/fastpso.h declares

@@ -479,12 +479,15 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
                   "PSO_FLAG_COLUMN_SPLIT", d, PSO_D_MAX_ROW);
     colsplit = true;  // one GPU: rows longer than a cluster are tiled
   }
-  // One GPU, rows that would need a cluster of 8 or 16 CTAs: the column split is
-  // faster (Rastrigin 4096 x 49152: 942 -> 739 us/iteration, 4096 x 65536:
-  // 1073 -> 998; Griewank 8192 x 32768: 991 -> 937; at d = 16384 the 4-CTA
-  // cluster stays faster, 831 vs 934).  PSO_CLUSTER (tuning) keeps the cluster.
+  // One GPU, rows that need a cluster of 4-16 CTAs: the column split (pbest
+  // slots, G cache) is faster from d = 9728 up (Griewank 16384 x 16384: 806 ->
+  // 708 us/iteration, 12288 x 10240: 482 -> 440; Rastrigin 12288 x 9728: 522
+  // -> 484); at d <= 9216 the 4-CTA cluster stays (12288 x 9216: 473 vs 512).
+  // PSO_CLUSTER (tuning) keeps the cluster.
   if (!colsplit && !o.nccl_comm && o.world <= 1 && d > PSO_D_AUTO_COLSPLIT && !std::getenv("PSO_CLUSTER"))
     colsplit = true;
+  if (const char* cs = std::getenv("PSO_COLSPLIT"))  // tuning: 1 = column split for any d
+    if (*cs == '1') colsplit = true;
   if (colsplit && (o.flags & PSO_FLAG_ASYNC_GBEST))
     return fail(PSO_ERR_INVALID, "PSO_FLAG_COLUMN_SPLIT excludes PSO_FLAG_ASYNC_GBEST");
   if (!finite(w) || !finite(c1) || !finite(c2))
@@ -688,6 +691,7 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
   if (const char* v = std::getenv("PSO_L2PF")) A.l2pf = std::atoi(v);
   if (A.l2pf < 0 || A.l2pf > 64) A.l2pf = 0;
   if (!lazy) A.l2pf = 0;
+  if (colsplit) A.l2pf = 0;  // (an L2 prefetch of row tiles ahead measured slower: W16K 767 -> 847 us)
   if (const char* v = std::getenv("PSO_L2PF_ALL")) A.l2pf_all = std::atoi(v) != 0;
   // dynamic row claims (bit 0: streaming and column-split kernels; bit 1: the
   // cluster kernel, where they measured slower).  NS 628 -> 591 us, W64K 912 -> 878.
@@ -895,13 +899,15 @@ pso_status pso_get_state(pso_handle h, float* x, float* v, float* pb, float* pf,
   if ((st = use_device(h)) != PSO_OK) return st;
   const size_t w = (size_t)h->d_local * 4, sp = (size_t)h->pitch * 4, rows = (size_t)h->n_local;
   if (rows > 0) {
+    // the plain layout first: deferred pbest rows (PB == X) written out; on the
+    // column split also rows whose x lives in the PB array (swarm_colsplit.cuh)
+    if (h->args.lazy_pb && (pb || (x && h->colsplit))) {
+      PSO_CUDA(h, launch_materialize_pb(h->args, h->stream));
+      ++h->launches;
+    }
     if (x) PSO_CUDA(h, cudaMemcpy2DAsync(x, w, h->args.X, sp, w, rows, cudaMemcpyDeviceToHost, h->stream));
     if (v) PSO_CUDA(h, cudaMemcpy2DAsync(v, w, h->args.V, sp, w, rows, cudaMemcpyDeviceToHost, h->stream));
     if (pb) {
-      if (h->args.lazy_pb) {  // write out the deferred pbest rows (PB == X) first
-        PSO_CUDA(h, launch_materialize_pb(h->args, h->stream));
-        ++h->launches;
-      }
       PSO_CUDA(h, cudaMemcpy2DAsync(pb, w, h->args.PB, sp, w, rows, cudaMemcpyDeviceToHost, h->stream));
     }
     if (pf) PSO_CUDA(h, cudaMemcpyAsync(pf, h->args.pf, rows * 4, cudaMemcpyDeviceToHost, h->stream));
@@ -922,26 +928,24 @@ pso_status pso_get_rows(pso_handle h, const int64_t* rows, int64_t m, float* x, 
       return fail(PSO_ERR_INVALID, "row %lld outside [0, %lld)", (long long)rows[k], (long long)h->n_local);
   if ((st = use_device(h)) != PSO_OK) return st;
   if ((st = sync_and_check(h)) != PSO_OK) return st;
-  // lazy pbest rows (PB == X, not stored): their pbest is read from X
+  // lazy pbest rows (pbx bit 0: PB == x, not stored) read their pbest where x
+  // is; column-split rows with pbx bit 1 hold x in PB and pb in X
   std::vector<unsigned char> lazy;
-  if (pb && h->args.lazy_pb && m > 0) {
+  if ((pb || x) && h->args.lazy_pb && m > 0) {
     lazy.resize((size_t)h->n_local);
     PSO_CUDA(h, cudaMemcpy(lazy.data(), h->args.pbx, lazy.size(), cudaMemcpyDeviceToHost));
   }
   const size_t w = (size_t)h->d_local * 4, sp = (size_t)h->pitch * 4;
   for (int64_t k = 0; k < m; ++k) {
     const size_t r = (size_t)rows[k], o = (size_t)k * h->d_local;
-    const unsigned char* xr = reinterpret_cast<const unsigned char*>(h->args.X) + r * sp;
+    const unsigned char fl = lazy.empty() ? 0 : lazy[r];
+    const unsigned char* xr = reinterpret_cast<const unsigned char*>((fl & 2) ? h->args.PB : h->args.X) + r * sp;
+    const unsigned char* pr = reinterpret_cast<const unsigned char*>((fl & 2) ? h->args.X : h->args.PB) + r * sp;
     if (x) PSO_CUDA(h, cudaMemcpyAsync(x + o, xr, w, cudaMemcpyDeviceToHost, h->stream));
     if (v)
       PSO_CUDA(h, cudaMemcpyAsync(v + o, reinterpret_cast<const unsigned char*>(h->args.V) + r * sp, w,
                                   cudaMemcpyDeviceToHost, h->stream));
-    if (pb) {
-      const unsigned char* src = (!lazy.empty() && lazy[r])
-                                     ? xr
-                                     : reinterpret_cast<const unsigned char*>(h->args.PB) + r * sp;
-      PSO_CUDA(h, cudaMemcpyAsync(pb + o, src, w, cudaMemcpyDeviceToHost, h->stream));
-    }
+    if (pb) PSO_CUDA(h, cudaMemcpyAsync(pb + o, (fl & 1) ? xr : pr, w, cudaMemcpyDeviceToHost, h->stream));
     if (pf) PSO_CUDA(h, cudaMemcpyAsync(pf + k, h->args.pf + r, 4, cudaMemcpyDeviceToHost, h->stream));
   }
   return sync_and_check(h);

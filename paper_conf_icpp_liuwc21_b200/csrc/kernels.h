@@ -57,7 +57,8 @@ struct SwarmArgs {
   float* cand;                // grid-resident kernel: [2][grid][pitch] candidate rows
   unsigned long long* cand_key;  // grid-resident kernel: [2][grid] candidate keys (~0: none)
   const float* bounds;        // per-dimension bounds [vlo | vhi | xlo | xhi] (4 x pitch), or null
-  unsigned char* pbx;         // lazy pbest: 1 = the row's PB equals its X (PB not stored)
+  unsigned char* pbx;         // lazy pbest: bit 0 = the row's pbest equals its x (PB not stored);
+                              // bit 1 (column split) = x in the PB array, pb in X
   int lazy_pb;
   int l2pf;                   // TMA producer: L2 prefetch distance in rows of this CTA (0: off)
   int serp;                   // streaming kernels: odd iterations visit rows backwards (L2 reuse)

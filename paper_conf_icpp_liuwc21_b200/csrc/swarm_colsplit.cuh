@@ -23,11 +23,19 @@
 //                 winner's x (this rank's block) into G.
 //
 // The pbest copy cannot wait for the decision (x' is stored before f is
-// known), so pbest rows use the lazy form: pbx[r] = 1 records "row r improved
-// in the last decision, its pbest is its current X".  The next k_col_step then
-// uses pb = x and stores the old x into PB (the deferred copy); a row that
-// never improves only reads PB.  Bytes per element: 16 (x, v in and out) + 4
-// (PB read, or PB written after an improvement).
+// known), so a row's position and pbest live in two slots, the X and the PB
+// array, and pbx[r] records where (round 3 of the design):
+//   bit 0 (lazy)  the row improved in the last decision: its pbest IS its
+//                 position (one slot holds both, the other is stale);
+//   bit 1 (swap)  the position lives in the PB array (and a non-lazy row's
+//                 pbest in the X array).
+// A non-lazy row reads x and pb and stores x' over x (same slot).  A lazy row
+// reads only x (= pb) and stores x' into the OTHER slot, so the old x stays
+// in place as the pbest should the row not improve -- no copy, ever:
+//   new swap bit = lazy ? !swap : swap,   new lazy bit = improved.
+// Bytes per element: 16 (x, v in and out) + 4 for a row that did not improve
+// in the last decision (its pb read).  k_materialize_pb restores the plain
+// layout (X = x, PB = pb) before the host reads whole matrices.
 //
 // Init (init = 1, Alg. 1 lines 1-3): the producer loads nothing; the compute
 // warps draw x0, v0 (Philox X0 / V0 at the global column), the finaliser stores
@@ -49,14 +57,22 @@ __global__ void __launch_bounds__(kColCompute + 64, 2)
   static_assert(Obj::kAcc <= 2, "the tile partial carries two accumulators");
   extern __shared__ __align__(128) unsigned char dsmem[];
   constexpr int nthr = kColCompute, nwarps = nthr / 32;
-  constexpr int per = kB ? 8 : 4;  // stage arrays: x, v, pb, g [, vlo, vhi, xlo, xhi]
+  // Shared memory: [G cache: 2 slots x gper tiles][ring: stages x {x, v, pb}].
+  // Items are visited tile-major, so a CTA's consecutive items mostly share
+  // their column tile: the G tile (and the bounds tiles) is loaded into one of
+  // two cache slots only when the tile changes, and the stages hold just the
+  // row arrays -- 4 stages of 24 KB instead of 3 of 32 KB at 512-float4 tiles.
+  constexpr int per = 3;            // stage arrays: x, v, pb
+  constexpr int gper = kB ? 5 : 1;  // cache slot arrays: g [, vlo, vhi, xlo, xhi]
   const int chunk = a.col_chunk, nb = a.col_nb, nvl = a.nvec, d = a.d;
-  float4* ring = reinterpret_cast<float4*>(dsmem);
+  float4* gcache = reinterpret_cast<float4*>(dsmem);
+  float4* ring = gcache + 2 * gper * chunk;
   __shared__ float red[kMaxStages][nwarps * 2];
   __shared__ unsigned long long full[kMaxStages], empty[kMaxStages], done[kMaxStages];
   __shared__ int sflag[kMaxStages];
   __shared__ long long s_r[kMaxStages];  // the stage's item: row (-1: no more items) ...
   __shared__ int s_b[kMaxStages];        // ... and tile
+  __shared__ int s_g[kMaxStages];        // ... and the G cache slot holding the tile
   // the tile's first and last x' for the neighbour terms across tiles, handed to
   // the finaliser by the arriving lanes themselves (ordered by their own release)
   __shared__ float s_edge[kMaxStages][2];
@@ -79,22 +95,26 @@ __global__ void __launch_bounds__(kColCompute + 64, 2)
       int s = 0;
       unsigned ph = 0;
       long long i = 0;
-      // Item schedule as k_step_tma's rows: round robin, or (a.dyn_rows) the
-      // first item is blockIdx.x and every further one is claimed from
-      // ctl->row_claim two items ahead, each claim's value consumed before the
-      // sentinel (the last CTA resets the counter).  The producer passes the
-      // item's (row, tile) to the other warps with the stage.
+      // Item schedule: tile-major (item k = tile k / n, row k mod n), round
+      // robin or (a.dyn_rows) the first item is blockIdx.x and every further
+      // one is claimed from ctl->row_claim two items ahead, each claim's value
+      // consumed before the sentinel (the last CTA resets the counter).  The
+      // producer passes the item's (row, tile, cache slot) with the stage.
       unsigned long long* claim_ctr = &a.ctl->row_claim;
       const bool dyn = (a.dyn_rows & 1) != 0;
+      const long long n = a.n_local;
       long long k = blockIdx.x;
       long long k_next =
           k >= items ? items : (dyn ? (long long)atomicAdd(claim_ctr, 1ull) + gridDim.x : k + gridDim.x);
       // the lazy-pbest flag of the next item is loaded one item ahead, so its L2
       // latency overlaps the wait for a free stage instead of delaying the copies
-      int fl_next = (!init && k < items) ? a.pbx[k / nb] : 0;
+      int fl_next = (!init && k < items) ? a.pbx[k % n] : 0;
+      // G cache: the tile each slot holds (-1: none) and the last item using it
+      int g_tile0 = -1, g_tile1 = -1;
+      long long g_last0 = -1, g_last1 = -1;
       for (; k < items; ++i) {
-        const long long r = k / nb;
-        const int b = (int)(k - r * nb);
+        const int b = (int)(k / n);
+        const long long r = k - (long long)b * n;
         const int q0 = b * chunk;
         const int cnt = min(chunk, nvl - q0);
         const unsigned bytes = (unsigned)cnt * 16u;
@@ -102,7 +122,7 @@ __global__ void __launch_bounds__(kColCompute + 64, 2)
         const long long k_nn = k_next >= items ? items
                                : (dyn ? (long long)atomicAdd(claim_ctr, 1ull) + gridDim.x
                                       : k_next + gridDim.x);
-        if (!init && k_next < items) fl_next = a.pbx[k_next / nb];
+        if (!init && k_next < items) fl_next = a.pbx[k_next % n];
         k = k_next;
         k_next = k_nn;
         if (i >= stages) mbar_wait(&empty[s], ph ^ 1u);
@@ -111,18 +131,37 @@ __global__ void __launch_bounds__(kColCompute + 64, 2)
         s_b[s] = b;
         if (init) {
           sflag[s] = 0;
+          s_g[s] = 0;
           mbar_arrive(&full[s]);
         } else {
+          int gs = g_tile0 == b ? 0 : g_tile1 == b ? 1 : -1;
+          const bool load_g = gs < 0;
+          if (load_g) {  // the least recently used slot, once no stage in flight reads it
+            gs = g_last0 <= g_last1 ? 0 : 1;
+            // (stages are released in item order, and the LRU slot's last item is
+            // at most i - 2, whose release needs only items up to i - 1)
+            const long long m = gs ? g_last1 : g_last0;
+            if (m >= 0 && m > i - stages) mbar_wait(&empty[m % stages], (unsigned)((m / stages) & 1));
+            if (gs) g_tile1 = b; else g_tile0 = b;
+          }
+          if (gs) g_last1 = i; else g_last0 = i;
+          s_g[s] = gs;
           sflag[s] = fl;
-          mbar_expect_tx(&full[s], bytes * ((fl ? 3u : 4u) + (kB ? 4u : 0u)));
+          const bool lazy = (fl & 1) != 0;
+          mbar_expect_tx(&full[s], bytes * ((lazy ? 2u : 3u) + (load_g ? (unsigned)gper : 0u)));
           const size_t off = ((size_t)r * nvl + q0) * 4;
-          bulk_g2s(st, a.X + off, bytes, &full[s]);
+          const float* xs = (fl & 2) ? a.PB : a.X;  // the slot of the position
+          const float* ps = (fl & 2) ? a.X : a.PB;  // ... and of a non-lazy pbest
+          bulk_g2s(st, xs + off, bytes, &full[s]);
           bulk_g2s(st + chunk, a.V + off, bytes, &full[s]);
-          if (!fl) bulk_g2s(st + 2 * chunk, a.PB + off, bytes, &full[s]);
-          bulk_g2s(st + 3 * chunk, a.G + (size_t)q0 * 4, bytes, &full[s]);
-          if (kB)
-            for (int m = 0; m < 4; ++m)
-              bulk_g2s(st + (4 + m) * chunk, a.bounds + ((size_t)m * nvl + q0) * 4, bytes, &full[s]);
+          if (!lazy) bulk_g2s(st + 2 * chunk, ps + off, bytes, &full[s]);
+          if (load_g) {
+            float4* gc = gcache + (size_t)gs * gper * chunk;
+            bulk_g2s(gc, a.G + (size_t)q0 * 4, bytes, &full[s]);
+            if (kB)
+              for (int m = 0; m < 4; ++m)
+                bulk_g2s(gc + (1 + m) * chunk, a.bounds + ((size_t)m * nvl + q0) * 4, bytes, &full[s]);
+          }
         }
         if (++s == stages) {
           s = 0;
@@ -143,7 +182,7 @@ __global__ void __launch_bounds__(kColCompute + 64, 2)
       // byte offset of this iteration's partial table within every rank's region
       const size_t parts_off =  // = col_parts(region, a, par) - region
           col_tag_bytes(a.world) + (size_t)par * (size_t)a.n_local * (size_t)a.col_nbt * sizeof(float4);
-      unsigned n_pbl = 0, n_pbs = 0;
+      unsigned n_pbl = 0;
       int s = 0, prev = -1;
       unsigned ph = 0;
       for (;;) {
@@ -165,7 +204,7 @@ __global__ void __launch_bounds__(kColCompute + 64, 2)
         }
         const float4* st = ring + (size_t)s * per * chunk;
         const int fl = sflag[s];
-        const float4* xnew = fl ? st + 2 * chunk : st;  // where the compute warps put x'
+        const float4* xnew = st;  // the compute warps put x' over x
         const float4 msg = make_float4(c[0], Obj::kAcc > 1 ? c[Obj::kAcc - 1] : 0.f,
                                        Obj::kNeighbor ? s_edge[s][0] : 0.f,
                                        Obj::kNeighbor ? s_edge[s][1] : 0.f);
@@ -176,13 +215,13 @@ __global__ void __launch_bounds__(kColCompute + 64, 2)
           reinterpret_cast<float4*>(const_cast<unsigned char*>(a.recv) + parts_off)[pidx] = msg;
         }
         const size_t off = ((size_t)r * nvl + q0) * 4;
-        bulk_s2g(a.X + off, xnew, bytes);
+        // x' over x (non-lazy row), or into the other slot (lazy row: the old x
+        // stays as the pbest until the decision says otherwise)
+        const bool to_pb = ((fl >> 1) ^ (fl & 1)) != 0;
+        bulk_s2g((to_pb ? a.PB : a.X) + off, xnew, bytes);
         bulk_s2g(a.V + off, st + chunk, bytes);
-        if (init || fl) bulk_s2g(a.PB + off, st, bytes);  // x0, or the deferred pbest (old x)
-        if (b == 0 && !init) {  // per row: PB read, or PB written
-          n_pbl += fl ? 0u : 1u;
-          n_pbs += fl ? 1u : 0u;
-        }
+        if (init) bulk_s2g(a.PB + off, xnew, bytes);  // PB = x0
+        if (b == 0 && !init) n_pbl += (fl & 1) ? 0u : 1u;  // per row: PB read
         bulk_commit();
         if (prev >= 0) {
           bulk_wait_read<1>();
@@ -197,7 +236,6 @@ __global__ void __launch_bounds__(kColCompute + 64, 2)
       bulk_wait_all();
       fence_proxy_async_global();
       if (n_pbl) atomicAdd(&a.ctl->pb_loads, (unsigned long long)n_pbl);
-      if (n_pbs) atomicAdd(&a.ctl->pb_stores, (unsigned long long)n_pbs);
       __threadfence_system();  // this CTA's partials (local and peer stores) before the ticket
       if (atomicAdd(&a.ctl->done, 1u) == gridDim.x - 1) {
         __threadfence_system();
@@ -227,8 +265,10 @@ __global__ void __launch_bounds__(kColCompute + 64, 2)
     const int q0 = s_b[s] * chunk;
     const int cnt = min(chunk, nvl - q0);
     const uint32_t gi = (uint32_t)(a.row_begin + r);
-    const int fl = sflag[s];
-    float4* xdst = fl ? st + 2 * chunk : st;  // keep the old x for the deferred pbest copy
+    const int fl = sflag[s] & 1;  // lazy row: pb = x (its pb slot is not loaded)
+    // x' over x: the old x of a lazy row stays in HBM (the other slot)
+    float4* xdst = st;
+    const float4* gc = gcache + (size_t)s_g[s] * gper * chunk;
     float acc[Obj::kAcc];
     Obj::init(acc);
     float e_first = 0.f, e_last = 0.f;  // x' of the tile's first / last float4 (owners only)
@@ -260,9 +300,9 @@ __global__ void __launch_bounds__(kColCompute + 64, 2)
         if (ql < cnt) {
           const int qg = a.col_q0 + q0 + ql;
           float4 x = st[ql], v = st[chunk + ql];
-          const float4 g = st[3 * chunk + ql];
-          move4_draw<kB>(mp, key, t, gi, (uint32_t)qg, fl, x, v, st + 2 * chunk + ql, g,
-                         st + 4 * chunk, chunk, ql);
+          const float4 g = gc[ql];
+          move4_draw<kB>(mp, key, t, gi, (uint32_t)qg, fl, x, v, st + 2 * chunk + ql, g, gc + chunk,
+                         chunk, ql);
           if ((d & 3) && qg == a.nvec_glob - 1) {
             const int jj = 4 * qg;
             if (jj + 1 >= d) x.y = v.y = 0.f;
@@ -350,6 +390,7 @@ __global__ void __launch_bounds__(kColDecideThreads) k_col_decide(const __grid_c
   for (long long r = blockIdx.x * wpc + warp; r < a.n_local; r += (long long)gridDim.x * wpc) {
     const float4* Pr = P + (size_t)r * nbt;
     const float pf_old = (lane == 0 && !init) ? a.pf[r] : 0.f;  // in flight with the partials
+    const int fo = (lane == 0 && !init) ? a.pbx[r] : 0;
     float c[Obj::kAcc];
     Obj::init(c);
     for (int bt = lane; bt < nbt; bt += 32) {
@@ -378,7 +419,9 @@ __global__ void __launch_bounds__(kColDecideThreads) k_col_decide(const __grid_c
           a.pf[r] = f;
           ++nimp;
         }
-        a.pbx[r] = imp ? 1 : 0;
+        // x' went to the other slot iff the row was lazy (see k_col_step)
+        const int sw = (fo >> 1) ^ (fo & 1);
+        a.pbx[r] = (unsigned char)((sw << 1) | (imp ? 1 : 0));
       }
       if (val == val && ord_f32(val) < inc_ord) {  // strictly below gf (Alg. 1 line 10)
         const unsigned long long key = pack_key(val, gi);
@@ -408,11 +451,14 @@ __global__ void __launch_bounds__(kColDecideThreads) k_col_decide(const __grid_c
     __threadfence();
     s_best[0] = *(volatile unsigned long long*)&a.ctl->key_acc;
     s_best[1] = a.ctl->key_cur;
+    s_nimp[0] = s_best[0] < s_best[1]  // the winner's slot (its decision is visible: ticket order)
+                    ? *(volatile unsigned char*)&a.pbx[(long long)(uint32_t)s_best[0] - a.row_begin]
+                    : 0u;
   }
   __syncthreads();
   const unsigned long long acc = s_best[0], cur = s_best[1];
   if (acc < cur) {  // the block is up to 1 MB: 8 independent loads in flight per thread
-    const float4* x = reinterpret_cast<const float4*>(a.X) +
+    const float4* x = reinterpret_cast<const float4*>((s_nimp[0] & 2u) ? a.PB : a.X) +
                       ((long long)(uint32_t)acc - a.row_begin) * a.nvec;
     float4* G4 = reinterpret_cast<float4*>(a.G);
     const int nt = blockDim.x;

@@ -190,16 +190,30 @@ __global__ void __launch_bounds__(32) k_p2p_probe(const SwarmArgs a, int phase, 
 }
 
 // ---------------------------------------------------------- materialize PB
-// Lazy pbest rows (PB == X, not stored): one warp per flagged row copies X -> PB.
+// Restores the plain layout (X holds x, PB holds pb, pbx = 0) before the host
+// reads whole matrices.  pbx bit 0: lazy pbest row (PB == x, not stored);
+// bit 1 (column split only): x lives in the PB array, a non-lazy pbest in the
+// X array (swarm_colsplit.cuh).  One warp per flagged row.
 __global__ void __launch_bounds__(256) k_materialize_pb(const SwarmArgs a) {
   const int lane = threadIdx.x & 31;
   const long long warps = (long long)gridDim.x * (blockDim.x >> 5);
   for (long long r = blockIdx.x * (long long)(blockDim.x >> 5) + (threadIdx.x >> 5); r < a.n_local;
        r += warps) {
-    if (!a.pbx[r]) continue;
-    const float4* x = reinterpret_cast<const float4*>(a.X) + r * a.nvec;
+    const int fl = a.pbx[r];
+    if (!fl) continue;
+    float4* x = reinterpret_cast<float4*>(a.X) + r * a.nvec;
     float4* pb = reinterpret_cast<float4*>(a.PB) + r * a.nvec;
-    for (int q = lane; q < a.nvec; q += 32) pb[q] = x[q];
+    for (int q = lane; q < a.nvec; q += 32) {
+      if (fl == 1) {
+        pb[q] = x[q];
+      } else if (fl == 3) {
+        x[q] = pb[q];
+      } else {  // 2: swap the slots
+        const float4 t = x[q];
+        x[q] = pb[q];
+        pb[q] = t;
+      }
+    }
     __syncwarp();
     if (lane == 0) a.pbx[r] = 0;
   }
@@ -637,18 +651,33 @@ cudaError_t plan_colsplit(int objective, int tile, int tiles_local, long long n,
   const KernelTable* t = kernel_table(objective);
   if (!t) return cudaErrorInvalidDeviceFunction;
   if (tile < 1 || tiles_local < 1 || n < 1) return cudaErrorInvalidConfiguration;
-  const int per = bounds ? 8 : 4;
-  const size_t stage = (size_t)per * tile * 16;
+  // k_col_step's shared memory: a G cache of 2 slots x {g [, 4 bounds tiles]},
+  // then the ring of {x, v, pb} stages
+  const size_t stage = (size_t)3 * tile * 16, gcache = (size_t)2 * (bounds ? 5 : 1) * tile * 16;
   int ctas = bounds ? 1 : 2;  // ~100 registers x 320 threads: 2 CTAs per SM
   if (const char* v = std::getenv("PSO_COL_CTAS")) ctas = std::max(1, std::min(2, std::atoi(v)));
-  int stages = ring_stages(0, stage, ctas);
+  const void* fn = t->col_step[bounds ? 1 : 0];
+  // the exact budget: the SM's shared memory over its CTAs, less the per-CTA
+  // reservation and the kernel's static shared memory (512-float4 tiles: 16 KB
+  // of cache + 4 stages of 24 KB fit two CTAs with 128 B to spare)
+  cudaFuncAttributes fa{};
+  cudaError_t e = cudaFuncGetAttributes(&fa, fn);
+  if (e != cudaSuccess) return e;
+  int dev = 0, per_sm = 0, reserved = 0, optin = 0;
+  if ((e = cudaGetDevice(&dev)) != cudaSuccess) return e;
+  if ((e = cudaDeviceGetAttribute(&per_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, dev)) != cudaSuccess ||
+      (e = cudaDeviceGetAttribute(&reserved, cudaDevAttrReservedSharedMemoryPerBlock, dev)) != cudaSuccess ||
+      (e = cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev)) != cudaSuccess)
+    return e;
+  long long budget = (long long)per_sm / ctas - reserved - (long long)fa.sharedSizeBytes;
+  budget = std::min(budget, (long long)optin - (long long)fa.sharedSizeBytes);
+  int stages = budget > (long long)gcache ? (int)((budget - (long long)gcache) / (long long)stage) : 0;
   int max_st = 4;  // 4 tiles in flight per CTA cover the HBM latency
   if (const char* v = std::getenv("PSO_COL_STAGES")) max_st = std::max(2, std::min(kMaxStages, std::atoi(v)));
   if (stages > max_st) stages = max_st;
   if (stages < 2) return cudaErrorInvalidConfiguration;
-  const void* fn = t->col_step[bounds ? 1 : 0];
-  const size_t smem = (size_t)stages * stage;
-  cudaError_t e = allow_dynamic_smem(fn, smem);
+  const size_t smem = gcache + (size_t)stages * stage;
+  e = allow_dynamic_smem(fn, smem);
   if (e != cudaSuccess) return e;
   const long long items = n * tiles_local;
   long long grid = (long long)sm_count * ctas;

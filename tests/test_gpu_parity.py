@@ -10,6 +10,8 @@ Acceptance (north_star):
 Sizes span several CTA tiles, ragged d (d % 4 != 0), every CTA shape
 (VPT 1/2/4/8) and the degenerate n = 1, d = 1.
 """
+import os
+
 import numpy as np
 import pytest
 
@@ -35,6 +37,14 @@ def gpu_swarm(n, d, obj, seed=2021, w=0.9, c1=2.0, c2=2.0, vmax=0.0, **kw):
 def cpu_swarm(n, d, obj, seed=2021, w=0.9, c1=2.0, c2=2.0, vmax=0.0, create=True):
     lo, hi = DOMAINS[obj]
     return orc.OracleSwarm(n, d, w, c1, c2, lo, hi, obj, seed, vmax=vmax, create=create)
+
+
+def keep_cluster(monkeypatch, d):
+    """Rows of d in (PSO_D_AUTO_COLSPLIT, 16384] take the column split on one
+    GPU; tests that exercise the row kernels there (the 4-CTA cluster: lazy vs
+    eager pbest, the exchanges against a single-GPU twin) ask for the cluster."""
+    if fp.PSO_D_AUTO_COLSPLIT < d <= 16384:
+        monkeypatch.setenv("PSO_CLUSTER", "4")
 
 
 # ------------------------------------------------------------------ Philox
@@ -333,6 +343,8 @@ def test_handles_sharing_a_kernel_keep_their_shared_memory(first, second, monkey
     not lower the limit the first one launches with (both keep stepping, each
     equal to a fresh single handle)."""
     monkeypatch.setenv("PSO_RESIDENT", "0")
+    if first > fp.PSO_D_AUTO_COLSPLIT:  # the cluster kernel (the column split's ring is d-free)
+        monkeypatch.setenv("PSO_CLUSTER", "4")
     a = gpu_swarm(300, first, RASTRIGIN, seed=1)
     b = gpu_swarm(300, second, RASTRIGIN, seed=2)
     ia, ib = a.info(), b.info()
@@ -345,18 +357,23 @@ def test_handles_sharing_a_kernel_keep_their_shared_memory(first, second, monkey
 
 
 # ------------------------------------------------------------------ full size, sampled
-@pytest.mark.parametrize("key", ["NS", "C4", "C3", "C2", "W16K", "W64K", "C5", "C5_2900K"])
-def test_full_size_sampled_rows(key):
+@pytest.mark.parametrize("key", ["NS", "C4", "C3", "C2", "W16K", "W16K@cluster", "W64K", "C5",
+                                 "C5_2900K"])
+def test_full_size_sampled_rows(key, monkeypatch):
     """Bench configurations at full size in the bench's launch shape (NS / C4
     streaming 100k x 2000, C3 streaming with a neighbour functor, C2 on the
-    grid-resident path, W16K on 4-CTA clusters, W64K on the automatic column
-    split, C5 1M x 4096 on the wide 16-warp instantiation, and the capacity
-    sweep's 2.9M x 4096 -- 142.5 GB of state): sampled rows read back with
+    grid-resident path, W16K and W64K on the automatic column split, W16K on
+    4-CTA clusters too, C5 1M x 4096 on the wide 16-warp instantiation, and the
+    capacity sweep's 2.9M x 4096 -- 142.5 GB of state): sampled rows read back with
     pso_get_rows are recomputed by the oracle exactly (rows are independent
     given G): init bit-exact, one iteration's X / V bit-exact, decisions as the
     oracle's; the gbest is min pf with the lowest index and G = PB[gi]."""
+    if key.endswith("@cluster"):
+        key = key.split("@")[0]
+        monkeypatch.setenv("PSO_CLUSTER", "4")
     w = WORKLOADS[key]
     g = gpu_swarm(w.n, w.d, w.objective, seed=w.seed)
+    assert g.info()["column_split"] == int(w.d > fp.PSO_D_AUTO_COLSPLIT and "PSO_CLUSTER" not in os.environ)
     idx = sample_rows(w.n, 48, seed=7)
     X0, V0, _, _ = g.get_rows(idx[:8])
     for k, i in enumerate(idx[:8]):  # init rows are bit-exact
@@ -427,6 +444,7 @@ def test_exchange_path_with_single_rank_comm(obj, n, d, mode, monkeypatch):
     iterations, or launched eagerly (PSO_GRAPH=0)."""
     import torch  # noqa: F401  (loads the NCCL the library resolves)
     monkeypatch.setenv("PSO_FORCE_EXCHANGE", "1")
+    keep_cluster(monkeypatch, d)
     if mode.endswith("-eager"):
         monkeypatch.setenv("PSO_GRAPH", "0")
     comm = fp.nccl_comm_init(1, fp.nccl_unique_id(), 0, 0)
@@ -577,7 +595,7 @@ def test_wide_rows_cluster_path(obj, n, d, monkeypatch):
     Above PSO_D_AUTO_COLSPLIT a single GPU picks the column split, so the
     cluster is requested there (PSO_CLUSTER)."""
     if d > fp.PSO_D_AUTO_COLSPLIT:
-        monkeypatch.setenv("PSO_CLUSTER", "16")
+        monkeypatch.setenv("PSO_CLUSTER", "4" if d <= 16384 else "16")
     g = gpu_swarm(n, d, obj, seed=d + obj)
     assert g.info()["cluster"] >= 2
     c = cpu_swarm(n, d, obj, seed=d + obj)
@@ -647,6 +665,7 @@ def test_nvlink_peer_exchange_single_rank(obj, n, d, monkeypatch):
     kernel per iteration."""
     import torch  # noqa: F401
     monkeypatch.setenv("PSO_FORCE_EXCHANGE", "1")
+    keep_cluster(monkeypatch, d)
     comm = fp.nccl_comm_init(1, fp.nccl_unique_id(), 0, 0)
     try:
         g = gpu_swarm(n, d, obj, seed=8, nccl_comm=comm)
@@ -714,6 +733,7 @@ def test_lazy_pbest_rows_lockstep(obj, n, d, monkeypatch):
     several iterations with both transitions, PB (materialised by get_state),
     pf and X/V equal the oracle's and the eager kernel's bit for bit."""
     monkeypatch.setenv("PSO_RESIDENT", "0")
+    keep_cluster(monkeypatch, d)
     g = gpu_swarm(n, d, obj, seed=77)
     assert g.info()["lazy_pb"] == 1
     monkeypatch.setenv("PSO_LAZY_PB", "0")
@@ -746,6 +766,8 @@ def test_lazy_rows_skip_r1_signed_zeros(w, c1, c2, obj, n, d, kw, monkeypatch):
     c = 0 (c2 = 0, or g == x).  Negative and zero c1 give b = -0 / +0.  Lazy and
     eager kernels and the oracle agree bit for bit (signs of zero included)."""
     monkeypatch.setenv("PSO_RESIDENT", "0")
+    if not kw:
+        keep_cluster(monkeypatch, d)
     g = gpu_swarm(n, d, obj, seed=5, w=w, c1=c1, c2=c2, **kw)
     c = cpu_swarm(n, d, obj, seed=5, w=w, c1=c1, c2=c2)
     if not kw:
@@ -777,6 +799,7 @@ def test_row_order_is_invisible(obj, n, d, monkeypatch):
     call (many rows per CTA, the wide 512-thread kernel at d = 4096, fewer rows
     than CTAs, the cluster kernel at d = 12000)."""
     monkeypatch.setenv("PSO_RESIDENT", "0")
+    keep_cluster(monkeypatch, d)
     monkeypatch.setenv("PSO_SERP", "1")
     monkeypatch.setenv("PSO_L2PF_ALL", "1")
     monkeypatch.setenv("PSO_DYN_ROWS", "3")  # claims on every streaming path, the cluster too
@@ -872,6 +895,59 @@ def test_column_split_lockstep_and_wide_rows(obj, n, d):
         assert_bitwise(G, PB2[gi], "G == PB[gi]")
     info = g.info()
     assert info["launches"] >= 2 + 2 * 4
+
+
+@pytest.mark.parametrize("obj,n,d,vmax", [(GRIEWANK, 48, 3001, 40.0), (ROSENBROCK, 24, 5003, 0.3),
+                                          (SPHERE, 40, 2049, 2.0), (RASTRIGIN, 6, 20001, 0.5)])
+def test_column_split_position_slots_lockstep(obj, n, d, vmax):
+    """The column split keeps a row's position and pbest in two slots (the X
+    and PB arrays, pbx bit 1) and never copies a pbest: a lazy row (improved
+    in the last decision) stores x' into the other slot, so its old x stays
+    as the pbest.  Step by step against the oracle with the state read by
+    get_rows, which resolves the slots without restoring the plain layout, so
+    every slot transition (plain -> lazy -> swapped -> lazy in the other slot
+    ...) runs on the device over several iterations; get_state (which
+    restores the plain layout) then returns the same bits, and a twin run
+    that was never read equals the read one after further steps."""
+    seed = 900 + d
+    g = gpu_swarm(n, d, obj, seed=seed, vmax=vmax, column_split=True)
+    twin = gpu_swarm(n, d, obj, seed=seed, vmax=vmax, column_split=True)
+    assert g.info()["column_split"] == 1
+    c = cpu_swarm(n, d, obj, seed=seed, vmax=vmax, create=False)
+    idx = np.arange(n)
+    imps, T = 0, 8
+    for it in range(T):
+        X, V, PB, pf = g.get_rows(idx)
+        c.set_state(X, V, PB, pf, t=it)
+        g.step(1)
+        c.step(1)
+        X2, V2, PB2, pf2 = g.get_rows(idx)
+        assert_bitwise(X2, c.X, f"X, iteration {it + 1}")
+        assert_bitwise(V2, c.V, f"V, iteration {it + 1}")
+        tol = fit_tol(obj, c.X, c.f)
+        amb = np.abs(c.f.astype(np.float64) - pf.astype(np.float64)) <= tol
+        c_imp = c.f < pf
+        g_imp = (pf2.view(np.uint32) != pf.view(np.uint32)) | (PB2 != PB).any(axis=1)
+        assert ((g_imp == c_imp) | amb).all()
+        agree = (g_imp == c_imp) & ~amb
+        assert_bitwise(PB2[agree], c.PB[agree], f"PB, iteration {it + 1}")
+        assert_fitness_close(obj, c.X[agree & c_imp], pf2[agree & c_imp], c.pf[agree & c_imp], "pf")
+        gf, gi, G = g.gbest()
+        assert_bitwise(G, PB2[gi], "G == PB[gi]")
+        imps += int(c_imp.sum())
+    assert 0 < imps < n * T  # both pbest branches, so lazy rows turn plain and plain rows lazy
+    twin.step(T)
+    Xr, Vr, PBr, pfr = g.get_rows(idx)
+    for a, b in zip(twin.get_rows(idx), (Xr, Vr, PBr, pfr)):
+        assert_bitwise(a, b, "a run read with get_rows equals one that was not")
+    X, V, PB, pf, t = g.get_state()
+    for a, b in zip((X, V, PB, pf), (Xr, Vr, PBr, pfr)):
+        assert_bitwise(a, b, "get_state (plain layout) equals get_rows (slots)")
+    g.step(3)
+    twin.step(3)
+    for a, b in zip(g.get_state()[:4], twin.get_state()[:4]):
+        assert_bitwise(a, b, "stepping after the layout was restored")
+    assert_bitwise(g.gbest()[2], twin.gbest()[2], "G")
 
 
 @pytest.mark.parametrize("n,d,forced", [(6, 6001, True), (3, 20001, False)])

@@ -45,10 +45,16 @@ for kernel in ("reg", "tma"):
 run("lazy+prefetch", 4, 300, 2000, steps=4, env={"PSO_RESIDENT": "0", "PSO_L2PF_ALL": "1"})
 run("cta-resident", 1, 32, 10, steps=10)
 run("grid-resident", 2, 256, 1000, steps=5)
-run("cluster", 3, 5, 12000, steps=3)
+run("cluster", 3, 5, 12000, steps=3, env={"PSO_CLUSTER": "4"})
 run("cluster-C16", 4, 3, 40000, steps=2, env={"PSO_CLUSTER": "16"})
 run("colsplit-auto", 2, 3, 20001, steps=3)
 run("colsplit", 3, 9, 999, steps=3, column_split=True)
+run("colsplit-auto2", 4, 6, 12000, steps=3)
+# position/pbest slots through every transition (mixed improvements), G cache over 9 tiles
+run("colsplit-slots", 1, 40, 2049, steps=8, column_split=True, vmax=2.0)
+bw = np.stack([np.full(12000, -0.5, np.float32), np.full(12000, 0.5, np.float32),
+               np.full(12000, -2.0, np.float32), np.full(12000, 2.0, np.float32)])
+run("colsplit-bounds", 3, 6, 12000, steps=3, bounds=bw)
 b = np.stack([np.full(1000, -0.5, np.float32), np.full(1000, 0.5, np.float32),
               np.full(1000, -3.0, np.float32), np.full(1000, 4.0, np.float32)])
 run("bounds", 2, 40, 1000, steps=3, bounds=b)
