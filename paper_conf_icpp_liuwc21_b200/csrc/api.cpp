@@ -484,10 +484,12 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
   // 708 us/iteration, 12288 x 10240: 482 -> 440; Rastrigin 12288 x 9728: 522
   // -> 484); at d <= 9216 the 4-CTA cluster stays (12288 x 9216: 473 vs 512).
   // PSO_CLUSTER (tuning) keeps the cluster.
-  if (!colsplit && !o.nccl_comm && o.world <= 1 && d > PSO_D_AUTO_COLSPLIT && !std::getenv("PSO_CLUSTER"))
+  // PSO_COLSPLIT (tuning): 1 = the column split for any d, 0 = never automatically
+  const char* cs = std::getenv("PSO_COLSPLIT");
+  if (!colsplit && !o.nccl_comm && o.world <= 1 && d > PSO_D_AUTO_COLSPLIT && !std::getenv("PSO_CLUSTER") &&
+      !(cs && *cs == '0'))
     colsplit = true;
-  if (const char* cs = std::getenv("PSO_COLSPLIT"))  // tuning: 1 = column split for any d
-    if (*cs == '1') colsplit = true;
+  if (cs && *cs == '1') colsplit = true;
   if (colsplit && (o.flags & PSO_FLAG_ASYNC_GBEST))
     return fail(PSO_ERR_INVALID, "PSO_FLAG_COLUMN_SPLIT excludes PSO_FLAG_ASYNC_GBEST");
   if (!finite(w) || !finite(c1) || !finite(c2))

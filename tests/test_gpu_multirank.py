@@ -147,7 +147,7 @@ WORLDS = [(2, RASTRIGIN, 300, 1000), (2, GRIEWANK, 41, 13), (2, ROSENBROCK, 6, 1
 
 
 @pytest.mark.parametrize("world,obj,n,d", WORLDS)
-def test_processes_nvlink_exchange_match_the_oracle(tmp_path, world, obj, n, d):
+def test_processes_nvlink_exchange_match_the_oracle(tmp_path, world, obj, n, d, monkeypatch):
     """Each rank's shard after every call equals the oracle run as `world`
     virtual particle shards (X, V, PB bitwise, pf within the
     fitness tolerance, (gi, G) the oracle's), replayed call by call from the
@@ -170,7 +170,9 @@ def test_processes_nvlink_exchange_match_the_oracle(tmp_path, world, obj, n, d):
     skip_state, skip_g = oracle_lockstep(make_oracle, obj, snaps, _oracle_ops(ops, snaps),
                                          f"world={world}")
     assert skip_state <= 1 and skip_g <= 2, (skip_state, skip_g)
-    # world invariance: the single-process run of the same ops
+    # world invariance: the single-process run of the same ops (on the ranks'
+    # row kernel: one GPU alone would take the column split above d = 9216)
+    monkeypatch.setenv("PSO_COLSPLIT", "0")
     ref = fp.Swarm(n, d, 0.9, 2.0, 2.0, lo, hi, obj, seed, device=0)
     rsnaps = _run_ops(ref, ops)
     for j, (a, b) in enumerate(zip(snaps, rsnaps)):

@@ -41,10 +41,11 @@ def cpu_swarm(n, d, obj, seed=2021, w=0.9, c1=2.0, c2=2.0, vmax=0.0, create=True
 
 def keep_cluster(monkeypatch, d):
     """Rows of d in (PSO_D_AUTO_COLSPLIT, 16384] take the column split on one
-    GPU; tests that exercise the row kernels there (the 4-CTA cluster: lazy vs
-    eager pbest, the exchanges against a single-GPU twin) ask for the cluster."""
+    GPU; tests that exercise the row kernels there (the cluster: lazy vs eager
+    pbest, the exchanges against a single-GPU twin) switch the automatic
+    column split off (PSO_COLSPLIT=0: the planner's own cluster)."""
     if fp.PSO_D_AUTO_COLSPLIT < d <= 16384:
-        monkeypatch.setenv("PSO_CLUSTER", "4")
+        monkeypatch.setenv("PSO_COLSPLIT", "0")
 
 
 # ------------------------------------------------------------------ Philox
