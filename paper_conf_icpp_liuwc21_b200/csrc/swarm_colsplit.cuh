@@ -127,6 +127,9 @@ __global__ void __launch_bounds__(kColCompute + 64, 2)
         k_next = k_nn;
         if (i >= stages) mbar_wait(&empty[s], ph ^ 1u);
         float4* st = ring + (size_t)s * per * chunk;
+        PSO_DCHECK(r >= 0 && r < n && b >= 0 && b < nb && cnt >= 1 && cnt <= chunk && s < stages);
+        PSO_DCHECK((size_t)((const unsigned char*)(st + per * chunk) - dsmem) <= dyn_smem_bytes());
+        PSO_DCHECK((size_t)q0 + cnt <= (size_t)nvl && stages <= kMaxStages);
         s_r[s] = r;
         s_b[s] = b;
         if (init) {
@@ -145,6 +148,8 @@ __global__ void __launch_bounds__(kColCompute + 64, 2)
             if (gs) g_tile1 = b; else g_tile0 = b;
           }
           if (gs) g_last1 = i; else g_last0 = i;
+          PSO_DCHECK(gs == 0 || gs == 1);
+          PSO_DCHECK((gs ? g_tile1 : g_tile0) == b);
           s_g[s] = gs;
           sflag[s] = fl;
           const bool lazy = (fl & 1) != 0;
@@ -457,6 +462,8 @@ __global__ void __launch_bounds__(kColDecideThreads) k_col_decide(const __grid_c
   }
   __syncthreads();
   const unsigned long long acc = s_best[0], cur = s_best[1];
+  PSO_DCHECK(acc >= cur || ((long long)(uint32_t)acc >= a.row_begin &&
+                            (long long)(uint32_t)acc - a.row_begin < a.n_local));
   if (acc < cur) {  // the block is up to 1 MB: 8 independent loads in flight per thread
     const float4* x = reinterpret_cast<const float4*>((s_nimp[0] & 2u) ? a.PB : a.X) +
                       ((long long)(uint32_t)acc - a.row_begin) * a.nvec;
