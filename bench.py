@@ -66,7 +66,7 @@ def _path_name(info) -> str:
         return "column-split (%d tiles per row)" % info["col_tiles"]
     if info["cluster"]:
         return "cluster (%d CTAs per row)" % info["cluster"]
-    return ["streaming", "cta-resident", "grid-resident"][info["resident"]]
+    return ["streaming", "cta-resident", "grid-resident", "persistent-streaming"][info["resident"]]
 
 
 def ncu_traffic(workload_name):
@@ -402,7 +402,7 @@ def run_gpu(args, w):
     # pbest equals x skips both); pf read + written on improvement
     pbl = info["pb_loads"] / max(n_local * K, 1)
     pbs = info["pb_stores"] / max(n_local * K, 1)
-    if info["resident"]:  # state held in shared memory: no per-iteration row traffic counted
+    if info["resident"] in (1, 2):  # state held in shared memory: no per-iteration row traffic counted
         pbl, pbs = 1.0, rho
     bytes_per_update = 16.0 + 4.0 * pbl + 4.0 * pbs
     alg_bytes = n_local * w.d * bytes_per_update + n_local * (4.0 + 4.0 * rho)

@@ -253,7 +253,10 @@ typedef struct {
   int32_t resident;              /* 0: streaming kernel, one launch per iteration;
                                     1: tiny swarm held in one CTA's shared memory,
                                     2: swarm held in the whole grid's shared memory
-                                    (cooperative launch); 1 and 2 run a whole
+                                    (cooperative launch), 3: persistent streaming
+                                    kernel (rows streamed from HBM every iteration,
+                                    a grid barrier per iteration; opt-in with the
+                                    PSO_PERSIST=1 tuning variable); 1-3 run a whole
                                     pso_step call in one launch (single GPU only) */
   int32_t bounds;                /* 1: per-dimension bounds in use */
   int32_t cluster;               /* > 0: each row is split in column blocks over a

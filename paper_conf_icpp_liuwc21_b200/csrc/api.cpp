@@ -320,6 +320,7 @@ pso_status reset_ctl(pso_swarm* h, uint32_t t) {
   DevCtl c{};
   c.key_cur = ~0ull;
   c.key_acc = ~0ull;
+  c.key_acc1 = ~0ull;
   c.improvements = 0;
   c.done = 0;
   c.t = t;
@@ -631,6 +632,7 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
   if (!colsplit) {
     const char* v = std::getenv("PSO_RESIDENT");
     hints.allow_resident = !h->xchg && hints.kernel == -1 && !(v && !std::strcmp(v, "0"));
+    if (const char* pv = std::getenv("PSO_PERSIST")) hints.persist = std::atoi(pv) ? 1 : 0;
     hints.bounds = o.bounds != nullptr;
   }
   if (!colsplit) {
@@ -659,8 +661,10 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
   const size_t pbxb = lazy ? align_up(rows, 256) : 0;
   const size_t rec = align_up(record_bytes(h->pitch), 256);
   // grid-resident kernel: [2 parities][grid] candidate rows, then their keys
-  const size_t cand_rows = h->cfg.gridres ? align_up(2 * (size_t)h->cfg.gridres_grid * h->pitch * 4, 256) : 0;
-  const size_t candb = h->cfg.gridres ? cand_rows + align_up(2 * (size_t)h->cfg.gridres_grid * 8, 256) : 0;
+  // grid-resident / persistent kernels: [2 parities][grid] candidate rows (+ keys for the former)
+  const int cand_grid = h->cfg.gridres ? h->cfg.gridres_grid : h->cfg.persist ? h->cfg.persist_grid : 0;
+  const size_t cand_rows = cand_grid ? align_up(2 * (size_t)cand_grid * h->pitch * 4, 256) : 0;
+  const size_t candb = h->cfg.gridres ? cand_rows + align_up(2 * (size_t)h->cfg.gridres_grid * 8, 256) : cand_rows;
   const size_t sendb = (h->xchg && !colsplit) ? rec : 0;
   const size_t recvb = colsplit ? col_tag_bytes(h->world) + 2 * rows * (size_t)col_nbt * 16
                        : h->xchg ? 4 * (size_t)h->world * record_bytes(h->pitch) : 0;
@@ -701,7 +705,7 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
   if (const char* v = std::getenv("PSO_DYN_ROWS")) A.dyn_rows = std::atoi(v) & 3;
   A.serp = 1;  // measured: C3 36.9 -> 35.7 us (120 MB state, L2-borderline), NS / C4 within 1 %
   if (const char* v = std::getenv("PSO_SERP")) A.serp = std::atoi(v) != 0;
-  A.cand = h->cfg.gridres ? (float*)p : nullptr;
+  A.cand = cand_grid ? (float*)p : nullptr;
   A.cand_key = h->cfg.gridres ? (unsigned long long*)(p + cand_rows) : nullptr;
   p += candb;
   A.G_view = async ? (float*)p : nullptr; p += viewb;
@@ -798,7 +802,7 @@ pso_status pso_step(pso_handle h, int64_t iters) {
     h->t += (uint64_t)iters;
     return PSO_OK;
   }
-  if (h->cfg.resident || h->cfg.gridres) {  // the whole call is one launch
+  if (h->cfg.resident || h->cfg.gridres || h->cfg.persist) {  // the whole call is one launch
     for (int64_t done = 0; done < iters;) {
       const int chunk = (int)((iters - done) < (1 << 30) ? (iters - done) : (1 << 30));
       pso_swarm::Timed* ev = nullptr;
@@ -806,6 +810,8 @@ pso_status pso_step(pso_handle h, int64_t iters) {
       if (ev) PSO_CUDA(h, cudaEventRecord(ev->start, h->stream));
       if (h->cfg.resident)
         PSO_CUDA(h, launch_resident(h->objective, h->args, h->cfg, chunk, h->stream));
+      else if (h->cfg.persist)
+        PSO_CUDA(h, launch_persist(h->objective, h->args, h->cfg, chunk, h->stream));
       else
         PSO_CUDA(h, launch_gridres(h->objective, h->args, h->cfg, chunk, h->stream));
       ++h->launches;
@@ -1122,7 +1128,7 @@ pso_status pso_get_info(pso_handle h, pso_info* info) {
   info->tma_pipeline = h->cfg.tma;
   info->pipeline_stages = h->cfg.stages;
   info->smem_bytes = (int32_t)(h->cfg.resident ? h->cfg.resident_smem : h->cfg.smem);
-  info->resident = h->cfg.resident ? 1 : (h->cfg.gridres ? 2 : 0);
+  info->resident = h->cfg.resident ? 1 : h->cfg.gridres ? 2 : h->cfg.persist ? 3 : 0;
   info->bounds = h->args.bounds ? 1 : 0;
   info->cluster = h->cfg.cluster;
   if (h->cfg.resident) {
@@ -1134,6 +1140,7 @@ pso_status pso_get_info(pso_handle h, pso_info* info) {
     info->grid = h->cfg.gridres_grid;
     info->smem_bytes = (int32_t)h->cfg.gridres_smem;
   }
+  if (h->cfg.persist) info->grid = h->cfg.persist_grid;
   info->vmax = h->vmax;
   info->t = h->t;
   info->launches = h->launches;

@@ -17,7 +17,7 @@ struct DevCtl {
   unsigned int t;                   // iterations done (low 32 bits; Philox ctr[2])
   unsigned long long row_claim;     // TMA streaming kernel, dynamic rows: rows claimed beyond the
                                     // grid's first (reset by the iteration's last CTA)
-  unsigned long long spare;
+  unsigned long long key_acc1;      // persistent kernel: the atomicMin slot of odd iterations
   unsigned int bar_count, bar_gen;  // grid-resident kernel: grid barrier
   unsigned long long pb_loads;      // streaming kernels: pbest rows read from HBM
   unsigned long long pb_stores;     // streaming kernels: pbest rows written to HBM
@@ -139,6 +139,8 @@ struct LaunchCfg {
   size_t smem = 0;    // dynamic shared memory bytes of the step kernel
   int resident = 0;   // 1: tiny swarm, whole pso_step in one single-CTA launch
   int gridres = 0;    // 1: swarm held in the grid's shared memory (cooperative launch)
+  int persist = 0;    // 1: persistent streaming kernel, a whole pso_step per cooperative launch
+  int persist_grid = 0;
   int cluster = 0;    // > 0: rows split across a thread-block cluster of this many CTAs
   int chunk = 0;      // float4 per CTA block in the cluster path
   int init_threads = 0;
@@ -163,6 +165,7 @@ struct PlanHints {
   int stages = 0;
   int ctas = 0;     // max CTAs per SM for the TMA pipeline (0: auto = 2)
   bool allow_resident = false;  // single-GPU tiny swarms (PSO_RESIDENT=0 disables)
+  int persist = -1;             // persistent streaming kernel: -1 auto, 0 off, 1 on (PSO_PERSIST)
   bool bounds = false;          // per-dimension bounds tables are in use
   int cluster = 0;              // force the cluster path with this many CTAs (PSO_CLUSTER)
 };
@@ -175,6 +178,7 @@ struct KernelTable {
   const void* step_tma_w[4][2];  // 512 compute threads, one CTA per SM (VPT 2 and 4 only)
   const void* gridres[4][2];
   const void* step_cluster[4][2];
+  const void* persist[4][2];     // persistent streaming kernel (swarm_persist.cuh)
   const void* resident[2];
   const void* init[4];
   const void* eval[4];
@@ -193,6 +197,8 @@ cudaError_t launch_step(int objective, const SwarmArgs& a, const LaunchCfg& c, c
 cudaError_t launch_resident(int objective, const SwarmArgs& a, const LaunchCfg& c, int iters,
                             cudaStream_t s);
 cudaError_t launch_gridres(int objective, const SwarmArgs& a, const LaunchCfg& c, int iters,
+                           cudaStream_t s);
+cudaError_t launch_persist(int objective, const SwarmArgs& a, const LaunchCfg& c, int iters,
                            cudaStream_t s);
 // Column split (NEXT-3): tile plan for this rank's block, and the two kernels
 // of an iteration (init = 1: Alg. 1 lines 1-3 instead of the move).

@@ -260,6 +260,12 @@ void shape_for(int nvec, int vpt_override, int* vpt, int* threads, int max_threa
 constexpr size_t kSmemPerSm = 228 * 1024;       // B200 unified L1/shared per SM
 constexpr size_t kSmemPerCtaMax = 227 * 1024;   // opt-in maximum per CTA
 constexpr size_t kStaticReserve = 4096;         // static shared (<= 3 KB) + per-CTA reservation
+// persistent streaming kernel: used automatically up to this many rows per CTA.
+// 0 = opt-in only (PSO_PERSIST=1): measured faster where most rows are lazy
+// (Griewank 10000 x 2000: 66.1 -> 56.6 us per iteration) but slower on C3
+// (Rosenbrock 10000 x 1000: 34.4 -> 37.3 us) and NS_R8 (75.9 -> 80.3 us), and
+// the lazy share is not known when the plan is made.
+constexpr long long kPersistMaxRowsPerCta = 0;
 constexpr long long kResidentElems = 8192;      // resident path: n d <= this
 
 }  // namespace
@@ -395,7 +401,7 @@ cudaError_t plan_launch(int objective, int d, long long n_local, int sm_count, c
   const size_t first = nb ? (size_t)nvec * 4 : 0;
   cfg->bounds = h.bounds ? 1 : 0;
   cfg->init_smem = 0;
-  cfg->resident = cfg->gridres = cfg->cluster = 0;
+  cfg->resident = cfg->gridres = cfg->cluster = cfg->persist = 0;
   cudaError_t e;
 
   // init kernel: one CTA per row, looping over the row's float4s
@@ -535,7 +541,7 @@ cudaError_t plan_launch(int objective, int d, long long n_local, int sm_count, c
   cfg->grid = (int)grid;
 
   // ---- grid-resident path: the whole swarm in the grid's shared memory
-  if (h.allow_resident && !cfg->resident && cfg->tma && nvec >= 64) {
+  if (h.allow_resident && !cfg->resident && cfg->tma && nvec >= 64 && h.persist != 1) {
     const void* fn = tab->gridres[vi][bi];
     for (int per = cfg->ctas_per_sm; per >= 1 && !cfg->gridres; --per) {
       long long g = (long long)per * sm_count;
@@ -559,6 +565,29 @@ cudaError_t plan_launch(int objective, int d, long long n_local, int sm_count, c
       cfg->gridres_grid = (int)g;
       cfg->gridres_rows = (int)rows;
       cfg->gridres_smem = smem;
+    }
+  }
+
+  // ---- persistent streaming kernel (swarm_persist.cuh): the narrow TMA shape,
+  // a whole pso_step call per cooperative launch, for swarms whose rows per CTA
+  // are few enough that the per-iteration kernel boundary shows (PSO_PERSIST=1
+  // forces it, 0 disables it)
+  if (h.allow_resident && !cfg->resident && !cfg->gridres && cfg->tma && !cfg->wide && h.persist != 0) {
+    const long long rows_per_cta = (n_local + cfg->grid - 1) / cfg->grid;
+    if (h.persist == 1 || rows_per_cta <= kPersistMaxRowsPerCta) {
+      const void* fn = tab->persist[vi][bi];
+      if ((e = allow_dynamic_smem(fn, cfg->smem)) != cudaSuccess) return e;
+      int occ = 0;
+      if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, cfg->threads, cfg->smem)) !=
+          cudaSuccess)
+        return e;
+      const int per = occ < cfg->ctas_per_sm ? occ : cfg->ctas_per_sm;
+      long long g = (long long)per * sm_count;
+      if (g > n_local) g = n_local;
+      if (per >= 1 && g >= 1) {
+        cfg->persist = 1;
+        cfg->persist_grid = (int)g;
+      }
     }
   }
   return cudaSuccess;
@@ -615,6 +644,16 @@ cudaError_t launch_gridres(int objective, const SwarmArgs& a, const LaunchCfg& c
   void* args[] = {const_cast<SwarmArgs*>(&a), &iters};
   return cudaLaunchCooperativeKernel(t->gridres[vpt_index(c.vpt)][c.bounds ? 1 : 0],
                                      dim3(c.gridres_grid), dim3(c.compute), args, c.gridres_smem, s);
+}
+
+cudaError_t launch_persist(int objective, const SwarmArgs& a, const LaunchCfg& c, int iters,
+                           cudaStream_t s) {
+  const KernelTable* t = kernel_table(objective);
+  if (!t) return cudaErrorInvalidDeviceFunction;
+  int stages = c.stages;
+  void* args[] = {const_cast<SwarmArgs*>(&a), &iters, &stages};
+  return cudaLaunchCooperativeKernel(t->persist[vpt_index(c.vpt)][c.bounds ? 1 : 0],
+                                     dim3(c.persist_grid), dim3(c.threads), args, c.smem, s);
 }
 
 cudaError_t launch_init(int objective, const SwarmArgs& a, const LaunchCfg& c, cudaStream_t s) {

@@ -2172,6 +2172,7 @@ __global__ void __launch_bounds__(kMaxThreads) k_eval(const float* X, long long 
 }
 
 #include "swarm_colsplit.cuh"
+#include "swarm_persist.cuh"
 
 template <class Obj>
 KernelTable make_kernel_table() {
@@ -2189,6 +2190,7 @@ KernelTable make_kernel_table() {
   t.step_tma_w[2][1] = (const void*)k_step_tma<Obj, 4, true, kMaxThreadsWide>;
   PSO_ALLV(gridres, k_gridres)
   PSO_ALLV(step_cluster, k_step_cluster)
+  PSO_ALLV(persist, k_step_persist)
 #undef PSO_ALLV
 #undef PSO_T
   t.resident[0] = (const void*)k_resident<Obj, false>;

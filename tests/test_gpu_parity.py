@@ -584,6 +584,75 @@ def test_set_bounds_requires_bounds_handle():
     assert e.value.status == 1
 
 
+# ------------------------------------------------------------------ persistent streaming kernel
+@pytest.mark.parametrize("obj,n,d,kw", [(ROSENBROCK, 3000, 1000, {}), (GRIEWANK, 2000, 2000, {}),
+                                        (RASTRIGIN, 1500, 4096, {}), (SPHERE, 60, 3001, {}),
+                                        (EASOM, 700, 999, {"bounds": True}), (ACKLEY, 5000, 256, {})])
+def test_persistent_kernel_bitwise_equals_streaming(obj, n, d, kw, monkeypatch):
+    """k_step_persist (a whole pso_step call per cooperative launch; every CTA
+    streams a fixed set of rows through the TMA ring for every iteration, the
+    gbest settled by a grid barrier and a candidate-row pull) against the
+    per-iteration streaming kernel: X, V, PB, pf, the gbest index and G bitwise
+    after calls of 1, 2, 5 and 3 iterations, across a set_state, and with fewer
+    rows than CTAs (n = 60: most CTAs own no row)."""
+    lo, hi = DOMAINS[obj]
+    bk = {}
+    if kw.get("bounds"):
+        bk["bounds"] = _dim_bounds(d, 7)
+    monkeypatch.setenv("PSO_PERSIST", "1")
+    g = fp.Swarm(n, d, 0.9, 2.0, 2.0, lo, hi, obj, 99, device=0, **bk)
+    monkeypatch.setenv("PSO_PERSIST", "0")
+    monkeypatch.setenv("PSO_RESIDENT", "0")
+    e = fp.Swarm(n, d, 0.9, 2.0, 2.0, lo, hi, obj, 99, device=0, **bk)
+    assert g.info()["resident"] == 3 and e.info()["resident"] == 0
+    assert g.info()["lazy_pb"] == e.info()["lazy_pb"]
+    for k in (1, 2, 5, 3):
+        g.step(k)
+        e.step(k)
+        for x, y, nm in zip(g.get_state(), e.get_state(), "X V PB pf t".split()):
+            if nm == "t":
+                assert x == y
+            else:
+                assert_bitwise(x, y, f"persistent vs streaming {nm}")
+        gf, gi, G = g.gbest()
+        ef, ei, EG = e.gbest()
+        assert (gf, gi) == (ef, ei)
+        assert_bitwise(G, EG, "G")
+    X, V, PB, pf, t = e.get_state()
+    rng = np.random.default_rng(5)
+    pf = (pf * rng.choice([0.5, 2.0], size=n)).astype(np.float32)  # both pbest branches
+    g.set_state(X, V, PB, pf, t=t)
+    e.set_state(X, V, PB, pf, t=t)
+    g.step(4)
+    e.step(4)
+    for x, y, nm in zip(g.get_state()[:4], e.get_state()[:4], "X V PB pf".split()):
+        assert_bitwise(x, y, f"after set_state {nm}")
+    assert g.gbest()[:2] == e.gbest()[:2]
+    # one step launch per call instead of one per iteration (15 iterations in 5 calls)
+    assert g.info()["launches"] <= e.info()["launches"] - 10
+
+
+def test_persistent_kernel_matches_the_oracle(monkeypatch):
+    """C3's shape at a tenth of its rows through k_step_persist against the
+    oracle run from the same seed: X bit-exact after 1 + 4 iterations, the
+    gbest index and fitness."""
+    monkeypatch.setenv("PSO_PERSIST", "1")
+    n, d, obj = 1000, 1000, ROSENBROCK
+    g = gpu_swarm(n, d, obj, seed=17)
+    assert g.info()["resident"] == 3
+    c = cpu_swarm(n, d, obj, seed=17)
+    for k in (1, 4):
+        g.step(k)
+        c.step(k)
+        X, V, PB, pf, t = g.get_state()
+        assert_bitwise(X, c.X, "X vs oracle")
+        assert_bitwise(V, c.V, "V vs oracle")
+        assert_fitness_close(obj, c.PB, pf, c.pf, "pf")
+        gf, gi, G = g.gbest()
+        assert gi == c.gi
+        assert_bitwise(G, PB[gi], "G == PB[gi]")
+
+
 # ------------------------------------------------------------------ wide rows (NEXT-3)
 WIDE = [(5, 8193), (3, 10000), (4, 16384), (2, 65536)]
 

@@ -60,7 +60,7 @@ def main():
             times.append(dt)
             fits.append(f)
         m = statistics.mean(times)
-        path = ["streaming", "cta-resident", "grid-resident"][info["resident"]]
+        path = ["streaming", "cta-resident", "grid-resident", "persistent-streaming"][info["resident"]]
         print(f"{NAMES[obj]:9s} {m * 1e3:8.2f} ms  ({N * D * T / m:.3e} updates/s; path {path}; "
               f"min {min(times) * 1e3:.2f} ms)  mean gbest {statistics.mean(fits):.6g}  |  "
               f"paper, V100: {PAPER_V100_S[obj]:.2f} s ({N * D * T / PAPER_V100_S[obj]:.3e} updates/s)"

@@ -26,7 +26,7 @@ def run(tag, obj, n, d, steps=3, env=None, **kw):
         X, V, PB, pf, t = s.get_state()
         info = s.info()
         path = ("colsplit" if info["column_split"] else "cluster" if info["cluster"] else
-                ["", "cta-resident", "grid-resident"][info["resident"]] if info["resident"] else
+                ["", "cta-resident", "grid-resident", "persistent"][info["resident"]] if info["resident"] else
                 "tma" if info["tma_pipeline"] else "reg")
         print(f"{tag:14s} obj={obj} n={n} d={d} path={path} lazy={info['lazy_pb']} f={f:.6g} i={i} "
               f"t={t}", flush=True)
