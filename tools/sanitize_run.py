@@ -45,6 +45,8 @@ for kernel in ("reg", "tma"):
 run("lazy+prefetch", 4, 300, 2000, steps=4, env={"PSO_RESIDENT": "0", "PSO_L2PF_ALL": "1"})
 run("cta-resident", 1, 32, 10, steps=10)
 run("grid-resident", 2, 256, 1000, steps=5)
+run("persistent", 3, 3000, 1000, steps=5, env={"PSO_PERSIST": "1"})
+run("persistent-few", 1, 60, 2001, steps=4, env={"PSO_PERSIST": "1"})
 run("cluster", 3, 5, 12000, steps=3, env={"PSO_CLUSTER": "4"})
 run("cluster-C16", 4, 3, 40000, steps=2, env={"PSO_CLUSTER": "16"})
 run("colsplit-auto", 2, 3, 20001, steps=3)
