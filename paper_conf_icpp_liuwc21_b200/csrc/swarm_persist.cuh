@@ -82,12 +82,20 @@ __global__ void __maxnreg__(80)
         // (a CTA without rows never waits: its finaliser's phases run ahead)
         if (it > 0 && myrows > 0) mbar_wait(&itdone, (unsigned)((it - 1) & 1));
         const uint32_t t = t0 + 1u + (uint32_t)it;
+        // lazy flags loaded one row ahead (their L2 latency overlaps the wait for
+        // a free stage instead of delaying the copies), as in k_step_tma
+        const bool lz = a.lazy_pb != 0;
+        int fl_next = (lz && myrows > 0) ? (int)a.pbx[row_of(t, 0)] : 0;
+        int pfl_next = (pd && lz && pd < myrows) ? (int)a.pbx[row_of(t, pd)] : 0;
         for (int m = 0; m < myrows; ++m, ++k) {
           const long long r = row_of(t, m);
-          const int fl = a.lazy_pb ? (int)a.pbx[r] : 0;
-          if (pd && a.lazy_pb && m + pd < myrows) {
+          const int fl = fl_next;
+          if (lz && m + 1 < myrows) fl_next = a.pbx[row_of(t, m + 1)];
+          if (pd && lz && m + pd < myrows) {
             const long long r2 = row_of(t, m + pd);
-            if (a.pbx[r2] || a.l2pf_all) {
+            const int pfl = pfl_next;
+            if (m + 1 + pd < myrows) pfl_next = a.pbx[row_of(t, m + 1 + pd)];
+            if (pfl || a.l2pf_all) {
               const size_t po = (size_t)r2 * 4 * nvec;
               bulk_prefetch_l2(a.X + po, row_bytes);
               bulk_prefetch_l2(a.V + po, row_bytes);
