@@ -223,7 +223,8 @@ pso_status pso_get_state(pso_handle h, float* x, float* v, float* pb, float* pf,
 /* Synchronise and copy m rank-local rows (local indices rows[k] in [0, n_local);
  * row k is particle row_begin + rows[k]) to host buffers (any may be NULL):
  * x, v, pb: m x d floats; pf: m floats.  The state is not changed (a pbest
- * deferred by the lazy rows is read from x).  For sampling swarms too large
+ * deferred by the lazy rows is read from x; on the column split each row is
+ * read from the slot that holds it).  For sampling swarms too large
  * to copy whole (e.g. 2.9M x 4096: 142 GB).  PSO_ERR_INVALID for an index
  * outside [0, n_local) or m < 0. */
 pso_status pso_get_rows(pso_handle h, const int64_t* rows, int64_t m, float* x, float* v, float* pb,

@@ -946,7 +946,7 @@ def test_column_split_single_gpu_matches_oracle(obj, n, d):
                                      (RASTRIGIN, 3, 70001), (ROSENBROCK, 2, 65537)])
 def test_column_split_lockstep_and_wide_rows(obj, n, d):
     """Several iterations in lockstep with the oracle (the lazy pbest rows of
-    the split: deferred PB copies, materialised by get_state); d > PSO_D_MAX_ROW
+    the split: position / pbest slots, the plain layout restored by get_state); d > PSO_D_MAX_ROW
     selects the column split automatically."""
     kw = {} if d > fp.PSO_D_MAX_ROW else {"column_split": True}
     g = gpu_swarm(n, d, obj, seed=31, **kw)
