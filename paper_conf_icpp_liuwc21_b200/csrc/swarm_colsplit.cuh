@@ -260,6 +260,14 @@ __global__ void __launch_bounds__(kColCompute + 64, 2)
   const PhiloxRoundKeys& key = a.rk;
   const MoveParams mp = move_params(a);
   const float4* B4 = reinterpret_cast<const float4*>(a.bounds);
+  // Row-invariant Philox rounds of this thread's two slots (k_step_tma's
+  // PhiloxSlot, the same draws bit for bit): with items visited tile-major a
+  // CTA's consecutive items mostly share their tile, so they are recomputed
+  // only when the tile changes
+  constexpr bool kSlotRng = PSO_SLOT_PHILOX && !Obj::kNeighbor && !kB;
+  const PhiloxIter pit = philox_iter(key, t);
+  PhiloxSlot ps1[2], ps2[2];
+  int slot_b = -1;
   int s = 0;
   unsigned ph = 0;
   for (;;) {
@@ -268,6 +276,17 @@ __global__ void __launch_bounds__(kColCompute + 64, 2)
     const long long r = s_r[s];
     if (r < 0) break;
     const int q0 = s_b[s] * chunk;
+    if constexpr (kSlotRng) {
+      if (!init && s_b[s] != slot_b) {
+        slot_b = s_b[s];
+#pragma unroll
+        for (int j = 0; j < 2; ++j) {
+          const uint32_t qg = (uint32_t)(a.col_q0 + q0 + tid + j * nthr);
+          ps1[j] = philox_slot(key, pit, qg, kTagR1);
+          ps2[j] = philox_slot(key, pit, qg, kTagR2);
+        }
+      }
+    }
     const int cnt = min(chunk, nvl - q0);
     const uint32_t gi = (uint32_t)(a.row_begin + r);
     const int fl = sflag[s] & 1;  // lazy row: pb = x (its pb slot is not loaded)
@@ -306,8 +325,12 @@ __global__ void __launch_bounds__(kColCompute + 64, 2)
           const int qg = a.col_q0 + q0 + ql;
           float4 x = st[ql], v = st[chunk + ql];
           const float4 g = gc[ql];
-          move4_draw<kB>(mp, key, t, gi, (uint32_t)qg, fl, x, v, st + 2 * chunk + ql, g, gc + chunk,
-                         chunk, ql);
+          if constexpr (kSlotRng)
+            move4_draw_slot<kB>(mp, key, pit, ps1[j], ps2[j], gi, fl, x, v, st + 2 * chunk + ql, g,
+                                gc + chunk, chunk, ql);
+          else
+            move4_draw<kB>(mp, key, t, gi, (uint32_t)qg, fl, x, v, st + 2 * chunk + ql, g, gc + chunk,
+                           chunk, ql);
           if ((d & 3) && qg == a.nvec_glob - 1) {
             const int jj = 4 * qg;
             if (jj + 1 >= d) x.y = v.y = 0.f;
