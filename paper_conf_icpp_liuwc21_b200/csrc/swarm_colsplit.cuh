@@ -265,8 +265,12 @@ __global__ void __launch_bounds__(kColCompute + 64, 2)
   // CTA's consecutive items mostly share their tile, so they are recomputed
   // only when the tile changes
   constexpr bool kSlotRng = PSO_SLOT_PHILOX && !Obj::kNeighbor && !kB;
+  // likewise the functor's per-dimension factors (Griewank's 1/sqrt(k): table4 /
+  // map4r, the same bits as map4)
+  constexpr bool kTab = HasRowTable<Obj>::value && !Obj::kNeighbor;
   const PhiloxIter pit = philox_iter(key, t);
   PhiloxSlot ps1[2], ps2[2];
+  float4 rtab[2];
   int slot_b = -1;
   int s = 0;
   unsigned ph = 0;
@@ -276,14 +280,18 @@ __global__ void __launch_bounds__(kColCompute + 64, 2)
     const long long r = s_r[s];
     if (r < 0) break;
     const int q0 = s_b[s] * chunk;
-    if constexpr (kSlotRng) {
+    if constexpr (kSlotRng || kTab) {
       if (!init && s_b[s] != slot_b) {
         slot_b = s_b[s];
 #pragma unroll
         for (int j = 0; j < 2; ++j) {
           const uint32_t qg = (uint32_t)(a.col_q0 + q0 + tid + j * nthr);
-          ps1[j] = philox_slot(key, pit, qg, kTagR1);
-          ps2[j] = philox_slot(key, pit, qg, kTagR2);
+          if constexpr (kSlotRng) {
+            ps1[j] = philox_slot(key, pit, qg, kTagR1);
+            ps2[j] = philox_slot(key, pit, qg, kTagR2);
+          }
+          if constexpr (kTab)
+            rtab[j] = (int)qg < a.nvec_glob ? Obj::table4(4 * (int)qg) : make_float4(0.f, 0.f, 0.f, 0.f);
         }
       }
     }
@@ -343,7 +351,10 @@ __global__ void __launch_bounds__(kColCompute + 64, 2)
           }
           xdst[ql] = x;
           st[chunk + ql] = v;
-          if constexpr (!Obj::kNeighbor) map4<Obj>(acc, x, 0.f, 4 * qg, d);
+          if constexpr (kTab)
+            Obj::map4r(acc, x, d, rtab[j]);
+          else if constexpr (!Obj::kNeighbor)
+            map4<Obj>(acc, x, 0.f, 4 * qg, d);
         }
       }
     }
