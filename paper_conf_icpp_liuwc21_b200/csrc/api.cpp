@@ -490,7 +490,7 @@ pso_status pso_create_ex(pso_handle* out, int64_t n, int32_t d, float w, float c
   if (!colsplit && !o.nccl_comm && o.world <= 1 && d > PSO_D_AUTO_COLSPLIT && !std::getenv("PSO_CLUSTER") &&
       !(cs && *cs == '0'))
     colsplit = true;
-  if (cs && *cs == '1') colsplit = true;
+  if (cs && *cs == '1' && !o.nccl_comm && o.world <= 1) colsplit = true;  // single GPU only
   if (colsplit && (o.flags & PSO_FLAG_ASYNC_GBEST))
     return fail(PSO_ERR_INVALID, "PSO_FLAG_COLUMN_SPLIT excludes PSO_FLAG_ASYNC_GBEST");
   if (!finite(w) || !finite(c1) || !finite(c2))
