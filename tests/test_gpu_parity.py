@@ -678,7 +678,7 @@ def test_wide_rows_cluster_path(obj, n, d, monkeypatch):
     _step_and_compare(obj, n, d, seed=5100 + d, pf_mode="inf", t0=0)
 
 
-@pytest.mark.parametrize("d", [16385, 40000, 65536])
+@pytest.mark.parametrize("d", [9217, 12000, 16385, 40000, 65536])
 def test_single_gpu_wide_rows_pick_the_column_split(d):
     """One GPU, d > PSO_D_AUTO_COLSPLIT: the column split is chosen (it beats
     8- and 16-CTA clusters); results as the oracle's (init bit-exact, one step
